@@ -1,0 +1,34 @@
+# Build: libfusedpat (the product, sm_100a), liboracle (host C, test infrastructure),
+# libsynth_{host,cuda} (seeded input generators).  `make -j` or __graft_entry__.build().
+NVCC     ?= nvcc
+CC       := gcc
+ARCH     := -gencode arch=compute_100a,code=sm_100a
+NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -shared --expt-relaxed-constexpr
+CFLAGS   := -O2 -fPIC -shared -fopenmp -ffp-contract=off -std=c11 -Wall
+PKG      := paper_conf_ppopp_asharitbrcks15_b200
+CSRC     := $(PKG)/csrc
+FP_SRCS  := $(wildcard $(CSRC)/*.cu)
+FP_HDRS  := $(wildcard $(CSRC)/*.cuh) include/fusedpat.h
+
+all: fusedpat oracle synth
+
+fusedpat: $(PKG)/libfusedpat.so
+oracle: oracle/liboracle.so
+synth: synth/libsynth_host.so synth/libsynth_cuda.so
+
+$(PKG)/libfusedpat.so: $(FP_SRCS) $(FP_HDRS)
+	$(NVCC) $(NVFLAGS) -Iinclude -Xptxas -v -o $@ $(FP_SRCS) -lnccl -lcudart 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
+
+oracle/liboracle.so: oracle/oracle.c
+	$(CC) $(CFLAGS) -o $@ $< -lm
+
+synth/libsynth_host.so: synth/synth_host.c synth/synth_core.h
+	$(CC) $(CFLAGS) -o $@ $< -lm
+
+synth/libsynth_cuda.so: synth/synth_cuda.cu synth/synth_core.h
+	$(NVCC) $(NVFLAGS) -o $@ $<
+
+clean:
+	rm -f $(PKG)/libfusedpat.so oracle/liboracle.so synth/libsynth_host.so synth/libsynth_cuda.so
+
+.PHONY: all fusedpat oracle synth clean
