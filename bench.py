@@ -1,0 +1,480 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of the fused pattern w = alpha X^T (v (.) (X y)) + beta z
+(Eq. 1) on B200, per BASELINE.json:
+
+  metric: "fused-pattern GB/s of X streamed and % of B200 HBM peak; evals/s at 1/2/4/8 GPU"
+
+A step is one pattern evaluation over the whole configured matrix (all SURVEY 8(a) rows:
+plan, w init, stage y, stream X once, dot, reduce+scale, scale-back, aggregation, and at
+N > 1 the NCCL allreduce of w).  Default workload: BASELINE.json configs[1] = C2, dense fp32
+10M x 128, X^T (X y) -- the config the metric is quoted on.  X (5.12 GB) is far larger than
+the 126 MB L2, so no L2 flush is needed between steps (C1, which fits in L2, is timed with
+an explicit flush).  Inputs are synthetic (synth/, seeded), generated directly in HBM.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...     (row-sharded, strong scaling)
+
+`--impl reference` times the fp64 CPU oracle (oracle/, the only reference this tier has) on
+a bounded sample of the same workload on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "fused-pattern GB/s of X streamed and % of B200 HBM peak; evals/s at 1/2/4/8 GPU"
+FALLBACK_HBM_GBS = 6650.0
+
+
+# ------------------------------------------------------------------------------ helpers
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs: copy, read+write bytes)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def traffic_for(config):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of the dominant kernel, from the
+    committed ncu --set full capture summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p))
+    e = d.get(config)
+    return None if e is None else e.get("dram_bytes_per_launch")
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, f[5:9]):
+                if val.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_info():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+# ------------------------------------------------------------------------------ workloads
+def algorithmic_bytes(cfg, m, nnz):
+    """X once + rowptr + v + y + [beta] z + w (bytes per evaluation)."""
+    s = 8 if cfg["dtype"] == "f64" else 4
+    n = cfg["n"]
+    vec = (m * s if cfg["use_v"] else 0) + n * s + (n * s if cfg["use_z"] else 0) + n * s
+    if cfg["fmt"] == "dense":
+        xb = m * n * s
+        return xb, xb + vec
+    xb = nnz * (s + 4) + (m + 1) * 8
+    return xb, xb + vec
+
+
+def build_inputs(name, rank, world, dev):
+    """This rank's row shard of config `name`, generated in HBM (bit-identical to the slice of
+    the full matrix, synth/ is counter-based)."""
+    cfg = synth.CONFIGS[name]
+    seed = synth.config_seed(name)
+    m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
+    import paper_conf_ppopp_asharitbrcks15_b200 as fp
+
+    if cfg["fmt"] == "dense":
+        b = fp.shard_rows_dense(m, world)
+        r0, r1 = b[rank], b[rank + 1]
+        X = _dense_shard(r0, r1, n, dt, cfg["xkind"], seed, dev)
+        inp = dict(X=X, m_local=r1 - r0, nnz_local=0, row0=r0)
+    else:
+        rp_full = None
+        if world > 1:
+            # shard bounds need the global rowptr (host); row lengths are cheap to regenerate
+            thr = synth.length_table(cfg["lengths"], n)
+            rp_full = _host_rowptr(m, thr, seed)
+            b = fp.shard_rows_csr(rp_full, world)
+        else:
+            b = [0, m]
+        r0, r1 = b[rank], b[rank + 1]
+        rp, ci, va = synth.csr(r1 - r0, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed, row0=r0, device=dev)
+        inp = dict(rowptr=rp, colidx=ci, val=va, m_local=r1 - r0, nnz_local=int(va.numel()), row0=r0)
+    inp["y"] = synth.vector(n, dt, seed=seed, stream=synth.S_Y, device=dev)
+    inp["v"] = synth.vector(inp["m_local"], dt, kind="pos", seed=seed, stream=synth.S_V, i0=inp["row0"],
+                            device=dev) if cfg["use_v"] else None
+    inp["z"] = synth.vector(n, dt, seed=seed, stream=synth.S_Z, device=dev) if cfg["use_z"] else None
+    inp["w"] = torch.empty(n, dtype=inp["y"].dtype, device=dev)
+    return cfg, inp
+
+
+def _dense_shard(r0, r1, n, dt, kind, seed, dev):
+    """Rows [r0, r1) of the seeded dense matrix (bit-identical to the slice of the full one)."""
+    return synth.dense(r1 - r0, n, dt, kind=kind, seed=seed, device=dev, row0=r0)
+
+
+def _host_rowptr(m, thr, seed):
+    lens = np.empty(m, np.int64)
+    import ctypes
+
+    lib = synth._host()
+    lib.synth_row_lengths(m, 0, thr.ctypes.data_as(ctypes.c_void_p), len(thr) - 1, seed,
+                          lens.ctypes.data_as(ctypes.c_void_p))
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    return torch.from_numpy(rp)
+
+
+# ------------------------------------------------------------------------------ main arm
+def run_gpu(args):
+    world, rank, local = dist_info()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    import paper_conf_ppopp_asharitbrcks15_b200 as fp
+
+    comm = None
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=dev)
+        comm = fp.Comm(device=local)
+    name = args.config
+    cfg, inp = build_inputs(name, rank, world, dev)
+    torch.cuda.synchronize()
+    alpha, beta = cfg["alpha"], cfg["beta"]
+    stream = torch.cuda.current_stream(dev)
+    n = cfg["n"]
+
+    if name == "C5":
+        iters = args.cg_iters
+
+        def step():
+            fp.cg_linreg_dense(inp["X"], inp["labels"], eps=1e-3, max_iter=iters, tol=0.0, comm=comm)
+        inp["labels"] = synth.vector(inp["m_local"], cfg["dtype"], seed=synth.config_seed(name),
+                                     stream=synth.S_LABEL, i0=inp["row0"], device=dev)
+        launches_per_step = 2 * iters + 2
+        passes_per_step = iters + 1
+    elif cfg["fmt"] == "dense":
+        def step():
+            if comm is None:
+                fp.dense(inp["X"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
+            else:
+                fp.dense_dist(comm, inp["X"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
+        launches_per_step = 1
+        passes_per_step = 1
+    else:
+        def step():
+            if comm is None:
+                fp.csr(inp["rowptr"], inp["colidx"], inp["val"], n, inp["y"], inp["v"], inp["z"], alpha, beta,
+                       w=inp["w"])
+            else:
+                fp.csr_dist(comm, inp["rowptr"], inp["colidx"], inp["val"], n, inp["y"], inp["v"], inp["z"], alpha,
+                            beta, w=inp["w"])
+        st = fp.fp_row_stats()
+        st.m, st.n, st.nnz = inp["m_local"], n, inp["nnz_local"]
+        st.mean = st.nnz / max(1, st.m)
+        plan = fp.choose(True, st, fp.FP_F64 if cfg["dtype"] == "f64" else fp.FP_F32, local)
+        launches_per_step = 1 if plan.variant == 3 else 2
+        passes_per_step = 1
+
+    flush = None
+    if name == "C1":  # X fits in L2: flush between timed iterations
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # global algorithmic bytes per evaluation (all ranks)
+    m_all, nnz_all = cfg["m"], None
+    if cfg["fmt"] == "csr":
+        t = torch.tensor([inp["nnz_local"]], dtype=torch.int64, device=dev)
+        if world > 1:
+            import torch.distributed as dist
+
+            dist.all_reduce(t)
+        nnz_all = int(t.item())
+    x_bytes, alg_bytes = algorithmic_bytes(cfg, m_all, nnz_all or 0)
+    x_local, alg_local = algorithmic_bytes(cfg, inp["m_local"], inp["nnz_local"])
+
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_begin = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_begin.record(stream)
+    for i in range(args.steps):
+        if flush is not None:
+            flush.zero_()
+        starts[i].record(stream)
+        step()
+        ends[i].record(stream)
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    total_ms = t_begin.elapsed_time(t_end)
+    kern_ms = float(np.mean(step_ms))
+    if flush is None:
+        ms_per_step = total_ms / args.steps
+    else:
+        ms_per_step = float(np.sum(step_ms)) / args.steps  # flush excluded
+    if world > 1:
+        t = torch.tensor([ms_per_step, kern_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_per_step, kern_ms = float(t[0]), float(t[1])
+
+    evals_per_s = 1e3 / ms_per_step
+    value = x_bytes * passes_per_step * evals_per_s / 1e9
+    peak, peak_src = peaks()
+    achieved = alg_local * passes_per_step / (kern_ms / 1e3) / 1e9   # per-GPU kernel bytes / kernel time
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": traffic_for(name),
+            "peak_source": peak_src,
+            "note": ("achieved = algorithmic bytes of one fp_* call (SURVEY 8(d): X once + rowptr + v + y + z + w) "
+                     "/ mean CUDA-event duration of that call on its launch stream")}
+
+    e2e = None
+    if not args.no_e2e and name != "C5":
+        e2e = run_e2e(args, cfg, inp, comm, world, rank, dev, x_bytes)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(name, args.cpu_seconds)
+
+    if rank == 0:
+        out = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"],
+            "data": "synthetic (counter-based seeded generator synth/, generated in HBM)",
+            "config": {"workload": f"{name}: {cfg['desc']}", "m": cfg["m"], "n": cfg["n"],
+                       "format": cfg["fmt"], "nnz": nnz_all, "alpha": alpha, "beta": beta, "v": cfg["use_v"],
+                       "z": cfg["use_z"], "parallelism": f"row-sharded x{world}, one NCCL allreduce of w",
+                       "l2": ("flushed (256 MiB memset) between timed steps" if flush is not None else
+                              f"inputs larger than L2 (X = {x_bytes / 1e9:.2f} GB >> 126 MB)"),
+                       "passes_per_step": passes_per_step},
+            "evals_per_s": round(evals_per_s * (1 if name != "C5" else 1), 3),
+            "pct_hbm_peak": round(100 * value / world / peak, 2),
+            "x_bytes_per_eval": x_bytes, "algorithmic_bytes_per_eval": alg_bytes,
+            "kernel_ms": round(kern_ms, 4),
+            "roofline": roof,
+            "gpu_launches": launches_per_step * args.steps,
+            "clocks": clk,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(out), flush=True)
+    if comm is not None:
+        comm.close()
+        import torch.distributed as dist
+
+        dist.destroy_process_group()
+
+
+def run_e2e(args, cfg, inp, comm, world, rank, dev, x_bytes):
+    """Same metric through the host-buffer C-ABI entry (fp_dense_host / fp_csr_host): inputs in
+    pinned host memory, H2D of the whole shard and D2H of w inside every timed step."""
+    import paper_conf_ppopp_asharitbrcks15_b200 as fp
+
+    host = {k: (t.cpu().pin_memory() if isinstance(t, torch.Tensor) else t) for k, t in inp.items()
+            if k in ("X", "rowptr", "colidx", "val", "y", "v", "z")}
+    n = cfg["n"]
+    z, beta = (host.get("z"), cfg["beta"]) if rank == 0 else (None, 0.0)
+    wh = torch.empty(n, dtype=host["y"].dtype).pin_memory()
+
+    def step():
+        if cfg["fmt"] == "dense":
+            fp.dense_host(host["X"], host["y"], host.get("v"), z, cfg["alpha"], beta, w=wh, device=dev.index)
+        else:
+            fp.csr_host(host["rowptr"], host["colidx"], host["val"], n, host["y"], host.get("v"), z, cfg["alpha"],
+                        beta, w=wh, device=dev.index)
+        if comm is not None:
+            wd = wh.to(dev, non_blocking=False)
+            comm.allreduce(wd)
+            wh.copy_(wd.cpu())
+
+    step()  # warm-up (allocates staging buffers)
+    steps = max(1, args.e2e_steps)
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        step()
+    dt = (time.perf_counter() - t0) / steps
+    if world > 1:
+        t = torch.tensor([dt], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dt = float(t[0])
+    h2d = sum(t.numel() * t.element_size() for k, t in host.items() if t is not None)
+    return {"value": round(x_bytes / dt / 1e9, 2), "unit": "GB/s", "h2d_bytes_per_step": int(h2d),
+            "d2h_bytes_per_step": int(wh.numel() * wh.element_size()), "steps": steps,
+            "ms_per_step": round(dt * 1e3, 3),
+            "api": "fp_dense_host / fp_csr_host (row chunks streamed through HBM, copy/compute overlapped)"}
+
+
+# ------------------------------------------------------------------------------ CPU oracle
+def _oracle_sample(name, target_s):
+    """Bounded sample of config `name` for the oracle: leading rows of the same seeded matrix
+    (the generator is counter-based, so they are the matrix's actual first rows)."""
+    cfg = synth.CONFIGS[name]
+    seed = synth.config_seed(name)
+    m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
+    # rows sized for ~target_s of oracle work at ~0.5-1 G entries/s on 16 cores
+    budget_entries = int(3e8 * target_s / 15)
+    if cfg["fmt"] == "dense":
+        rows = min(m, max(1, budget_entries // n))
+        X = synth.dense(rows, n, dt, kind=cfg["xkind"], seed=seed)
+        data = dict(X=X)
+        entries = rows * n
+    else:
+        mean = {"C3": 10.0, "C4": 40.0}.get(name, 10.0)
+        rows = min(m, max(1, int(budget_entries / mean)))
+        rp, ci, va = synth.csr(rows, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed)
+        data = dict(rp=rp, ci=ci, va=va)
+        entries = int(va.numel())
+    y = synth.vector(n, dt, seed=seed, stream=synth.S_Y)
+    v = synth.vector(rows, dt, kind="pos", seed=seed, stream=synth.S_V) if cfg["use_v"] else None
+    z = synth.vector(n, dt, seed=seed, stream=synth.S_Z) if cfg["use_z"] else None
+    return cfg, rows, entries, data, y, v, z
+
+
+def _oracle_eval(cfg, rows, data, y, v, z, threads):
+    import oracle
+
+    if cfg["fmt"] == "dense":
+        return oracle.dense(data["X"], y, v, z, cfg["alpha"], cfg["beta"], threads=threads)
+    return oracle.csr(rows, cfg["n"], data["rp"], data["ci"], data["va"], y, v, z, cfg["alpha"], cfg["beta"],
+                      threads=threads)
+
+
+def cpu_baseline(name, target_s=15.0):
+    cfg, rows, entries, data, y, v, z = _oracle_sample(name, target_s)
+    threads = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    _oracle_eval(cfg, rows, data, y, v, z, threads)
+    dt = time.perf_counter() - t0
+    xb, _ = algorithmic_bytes(cfg, rows, entries)
+    return {"value": round(xb / dt / 1e9, 4), "unit": "GB/s", "cores": threads, "kind": "oracle",
+            "sample": f"first {rows:,} of {cfg['m']:,} rows of {name} (same generator), 1 evaluation, "
+                      f"{dt:.1f} s, fp64 Neumaier oracle (oracle/oracle.c, OpenMP)"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as the reference arm (this tier has no reference code)."""
+    world, rank, _ = dist_info()
+    if rank != 0:
+        return
+    name = args.config
+    cfg, rows, entries, data, y, v, z = _oracle_sample(name, args.ref_seconds)
+    threads = os.cpu_count() or 1
+    for _ in range(args.warmup):
+        _oracle_eval(cfg, rows, data, y, v, z, threads)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        _oracle_eval(cfg, rows, data, y, v, z, threads)
+    dt = (time.perf_counter() - t0) / args.steps
+    xb, _ = algorithmic_bytes(cfg, rows, entries)
+    val = xb / dt / 1e9
+    sample = (f"first {rows:,} of {cfg['m']:,} rows of {name} per step (same generator); "
+              f"GB/s of X streamed by the fp64 oracle")
+    out = {"impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "GB/s", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f64 (oracle arithmetic; inputs " + cfg["dtype"] + ")",
+           "data": "synthetic", "config": {"workload": f"{name}: {cfg['desc']}", "m": cfg["m"], "n": cfg["n"]},
+           "cpu_baseline": {"value": round(val, 4), "unit": "GB/s", "kind": "oracle", "cores": threads,
+                            "sample": sample},
+           "e2e": {"value": round(val, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C2", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--impl", default="fusedpat", choices=["fusedpat", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--ref-seconds", type=float, default=4.0)
+    ap.add_argument("--cg-iters", type=int, default=20)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_gpu(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,387 @@
+"""Python binding of libfusedpat (include/fusedpat.h) -- argument marshalling only.
+
+The fused pattern of Ashari et al., PPoPP'15, Eq. (1):
+
+    w = alpha * X^T (v (.) (X y)) + beta * z
+
+Every step runs in the CUDA library (``libfusedpat.so``, sm_100a); this module only turns
+torch tensors into pointers/sizes and status codes into exceptions.  PyTorch provides device
+memory, streams and process groups.  There is no CPU fallback: importing works without a GPU
+(so the ABI can be inspected), but any compute call without a CUDA device fails loudly.
+
+Low-level names mirror the C ABI one to one (``fp_dense``, ``fp_csr``, ``fp_choose`` ...);
+the tensor-level helpers ``dense``, ``csr``, ``cg_linreg_*`` and the ``Comm`` class are thin
+conveniences over them.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libfusedpat.so")
+
+FP_F32, FP_F64 = 0, 1
+STATUS = {0: "FP_OK", 1: "FP_ERR_INVALID_ARG", 2: "FP_ERR_UNSUPPORTED", 3: "FP_ERR_ALIAS", 4: "FP_ERR_INVALID_CSR",
+          5: "FP_ERR_CUDA", 6: "FP_ERR_NCCL", 7: "FP_ERR_NOMEM"}
+VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2"}
+
+
+class FusedPatError(RuntimeError):
+    def __init__(self, status, where, detail):
+        self.status = status
+        super().__init__(f"{where}: {STATUS.get(status, status)}: {detail}")
+
+
+class fp_row_stats(ctypes.Structure):
+    _fields_ = [("m", ctypes.c_int64), ("n", ctypes.c_int64), ("nnz", ctypes.c_int64), ("mean", ctypes.c_double),
+                ("max_len", ctypes.c_int64), ("min_len", ctypes.c_int64), ("empty_rows", ctypes.c_int64),
+                ("hist_log2", ctypes.c_int64 * 64)]
+
+
+class fp_device_profile(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_int) for k in (
+        "sm_count", "max_threads_per_sm", "max_threads_per_block", "max_blocks_per_sm", "regs_per_sm",
+        "max_regs_per_thread", "reg_alloc_unit", "warp_alloc_granularity", "smem_per_sm", "smem_per_block",
+        "smem_alloc_unit", "warp_size")]
+
+
+class fp_launch(ctypes.Structure):
+    _fields_ = [("variant", ctypes.c_int), ("vs", ctypes.c_int), ("bs", ctypes.c_int), ("tl", ctypes.c_int),
+                ("grid", ctypes.c_int), ("blocks_per_sm", ctypes.c_int), ("rows_per_vector", ctypes.c_int64),
+                ("smem_bytes", ctypes.c_int), ("regs_per_thread", ctypes.c_int), ("concurrent_warps", ctypes.c_int)]
+
+    def as_dict(self):
+        d = {k: getattr(self, k) for k, _ in self._fields_}
+        d["variant_name"] = VARIANTS.get(self.variant, "?")
+        return d
+
+
+_i64, _dbl, _vp, _int = ctypes.c_int64, ctypes.c_double, ctypes.c_void_p, ctypes.c_int
+_P = ctypes.POINTER
+
+# name -> (restype, argtypes)
+_SIGS = {
+    "fp_status_string": (ctypes.c_char_p, [_int]),
+    "fp_last_error": (ctypes.c_char_p, []),
+    "fp_version": (ctypes.c_char_p, []),
+    "fp_dense": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp]),
+    "fp_csr": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp]),
+    "fp_dense_ex": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _P(fp_launch), _vp]),
+    "fp_csr_ex": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _P(fp_launch), _vp]),
+    "fp_device_profile_query": (_int, [_int, _P(fp_device_profile)]),
+    "fp_device_profile_kepler": (_int, [_P(fp_device_profile)]),
+    "fp_row_stats_host": (_int, [_i64, _vp, _P(fp_row_stats)]),
+    "fp_row_stats_device": (_int, [_i64, _vp, _P(fp_row_stats), _vp]),
+    "fp_row_stats_dense": (_int, [_i64, _i64, _P(fp_row_stats)]),
+    "fp_choose_paper": (_int, [_int, _P(fp_row_stats), _int, _P(fp_device_profile), _int, _int, _int, _P(fp_launch)]),
+    "fp_choose": (_int, [_int, _P(fp_row_stats), _int, _int, _P(fp_launch)]),
+    "fp_csr_validate": (_int, [_i64, _i64, _i64, _vp, _vp, _vp]),
+    "fp_dense_host": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
+    "fp_csr_host": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
+    "fp_release_workspace": (_int, []),
+    "fp_comm_get_unique_id": (_int, [_vp]),
+    "fp_comm_init": (_int, [_P(_vp), _int, _int, _vp, _int]),
+    "fp_comm_destroy": (_int, [_vp]),
+    "fp_comm_rank": (_int, [_vp]),
+    "fp_comm_size": (_int, [_vp]),
+    "fp_allreduce": (_int, [_vp, _vp, _i64, _int, _vp]),
+    "fp_shard_rows_dense": (_int, [_i64, _int, _vp]),
+    "fp_shard_rows_csr": (_int, [_i64, _vp, _int, _vp]),
+    "fp_dense_dist": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp, _vp]),
+    "fp_csr_dist": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp, _vp]),
+    "fp_cg_linreg_dense": (_int, [_i64, _i64, _vp, _i64, _vp, _dbl, _int, _dbl, _vp, _P(_int), _vp, _int, _vp, _vp]),
+    "fp_cg_linreg_csr": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _dbl, _int, _dbl, _vp, _P(_int), _vp, _int, _vp,
+                                _vp]),
+}
+
+_lib = None
+
+
+def lib():
+    """Load libfusedpat.so (raises if it was not built -- there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build it with __graft_entry__.build() (or `make fusedpat`)")
+        L = ctypes.CDLL(LIB_PATH, mode=ctypes.RTLD_GLOBAL)
+        for name, (res, args) in _SIGS.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def exported_symbols():
+    return sorted(_SIGS)
+
+
+def _check(status, where):
+    if status != 0:
+        detail = lib().fp_last_error().decode(errors="replace")
+        raise FusedPatError(status, where, detail)
+
+
+def _call(name, *args):
+    _check(getattr(lib(), name)(*args), name)
+
+
+# expose the raw C functions under their C names (checked: raise FusedPatError on failure)
+def _make_raw(name):
+    def f(*args):
+        r = getattr(lib(), name)(*args)
+        if _SIGS[name][0] is _int and name not in ("fp_comm_rank", "fp_comm_size"):
+            _check(r, name)
+        return r
+    f.__name__ = name
+    f.__doc__ = f"Checked ctypes call of the C ABI function {name} (include/fusedpat.h)."
+    return f
+
+
+for _n in _SIGS:
+    globals()[_n] = _make_raw(_n)
+
+
+# ------------------------------------------------------------------------------- tensor level
+def _dt(t):
+    if t.dtype == torch.float64:
+        return FP_F64
+    if t.dtype == torch.float32:
+        return FP_F32
+    raise TypeError(f"unsupported dtype {t.dtype} (float32 / float64)")
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(device, stream=None):
+    if stream is not None:
+        return ctypes.c_void_p(stream.cuda_stream)
+    return ctypes.c_void_p(torch.cuda.current_stream(device).cuda_stream)
+
+
+def _require_cuda(*ts):
+    for t in ts:
+        if t is not None and not t.is_cuda:
+            raise ValueError("libfusedpat device entry points take CUDA tensors (use fp_*_host for host buffers)")
+
+
+def _vec(t, length, dtype, name):
+    if t is None:
+        return None
+    if t.dim() != 1 or t.shape[0] != length or t.dtype != dtype or not t.is_contiguous():
+        raise ValueError(f"{name} must be a contiguous 1-D {dtype} tensor of length {length}")
+    return t
+
+
+def dense(X, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, launch=None, stream=None):
+    """w = alpha X^T (v (.) (X y)) + beta z for a dense row-major X (m x n, row stride >= n).
+    y=None selects alpha X^T v (Table 1 row 1); v=None means v = 1; returns w."""
+    _require_cuda(X, y, v, z, w)
+    if X.dim() != 2 or X.stride(1) != 1:
+        raise ValueError("X must be 2-D row-major (stride(1) == 1)")
+    m, n = X.shape
+    ld = X.stride(0) if m > 1 else n
+    y, v, z = _vec(y, n, X.dtype, "y"), _vec(v, m, X.dtype, "v"), _vec(z, n, X.dtype, "z")
+    if w is None:
+        w = torch.empty(n, dtype=X.dtype, device=X.device)
+    _vec(w, n, X.dtype, "w")
+    s = _stream(X.device, stream)
+    if launch is None:
+        _call("fp_dense", m, n, _ptr(X), ld, _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w), _dt(X), s)
+    else:
+        _call("fp_dense_ex", m, n, _ptr(X), ld, _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w), _dt(X),
+              ctypes.byref(launch), s)
+    return w
+
+
+def csr(rowptr, colidx, val, n, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, launch=None, stream=None):
+    """CSR variant: rowptr int64[m+1], colidx int32[nnz], val[nnz]."""
+    _require_cuda(rowptr, colidx, val, y, v, z, w)
+    if rowptr.dtype != torch.int64 or colidx.dtype != torch.int32:
+        raise TypeError("rowptr must be int64 and colidx int32")
+    m = rowptr.shape[0] - 1
+    nnz = val.shape[0]
+    y, v, z = _vec(y, n, val.dtype, "y"), _vec(v, m, val.dtype, "v"), _vec(z, n, val.dtype, "z")
+    if w is None:
+        w = torch.empty(n, dtype=val.dtype, device=val.device)
+    _vec(w, n, val.dtype, "w")
+    s = _stream(val.device, stream)
+    args = (m, n, nnz, _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta),
+            _ptr(w), _dt(val))
+    if launch is None:
+        _call("fp_csr", *args, s)
+    else:
+        _call("fp_csr_ex", *args, ctypes.byref(launch), s)
+    return w
+
+
+def dense_host(X, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, device=0):
+    """Host-buffer entry (fp_dense_host): X, y, v, z, w are CPU tensors; rows stream through HBM."""
+    for t in (X, y, v, z, w):
+        if t is not None and t.is_cuda:
+            raise ValueError("fp_dense_host takes host tensors")
+    m, n = X.shape
+    ld = X.stride(0) if m > 1 else n
+    if w is None:
+        w = torch.empty(n, dtype=X.dtype)
+    _call("fp_dense_host", m, n, _ptr(X), ld, _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w), _dt(X),
+          int(device))
+    return w
+
+
+def csr_host(rowptr, colidx, val, n, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, device=0):
+    m = rowptr.shape[0] - 1
+    if w is None:
+        w = torch.empty(n, dtype=val.dtype)
+    _call("fp_csr_host", m, n, val.shape[0], _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(y), _ptr(v), _ptr(z),
+          float(alpha), float(beta), _ptr(w), _dt(val), int(device))
+    return w
+
+
+# ------------------------------------------------------------------------------- chooser
+def row_stats_host(rowptr):
+    st = fp_row_stats()
+    rp = rowptr.detach().cpu().contiguous()
+    _call("fp_row_stats_host", rp.shape[0] - 1, _ptr(rp), ctypes.byref(st))
+    return st
+
+
+def row_stats_device(rowptr, stream=None):
+    st = fp_row_stats()
+    _call("fp_row_stats_device", rowptr.shape[0] - 1, _ptr(rowptr), ctypes.byref(st), _stream(rowptr.device, stream))
+    return st
+
+
+def row_stats_dense(m, n):
+    st = fp_row_stats()
+    _call("fp_row_stats_dense", m, n, ctypes.byref(st))
+    return st
+
+
+def kepler_profile():
+    p = fp_device_profile()
+    _call("fp_device_profile_kepler", ctypes.byref(p))
+    return p
+
+
+def device_profile(device=0):
+    p = fp_device_profile()
+    _call("fp_device_profile_query", int(device), ctypes.byref(p))
+    return p
+
+
+def choose_paper(is_csr, stats, dtype, profile, regs_per_thread=43, regs_dense_tl1=23, regs_dense_tl40=255):
+    """The paper's analytical model (Section 3.3) -- defaults are its profiled register counts."""
+    L = fp_launch()
+    _call("fp_choose_paper", int(bool(is_csr)), ctypes.byref(stats), dtype, ctypes.byref(profile),
+          int(regs_per_thread), int(regs_dense_tl1), int(regs_dense_tl40), ctypes.byref(L))
+    return L
+
+
+def choose(is_csr, stats, dtype, device=0):
+    """The B200 plan the kernels launch."""
+    L = fp_launch()
+    _call("fp_choose", int(bool(is_csr)), ctypes.byref(stats), dtype, int(device), ctypes.byref(L))
+    return L
+
+
+def csr_validate(rowptr, colidx, n, stream=None):
+    _call("fp_csr_validate", rowptr.shape[0] - 1, n, colidx.shape[0], _ptr(rowptr), _ptr(colidx),
+          _stream(rowptr.device, stream))
+
+
+# ------------------------------------------------------------------------------- multi-GPU
+def shard_rows_dense(m, nranks):
+    b = (ctypes.c_int64 * (nranks + 1))()
+    _call("fp_shard_rows_dense", m, nranks, ctypes.cast(b, ctypes.c_void_p))
+    return list(b)
+
+
+def shard_rows_csr(rowptr_host, nranks):
+    rp = rowptr_host.detach().cpu().contiguous()
+    if rp.dtype != torch.int64:
+        raise TypeError("rowptr must be int64")
+    b = (ctypes.c_int64 * (nranks + 1))()
+    _call("fp_shard_rows_csr", rp.shape[0] - 1, _ptr(rp), nranks, ctypes.cast(b, ctypes.c_void_p))
+    return list(b)
+
+
+class Comm:
+    """NCCL communicator owned by libfusedpat, bootstrapped through torch.distributed:
+    rank 0 creates the 128-byte unique id, broadcast_object_list ships it to every rank."""
+
+    def __init__(self, device=None, group=None):
+        import torch.distributed as dist
+
+        self.rank, self.size = dist.get_rank(group), dist.get_world_size(group)
+        self.device = torch.cuda.current_device() if device is None else int(device)
+        uid = (ctypes.c_ubyte * 128)()
+        if self.rank == 0:
+            _call("fp_comm_get_unique_id", ctypes.cast(uid, ctypes.c_void_p))
+        obj = [bytes(uid)]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = (ctypes.c_ubyte * 128).from_buffer_copy(obj[0])
+        h = ctypes.c_void_p()
+        _call("fp_comm_init", ctypes.byref(h), self.size, self.rank, ctypes.cast(uid, ctypes.c_void_p), self.device)
+        self.handle = h
+
+    def close(self):
+        if self.handle:
+            _call("fp_comm_destroy", self.handle)
+            self.handle = None
+
+    def allreduce(self, t, stream=None):
+        _call("fp_allreduce", self.handle, _ptr(t), t.numel(), _dt(t), _stream(t.device, stream))
+        return t
+
+
+def dense_dist(comm, X_local, y=None, v_local=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
+    m, n = X_local.shape
+    ld = X_local.stride(0) if m > 1 else n
+    if w is None:
+        w = torch.empty(n, dtype=X_local.dtype, device=X_local.device)
+    _call("fp_dense_dist", m, n, _ptr(X_local), ld, _ptr(y), _ptr(v_local), _ptr(z), float(alpha), float(beta),
+          _ptr(w), _dt(X_local), comm.handle, _stream(X_local.device, stream))
+    return w
+
+
+def csr_dist(comm, rowptr_local, colidx_local, val_local, n, y=None, v_local=None, z=None, alpha=1.0, beta=0.0,
+             w=None, stream=None):
+    m = rowptr_local.shape[0] - 1
+    if w is None:
+        w = torch.empty(n, dtype=val_local.dtype, device=val_local.device)
+    _call("fp_csr_dist", m, n, val_local.shape[0], _ptr(rowptr_local), _ptr(colidx_local), _ptr(val_local), _ptr(y),
+          _ptr(v_local), _ptr(z), float(alpha), float(beta), _ptr(w), _dt(val_local), comm.handle,
+          _stream(val_local.device, stream))
+    return w
+
+
+# ------------------------------------------------------------------------------- drivers
+def cg_linreg_dense(X, labels, eps=1e-3, max_iter=100, tol=1e-6, comm=None, stream=None):
+    """Listing 1 with the fused op.  Returns (w, iters, nr2_history)."""
+    _require_cuda(X, labels)
+    m, n = X.shape
+    ld = X.stride(0) if m > 1 else n
+    w = torch.empty(n, dtype=X.dtype, device=X.device)
+    it = ctypes.c_int(0)
+    hist = torch.zeros(max_iter + 1, dtype=torch.float64)
+    _call("fp_cg_linreg_dense", m, n, _ptr(X), ld, _ptr(labels), float(eps), int(max_iter), float(tol), _ptr(w),
+          ctypes.byref(it), _ptr(hist), _dt(X), comm.handle if comm else None, _stream(X.device, stream))
+    return w, it.value, hist[: it.value + 1]
+
+
+def cg_linreg_csr(rowptr, colidx, val, n, labels, eps=1e-3, max_iter=100, tol=1e-6, comm=None, stream=None):
+    _require_cuda(rowptr, colidx, val, labels)
+    m = rowptr.shape[0] - 1
+    w = torch.empty(n, dtype=val.dtype, device=val.device)
+    it = ctypes.c_int(0)
+    hist = torch.zeros(max_iter + 1, dtype=torch.float64)
+    _call("fp_cg_linreg_csr", m, n, val.shape[0], _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(labels), float(eps),
+          int(max_iter), float(tol), _ptr(w), ctypes.byref(it), _ptr(hist), _dt(val), comm.handle if comm else None,
+          _stream(val.device, stream))
+    return w, it.value, hist[: it.value + 1]

@@ -1,0 +1,40 @@
+// aggregate.cuh -- grid-level aggregation of per-CTA partial w (rows a9-a10 of SURVEY 8).
+//
+// The paper aggregates per-block partials with one global atomicAdd per element
+// (Alg. 1 l.15-16 P:195-196, Alg. 2 l.17-18 P:224-225, Alg. 3 l.26-27 P:286-287) into a w
+// that must first hold beta*z -- which needs either grid-stride atomics in every block or
+// a second kernel, because CUDA had no inter-block barrier.  On sm_100a we
+// instead: (1) every CTA adds its fp64 partial into an fp64 workspace accumulator with
+// fire-and-forget REDG.E.ADD.F64 (L2-resident, n*8 bytes), (2) takes a ticket on a
+// device counter, and (3) the LAST CTA (ticket == gridDim-1) applies alpha and beta*z once
+// and writes w -- one launch, no pre-zeroed w, no race on beta*z, and the workspace is
+// re-zeroed for the next call.
+#pragma once
+#include "common.cuh"
+
+namespace fpd {
+
+template <typename T, typename S>
+__device__ __forceinline__ void grid_finalize(const S* __restrict__ sw, int64_t n, double* acc,
+                                              unsigned long long* counter, double alpha, double beta,
+                                              const T* z, T* w, bool add_beta_z, bool accumulate) {
+  for (int64_t j = threadIdx.x; j < n; j += blockDim.x) atomicAdd(acc + j, (double)sw[j]);
+  __threadfence();
+  __syncthreads();
+  __shared__ int s_last;
+  if (threadIdx.x == 0) s_last = (atomicAdd(counter, 1ull) == (unsigned long long)gridDim.x - 1ull);
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  for (int64_t j = threadIdx.x; j < n; j += blockDim.x) {
+    double s = __ldcg(acc + j);
+    acc[j] = 0.0;
+    double r = alpha * s;
+    if (add_beta_z && beta != 0.0) r += beta * (double)z[j];
+    if (accumulate) r += (double)w[j];
+    w[j] = (T)r;
+  }
+  if (threadIdx.x == 0) *counter = 0ull;
+}
+
+}  // namespace fpd

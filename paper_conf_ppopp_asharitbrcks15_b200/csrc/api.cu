@@ -1,0 +1,161 @@
+// api.cu -- the C ABI entry points of fusedpat.h for the single-GPU pattern: argument
+// validation (every call), alias checks, the alpha == 0 / m == 0 path, plan + launch.
+#include <string.h>
+
+#include "kernels.cuh"
+
+namespace fp {
+
+static fp_status check_vec_alias(const void* w, size_t wb, const void* p, size_t pb, const char* what) {
+  FP_REQUIRE(!overlaps(w, wb, p, pb), FP_ERR_ALIAS, "w overlaps %s", what);
+  return FP_OK;
+}
+
+// Shared validation of the vector / scalar part (R2-R4 of DESIGN.md).
+static fp_status check_common(const PatternArgs& a) {
+  FP_REQUIRE(valid_dtype(a.dtype), FP_ERR_INVALID_ARG, "dtype must be FP_F32 or FP_F64");
+  FP_REQUIRE(a.m >= 0 && a.n >= 0, FP_ERR_INVALID_ARG, "negative size (m=%lld n=%lld)", (long long)a.m,
+             (long long)a.n);
+  if (a.n == 0) return FP_OK;
+  FP_REQUIRE(a.w != nullptr, FP_ERR_INVALID_ARG, "w is NULL");
+  FP_REQUIRE(a.beta == 0.0 || a.z != nullptr, FP_ERR_INVALID_ARG, "beta != 0 requires z");
+  const size_t s = dtype_size(a.dtype), wb = (size_t)a.n * s;
+  if (a.z && a.z != a.w) {
+    fp_status st = check_vec_alias(a.w, wb, a.z, wb, "z (only exact aliasing w == z is allowed)");
+    if (st != FP_OK) return st;
+  }
+  if (a.alpha != 0.0 && a.m > 0) {
+    fp_status st = check_vec_alias(a.w, wb, a.y, a.y ? wb : 0, "y");
+    if (st == FP_OK) st = check_vec_alias(a.w, wb, a.v, a.v ? (size_t)a.m * s : 0, "v");
+    if (st != FP_OK) return st;
+  }
+  return FP_OK;
+}
+
+static fp_status check_dense(const PatternArgs& a) {
+  fp_status st = check_common(a);
+  if (st != FP_OK || a.n == 0) return st;
+  FP_REQUIRE(a.ld >= a.n, FP_ERR_INVALID_ARG, "ld (%lld) < n (%lld)", (long long)a.ld, (long long)a.n);
+  if (a.alpha != 0.0 && a.m > 0) {
+    FP_REQUIRE(a.X != nullptr, FP_ERR_INVALID_ARG, "X is NULL");
+    const size_t s = dtype_size(a.dtype);
+    st = check_vec_alias(a.w, (size_t)a.n * s, a.X, (size_t)((a.m - 1) * a.ld + a.n) * s, "X");
+  }
+  return st;
+}
+
+static fp_status check_csr(const PatternArgs& a) {
+  FP_REQUIRE(a.n <= INT32_MAX, FP_ERR_UNSUPPORTED, "n exceeds int32 column indices");
+  fp_status st = check_common(a);
+  if (st != FP_OK || a.n == 0) return st;
+  FP_REQUIRE(a.nnz >= 0, FP_ERR_INVALID_ARG, "nnz < 0");
+  if (a.alpha != 0.0 && a.m > 0) {
+    FP_REQUIRE(a.rowptr != nullptr, FP_ERR_INVALID_ARG, "rowptr is NULL");
+    FP_REQUIRE(a.nnz == 0 || (a.colidx && a.val), FP_ERR_INVALID_ARG, "colidx/val is NULL");
+    const size_t s = dtype_size(a.dtype), wb = (size_t)a.n * s;
+    st = check_vec_alias(a.w, wb, a.val, (size_t)a.nnz * s, "val");
+    if (st == FP_OK) st = check_vec_alias(a.w, wb, a.colidx, (size_t)a.nnz * 4, "colidx");
+    if (st == FP_OK) st = check_vec_alias(a.w, wb, a.rowptr, (size_t)(a.m + 1) * 8, "rowptr");
+  }
+  return st;
+}
+
+fp_status run_dense(const PatternArgs& a, const fp_launch* override_, cudaStream_t s) {
+  fp_status st = check_dense(a);
+  if (st != FP_OK || a.n == 0) return st;
+  if (a.alpha == 0.0 || a.m == 0)
+    return launch_scale_z(a.n, a.add_beta_z ? a.z : nullptr, a.add_beta_z ? a.beta : 0.0, a.w, a.dtype, s);
+  fp_launch L;
+  if (override_) {
+    L = *override_;
+  } else {
+    st = plan_dense(a, current_device(), &L);
+    if (st != FP_OK) return st;
+  }
+  return launch_dense(a, L, s);
+}
+
+fp_status run_csr(const PatternArgs& a, const fp_launch* override_, cudaStream_t s) {
+  fp_status st = check_csr(a);
+  if (st != FP_OK || a.n == 0) return st;
+  if (a.alpha == 0.0 || a.m == 0)
+    return launch_scale_z(a.n, a.add_beta_z ? a.z : nullptr, a.add_beta_z ? a.beta : 0.0, a.w, a.dtype, s);
+  fp_launch L;
+  if (override_) {
+    L = *override_;
+  } else {
+    st = plan_csr(a, current_device(), &L);
+    if (st != FP_OK) return st;
+  }
+  return launch_csr(a, L, s);
+}
+
+PatternArgs dense_args(int64_t m, int64_t n, const void* X, int64_t ld, const void* y, const void* v, const void* z,
+                       double alpha, double beta, void* w, fp_dtype dtype) {
+  PatternArgs a;
+  a.m = m; a.n = n; a.X = X; a.ld = ld; a.y = y; a.v = v; a.z = z;
+  a.alpha = alpha; a.beta = beta; a.w = w; a.dtype = dtype;
+  return a;
+}
+
+PatternArgs csr_args(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                     const void* val, const void* y, const void* v, const void* z, double alpha, double beta, void* w,
+                     fp_dtype dtype) {
+  PatternArgs a;
+  a.m = m; a.n = n; a.nnz = nnz; a.rowptr = rowptr; a.colidx = colidx; a.val = val;
+  a.y = y; a.v = v; a.z = z; a.alpha = alpha; a.beta = beta; a.w = w; a.dtype = dtype;
+  return a;
+}
+
+}  // namespace fp
+
+extern "C" {
+
+const char* fp_status_string(fp_status s) {
+  switch (s) {
+    case FP_OK: return "FP_OK";
+    case FP_ERR_INVALID_ARG: return "FP_ERR_INVALID_ARG";
+    case FP_ERR_UNSUPPORTED: return "FP_ERR_UNSUPPORTED";
+    case FP_ERR_ALIAS: return "FP_ERR_ALIAS";
+    case FP_ERR_INVALID_CSR: return "FP_ERR_INVALID_CSR";
+    case FP_ERR_CUDA: return "FP_ERR_CUDA";
+    case FP_ERR_NCCL: return "FP_ERR_NCCL";
+    case FP_ERR_NOMEM: return "FP_ERR_NOMEM";
+  }
+  return "FP_ERR_UNKNOWN";
+}
+
+const char* fp_version(void) { return "0.1.0 sm_100a"; }
+
+fp_status fp_dense(int64_t m, int64_t n, const void* X, int64_t ld, const void* y, const void* v, const void* z,
+                   double alpha, double beta, void* w, fp_dtype dtype, fp_stream stream) {
+  return fp::run_dense(fp::dense_args(m, n, X, ld, y, v, z, alpha, beta, w, dtype), nullptr, (cudaStream_t)stream);
+}
+
+fp_status fp_dense_ex(int64_t m, int64_t n, const void* X, int64_t ld, const void* y, const void* v, const void* z,
+                      double alpha, double beta, void* w, fp_dtype dtype, const fp_launch* override_,
+                      fp_stream stream) {
+  return fp::run_dense(fp::dense_args(m, n, X, ld, y, v, z, alpha, beta, w, dtype), override_,
+                       (cudaStream_t)stream);
+}
+
+fp_status fp_csr(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx, const void* val,
+                 const void* y, const void* v, const void* z, double alpha, double beta, void* w, fp_dtype dtype,
+                 fp_stream stream) {
+  return fp::run_csr(fp::csr_args(m, n, nnz, rowptr, colidx, val, y, v, z, alpha, beta, w, dtype), nullptr,
+                     (cudaStream_t)stream);
+}
+
+fp_status fp_csr_ex(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx, const void* val,
+                    const void* y, const void* v, const void* z, double alpha, double beta, void* w, fp_dtype dtype,
+                    const fp_launch* override_, fp_stream stream) {
+  return fp::run_csr(fp::csr_args(m, n, nnz, rowptr, colidx, val, y, v, z, alpha, beta, w, dtype), override_,
+                     (cudaStream_t)stream);
+}
+
+fp_status fp_release_workspace(void) {
+  fp::release_all_workspaces();
+  return FP_OK;
+}
+
+}  // extern "C"

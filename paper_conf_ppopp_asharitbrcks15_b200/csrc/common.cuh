@@ -1,0 +1,149 @@
+// common.cuh -- shared internals of libfusedpat (error state, device info, per-stream
+// workspace, sm_100a load/reduce primitives).  Product code only; no oracle code here.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "fusedpat.h"
+
+namespace fp {
+
+// ---------------------------------------------------------------------------- errors
+void set_error(const char* fmt, ...);
+const char* last_error_text();
+fp_status cuda_fail(cudaError_t e, const char* what);
+
+#define FP_CUDA(call)                                          \
+  do {                                                         \
+    cudaError_t e_ = (call);                                   \
+    if (e_ != cudaSuccess) return ::fp::cuda_fail(e_, #call);  \
+  } while (0)
+
+#define FP_REQUIRE(cond, status, ...)      \
+  do {                                     \
+    if (!(cond)) {                         \
+      ::fp::set_error(__VA_ARGS__);        \
+      return status;                       \
+    }                                      \
+  } while (0)
+
+// ---------------------------------------------------------------------------- device info
+struct DeviceInfo {
+  int ordinal;
+  int sm_count;
+  int max_threads_per_sm;
+  int max_blocks_per_sm;
+  int regs_per_sm;
+  size_t smem_per_sm;
+  size_t smem_optin_per_block;
+  size_t l2_bytes;
+};
+const DeviceInfo& device_info(int ordinal);
+int current_device();
+
+// ---------------------------------------------------------------------------- workspace
+// One per (device, stream).  acc: fp64 grid accumulator, ALWAYS all-zero between launches
+// (the finalising CTA re-zeroes what it consumed).  counters: [0] CTA-done ticket,
+// [1] dynamic row-chunk counter; both reset to 0 by the finalising CTA.
+struct Workspace {
+  double* acc = nullptr;
+  size_t acc_cap = 0;          // elements
+  unsigned long long* counters = nullptr;
+  void* scratch = nullptr;     // general device scratch (row stats, CG scalars)
+  size_t scratch_cap = 0;      // bytes
+};
+// Returns nullptr (and sets the error) on allocation failure.  Growing reallocates, which
+// synchronises the device; steady-state calls never allocate.
+Workspace* workspace(cudaStream_t s, size_t acc_elems, size_t scratch_bytes);
+void release_all_workspaces();
+
+// ---------------------------------------------------------------------------- helpers
+inline size_t dtype_size(fp_dtype t) { return t == FP_F64 ? 8 : 4; }
+inline bool valid_dtype(fp_dtype t) { return t == FP_F32 || t == FP_F64; }
+
+// [a, a+na) and [b, b+nb) byte ranges overlap?
+inline bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
+  if (!a || !b || na == 0 || nb == 0) return false;
+  uintptr_t x = (uintptr_t)a, y = (uintptr_t)b;
+  return x < y + nb && y < x + na;
+}
+
+}  // namespace fp
+
+// ------------------------------------------------------------------------------------------
+// Device primitives (sm_100a).
+// ------------------------------------------------------------------------------------------
+#ifdef __CUDACC__
+namespace fpd {
+
+// Streaming read-once loads of X: bypass L1 allocation, evict-first in L2 (X is far larger
+// than L2 and never re-read within a call).  256-bit loads are sm_100 LDG.E.256.
+__device__ __forceinline__ void ld_stream32(const float* p, float (&r)[8]) {
+  asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]), "=f"(r[7])
+               : "l"(p));
+}
+__device__ __forceinline__ void ld_stream32(const double* p, double (&r)[4]) {
+  asm("ld.global.nc.L1::no_allocate.L2::evict_first.v4.f64 {%0,%1,%2,%3}, [%4];"
+               : "=d"(r[0]), "=d"(r[1]), "=d"(r[2]), "=d"(r[3])
+               : "l"(p));
+}
+__device__ __forceinline__ void ld_stream16(const float* p, float (&r)[4]) {
+  asm("ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3])
+               : "l"(p));
+}
+__device__ __forceinline__ void ld_stream16(const double* p, double (&r)[2]) {
+  asm("ld.global.nc.L1::no_allocate.L2::256B.v2.f64 {%0,%1}, [%2];" : "=d"(r[0]), "=d"(r[1]) : "l"(p));
+}
+__device__ __forceinline__ void ld_stream4(const float* p, float (&r)[1]) {
+  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r[0]) : "l"(p));
+}
+__device__ __forceinline__ void ld_stream4(const double* p, double (&r)[1]) {
+  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(r[0]) : "l"(p));
+}
+
+// Load E = CB/sizeof(T) consecutive elements (CB-byte aligned).
+template <int CB, typename T, int E>
+__device__ __forceinline__ void ld_chunk(const T* p, T (&r)[E]) {
+  if constexpr (CB == 32) {
+    ld_stream32(p, r);
+  } else if constexpr (CB == 16) {
+    ld_stream16(p, r);
+  } else {
+    ld_stream4(p, r);
+  }
+}
+
+// Read-once streaming loads for CSR structure (colidx / val / rowptr).
+__device__ __forceinline__ int ld_once(const int* p) {
+  int r;
+  asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float ld_once(const float* p) {
+  float r;
+  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ double ld_once(const double* p) {
+  double r;
+  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(r) : "l"(p));
+  return r;
+}
+
+// Fire-and-forget fp reduction into global memory (SASS REDG.E.ADD.F32/F64).
+__device__ __forceinline__ void red_add(float* p, float v) { atomicAdd(p, v); }
+__device__ __forceinline__ void red_add(double* p, double v) { atomicAdd(p, v); }
+
+// Sum over the VS lanes of a vector (VS a power of two <= 32, vectors aligned in the warp);
+// every lane of the vector receives the total.
+template <int VS, typename T>
+__device__ __forceinline__ T vector_allreduce(T x) {
+#pragma unroll
+  for (int off = VS / 2; off > 0; off >>= 1) x += __shfl_xor_sync(0xffffffffu, x, off);
+  return x;
+}
+
+}  // namespace fpd
+#endif

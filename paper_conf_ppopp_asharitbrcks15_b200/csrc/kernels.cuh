@@ -1,0 +1,44 @@
+// kernels.cuh -- launcher interfaces between the C-ABI layer (api.cu) and the kernel files.
+#pragma once
+#include "common.cuh"
+
+namespace fp {
+
+struct PatternArgs {
+  int64_t m = 0, n = 0;
+  // dense
+  const void* X = nullptr;
+  int64_t ld = 0;
+  // csr
+  int64_t nnz = 0;
+  const int64_t* rowptr = nullptr;
+  const int32_t* colidx = nullptr;
+  const void* val = nullptr;
+  // vectors / scalars
+  const void* y = nullptr;
+  const void* v = nullptr;
+  const void* z = nullptr;
+  double alpha = 1.0, beta = 0.0;
+  void* w = nullptr;
+  fp_dtype dtype = FP_F64;
+  // when false the CTA-finalise does NOT add beta*z (multi-GPU ranks != 0); set by dist layer
+  bool add_beta_z = true;
+  // when true the result is ADDED to the current w (w += alpha X^T(v (.) X y) [+ beta z]);
+  // used by the host-streaming (out-of-core) path to sum row chunks
+  bool accumulate = false;
+};
+
+// Dense chooser (B200 plan): fills vs, tl, bs, grid, variant ... for the kernels in dense.cu.
+fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out);
+fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s);
+
+fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out);
+fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s);
+
+// w = beta*z (or 0): the alpha == 0 / m == 0 path, and the pre-initialisation of the L2 path.
+fp_status launch_scale_z(int64_t n, const void* z, double beta, void* w, fp_dtype dt, cudaStream_t s);
+
+// Register count of the kernel instantiation a plan selects (0 if unknown).
+int dense_kernel_regs(const PatternArgs& a, const fp_launch& L);
+
+}  // namespace fp

@@ -35,7 +35,7 @@ def _host():
         if not os.path.exists(path):
             raise RuntimeError(f"{path} missing: run __graft_entry__.build()")
         lib = ctypes.CDLL(path)
-        lib.synth_dense.argtypes = [i64, i64, i64, ci, ci, u64, u64, vp]
+        lib.synth_dense.argtypes = [i64, i64, i64, i64, ci, ci, u64, u64, vp]
         lib.synth_vector.argtypes = [i64, i64, ci, ci, u64, u64, vp]
         lib.synth_row_lengths.argtypes = [i64, i64, vp, i64, u64, vp]
         lib.synth_rowptr.argtypes = [i64, vp, vp]
@@ -53,7 +53,7 @@ def _cuda():
         if not os.path.exists(path):
             raise RuntimeError(f"{path} missing: run __graft_entry__.build()")
         lib = ctypes.CDLL(path)
-        lib.synth_dense_cuda.argtypes = [i64, i64, i64, ci, ci, u64, u64, vp, vp]
+        lib.synth_dense_cuda.argtypes = [i64, i64, i64, i64, ci, ci, u64, u64, vp, vp]
         lib.synth_vector_cuda.argtypes = [i64, i64, ci, ci, u64, u64, vp, vp]
         lib.synth_row_lengths_cuda.argtypes = [i64, i64, vp, i64, u64, vp, vp]
         lib.synth_rowptr_cuda.argtypes = [i64, vp, vp, vp, ctypes.POINTER(ctypes.c_size_t), vp]
@@ -79,17 +79,17 @@ def _check(rc, what):
         raise RuntimeError(f"{what} failed rc={rc}")
 
 
-def dense(m, n, dtype, kind="uniform", seed=BASE_SEED, stream=S_X, ld=None, device="cpu"):
-    """Row-major (m, ld) matrix; logical element (r, c) = value(hash(seed, stream, r*n+c));
-    padding columns (c >= n) are NaN."""
+def dense(m, n, dtype, kind="uniform", seed=BASE_SEED, stream=S_X, ld=None, device="cpu", row0=0):
+    """Rows [row0, row0+m) of the seeded matrix as a row-major (m, ld) tensor; element (r, c) =
+    value(hash(seed, stream, r*n+c)) (global r); padding columns (c >= n) are NaN."""
     ld = n if ld is None else ld
     tdt, code = _tdt(dtype)
     out = torch.empty((m, ld), dtype=tdt, device=device)
     if out.is_cuda:
-        _check(_cuda().synth_dense_cuda(m, n, ld, code, KINDS[kind], seed, stream, ctypes.c_void_p(out.data_ptr()),
+        _check(_cuda().synth_dense_cuda(m, n, ld, row0, code, KINDS[kind], seed, stream, ctypes.c_void_p(out.data_ptr()),
                                         _stream_ptr(out.device)), "synth_dense_cuda")
     else:
-        _check(_host().synth_dense(m, n, ld, code, KINDS[kind], seed, stream, ctypes.c_void_p(out.data_ptr())),
+        _check(_host().synth_dense(m, n, ld, row0, code, KINDS[kind], seed, stream, ctypes.c_void_p(out.data_ptr())),
                "synth_dense")
     return out
 

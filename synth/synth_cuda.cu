@@ -21,11 +21,11 @@ template <>
 __device__ __forceinline__ float syn_value<float>(uint64_t h, int kind, int colexp) { return syn_value_f32(h, kind, colexp); }
 
 template <typename T>
-__global__ void k_dense(int64_t m, int64_t n, int64_t ld, int kind, uint64_t seed, uint64_t stream, T* out) {
+__global__ void k_dense(int64_t m, int64_t n, int64_t ld, int64_t row0, int kind, uint64_t seed, uint64_t stream, T* out) {
   int64_t total = m * ld;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     int64_t r = i / ld, c = i - r * ld;
-    out[i] = c < n ? syn_value<T>(syn_hash(seed, stream, (uint64_t)(r * n + c)), kind, syn_colscale_exp(seed, (uint64_t)c))
+    out[i] = c < n ? syn_value<T>(syn_hash(seed, stream, (uint64_t)((row0 + r) * n + c)), kind, syn_colscale_exp(seed, (uint64_t)c))
                    : (T)NAN;
   }
 }
@@ -68,12 +68,12 @@ static int grid_for(int64_t work) {
 
 extern "C" {
 
-int synth_dense_cuda(int64_t m, int64_t n, int64_t ld, int dtype, int kind, uint64_t seed, uint64_t stream, void* out,
+int synth_dense_cuda(int64_t m, int64_t n, int64_t ld, int64_t row0, int dtype, int kind, uint64_t seed, uint64_t stream, void* out,
                      cudaStream_t s) {
   if (m < 0 || n < 0 || ld < n) return 1;
   if (m == 0 || ld == 0) return 0;
-  if (dtype == SYN_F64) k_dense<double><<<grid_for(m * ld), 256, 0, s>>>(m, n, ld, kind, seed, stream, (double*)out);
-  else k_dense<float><<<grid_for(m * ld), 256, 0, s>>>(m, n, ld, kind, seed, stream, (float*)out);
+  if (dtype == SYN_F64) k_dense<double><<<grid_for(m * ld), 256, 0, s>>>(m, n, ld, row0, kind, seed, stream, (double*)out);
+  else k_dense<float><<<grid_for(m * ld), 256, 0, s>>>(m, n, ld, row0, kind, seed, stream, (float*)out);
   return cudaGetLastError() == cudaSuccess ? 0 : 2;
 }
 

@@ -11,10 +11,10 @@
 #define SYN_F32 0
 #define SYN_F64 1
 
-/* Dense row-major matrix, m rows, n logical columns, row stride ld >= n (elements).
-   Element (r, c) = value(hash(seed, stream, r*n + c)); padding columns c >= n hold NaN
+/* Dense row-major matrix: rows [row0, row0+m) of the seeded matrix, n logical columns, row
+   stride ld >= n (elements).  Element (r, c) = value(hash(seed, stream, r*n + c)); padding columns c >= n hold NaN
    so that any read of padding by a consumer shows up in its result. */
-int synth_dense(int64_t m, int64_t n, int64_t ld, int dtype, int kind, uint64_t seed,
+int synth_dense(int64_t m, int64_t n, int64_t ld, int64_t row0, int dtype, int kind, uint64_t seed,
                 uint64_t stream, void* out) {
   if (m < 0 || n < 0 || ld < n) return 1;
 #pragma omp parallel for schedule(static)
@@ -22,12 +22,12 @@ int synth_dense(int64_t m, int64_t n, int64_t ld, int dtype, int kind, uint64_t 
     for (int64_t c = 0; c < ld; ++c) {
       if (dtype == SYN_F64) {
         double* o = (double*)out;
-        o[r * ld + c] = c < n ? syn_value_f64(syn_hash(seed, stream, (uint64_t)(r * n + c)), kind,
+        o[r * ld + c] = c < n ? syn_value_f64(syn_hash(seed, stream, (uint64_t)((row0 + r) * n + c)), kind,
                                               syn_colscale_exp(seed, (uint64_t)c))
                               : NAN;
       } else {
         float* o = (float*)out;
-        o[r * ld + c] = c < n ? syn_value_f32(syn_hash(seed, stream, (uint64_t)(r * n + c)), kind,
+        o[r * ld + c] = c < n ? syn_value_f32(syn_hash(seed, stream, (uint64_t)((row0 + r) * n + c)), kind,
                                               syn_colscale_exp(seed, (uint64_t)c))
                               : NAN;
       }
