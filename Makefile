@@ -3,11 +3,13 @@
 NVCC     ?= nvcc
 CC       := gcc
 ARCH     := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -shared --expt-relaxed-constexpr
+NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC --expt-relaxed-constexpr
 CFLAGS   := -O2 -fPIC -shared -fopenmp -ffp-contract=off -std=c11 -Wall
 PKG      := paper_conf_ppopp_asharitbrcks15_b200
 CSRC     := $(PKG)/csrc
+OBJDIR   := build/obj
 FP_SRCS  := $(wildcard $(CSRC)/*.cu)
+FP_OBJS  := $(patsubst $(CSRC)/%.cu,$(OBJDIR)/%.o,$(FP_SRCS))
 FP_HDRS  := $(wildcard $(CSRC)/*.cuh) include/fusedpat.h
 
 all: fusedpat oracle synth
@@ -16,8 +18,13 @@ fusedpat: $(PKG)/libfusedpat.so
 oracle: oracle/liboracle.so
 synth: synth/libsynth_host.so synth/libsynth_cuda.so
 
-$(PKG)/libfusedpat.so: $(FP_SRCS) $(FP_HDRS)
-	$(NVCC) $(NVFLAGS) -Iinclude -Xptxas -v -o $@ $(FP_SRCS) -lnccl -lcudart 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
+$(OBJDIR)/%.o: $(CSRC)/%.cu $(FP_HDRS)
+	@mkdir -p $(OBJDIR)
+	$(NVCC) $(NVFLAGS) -Iinclude -Xptxas -v -c -o $@ $< 2> $@.ptxas.log || (cat $@.ptxas.log; exit 1)
+
+$(PKG)/libfusedpat.so: $(FP_OBJS)
+	$(NVCC) $(ARCH) -shared -o $@ $(FP_OBJS) -lnccl -lcudart
+	@cat $(OBJDIR)/*.ptxas.log > $(PKG)/ptxas.log
 
 oracle/liboracle.so: oracle/oracle.c
 	$(CC) $(CFLAGS) -o $@ $< -lm
@@ -26,9 +33,9 @@ synth/libsynth_host.so: synth/synth_host.c synth/synth_core.h
 	$(CC) $(CFLAGS) -o $@ $< -lm
 
 synth/libsynth_cuda.so: synth/synth_cuda.cu synth/synth_core.h
-	$(NVCC) $(NVFLAGS) -o $@ $<
+	$(NVCC) $(NVFLAGS) -shared -o $@ $<
 
 clean:
-	rm -f $(PKG)/libfusedpat.so oracle/liboracle.so synth/libsynth_host.so synth/libsynth_cuda.so
+	rm -rf $(OBJDIR) $(PKG)/libfusedpat.so oracle/liboracle.so synth/libsynth_host.so synth/libsynth_cuda.so
 
 .PHONY: all fusedpat oracle synth clean

@@ -1,0 +1,300 @@
+// dense_kernels.cuh -- fused dense kernels for Eq. (1), re-designing Algorithm 3
+// and its generated form, Listing 2, for sm_100a.
+//
+// What is kept from the paper: a "vector" of VS threads per row, TL elements of the row per
+// thread held in registers (l_X), y held in registers (l_y), the row's partial dot
+// reduced inside the vector and scaled by v[row] (Alg. 3 l.10-22), the row immediately
+// streamed back from the same registers into the thread's register partial of w (l_w,
+// l.23-24), coarsening over rows (l.25), and full unrolling of every TL loop, which the
+// paper obtains by code generation and we obtain by C++ template instantiation.
+// What changed for B200:
+//   - rows are fetched with 256-bit LDG.E.256 streaming loads (L1 no-allocate, L2
+//     evict-first); RPV rows per vector are loaded before any is reduced, so each lane keeps
+//     RPV*32 bytes in flight (memory-level parallelism instead of occupancy alone);
+//   - the vector reduction is an xor-shuffle all-reduce, so every lane gets p[r]*v[r]
+//     without the warp-synchronous volatile smem broadcast of Listing 2, which
+//     is a race on Volta+ independent thread scheduling;
+//   - no zero padding of X or y: predicated tails;
+//   - aggregation: warp xor-shuffle across vectors -> CTA smem (fixed warp order) ->
+//     fp64 grid accumulator + last-CTA finalize (aggregate.cuh) instead of per-thread
+//     atomicAdd into a w pre-initialised with beta*z (Alg. 3 l.6-7, l.26-27).
+//   - VS > 32 (Alg. 3 l.16-22) is the CTA variant: warp shuffle + smem across warps.
+#pragma once
+#include "aggregate.cuh"
+#include "kernels.cuh"
+
+namespace fp {
+
+struct DenseKArgs {
+  int64_t m, n, ld;
+  const void* X;
+  const void* y;
+  const void* v;
+  const void* z;
+  double alpha, beta;
+  void* w;
+  double* acc;
+  unsigned long long* counter;
+  int add_beta_z;
+  int accumulate;
+};
+
+// Warp-granular vector kernel: VS in {1,2,4,8,16,32} lanes per row, NCH chunks of E
+// elements per lane (thread load TL = NCH*E), RPV rows per vector per iteration.
+template <typename T, int VS, int NCH, int E, int RPV, bool HAS_Y, int BS>
+__global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
+  constexpr int VPW = 32 / VS;       // vectors per warp
+  constexpr int NW = BS / 32;        // warps per CTA
+  constexpr int RPW = VPW * RPV;     // rows per warp iteration
+  const T* __restrict__ X = (const T*)a.X;
+  const T* __restrict__ y = (const T*)a.y;
+  const T* __restrict__ v = (const T*)a.v;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int lid = lane & (VS - 1), vid = lane / VS;
+  const int64_t m = a.m, n = a.n, ld = a.ld;
+  const int64_t nfull = n / E;  // chunks lying completely inside the row
+
+  T ly[NCH][E], lw[NCH][E];
+#pragma unroll
+  for (int k = 0; k < NCH; ++k)
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const int64_t col = (int64_t)(k * VS + lid) * E + e;
+      ly[k][e] = (HAS_Y && col < n) ? y[col] : T(0);
+      lw[k][e] = T(0);
+    }
+
+  const int64_t nwarps = (int64_t)gridDim.x * NW;
+  for (int64_t base = ((int64_t)blockIdx.x * NW + warp) * RPW; base < m; base += nwarps * RPW) {
+    T x[RPV][NCH][E];
+    T vr[RPV];
+    bool okr[RPV];
+#pragma unroll
+    for (int i = 0; i < RPV; ++i) {
+      const int64_t row = base + vid * RPV + i;
+      const bool ok = row < m;
+      okr[i] = ok;
+      vr[i] = ok ? (v ? v[row] : T(1)) : T(0);
+      const T* xr = X + (ok ? row : 0) * ld;
+#pragma unroll
+      for (int k = 0; k < NCH; ++k) {
+        const int64_t c = k * VS + lid;
+        if (ok && c < nfull) {
+          fpd::ld_chunk<E * (int)sizeof(T)>(xr + c * E, x[i][k]);
+        } else {
+#pragma unroll
+          for (int e = 0; e < E; ++e) {
+            const int64_t col = c * E + e;
+            x[i][k][e] = (ok && col < n) ? xr[col] : T(0);
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < RPV; ++i) {
+      T q;
+      if constexpr (HAS_Y) {
+        T p = T(0);  // Eq. (2): X[r,:] . y, TL products per lane
+#pragma unroll
+        for (int k = 0; k < NCH; ++k)
+#pragma unroll
+          for (int e = 0; e < E; ++e) p = fma(x[i][k][e], ly[k][e], p);
+        p = fpd::vector_allreduce<VS>(p);  // intra-vector reduce, every lane gets p[r]
+        q = okr[i] ? p * vr[i] : T(0);     // rows past m contribute nothing (even if y has Inf)
+      } else {
+        q = vr[i];  // Table 1 row 1: alpha X^T v
+      }
+#pragma unroll
+      for (int k = 0; k < NCH; ++k)  // Eq. (3): l_w += X[r,:]^T q, same registers
+#pragma unroll
+        for (int e = 0; e < E; ++e) lw[k][e] = fma(x[i][k][e], q, lw[k][e]);
+    }
+  }
+
+  // ---- aggregation: vectors of a warp (xor over the vector-id lane bits) -> CTA -> grid
+#pragma unroll
+  for (int k = 0; k < NCH; ++k)
+#pragma unroll
+    for (int e = 0; e < E; ++e)
+#pragma unroll
+      for (int off = VS; off < 32; off <<= 1) lw[k][e] += __shfl_xor_sync(0xffffffffu, lw[k][e], off);
+
+  extern __shared__ double sw[];  // n doubles
+  for (int64_t j = threadIdx.x; j < n; j += BS) sw[j] = 0.0;
+  __syncthreads();
+  for (int ww = 0; ww < NW; ++ww) {  // fixed warp order: deterministic within the CTA
+    if (warp == ww && vid == 0) {
+#pragma unroll
+      for (int k = 0; k < NCH; ++k)
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          const int64_t col = (int64_t)(k * VS + lid) * E + e;
+          if (col < n) sw[col] += (double)lw[k][e];
+        }
+    }
+    __syncthreads();
+  }
+  fpd::grid_finalize<T, double>(sw, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z, a.accumulate);
+}
+
+// CTA-wide vector (VS = BS > 32; Alg. 3 l.16-22): all BS threads share one row at a time;
+// intra-warp shuffle reduce, then the NW warp sums through double-buffered smem (one
+// barrier per row).  Thread t owns chunks t, t+BS, ... (NCH of them).
+template <typename T, int NCH, int E, bool HAS_Y, int BS>
+__global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
+  constexpr int NW = BS / 32;
+  const T* __restrict__ X = (const T*)a.X;
+  const T* __restrict__ y = (const T*)a.y;
+  const T* __restrict__ v = (const T*)a.v;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t m = a.m, n = a.n, ld = a.ld;
+  const int64_t nfull = n / E;
+  __shared__ T red[2][NW];
+
+  T ly[NCH][E], lw[NCH][E];
+#pragma unroll
+  for (int k = 0; k < NCH; ++k)
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const int64_t col = (int64_t)(k * BS + tid) * E + e;
+      ly[k][e] = (HAS_Y && col < n) ? y[col] : T(0);
+      lw[k][e] = T(0);
+    }
+  int buf = 0;
+  for (int64_t row = blockIdx.x; row < m; row += gridDim.x) {
+    T x[NCH][E];
+    const T* xr = X + row * ld;
+    const T vr = v ? v[row] : T(1);
+#pragma unroll
+    for (int k = 0; k < NCH; ++k) {
+      const int64_t c = k * BS + tid;
+      if (c < nfull) {
+        fpd::ld_chunk<E * (int)sizeof(T)>(xr + c * E, x[k]);
+      } else {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          const int64_t col = c * E + e;
+          x[k][e] = col < n ? xr[col] : T(0);
+        }
+      }
+    }
+    T q;
+    if constexpr (HAS_Y) {
+      T p = T(0);
+#pragma unroll
+      for (int k = 0; k < NCH; ++k)
+#pragma unroll
+        for (int e = 0; e < E; ++e) p = fma(x[k][e], ly[k][e], p);
+      p = fpd::vector_allreduce<32>(p);  // intra-warp (Alg. 3 l.17)
+      if (lane == 0) red[buf][warp] = p;
+      __syncthreads();                   // l.18-19
+      p = T(0);
+#pragma unroll
+      for (int i = 0; i < NW; ++i) p += red[buf][i];  // inter-warp (l.20), same order everywhere
+      buf ^= 1;
+      q = p * vr;
+    } else {
+      q = vr;
+    }
+#pragma unroll
+    for (int k = 0; k < NCH; ++k)
+#pragma unroll
+      for (int e = 0; e < E; ++e) lw[k][e] = fma(x[k][e], q, lw[k][e]);
+  }
+  extern __shared__ double sw[];
+  __syncthreads();
+  // every column has exactly one owner thread in the CTA: no intra-CTA reduction needed
+  for (int64_t j = tid; j < n; j += BS) sw[j] = 0.0;
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < NCH; ++k)
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const int64_t col = (int64_t)(k * BS + tid) * E + e;
+      if (col < n) sw[col] = (double)lw[k][e];
+    }
+  __syncthreads();
+  fpd::grid_finalize<T, double>(sw, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z, a.accumulate);
+}
+
+// ------------------------------------------------------------------------------ dispatch
+// Instantiation sets.  Thread load TL = NCH * E elements is capped at 256 bytes per thread
+// (x, y and w partial all live in registers: 3 x 256 B = 192 registers).  E is the elements
+// of one load: 32 bytes (LDG.256) when X and ld*sizeof(T) are 32-byte aligned, 16 bytes
+// (LDG.128) when 16-byte aligned, else 1 element.
+constexpr int kBS = 256;     // vector-kernel block size
+constexpr int kBSCta = 256;  // CTA-kernel block size
+using DenseKFn = void (*)(const DenseKArgs);
+
+constexpr int rpv_for(int nch, int eb) { return nch * eb <= 32 ? 4 : (nch * eb <= 64 ? 2 : 1); }
+
+template <typename T, int VS, int NCH, int E, bool HY>
+DenseKFn vec_k() {
+  constexpr int EB = E * (int)sizeof(T);
+  if constexpr (NCH * EB <= 256) return k_dense_vector<T, VS, NCH, E, rpv_for(NCH, EB), HY, kBS>;
+  else return nullptr;
+}
+
+template <typename T, int NCH, int E, bool HY>
+DenseKFn cta_k() {
+  if constexpr (NCH * E * (int)sizeof(T) <= 256) return k_dense_cta<T, NCH, E, HY, kBSCta>;
+  else return nullptr;
+}
+
+template <typename T, int E, bool HY>
+DenseKFn pick_vector(int vs, int nch) {
+  if (vs < 32 && nch != 1) return nullptr;
+  switch (vs) {
+    case 1: return vec_k<T, 1, 1, E, HY>();
+    case 2: return vec_k<T, 2, 1, E, HY>();
+    case 4: return vec_k<T, 4, 1, E, HY>();
+    case 8: return vec_k<T, 8, 1, E, HY>();
+    case 16: return vec_k<T, 16, 1, E, HY>();
+    case 32: break;
+    default: return nullptr;
+  }
+  switch (nch) {
+    case 1: return vec_k<T, 32, 1, E, HY>();
+    case 2: return vec_k<T, 32, 2, E, HY>();
+    case 3: return vec_k<T, 32, 3, E, HY>();
+    case 4: return vec_k<T, 32, 4, E, HY>();
+    case 6: return vec_k<T, 32, 6, E, HY>();
+    case 8: return vec_k<T, 32, 8, E, HY>();
+    case 12: return vec_k<T, 32, 12, E, HY>();
+    case 16: return vec_k<T, 32, 16, E, HY>();
+    case 32: return vec_k<T, 32, 32, E, HY>();
+    case 64: return vec_k<T, 32, 64, E, HY>();
+    default: return nullptr;
+  }
+}
+
+template <typename T, int E, bool HY>
+DenseKFn pick_cta(int nch) {
+  switch (nch) {
+    case 1: return cta_k<T, 1, E, HY>();
+    case 2: return cta_k<T, 2, E, HY>();
+    case 4: return cta_k<T, 4, E, HY>();
+    case 8: return cta_k<T, 8, E, HY>();
+    case 16: return cta_k<T, 16, E, HY>();
+    case 32: return cta_k<T, 32, E, HY>();
+    case 64: return cta_k<T, 64, E, HY>();
+    default: return nullptr;
+  }
+}
+
+template <typename T, bool HY>
+DenseKFn pick_t(int variant, int chunk_bytes, int vs, int nch) {
+  constexpr int E32 = 32 / (int)sizeof(T), E16 = 16 / (int)sizeof(T);
+  const bool cta = variant == FP_VAR_DENSE_CTA;
+  if (variant != FP_VAR_DENSE_VECTOR && !cta) return nullptr;
+  if (chunk_bytes == 32) return cta ? pick_cta<T, E32, HY>(nch) : pick_vector<T, E32, HY>(vs, nch);
+  if (chunk_bytes == 16) return cta ? pick_cta<T, E16, HY>(nch) : pick_vector<T, E16, HY>(vs, nch);
+  if (chunk_bytes == (int)sizeof(T)) return cta ? pick_cta<T, 1, HY>(nch) : pick_vector<T, 1, HY>(vs, nch);
+  return nullptr;
+}
+
+// defined in dense_f32.cu / dense_f64.cu (separate translation units: parallel build)
+DenseKFn dense_pick_f32(bool has_y, int variant, int chunk_bytes, int vs, int nch);
+DenseKFn dense_pick_f64(bool has_y, int variant, int chunk_bytes, int vs, int nch);
+
+}  // namespace fp

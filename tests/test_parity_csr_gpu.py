@@ -110,7 +110,7 @@ def test_duplicates_and_unsorted_columns(cuda_dev):
     ci = rng.integers(0, n, rp[-1]).astype(np.int32)               # unsorted, with duplicates
     va = rng.integers(-2, 3, rp[-1]).astype(np.float64)
     y, v, z = rng.integers(-3, 4, n).astype(np.float64), rng.integers(1, 4, m).astype(np.float64), np.ones(n)
-    A = sp.csr_matrix((va, ci, rp), shape=(m, n))
+    A = sp.csr_matrix((va.copy(), ci.copy(), rp.copy()), shape=(m, n))  # scipy dedups in place
     A.sum_duplicates()
     ref = A.T @ (v * (A @ y)) + z
     w = gpu_csr(cuda_dev, torch.from_numpy(rp), torch.from_numpy(ci), torch.from_numpy(va), n, torch.from_numpy(y),
