@@ -385,3 +385,14 @@ def cg_linreg_csr(rowptr, colidx, val, n, labels, eps=1e-3, max_iter=100, tol=1e
           int(max_iter), float(tol), _ptr(w), ctypes.byref(it), _ptr(hist), _dt(val), comm.handle if comm else None,
           _stream(val.device, stream))
     return w, it.value, hist[: it.value + 1]
+
+
+# ------------------------------------------------------------------------------- host sharding
+def shard_slice_csr(rowptr, colidx, val, v, bounds, rank):
+    """Rank `rank`'s rows [bounds[rank], bounds[rank+1]) of a CSR matrix: rowptr rebased to 0,
+    colidx/val/v sliced (views where possible).  Pure host/tensor indexing, no arithmetic of
+    the method."""
+    r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
+    a, b = int(rowptr[r0]), int(rowptr[r1])
+    rp = rowptr[r0:r1 + 1] - a
+    return rp, colidx[a:b], val[a:b], (None if v is None else v[r0:r1])
