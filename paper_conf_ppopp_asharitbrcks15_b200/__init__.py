@@ -26,7 +26,7 @@ LIB_PATH = os.path.join(_HERE, "libfusedpat.so")
 FP_F32, FP_F64 = 0, 1
 STATUS = {0: "FP_OK", 1: "FP_ERR_INVALID_ARG", 2: "FP_ERR_UNSUPPORTED", 3: "FP_ERR_ALIAS", 4: "FP_ERR_INVALID_CSR",
           5: "FP_ERR_CUDA", 6: "FP_ERR_NCCL", 7: "FP_ERR_NOMEM"}
-VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2"}
+VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2", 5: "csr_vector_private"}
 
 
 class FusedPatError(RuntimeError):

@@ -1,0 +1,6 @@
+// csr_f32.cu -- float instantiations of the CSR kernels (csr_kernels.cuh).
+#include "csr_kernels.cuh"
+
+namespace fp {
+CsrKFn csr_pick_f32(bool has_y, int mode, int vs) { return csr_pick_t<float>(has_y, mode, vs); }
+}  // namespace fp

@@ -1,0 +1,305 @@
+// csr_kernels.cuh -- fused CSR kernels for Eq. (1), re-designing
+// Algorithms 1-2 for sm_100a.
+//
+// Kept from the paper: CSR-vector ([3]) -- a vector of VS lanes per row, VS from the
+// mean row length (Eq. 4); the row's dot with y reduced inside the vector
+// (Alg. 2 l.10-12) and multiplied by v[row] by the vector; the same lanes then
+// scatter X[r,:]^T q into a partial w (l.13-14) -- the second touch of the row comes from the
+// registers that loaded it, not from HBM; partial w in shared memory when n fits
+// ("inter-vector aggregation") and in global memory for large n.
+// Changed for B200:
+//   - each warp owns a contiguous row range balanced by nnz + per-row cost, found with a
+//     32-ary warp-cooperative search of rowptr (no coarsening factor C to tune, no tail
+//     imbalance on power-law rows; correctness never depends on it);
+//   - rowptr is fetched 32 rows at a time with one coalesced load and broadcast by shuffle;
+//     RPV row groups are in flight per warp iteration;
+//   - y is staged in shared memory when it fits (the paper bound y to texture);
+//   - the inter-vector aggregation has three modes:
+//       MODE_PRIVATE: one partial w per WARP in shared memory, updated with plain
+//         load-add-store (no atomics: float shared atomics are CAS loops on sm_100a); lanes of
+//         different vectors that hit the same column in one instruction are serialised with
+//         __match_any_sync; the NW warp partials are summed in fixed order at the end;
+//       MODE_SHARED: one partial w per CTA, shared-memory atomicAdd (the paper's SD);
+//       MODE_L2: fire-and-forget red.global.add into the L2-resident w, alpha folded
+//         into q, w pre-written with beta*z by a tiny kernel.
+//     Small-n modes finish with the fp64 grid accumulator + last-CTA finalize (aggregate.cuh).
+#pragma once
+#include "aggregate.cuh"
+#include "kernels.cuh"
+
+namespace fp {
+
+struct CsrKArgs {
+  int64_t m, n, nnz;
+  const int64_t* rowptr;
+  const int32_t* colidx;
+  const void* val;
+  const void* y;
+  const void* v;
+  const void* z;
+  double alpha, beta;
+  void* w;
+  double* acc;
+  unsigned long long* counter;
+  int add_beta_z;
+  int accumulate;
+  int y_in_smem;  // MODE_L2 only: stage y in shared memory (n*s bytes) for the gathers
+};
+
+enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2 };
+
+constexpr int64_t kRowCost = 4;  // a row costs about as much as 4 nonzeros (rowptr, v, reduce)
+
+// First row r in [0, m] with rowptr[r] + kRowCost*r >= t (monotone in r).  Warp-cooperative
+// 32-ary search: ~log32(m) dependent loads instead of log2(m).
+__device__ __forceinline__ int64_t warp_search_rows(const int64_t* __restrict__ rowptr, int64_t m, int64_t t,
+                                                    int lane) {
+  int64_t lo = 0, hi = m;  // answer in [lo, hi]
+  while (hi - lo > 32) {
+    const int64_t span = hi - lo;
+    const int64_t p = lo + (span * (lane + 1)) / 33;
+    const bool below = __ldg(rowptr + p) + kRowCost * p < t;
+    const unsigned bal = __ballot_sync(0xffffffffu, below);
+    const int cnt = __popc(bal);
+    const int64_t plo = __shfl_sync(0xffffffffu, p, cnt > 0 ? cnt - 1 : 0);
+    const int64_t phi = __shfl_sync(0xffffffffu, p, cnt < 32 ? cnt : 31);
+    if (cnt > 0) lo = plo + 1;
+    if (cnt < 32) hi = phi;
+  }
+  const int64_t p = lo + lane;
+  const bool below = p < hi && (__ldg(rowptr + p) + kRowCost * p < t);
+  const unsigned bal = __ballot_sync(0xffffffffu, below);
+  return lo + __popc(bal);
+}
+
+// Warp-private partial update wp[c] += val for the active lanes of a warp; lanes sharing a
+// column in this instruction are serialised in rounds (rare for distinct rows' columns).
+template <typename T>
+__device__ __forceinline__ void warp_private_add(T* wp, int c, T val, bool act, int lane) {
+  const unsigned key = act ? (unsigned)c : (0x80000000u | (unsigned)lane);
+  const unsigned grp = __match_any_sync(0xffffffffu, key);
+  const unsigned cnt = act ? (unsigned)__popc(grp) : 0u;
+  const unsigned rounds = __reduce_max_sync(0xffffffffu, cnt);
+  if (rounds <= 1) {
+    if (act) wp[c] += val;
+  } else {
+    const unsigned rank = __popc(grp & ((1u << lane) - 1u));
+    for (unsigned r = 0; r < rounds; ++r) {
+      if (act && rank == r) wp[c] += val;
+      __syncwarp();
+    }
+  }
+  __syncwarp();
+}
+
+// VS lanes per row, K nonzeros per lane cached in registers (rows up to VS*K are read from
+// HBM exactly once; longer rows re-read their tail from L1/L2 for the scatter, the paper's
+// "likely a cache hit"), RPV row groups per warp iteration.
+template <typename T, int VS, int K, int RPV, bool HAS_Y, int MODE, int BS>
+__global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
+  constexpr int VPW = 32 / VS;
+  constexpr int NW = BS / 32;
+  constexpr int GROUP = VPW * RPV;  // rows per warp iteration
+  static_assert(GROUP <= 32, "rowptr batch holds 32 rows");
+  const int64_t* __restrict__ rowptr = a.rowptr;
+  const int32_t* __restrict__ colidx = a.colidx;
+  const T* __restrict__ val = (const T*)a.val;
+  const T* __restrict__ y = (const T*)a.y;
+  const T* __restrict__ v = (const T*)a.v;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int lid = lane & (VS - 1), vid = lane / VS;
+  const int64_t m = a.m, n = a.n;
+
+  // shared memory: [y_s: n] [w partials: n (SHARED) or NW*n (PRIVATE)]
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* y_s = reinterpret_cast<T*>(smem_raw);
+  const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
+  T* w_s = y_s + (ysm ? n : 0);
+  T* w_mine = MODE == MODE_PRIVATE ? w_s + (int64_t)warp * n : w_s;
+  {
+    const int64_t nw_copies = MODE == MODE_PRIVATE ? NW : (MODE == MODE_SHARED ? 1 : 0);
+    for (int64_t j = threadIdx.x; j < nw_copies * n; j += BS) w_s[j] = T(0);
+    if (ysm)
+      for (int64_t j = threadIdx.x; j < n; j += BS) y_s[j] = y[j];
+    if (nw_copies > 0 || ysm) __syncthreads();
+  }
+  // alpha: folded into q on the L2 path, applied once by the finaliser on the smem paths
+  const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
+  auto Y = [&](int c) -> T { return ysm ? y_s[c] : __ldg(y + c); };
+  auto W_ADD = [&](int c, T val_, bool act) {
+    if constexpr (MODE == MODE_PRIVATE) {
+      warp_private_add(w_mine, c, val_, act, lane);
+    } else if constexpr (MODE == MODE_SHARED) {
+      if (act) atomicAdd(w_s + c, val_);
+    } else {
+      if (act) fpd::red_add((T*)a.w + c, val_);
+    }
+  };
+
+  // ---- this warp's row range, balanced by nnz + kRowCost*rows
+  const int64_t gw = (int64_t)blockIdx.x * NW + warp, tw = (int64_t)gridDim.x * NW;
+  const int64_t total = a.nnz + kRowCost * m;
+  const int64_t r0 = warp_search_rows(rowptr, m, (total * gw) / tw, lane);
+  const int64_t r1 = warp_search_rows(rowptr, m, (total * (gw + 1)) / tw, lane);
+
+  int64_t bstart = r0;  // rows [bstart, bstart+32) have their rowptr in `rp` (lane i: row bstart+i)
+  int64_t rp = (bstart + lane <= m) ? __ldg(rowptr + bstart + lane) : 0;
+  int64_t rp32 = (bstart + 32 <= m) ? __ldg(rowptr + bstart + 32) : 0;
+
+  for (int64_t rb = r0; rb < r1; rb += GROUP) {
+    if (rb + GROUP > bstart + 32) {  // refill the rowptr batch (warp-uniform)
+      bstart = rb;
+      rp = (bstart + lane <= m) ? __ldg(rowptr + bstart + lane) : 0;
+      rp32 = (bstart + 32 <= m) ? __ldg(rowptr + bstart + 32) : 0;
+    }
+    int64_t start[RPV], len[RPV];
+    T vr[RPV];
+    bool any_long = false;
+#pragma unroll
+    for (int i = 0; i < RPV; ++i) {
+      const int64_t row = rb + i * VPW + vid;
+      const int o = (int)(row - bstart);
+      const int64_t s0 = __shfl_sync(0xffffffffu, rp, o & 31);
+      const int64_t s1n = __shfl_sync(0xffffffffu, rp, (o + 1) & 31);
+      const int64_t s1 = (o + 1 == 32) ? rp32 : s1n;
+      const bool ok = row < r1;
+      start[i] = ok ? s0 : 0;
+      len[i] = ok ? s1 - s0 : 0;
+      vr[i] = ok ? (v ? v[row] : T(1)) : T(0);
+      any_long |= len[i] > VS * K;
+    }
+    any_long = __any_sync(0xffffffffu, any_long);
+
+    // ---- first touch: (col, val) into registers
+    int cc[RPV][K];
+    T xv[RPV][K];
+#pragma unroll
+    for (int i = 0; i < RPV; ++i)
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const int64_t idx = lid + k * VS;
+        if (idx < len[i]) {
+          cc[i][k] = fpd::ld_once(colidx + start[i] + idx);
+          xv[i][k] = fpd::ld_once(val + start[i] + idx);
+        } else {
+          cc[i][k] = 0;
+          xv[i][k] = T(0);
+        }
+      }
+    int64_t lmax = 0;
+    if (any_long) {
+#pragma unroll
+      for (int i = 0; i < RPV; ++i) lmax = len[i] > lmax ? len[i] : lmax;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        const int64_t o = __shfl_xor_sync(0xffffffffu, lmax, off);
+        lmax = o > lmax ? o : lmax;
+      }
+    }
+
+    T q[RPV];
+    if constexpr (HAS_Y) {
+      T p[RPV];
+#pragma unroll
+      for (int i = 0; i < RPV; ++i) {  // Eq. (2) / Alg. 2 l.10-11
+        p[i] = T(0);
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (lid + k * VS < len[i]) p[i] = fma(xv[i][k], Y(cc[i][k]), p[i]);
+      }
+      if (any_long) {  // tails of rows longer than VS*K (warp-uniform loop)
+        for (int64_t seg = VS * K; seg < lmax; seg += VS * K) {
+#pragma unroll
+          for (int i = 0; i < RPV; ++i)
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+              const int64_t idx = seg + lid + k * VS;
+              if (idx < len[i]) {
+                const int c = __ldg(colidx + start[i] + idx);
+                p[i] = fma(__ldg(val + start[i] + idx), Y(c), p[i]);
+              }
+            }
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < RPV; ++i) q[i] = fpd::vector_allreduce<VS>(p[i]) * vr[i] * qscale;  // l.12
+    } else {
+#pragma unroll
+      for (int i = 0; i < RPV; ++i) q[i] = vr[i] * qscale;
+    }
+
+    // ---- second touch from registers: Eq. (3) / Alg. 2 l.13-14
+#pragma unroll
+    for (int i = 0; i < RPV; ++i)
+#pragma unroll
+      for (int k = 0; k < K; ++k) W_ADD(cc[i][k], xv[i][k] * q[i], lid + k * VS < len[i]);
+    if (any_long) {
+      for (int64_t seg = VS * K; seg < lmax; seg += VS * K) {
+#pragma unroll
+        for (int i = 0; i < RPV; ++i)
+#pragma unroll
+          for (int k = 0; k < K; ++k) {
+            const int64_t idx = seg + lid + k * VS;
+            const bool act = idx < len[i];
+            int c = 0;
+            T x = T(0);
+            if (act) {
+              c = __ldg(colidx + start[i] + idx);
+              x = __ldg(val + start[i] + idx);
+            }
+            W_ADD(c, x * q[i], act);
+          }
+      }
+    }
+  }
+
+  if constexpr (MODE == MODE_PRIVATE) {
+    __syncthreads();
+    for (int64_t j = threadIdx.x; j < n; j += BS) {  // fixed warp order: deterministic in the CTA
+      T s = w_s[j];
+#pragma unroll
+      for (int ww = 1; ww < NW; ++ww) s += w_s[(int64_t)ww * n + j];
+      w_s[j] = s;
+    }
+    __syncthreads();
+    fpd::grid_finalize<T, T>(w_s, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
+                             a.accumulate);
+  } else if constexpr (MODE == MODE_SHARED) {
+    __syncthreads();
+    fpd::grid_finalize<T, T>(w_s, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
+                             a.accumulate);
+  }
+}
+
+// ------------------------------------------------------------------------------ dispatch
+constexpr int kCsrBS = 256;
+using CsrKFn = void (*)(const CsrKArgs);
+
+// VS -> (K, RPV): a vector caches VS*K nonzeros per row; RPV row groups per iteration.
+template <typename T, bool HY, int MODE>
+CsrKFn csr_pick_vs(int vs) {
+  switch (vs) {
+    case 1: return k_csr_vector<T, 1, 2, 1, HY, MODE, kCsrBS>;
+    case 2: return k_csr_vector<T, 2, 2, 1, HY, MODE, kCsrBS>;
+    case 4: return k_csr_vector<T, 4, 2, 2, HY, MODE, kCsrBS>;
+    case 8: return k_csr_vector<T, 8, 2, 2, HY, MODE, kCsrBS>;
+    case 16: return k_csr_vector<T, 16, 2, 2, HY, MODE, kCsrBS>;
+    case 32: return k_csr_vector<T, 32, 4, 2, HY, MODE, kCsrBS>;
+    default: return nullptr;
+  }
+}
+
+template <typename T>
+CsrKFn csr_pick_t(bool hy, int mode, int vs) {
+  switch (mode) {
+    case MODE_L2: return hy ? csr_pick_vs<T, true, MODE_L2>(vs) : csr_pick_vs<T, false, MODE_L2>(vs);
+    case MODE_SHARED: return hy ? csr_pick_vs<T, true, MODE_SHARED>(vs) : csr_pick_vs<T, false, MODE_SHARED>(vs);
+    case MODE_PRIVATE: return hy ? csr_pick_vs<T, true, MODE_PRIVATE>(vs) : csr_pick_vs<T, false, MODE_PRIVATE>(vs);
+    default: return nullptr;
+  }
+}
+
+CsrKFn csr_pick_f32(bool has_y, int mode, int vs);  // csr_f32.cu
+CsrKFn csr_pick_f64(bool has_y, int mode, int vs);  // csr_f64.cu
+
+}  // namespace fp
