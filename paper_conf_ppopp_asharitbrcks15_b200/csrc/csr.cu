@@ -14,11 +14,15 @@ int mode_of(int variant) {
   }
 }
 
+// entries per lane cached in registers: VS*K covers ~1.6x the mean row for the VS Eq. (4) picks
+int default_k(int vs) { return (vs == 8 || vs == 16) ? 2 : (vs == 32 ? 4 : 4); }
+
 CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int mode = mode_of(L.variant);
   if (mode < 0) return nullptr;
   const bool hy = a.y != nullptr;
-  return a.dtype == FP_F64 ? csr_pick_f64(hy, mode, L.vs) : csr_pick_f32(hy, mode, L.vs);
+  const int k = L.tl > 0 ? L.tl : default_k(L.vs);
+  return a.dtype == FP_F64 ? csr_pick_f64(hy, mode, L.vs, k) : csr_pick_f32(hy, mode, L.vs, k);
 }
 
 constexpr size_t kPrivateBudget = 100 * 1024;  // y + NW warp partials per CTA
@@ -73,7 +77,7 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   L.regs_per_thread = fa.numRegs;
   L.blocks_per_sm = per_sm;
   L.concurrent_warps = per_sm * L.bs / 32;
-  L.tl = 0;
+  L.tl = default_k(L.vs);
   int64_t grid = (int64_t)di.sm_count * per_sm;
   int64_t need = (a.m + (L.bs / L.vs) - 1) / (L.bs / L.vs);  // one row per vector at least
   if (need < 1) need = 1;

@@ -72,24 +72,33 @@ __device__ __forceinline__ int64_t warp_search_rows(const int64_t* __restrict__ 
   return lo + __popc(bal);
 }
 
-// Warp-private partial update wp[c] += val for the active lanes of a warp; lanes sharing a
-// column in this instruction are serialised in rounds (rare for distinct rows' columns).
-template <typename T>
+// Warp-private partial update wp[c] += val (plain load-add-store, no atomics).  Lanes of
+// DIFFERENT vectors may hit the same column, so the VPW vectors of the warp update one after
+// the other.  Inside a vector the lanes hold one row's entries; their columns are distinct
+// when the row is canonical (strictly increasing across lanes -- one shuffle + vote checks
+// it); a non-canonical row (duplicates, reading R7) is serialised lane by lane.
+template <int VS, typename T>
 __device__ __forceinline__ void warp_private_add(T* wp, int c, T val, bool act, int lane) {
-  const unsigned key = act ? (unsigned)c : (0x80000000u | (unsigned)lane);
-  const unsigned grp = __match_any_sync(0xffffffffu, key);
-  const unsigned cnt = act ? (unsigned)__popc(grp) : 0u;
-  const unsigned rounds = __reduce_max_sync(0xffffffffu, cnt);
-  if (rounds <= 1) {
-    if (act) wp[c] += val;
+  constexpr int VPW = 32 / VS;
+  const int lid = lane & (VS - 1), vid = lane / VS;
+  bool ok = true;
+  if constexpr (VS > 1) {
+    const int cn = __shfl_down_sync(0xffffffffu, c, 1);
+    const bool nact = __shfl_down_sync(0xffffffffu, (int)act, 1) != 0;
+    ok = !(act && nact && lid + 1 < VS && cn <= c);
+  }
+  if (__all_sync(0xffffffffu, ok)) {
+#pragma unroll
+    for (int u = 0; u < VPW; ++u) {
+      if (act && vid == u) wp[c] += val;
+      __syncwarp();
+    }
   } else {
-    const unsigned rank = __popc(grp & ((1u << lane) - 1u));
-    for (unsigned r = 0; r < rounds; ++r) {
-      if (act && rank == r) wp[c] += val;
+    for (int l = 0; l < 32; ++l) {
+      if (act && lane == l) wp[c] += val;
       __syncwarp();
     }
   }
-  __syncwarp();
 }
 
 // VS lanes per row, K nonzeros per lane cached in registers (rows up to VS*K are read from
@@ -128,7 +137,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   auto Y = [&](int c) -> T { return ysm ? y_s[c] : __ldg(y + c); };
   auto W_ADD = [&](int c, T val_, bool act) {
     if constexpr (MODE == MODE_PRIVATE) {
-      warp_private_add(w_mine, c, val_, act, lane);
+      warp_private_add<VS>(w_mine, c, val_, act, lane);
     } else if constexpr (MODE == MODE_SHARED) {
       if (act) atomicAdd(w_s + c, val_);
     } else {
@@ -275,31 +284,32 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
 constexpr int kCsrBS = 256;
 using CsrKFn = void (*)(const CsrKArgs);
 
-// VS -> (K, RPV): a vector caches VS*K nonzeros per row; RPV row groups per iteration.
+// (VS, K) -> kernel: a vector caches VS*K nonzeros of a row in registers; RPV row groups per
+// warp iteration (1 for VS <= 2, else 2).  K is fp_launch.tl for the CSR variants.
 template <typename T, bool HY, int MODE>
-CsrKFn csr_pick_vs(int vs) {
-  switch (vs) {
-    case 1: return k_csr_vector<T, 1, 2, 1, HY, MODE, kCsrBS>;
-    case 2: return k_csr_vector<T, 2, 2, 1, HY, MODE, kCsrBS>;
-    case 4: return k_csr_vector<T, 4, 2, 2, HY, MODE, kCsrBS>;
-    case 8: return k_csr_vector<T, 8, 2, 2, HY, MODE, kCsrBS>;
-    case 16: return k_csr_vector<T, 16, 2, 2, HY, MODE, kCsrBS>;
-    case 32: return k_csr_vector<T, 32, 4, 2, HY, MODE, kCsrBS>;
-    default: return nullptr;
-  }
+CsrKFn csr_pick_vs(int vs, int k) {
+#define FP_CSR_K(VS_, K_, RPV_) \
+  if (vs == VS_ && k == K_) return k_csr_vector<T, VS_, K_, RPV_, HY, MODE, kCsrBS>;
+  FP_CSR_K(1, 2, 1) FP_CSR_K(1, 4, 1) FP_CSR_K(2, 2, 1) FP_CSR_K(2, 4, 1)
+  FP_CSR_K(4, 2, 2) FP_CSR_K(4, 4, 2) FP_CSR_K(8, 1, 2) FP_CSR_K(8, 2, 2)
+  FP_CSR_K(16, 1, 2) FP_CSR_K(16, 2, 2) FP_CSR_K(32, 2, 2) FP_CSR_K(32, 4, 2)
+#undef FP_CSR_K
+  return nullptr;
 }
 
 template <typename T>
-CsrKFn csr_pick_t(bool hy, int mode, int vs) {
+CsrKFn csr_pick_t(bool hy, int mode, int vs, int k) {
   switch (mode) {
-    case MODE_L2: return hy ? csr_pick_vs<T, true, MODE_L2>(vs) : csr_pick_vs<T, false, MODE_L2>(vs);
-    case MODE_SHARED: return hy ? csr_pick_vs<T, true, MODE_SHARED>(vs) : csr_pick_vs<T, false, MODE_SHARED>(vs);
-    case MODE_PRIVATE: return hy ? csr_pick_vs<T, true, MODE_PRIVATE>(vs) : csr_pick_vs<T, false, MODE_PRIVATE>(vs);
+    case MODE_L2: return hy ? csr_pick_vs<T, true, MODE_L2>(vs, k) : csr_pick_vs<T, false, MODE_L2>(vs, k);
+    case MODE_SHARED:
+      return hy ? csr_pick_vs<T, true, MODE_SHARED>(vs, k) : csr_pick_vs<T, false, MODE_SHARED>(vs, k);
+    case MODE_PRIVATE:
+      return hy ? csr_pick_vs<T, true, MODE_PRIVATE>(vs, k) : csr_pick_vs<T, false, MODE_PRIVATE>(vs, k);
     default: return nullptr;
   }
 }
 
-CsrKFn csr_pick_f32(bool has_y, int mode, int vs);  // csr_f32.cu
-CsrKFn csr_pick_f64(bool has_y, int mode, int vs);  // csr_f64.cu
+CsrKFn csr_pick_f32(bool has_y, int mode, int vs, int k);  // csr_f32.cu
+CsrKFn csr_pick_f64(bool has_y, int mode, int vs, int k);  // csr_f64.cu
 
 }  // namespace fp
