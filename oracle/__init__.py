@@ -38,7 +38,13 @@ def _lib():
         lib.oracle_csr.argtypes = [i64, i64, vp, vp, vp, vp, vp, vp, dbl, dbl, ci, ci, vp, vp]
         lib.oracle_cg_linreg_dense.argtypes = [i64, i64, vp, i64, vp, dbl, ci, dbl, ci, ci, vp, vp, vp]
         lib.oracle_cg_linreg_csr.argtypes = [i64, i64, vp, vp, vp, vp, dbl, ci, dbl, ci, ci, vp, vp, vp]
-        for f in (lib.oracle_dense, lib.oracle_csr, lib.oracle_cg_linreg_dense, lib.oracle_cg_linreg_csr):
+        lib.oracle_logreg_fgd_dense.argtypes = [i64, i64, vp, i64, vp, dbl, vp, ci, ci, vp, vp, vp]
+        lib.oracle_logreg_fgd_csr.argtypes = [i64, i64, vp, vp, vp, vp, dbl, vp, ci, ci, vp, vp, vp]
+        lib.oracle_logreg_tron_dense.argtypes = [i64, i64, vp, i64, vp, dbl, dbl, ci, ci, ci, ci, vp, vp, vp]
+        lib.oracle_logreg_tron_csr.argtypes = [i64, i64, vp, vp, vp, vp, dbl, dbl, ci, ci, ci, ci, vp, vp, vp]
+        for f in (lib.oracle_dense, lib.oracle_csr, lib.oracle_cg_linreg_dense, lib.oracle_cg_linreg_csr,
+                  lib.oracle_logreg_fgd_dense, lib.oracle_logreg_fgd_csr, lib.oracle_logreg_tron_dense,
+                  lib.oracle_logreg_tron_csr):
             f.restype = ci
         _LIB = lib
     return _LIB
@@ -122,6 +128,65 @@ def cg_linreg_dense(X, labels, eps=1e-3, max_iter=100, tol=1e-6, threads=None):
                                        _ptr(hist))
     if rc != 0:
         raise ValueError(f"oracle_cg_linreg_dense rc={rc}")
+    return w, it.value, hist[: it.value + 1]
+
+
+def logreg_fgd_dense(X, labels, C, w, threads=None):
+    """(f, g, D) of L2-regularised logistic regression at w (reading R20)."""
+    X, labels = _np(X), _np(labels)
+    m, n = X.shape
+    w = np.ascontiguousarray(w, dtype=np.float64)
+    f = ctypes.c_double(0.0)
+    g, D = np.zeros(n), np.zeros(m)
+    rc = _lib().oracle_logreg_fgd_dense(m, n, _ptr(X), n, _ptr(labels), float(C), _ptr(w), _dtype_code(X),
+                                        threads or default_threads(), ctypes.byref(f), _ptr(g), _ptr(D))
+    if rc != 0:
+        raise ValueError(f"oracle_logreg_fgd_dense rc={rc}")
+    return f.value, g, D
+
+
+def logreg_fgd_csr(m, n, rowptr, colidx, val, labels, C, w, threads=None):
+    rowptr = _np(rowptr).astype(np.int64, copy=False)
+    colidx = _np(colidx).astype(np.int32, copy=False)
+    val, labels = _np(val), _np(labels)
+    w = np.ascontiguousarray(w, dtype=np.float64)
+    f = ctypes.c_double(0.0)
+    g, D = np.zeros(n), np.zeros(m)
+    rc = _lib().oracle_logreg_fgd_csr(m, n, _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(labels), float(C), _ptr(w),
+                                      _dtype_code(val), threads or default_threads(), ctypes.byref(f), _ptr(g),
+                                      _ptr(D))
+    if rc != 0:
+        raise ValueError(f"oracle_logreg_fgd_csr rc={rc}")
+    return f.value, g, D
+
+
+def logreg_tron_dense(X, labels, C=1.0, eps=1e-3, max_iter=50, max_cg=250, threads=None):
+    """TRON (reading R20).  Returns (w, iters, f_history)."""
+    X, labels = _np(X), _np(labels)
+    m, n = X.shape
+    w = np.zeros(n)
+    it = ctypes.c_int(0)
+    hist = np.full(max_iter + 1, np.nan)
+    rc = _lib().oracle_logreg_tron_dense(m, n, _ptr(X), n, _ptr(labels), float(C), float(eps), int(max_iter),
+                                         int(max_cg), _dtype_code(X), threads or default_threads(), _ptr(w),
+                                         ctypes.byref(it), _ptr(hist))
+    if rc != 0:
+        raise ValueError(f"oracle_logreg_tron_dense rc={rc}")
+    return w, it.value, hist[: it.value + 1]
+
+
+def logreg_tron_csr(m, n, rowptr, colidx, val, labels, C=1.0, eps=1e-3, max_iter=50, max_cg=250, threads=None):
+    rowptr = _np(rowptr).astype(np.int64, copy=False)
+    colidx = _np(colidx).astype(np.int32, copy=False)
+    val, labels = _np(val), _np(labels)
+    w = np.zeros(n)
+    it = ctypes.c_int(0)
+    hist = np.full(max_iter + 1, np.nan)
+    rc = _lib().oracle_logreg_tron_csr(m, n, _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(labels), float(C),
+                                       float(eps), int(max_iter), int(max_cg), _dtype_code(val),
+                                       threads or default_threads(), _ptr(w), ctypes.byref(it), _ptr(hist))
+    if rc != 0:
+        raise ValueError(f"oracle_logreg_tron_csr rc={rc}")
     return w, it.value, hist[: it.value + 1]
 
 

@@ -92,6 +92,13 @@ _SIGS = {
     "fp_shard_rows_csr": (_int, [_i64, _vp, _int, _vp]),
     "fp_dense_dist": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp, _vp]),
     "fp_csr_dist": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp, _vp]),
+    "fp_dense_epi": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int, _dbl, _vp, _vp, _vp]),
+    "fp_csr_epi": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int, _dbl, _vp, _vp,
+                          _vp]),
+    "fp_logreg_tron_dense": (_int, [_i64, _i64, _vp, _i64, _vp, _dbl, _dbl, _int, _int, _vp, _P(_int), _vp, _int, _vp,
+                                    _vp]),
+    "fp_logreg_tron_csr": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _dbl, _dbl, _int, _int, _vp, _P(_int), _vp,
+                                  _int, _vp, _vp]),
     "fp_cg_linreg_dense": (_int, [_i64, _i64, _vp, _i64, _vp, _dbl, _int, _dbl, _vp, _P(_int), _vp, _int, _vp, _vp]),
     "fp_cg_linreg_csr": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _dbl, _int, _dbl, _vp, _P(_int), _vp, _int, _vp,
                                 _vp]),
@@ -396,3 +403,57 @@ def shard_slice_csr(rowptr, colidx, val, v, bounds, rank):
     a, b = int(rowptr[r0]), int(rowptr[r1])
     rp = rowptr[r0:r1 + 1] - a
     return rp, colidx[a:b], val[a:b], (None if v is None else v[r0:r1])
+
+
+# ------------------------------------------------------------------------------- row epilogues
+FP_EPI_LINEAR, FP_EPI_LOGISTIC = 0, 1
+
+
+def dense_epi(X, y, v, z, alpha, beta, epilogue, c=1.0, row_out=None, scalar_out=None, w=None, stream=None):
+    """fp_dense_epi: the fused pass with a row epilogue (see include/fusedpat.h)."""
+    _require_cuda(X, y, v, z, w, row_out, scalar_out)
+    m, n = X.shape
+    ld = X.stride(0) if m > 1 else n
+    if w is None:
+        w = torch.empty(n, dtype=X.dtype, device=X.device)
+    _call("fp_dense_epi", m, n, _ptr(X), ld, _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w), _dt(X),
+          int(epilogue), float(c), _ptr(row_out), _ptr(scalar_out), _stream(X.device, stream))
+    return w
+
+
+def csr_epi(rowptr, colidx, val, n, y, v, z, alpha, beta, epilogue, c=1.0, row_out=None, scalar_out=None, w=None,
+            stream=None):
+    _require_cuda(rowptr, colidx, val, y, v, z, w, row_out, scalar_out)
+    m = rowptr.shape[0] - 1
+    if w is None:
+        w = torch.empty(n, dtype=val.dtype, device=val.device)
+    _call("fp_csr_epi", m, n, val.shape[0], _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(y), _ptr(v), _ptr(z),
+          float(alpha), float(beta), _ptr(w), _dt(val), int(epilogue), float(c), _ptr(row_out), _ptr(scalar_out),
+          _stream(val.device, stream))
+    return w
+
+
+def logreg_tron_dense(X, labels, C=1.0, eps=1e-3, max_iter=50, max_cg=250, comm=None, stream=None):
+    """TRON logistic regression (reading R20).  Returns (w, iters, f_history)."""
+    _require_cuda(X, labels)
+    m, n = X.shape
+    ld = X.stride(0) if m > 1 else n
+    w = torch.empty(n, dtype=X.dtype, device=X.device)
+    it = ctypes.c_int(0)
+    hist = torch.full((max_iter + 1,), float("nan"), dtype=torch.float64)
+    _call("fp_logreg_tron_dense", m, n, _ptr(X), ld, _ptr(labels), float(C), float(eps), int(max_iter), int(max_cg),
+          _ptr(w), ctypes.byref(it), _ptr(hist), _dt(X), comm.handle if comm else None, _stream(X.device, stream))
+    return w, it.value, hist[: it.value + 1]
+
+
+def logreg_tron_csr(rowptr, colidx, val, n, labels, C=1.0, eps=1e-3, max_iter=50, max_cg=250, comm=None,
+                    stream=None):
+    _require_cuda(rowptr, colidx, val, labels)
+    m = rowptr.shape[0] - 1
+    w = torch.empty(n, dtype=val.dtype, device=val.device)
+    it = ctypes.c_int(0)
+    hist = torch.full((max_iter + 1,), float("nan"), dtype=torch.float64)
+    _call("fp_logreg_tron_csr", m, n, val.shape[0], _ptr(rowptr), _ptr(colidx), _ptr(val), _ptr(labels), float(C),
+          float(eps), int(max_iter), int(max_cg), _ptr(w), ctypes.byref(it), _ptr(hist), _dt(val),
+          comm.handle if comm else None, _stream(val.device, stream))
+    return w, it.value, hist[: it.value + 1]

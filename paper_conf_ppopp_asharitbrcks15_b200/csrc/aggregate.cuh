@@ -38,3 +38,44 @@ __device__ __forceinline__ void grid_finalize(const S* __restrict__ sw, int64_t 
 }
 
 }  // namespace fpd
+
+namespace fpd {
+
+// Row epilogue: what the fused kernels do with a row's dot p = X[r,:] . y before the scale-
+// back (Eq. 2).  kind 0: q = v[r] p (Eq. 1), optionally writing p (X y, the margins)
+// to row_out.  kind 1 (logistic-regression gradient, reading R20): v[r] = label in {-1,+1},
+// t = v[r] p, sigma = 1/(1+e^-t); q = C (sigma - 1) v[r]; row_out <- C sigma (1 - sigma) (the
+// Hessian weights D); loss += log(1 + e^-t).  One pass over X gives gradient, D and loss.
+struct RowEpi {
+  int kind;
+  double c;
+  void* row_out;
+  double* loss;
+};
+
+template <typename T>
+__device__ __forceinline__ T row_epilogue(T p, T vr, bool ok, int64_t row, bool writer, const RowEpi& e,
+                                          double& loss_acc) {
+  if (e.kind == 0) {
+    if (writer && ok && e.row_out) ((T*)e.row_out)[row] = p;
+    return ok ? p * vr : T(0);
+  }
+  if (!ok) return T(0);
+  const double t = (double)vr * (double)p;
+  const double sg = 1.0 / (1.0 + exp(-t));
+  if (writer) {
+    if (e.row_out) ((T*)e.row_out)[row] = (T)(e.c * sg * (1.0 - sg));
+    loss_acc += t > 0.0 ? log1p(exp(-t)) : (-t + log1p(exp(t)));
+  }
+  return (T)(e.c * (sg - 1.0) * (double)vr);
+}
+
+// warp-sum the per-thread loss and add it to the global scalar (fp64 atomic)
+__device__ __forceinline__ void flush_loss(const RowEpi& e, double loss_acc) {
+  if (e.kind != 1 || !e.loss) return;
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) loss_acc += __shfl_xor_sync(0xffffffffu, loss_acc, off);
+  if ((threadIdx.x & 31) == 0 && loss_acc != 0.0) atomicAdd(e.loss, loss_acc);
+}
+
+}  // namespace fpd

@@ -60,8 +60,20 @@ static fp_status check_csr(const PatternArgs& a) {
   return st;
 }
 
+// Row-epilogue arguments (fp_*_epi): kind 1 needs y (the margins' weights) and v (labels);
+// row_out / scalar_out need alpha != 0 (X must be read).  scalar_out is zeroed here.
+static fp_status prepare_epilogue(const PatternArgs& a, cudaStream_t s) {
+  FP_REQUIRE(a.epi_kind == 0 || a.epi_kind == 1, FP_ERR_INVALID_ARG, "unknown epilogue %d", a.epi_kind);
+  if (a.epi_kind == 1) FP_REQUIRE(a.y && a.v, FP_ERR_INVALID_ARG, "logistic epilogue needs y (w) and v (labels)");
+  if (a.epi_kind == 1 || a.row_out)
+    FP_REQUIRE(a.alpha != 0.0, FP_ERR_INVALID_ARG, "row epilogue outputs need alpha != 0");
+  if (a.scalar_out && !a.accumulate) FP_CUDA(cudaMemsetAsync(a.scalar_out, 0, sizeof(double), s));
+  return FP_OK;
+}
+
 fp_status run_dense(const PatternArgs& a, const fp_launch* override_, cudaStream_t s) {
   fp_status st = check_dense(a);
+  if (st == FP_OK) st = prepare_epilogue(a, s);
   if (st != FP_OK || a.n == 0) return st;
   if (a.alpha == 0.0 || a.m == 0)
     return launch_scale_z(a.n, a.add_beta_z ? a.z : nullptr, a.add_beta_z ? a.beta : 0.0, a.w, a.dtype, s);
@@ -77,6 +89,7 @@ fp_status run_dense(const PatternArgs& a, const fp_launch* override_, cudaStream
 
 fp_status run_csr(const PatternArgs& a, const fp_launch* override_, cudaStream_t s) {
   fp_status st = check_csr(a);
+  if (st == FP_OK) st = prepare_epilogue(a, s);
   if (st != FP_OK || a.n == 0) return st;
   if (a.alpha == 0.0 || a.m == 0)
     return launch_scale_z(a.n, a.add_beta_z ? a.z : nullptr, a.add_beta_z ? a.beta : 0.0, a.w, a.dtype, s);
@@ -151,6 +164,28 @@ fp_status fp_csr_ex(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, co
                     const fp_launch* override_, fp_stream stream) {
   return fp::run_csr(fp::csr_args(m, n, nnz, rowptr, colidx, val, y, v, z, alpha, beta, w, dtype), override_,
                      (cudaStream_t)stream);
+}
+
+fp_status fp_dense_epi(int64_t m, int64_t n, const void* X, int64_t ld, const void* y, const void* v, const void* z,
+                       double alpha, double beta, void* w, fp_dtype dtype, int epilogue, double c, void* row_out,
+                       double* scalar_out, fp_stream stream) {
+  fp::PatternArgs a = fp::dense_args(m, n, X, ld, y, v, z, alpha, beta, w, dtype);
+  a.epi_kind = epilogue;
+  a.epi_c = c;
+  a.row_out = row_out;
+  a.scalar_out = scalar_out;
+  return fp::run_dense(a, nullptr, (cudaStream_t)stream);
+}
+
+fp_status fp_csr_epi(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                     const void* val, const void* y, const void* v, const void* z, double alpha, double beta, void* w,
+                     fp_dtype dtype, int epilogue, double c, void* row_out, double* scalar_out, fp_stream stream) {
+  fp::PatternArgs a = fp::csr_args(m, n, nnz, rowptr, colidx, val, y, v, z, alpha, beta, w, dtype);
+  a.epi_kind = epilogue;
+  a.epi_c = c;
+  a.row_out = row_out;
+  a.scalar_out = scalar_out;
+  return fp::run_csr(a, nullptr, (cudaStream_t)stream);
 }
 
 fp_status fp_release_workspace(void) {

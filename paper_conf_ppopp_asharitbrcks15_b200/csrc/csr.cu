@@ -105,7 +105,8 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
     if (st != FP_OK) return st;
   }
   CsrKArgs k{a.m, a.n, a.nnz, a.rowptr, a.colidx, a.val, a.y, a.v, a.z, a.alpha, a.beta, a.w,
-             ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (l2 && y_in_smem_l2(a)) ? 1 : 0};
+             ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (l2 && y_in_smem_l2(a)) ? 1 : 0,
+             {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}};
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   f<<<L.grid, L.bs, smem, s>>>(k);
   FP_CUDA(cudaGetLastError());

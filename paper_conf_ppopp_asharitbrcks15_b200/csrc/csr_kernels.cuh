@@ -44,6 +44,7 @@ struct CsrKArgs {
   int add_beta_z;
   int accumulate;
   int y_in_smem;  // MODE_L2 only: stage y in shared memory (n*s bytes) for the gathers
+  fpd::RowEpi epi;
 };
 
 enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2 };
@@ -155,6 +156,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   int64_t rp = (bstart + lane <= m) ? __ldg(rowptr + bstart + lane) : 0;
   int64_t rp32 = (bstart + 32 <= m) ? __ldg(rowptr + bstart + 32) : 0;
 
+  double loss_acc = 0.0;  // logistic epilogue only
   for (int64_t rb = r0; rb < r1; rb += GROUP) {
     if (rb + GROUP > bstart + 32) {  // refill the rowptr batch (warp-uniform)
       bstart = rb;
@@ -163,6 +165,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
     }
     int64_t start[RPV], len[RPV];
     T vr[RPV];
+    bool okr[RPV];
     bool any_long = false;
 #pragma unroll
     for (int i = 0; i < RPV; ++i) {
@@ -172,6 +175,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
       const int64_t s1n = __shfl_sync(0xffffffffu, rp, (o + 1) & 31);
       const int64_t s1 = (o + 1 == 32) ? rp32 : s1n;
       const bool ok = row < r1;
+      okr[i] = ok;
       start[i] = ok ? s0 : 0;
       len[i] = ok ? s1 - s0 : 0;
       vr[i] = ok ? (v ? v[row] : T(1)) : T(0);
@@ -231,7 +235,10 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
         }
       }
 #pragma unroll
-      for (int i = 0; i < RPV; ++i) q[i] = fpd::vector_allreduce<VS>(p[i]) * vr[i] * qscale;  // l.12
+      for (int i = 0; i < RPV; ++i)  // l.12: q = v[r] * reduce(p) (or the row epilogue)
+        q[i] = fpd::row_epilogue<T>(fpd::vector_allreduce<VS>(p[i]), vr[i], okr[i], rb + i * VPW + vid, lid == 0,
+                                    a.epi, loss_acc) *
+               qscale;
     } else {
 #pragma unroll
       for (int i = 0; i < RPV; ++i) q[i] = vr[i] * qscale;
@@ -261,6 +268,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
       }
     }
   }
+  fpd::flush_loss(a.epi, loss_acc);
 
   if constexpr (MODE == MODE_PRIVATE) {
     __syncthreads();

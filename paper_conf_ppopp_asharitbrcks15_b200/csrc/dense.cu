@@ -134,7 +134,7 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
   Workspace* ws = workspace(s, (size_t)a.n, 0);
   if (!ws) return FP_ERR_NOMEM;
   DenseKArgs k{a.m, a.n, a.ld, a.X, a.y, a.v, a.z, a.alpha, a.beta, a.w, ws->acc, ws->counters, a.add_beta_z ? 1 : 0,
-               a.accumulate ? 1 : 0};
+               a.accumulate ? 1 : 0, {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}};
   const size_t smem = (size_t)a.n * sizeof(double);
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   f<<<L.grid, L.bs, smem, s>>>(k);

@@ -37,6 +37,7 @@ struct DenseKArgs {
   unsigned long long* counter;
   int add_beta_z;
   int accumulate;
+  fpd::RowEpi epi;
 };
 
 // Warp-granular vector kernel: VS in {1,2,4,8,16,32} lanes per row, NCH chunks of E
@@ -65,6 +66,7 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
     }
 
   const int64_t nwarps = (int64_t)gridDim.x * NW;
+  double loss_acc = 0.0;  // logistic epilogue only
   for (int64_t base = ((int64_t)blockIdx.x * NW + warp) * RPW; base < m; base += nwarps * RPW) {
     T x[RPV][NCH][E];
     T vr[RPV];
@@ -100,7 +102,8 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 #pragma unroll
           for (int e = 0; e < E; ++e) p = fma(x[i][k][e], ly[k][e], p);
         p = fpd::vector_allreduce<VS>(p);  // intra-vector reduce, every lane gets p[r]
-        q = okr[i] ? p * vr[i] : T(0);     // rows past m contribute nothing (even if y has Inf)
+        // q = v[r] p (rows past m contribute nothing, even if y has Inf), or the row epilogue
+        q = fpd::row_epilogue<T>(p, vr[i], okr[i], base + vid * RPV + i, lid == 0, a.epi, loss_acc);
       } else {
         q = vr[i];  // Table 1 row 1: alpha X^T v
       }
@@ -119,6 +122,7 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 #pragma unroll
       for (int off = VS; off < 32; off <<= 1) lw[k][e] += __shfl_xor_sync(0xffffffffu, lw[k][e], off);
 
+  fpd::flush_loss(a.epi, loss_acc);
   extern __shared__ double sw[];  // n doubles
   for (int64_t j = threadIdx.x; j < n; j += BS) sw[j] = 0.0;
   __syncthreads();
@@ -161,6 +165,7 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
       lw[k][e] = T(0);
     }
   int buf = 0;
+  double loss_acc = 0.0;
   for (int64_t row = blockIdx.x; row < m; row += gridDim.x) {
     T x[NCH][E];
     const T* xr = X + row * ld;
@@ -192,7 +197,7 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
 #pragma unroll
       for (int i = 0; i < NW; ++i) p += red[buf][i];  // inter-warp (l.20), same order everywhere
       buf ^= 1;
-      q = p * vr;
+      q = fpd::row_epilogue<T>(p, vr, true, row, tid == 0, a.epi, loss_acc);
     } else {
       q = vr;
     }
@@ -201,6 +206,7 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
 #pragma unroll
       for (int e = 0; e < E; ++e) lw[k][e] = fma(x[k][e], q, lw[k][e]);
   }
+  fpd::flush_loss(a.epi, loss_acc);
   extern __shared__ double sw[];
   __syncthreads();
   // every column has exactly one owner thread in the CTA: no intra-CTA reduction needed

@@ -26,6 +26,12 @@ struct PatternArgs {
   // when true the result is ADDED to the current w (w += alpha X^T(v (.) X y) [+ beta z]);
   // used by the host-streaming (out-of-core) path to sum row chunks
   bool accumulate = false;
+  // row epilogue (aggregate.cuh fpd::RowEpi): 0 = Eq. (1) (optionally writing X y to row_out),
+  // 1 = logistic-regression gradient (v = labels, writes D to row_out, loss to scalar_out)
+  int epi_kind = 0;
+  double epi_c = 1.0;
+  void* row_out = nullptr;
+  double* scalar_out = nullptr;
 };
 
 // Dense chooser (B200 plan): fills vs, tl, bs, grid, variant ... for the kernels in dense.cu.
