@@ -20,9 +20,9 @@ int default_k(int vs) { return (vs == 8 || vs == 16) ? 2 : (vs == 32 ? 4 : 4); }
 CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int mode = mode_of(L.variant);
   if (mode < 0) return nullptr;
-  const bool hy = a.y != nullptr;
+  const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
   const int k = L.tl > 0 ? L.tl : default_k(L.vs);
-  return a.dtype == FP_F64 ? csr_pick_f64(hy, mode, L.vs, k) : csr_pick_f32(hy, mode, L.vs, k);
+  return a.dtype == FP_F64 ? csr_pick_f64(ym, mode, L.vs, k) : csr_pick_f32(ym, mode, L.vs, k);
 }
 
 constexpr size_t kPrivateBudget = 100 * 1024;  // y + NW warp partials per CTA

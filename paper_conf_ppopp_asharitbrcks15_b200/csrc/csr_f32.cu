@@ -2,5 +2,5 @@
 #include "csr_kernels.cuh"
 
 namespace fp {
-CsrKFn csr_pick_f32(bool has_y, int mode, int vs, int k) { return csr_pick_t<float>(has_y, mode, vs, k); }
+CsrKFn csr_pick_f32(int ym, int mode, int vs, int k) { return csr_pick_t<float>(ym, mode, vs, k); }
 }  // namespace fp

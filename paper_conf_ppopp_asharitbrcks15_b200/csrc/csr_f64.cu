@@ -2,5 +2,5 @@
 #include "csr_kernels.cuh"
 
 namespace fp {
-CsrKFn csr_pick_f64(bool has_y, int mode, int vs, int k) { return csr_pick_t<double>(has_y, mode, vs, k); }
+CsrKFn csr_pick_f64(int ym, int mode, int vs, int k) { return csr_pick_t<double>(ym, mode, vs, k); }
 }  // namespace fp

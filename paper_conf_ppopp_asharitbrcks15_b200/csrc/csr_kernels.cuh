@@ -105,7 +105,7 @@ __device__ __forceinline__ void warp_private_add(T* wp, int c, T val, bool act, 
 // VS lanes per row, K nonzeros per lane cached in registers (rows up to VS*K are read from
 // HBM exactly once; longer rows re-read their tail from L1/L2 for the scatter, the paper's
 // "likely a cache hit"), RPV row groups per warp iteration.
-template <typename T, int VS, int K, int RPV, bool HAS_Y, int MODE, int BS>
+template <typename T, int VS, int K, int RPV, int YM, int MODE, int BS>
 __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   constexpr int VPW = 32 / VS;
   constexpr int NW = BS / 32;
@@ -123,6 +123,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   // shared memory: [y_s: n] [w partials: n (SHARED) or NW*n (PRIVATE)]
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* y_s = reinterpret_cast<T*>(smem_raw);
+  constexpr bool HAS_Y = YM != 0;
   const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
   T* w_s = y_s + (ysm ? n : 0);
   T* w_mine = MODE == MODE_PRIVATE ? w_s + (int64_t)warp * n : w_s;
@@ -236,9 +237,12 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
       }
 #pragma unroll
       for (int i = 0; i < RPV; ++i)  // l.12: q = v[r] * reduce(p) (or the row epilogue)
-        q[i] = fpd::row_epilogue<T>(fpd::vector_allreduce<VS>(p[i]), vr[i], okr[i], rb + i * VPW + vid, lid == 0,
-                                    a.epi, loss_acc) *
-               qscale;
+        if constexpr (YM == 2)
+          q[i] = fpd::row_epilogue<T>(fpd::vector_allreduce<VS>(p[i]), vr[i], okr[i], rb + i * VPW + vid, lid == 0,
+                                      a.epi, loss_acc) *
+                 qscale;
+        else
+          q[i] = fpd::vector_allreduce<VS>(p[i]) * vr[i] * qscale;
     } else {
 #pragma unroll
       for (int i = 0; i < RPV; ++i) q[i] = vr[i] * qscale;
@@ -268,7 +272,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
       }
     }
   }
-  fpd::flush_loss(a.epi, loss_acc);
+  if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
 
   if constexpr (MODE == MODE_PRIVATE) {
     __syncthreads();
@@ -294,10 +298,10 @@ using CsrKFn = void (*)(const CsrKArgs);
 
 // (VS, K) -> kernel: a vector caches VS*K nonzeros of a row in registers; RPV row groups per
 // warp iteration (1 for VS <= 2, else 2).  K is fp_launch.tl for the CSR variants.
-template <typename T, bool HY, int MODE>
+template <typename T, int YM, int MODE>
 CsrKFn csr_pick_vs(int vs, int k) {
 #define FP_CSR_K(VS_, K_, RPV_) \
-  if (vs == VS_ && k == K_) return k_csr_vector<T, VS_, K_, RPV_, HY, MODE, kCsrBS>;
+  if (vs == VS_ && k == K_) return k_csr_vector<T, VS_, K_, RPV_, YM, MODE, kCsrBS>;
   FP_CSR_K(1, 2, 1) FP_CSR_K(1, 4, 1) FP_CSR_K(2, 2, 1) FP_CSR_K(2, 4, 1)
   FP_CSR_K(4, 2, 2) FP_CSR_K(4, 4, 2) FP_CSR_K(8, 1, 2) FP_CSR_K(8, 2, 2)
   FP_CSR_K(16, 1, 2) FP_CSR_K(16, 2, 2) FP_CSR_K(32, 2, 2) FP_CSR_K(32, 4, 2)
@@ -305,19 +309,28 @@ CsrKFn csr_pick_vs(int vs, int k) {
   return nullptr;
 }
 
-template <typename T>
-CsrKFn csr_pick_t(bool hy, int mode, int vs, int k) {
+template <typename T, int YM>
+CsrKFn csr_pick_m(int mode, int vs, int k) {
   switch (mode) {
-    case MODE_L2: return hy ? csr_pick_vs<T, true, MODE_L2>(vs, k) : csr_pick_vs<T, false, MODE_L2>(vs, k);
-    case MODE_SHARED:
-      return hy ? csr_pick_vs<T, true, MODE_SHARED>(vs, k) : csr_pick_vs<T, false, MODE_SHARED>(vs, k);
-    case MODE_PRIVATE:
-      return hy ? csr_pick_vs<T, true, MODE_PRIVATE>(vs, k) : csr_pick_vs<T, false, MODE_PRIVATE>(vs, k);
+    case MODE_L2: return csr_pick_vs<T, YM, MODE_L2>(vs, k);
+    case MODE_SHARED: return csr_pick_vs<T, YM, MODE_SHARED>(vs, k);
+    case MODE_PRIVATE: return csr_pick_vs<T, YM, MODE_PRIVATE>(vs, k);
     default: return nullptr;
   }
 }
 
-CsrKFn csr_pick_f32(bool has_y, int mode, int vs, int k);  // csr_f32.cu
-CsrKFn csr_pick_f64(bool has_y, int mode, int vs, int k);  // csr_f64.cu
+// ym: 0 = no y (Table 1 row 1), 1 = Eq. (1), 2 = Eq. (1) with a row epilogue
+template <typename T>
+CsrKFn csr_pick_t(int ym, int mode, int vs, int k) {
+  switch (ym) {
+    case 0: return csr_pick_m<T, 0>(mode, vs, k);
+    case 1: return csr_pick_m<T, 1>(mode, vs, k);
+    case 2: return csr_pick_m<T, 2>(mode, vs, k);
+    default: return nullptr;
+  }
+}
+
+CsrKFn csr_pick_f32(int ym, int mode, int vs, int k);  // csr_f32.cu
+CsrKFn csr_pick_f64(int ym, int mode, int vs, int k);  // csr_f64.cu
 
 }  // namespace fp

@@ -36,8 +36,9 @@ DenseKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int ce = cb / (int)dtype_size(a.dtype);
   if (L.tl <= 0 || L.tl % ce != 0) return nullptr;
   const int nch = L.tl / ce;
-  const bool hy = a.y != nullptr;
-  return a.dtype == FP_F64 ? dense_pick_f64(hy, L.variant, cb, L.vs, nch) : dense_pick_f32(hy, L.variant, cb, L.vs, nch);
+  // 0: no y (Table 1 row 1); 1: Eq. (1) fast path; 2: Eq. (1) + row epilogue (outputs / logistic)
+  const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
+  return a.dtype == FP_F64 ? dense_pick_f64(ym, L.variant, cb, L.vs, nch) : dense_pick_f32(ym, L.variant, cb, L.vs, nch);
 }
 
 int round_up_in(int need, const int* set, int cnt) {

@@ -1,8 +1,14 @@
-// dense_f64.cu -- fp64 instantiations of the dense kernels (dense_kernels.cuh).
+// dense_f64.cu -- double instantiations of the dense kernels (dense_kernels.cuh).
 #include "dense_kernels.cuh"
 
 namespace fp {
-DenseKFn dense_pick_f64(bool has_y, int variant, int chunk_bytes, int vs, int nch) {
-  return has_y ? pick_t<double, true>(variant, chunk_bytes, vs, nch) : pick_t<double, false>(variant, chunk_bytes, vs, nch);
+// ym: 0 = no y (Table 1 row 1), 1 = Eq. (1), 2 = Eq. (1) with a row epilogue
+DenseKFn dense_pick_f64(int ym, int variant, int chunk_bytes, int vs, int nch) {
+  switch (ym) {
+    case 0: return pick_t<double, 0>(variant, chunk_bytes, vs, nch);
+    case 1: return pick_t<double, 1>(variant, chunk_bytes, vs, nch);
+    case 2: return pick_t<double, 2>(variant, chunk_bytes, vs, nch);
+    default: return nullptr;
+  }
 }
 }  // namespace fp

@@ -42,7 +42,7 @@ struct DenseKArgs {
 
 // Warp-granular vector kernel: VS in {1,2,4,8,16,32} lanes per row, NCH chunks of E
 // elements per lane (thread load TL = NCH*E), RPV rows per vector per iteration.
-template <typename T, int VS, int NCH, int E, int RPV, bool HAS_Y, int BS>
+template <typename T, int VS, int NCH, int E, int RPV, int YM, int BS>
 __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
   constexpr int VPW = 32 / VS;       // vectors per warp
   constexpr int NW = BS / 32;        // warps per CTA
@@ -61,7 +61,7 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 #pragma unroll
     for (int e = 0; e < E; ++e) {
       const int64_t col = (int64_t)(k * VS + lid) * E + e;
-      ly[k][e] = (HAS_Y && col < n) ? y[col] : T(0);
+      ly[k][e] = (YM != 0 && col < n) ? y[col] : T(0);
       lw[k][e] = T(0);
     }
 
@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 #pragma unroll
     for (int i = 0; i < RPV; ++i) {
       T q;
-      if constexpr (HAS_Y) {
+      if constexpr (YM != 0) {
         T p = T(0);  // Eq. (2): X[r,:] . y, TL products per lane
 #pragma unroll
         for (int k = 0; k < NCH; ++k)
@@ -103,7 +103,8 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
           for (int e = 0; e < E; ++e) p = fma(x[i][k][e], ly[k][e], p);
         p = fpd::vector_allreduce<VS>(p);  // intra-vector reduce, every lane gets p[r]
         // q = v[r] p (rows past m contribute nothing, even if y has Inf), or the row epilogue
-        q = fpd::row_epilogue<T>(p, vr[i], okr[i], base + vid * RPV + i, lid == 0, a.epi, loss_acc);
+        if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr[i], okr[i], base + vid * RPV + i, lid == 0, a.epi, loss_acc);
+        else q = okr[i] ? p * vr[i] : T(0);
       } else {
         q = vr[i];  // Table 1 row 1: alpha X^T v
       }
@@ -122,7 +123,7 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 #pragma unroll
       for (int off = VS; off < 32; off <<= 1) lw[k][e] += __shfl_xor_sync(0xffffffffu, lw[k][e], off);
 
-  fpd::flush_loss(a.epi, loss_acc);
+  if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
   extern __shared__ double sw[];  // n doubles
   for (int64_t j = threadIdx.x; j < n; j += BS) sw[j] = 0.0;
   __syncthreads();
@@ -144,7 +145,7 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 // CTA-wide vector (VS = BS > 32; Alg. 3 l.16-22): all BS threads share one row at a time;
 // intra-warp shuffle reduce, then the NW warp sums through double-buffered smem (one
 // barrier per row).  Thread t owns chunks t, t+BS, ... (NCH of them).
-template <typename T, int NCH, int E, bool HAS_Y, int BS>
+template <typename T, int NCH, int E, int YM, int BS>
 __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
   constexpr int NW = BS / 32;
   const T* __restrict__ X = (const T*)a.X;
@@ -161,7 +162,7 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
 #pragma unroll
     for (int e = 0; e < E; ++e) {
       const int64_t col = (int64_t)(k * BS + tid) * E + e;
-      ly[k][e] = (HAS_Y && col < n) ? y[col] : T(0);
+      ly[k][e] = (YM != 0 && col < n) ? y[col] : T(0);
       lw[k][e] = T(0);
     }
   int buf = 0;
@@ -184,7 +185,7 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
       }
     }
     T q;
-    if constexpr (HAS_Y) {
+    if constexpr (YM != 0) {
       T p = T(0);
 #pragma unroll
       for (int k = 0; k < NCH; ++k)
@@ -197,7 +198,8 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
 #pragma unroll
       for (int i = 0; i < NW; ++i) p += red[buf][i];  // inter-warp (l.20), same order everywhere
       buf ^= 1;
-      q = fpd::row_epilogue<T>(p, vr, true, row, tid == 0, a.epi, loss_acc);
+      if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr, true, row, tid == 0, a.epi, loss_acc);
+      else q = p * vr;
     } else {
       q = vr;
     }
@@ -206,7 +208,7 @@ __global__ void __launch_bounds__(BS) k_dense_cta(const DenseKArgs a) {
 #pragma unroll
       for (int e = 0; e < E; ++e) lw[k][e] = fma(x[k][e], q, lw[k][e]);
   }
-  fpd::flush_loss(a.epi, loss_acc);
+  if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
   extern __shared__ double sw[];
   __syncthreads();
   // every column has exactly one owner thread in the CTA: no intra-CTA reduction needed
@@ -234,73 +236,73 @@ using DenseKFn = void (*)(const DenseKArgs);
 
 constexpr int rpv_for(int nch, int eb) { return nch * eb <= 32 ? 4 : (nch * eb <= 64 ? 2 : 1); }
 
-template <typename T, int VS, int NCH, int E, bool HY>
+template <typename T, int VS, int NCH, int E, int YM>
 DenseKFn vec_k() {
   constexpr int EB = E * (int)sizeof(T);
-  if constexpr (NCH * EB <= 256) return k_dense_vector<T, VS, NCH, E, rpv_for(NCH, EB), HY, kBS>;
+  if constexpr (NCH * EB <= 256) return k_dense_vector<T, VS, NCH, E, rpv_for(NCH, EB), YM, kBS>;
   else return nullptr;
 }
 
-template <typename T, int NCH, int E, bool HY>
+template <typename T, int NCH, int E, int YM>
 DenseKFn cta_k() {
-  if constexpr (NCH * E * (int)sizeof(T) <= 256) return k_dense_cta<T, NCH, E, HY, kBSCta>;
+  if constexpr (NCH * E * (int)sizeof(T) <= 256) return k_dense_cta<T, NCH, E, YM, kBSCta>;
   else return nullptr;
 }
 
-template <typename T, int E, bool HY>
+template <typename T, int E, int YM>
 DenseKFn pick_vector(int vs, int nch) {
   if (vs < 32 && nch != 1) return nullptr;
   switch (vs) {
-    case 1: return vec_k<T, 1, 1, E, HY>();
-    case 2: return vec_k<T, 2, 1, E, HY>();
-    case 4: return vec_k<T, 4, 1, E, HY>();
-    case 8: return vec_k<T, 8, 1, E, HY>();
-    case 16: return vec_k<T, 16, 1, E, HY>();
+    case 1: return vec_k<T, 1, 1, E, YM>();
+    case 2: return vec_k<T, 2, 1, E, YM>();
+    case 4: return vec_k<T, 4, 1, E, YM>();
+    case 8: return vec_k<T, 8, 1, E, YM>();
+    case 16: return vec_k<T, 16, 1, E, YM>();
     case 32: break;
     default: return nullptr;
   }
   switch (nch) {
-    case 1: return vec_k<T, 32, 1, E, HY>();
-    case 2: return vec_k<T, 32, 2, E, HY>();
-    case 3: return vec_k<T, 32, 3, E, HY>();
-    case 4: return vec_k<T, 32, 4, E, HY>();
-    case 6: return vec_k<T, 32, 6, E, HY>();
-    case 8: return vec_k<T, 32, 8, E, HY>();
-    case 12: return vec_k<T, 32, 12, E, HY>();
-    case 16: return vec_k<T, 32, 16, E, HY>();
-    case 32: return vec_k<T, 32, 32, E, HY>();
-    case 64: return vec_k<T, 32, 64, E, HY>();
+    case 1: return vec_k<T, 32, 1, E, YM>();
+    case 2: return vec_k<T, 32, 2, E, YM>();
+    case 3: return vec_k<T, 32, 3, E, YM>();
+    case 4: return vec_k<T, 32, 4, E, YM>();
+    case 6: return vec_k<T, 32, 6, E, YM>();
+    case 8: return vec_k<T, 32, 8, E, YM>();
+    case 12: return vec_k<T, 32, 12, E, YM>();
+    case 16: return vec_k<T, 32, 16, E, YM>();
+    case 32: return vec_k<T, 32, 32, E, YM>();
+    case 64: return vec_k<T, 32, 64, E, YM>();
     default: return nullptr;
   }
 }
 
-template <typename T, int E, bool HY>
+template <typename T, int E, int YM>
 DenseKFn pick_cta(int nch) {
   switch (nch) {
-    case 1: return cta_k<T, 1, E, HY>();
-    case 2: return cta_k<T, 2, E, HY>();
-    case 4: return cta_k<T, 4, E, HY>();
-    case 8: return cta_k<T, 8, E, HY>();
-    case 16: return cta_k<T, 16, E, HY>();
-    case 32: return cta_k<T, 32, E, HY>();
-    case 64: return cta_k<T, 64, E, HY>();
+    case 1: return cta_k<T, 1, E, YM>();
+    case 2: return cta_k<T, 2, E, YM>();
+    case 4: return cta_k<T, 4, E, YM>();
+    case 8: return cta_k<T, 8, E, YM>();
+    case 16: return cta_k<T, 16, E, YM>();
+    case 32: return cta_k<T, 32, E, YM>();
+    case 64: return cta_k<T, 64, E, YM>();
     default: return nullptr;
   }
 }
 
-template <typename T, bool HY>
+template <typename T, int YM>
 DenseKFn pick_t(int variant, int chunk_bytes, int vs, int nch) {
   constexpr int E32 = 32 / (int)sizeof(T), E16 = 16 / (int)sizeof(T);
   const bool cta = variant == FP_VAR_DENSE_CTA;
   if (variant != FP_VAR_DENSE_VECTOR && !cta) return nullptr;
-  if (chunk_bytes == 32) return cta ? pick_cta<T, E32, HY>(nch) : pick_vector<T, E32, HY>(vs, nch);
-  if (chunk_bytes == 16) return cta ? pick_cta<T, E16, HY>(nch) : pick_vector<T, E16, HY>(vs, nch);
-  if (chunk_bytes == (int)sizeof(T)) return cta ? pick_cta<T, 1, HY>(nch) : pick_vector<T, 1, HY>(vs, nch);
+  if (chunk_bytes == 32) return cta ? pick_cta<T, E32, YM>(nch) : pick_vector<T, E32, YM>(vs, nch);
+  if (chunk_bytes == 16) return cta ? pick_cta<T, E16, YM>(nch) : pick_vector<T, E16, YM>(vs, nch);
+  if (chunk_bytes == (int)sizeof(T)) return cta ? pick_cta<T, 1, YM>(nch) : pick_vector<T, 1, YM>(vs, nch);
   return nullptr;
 }
 
 // defined in dense_f32.cu / dense_f64.cu (separate translation units: parallel build)
-DenseKFn dense_pick_f32(bool has_y, int variant, int chunk_bytes, int vs, int nch);
-DenseKFn dense_pick_f64(bool has_y, int variant, int chunk_bytes, int vs, int nch);
+DenseKFn dense_pick_f32(int ym, int variant, int chunk_bytes, int vs, int nch);
+DenseKFn dense_pick_f64(int ym, int variant, int chunk_bytes, int vs, int nch);
 
 }  // namespace fp
