@@ -10,6 +10,8 @@ int mode_of(int variant) {
     case FP_VAR_CSR_VECTOR: return MODE_SHARED;
     case FP_VAR_CSR_VECTOR_L2: return MODE_L2;
     case FP_VAR_CSR_VECTOR_PRIVATE: return MODE_PRIVATE;
+    case FP_VAR_CSR_FLAT: return DMODE_FLAT_SHARED;
+    case FP_VAR_CSR_FLAT_L2: return DMODE_FLAT_L2;
     default: return -1;
   }
 }
@@ -21,7 +23,8 @@ CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int mode = mode_of(L.variant);
   if (mode < 0) return nullptr;
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
-  const int k = L.tl > 0 ? L.tl : default_k(L.vs);
+  const bool flat = L.variant == FP_VAR_CSR_FLAT || L.variant == FP_VAR_CSR_FLAT_L2;
+  const int k = L.tl > 0 ? L.tl : (flat ? 4 : default_k(L.vs));
   return a.dtype == FP_F64 ? csr_pick_f64(ym, mode, L.vs, k) : csr_pick_f32(ym, mode, L.vs, k);
 }
 
@@ -36,8 +39,10 @@ size_t smem_for(const PatternArgs& a, int variant) {
   const size_t yb = a.y ? vb : 0;
   switch (variant) {
     case FP_VAR_CSR_VECTOR_PRIVATE: return yb + (size_t)(kCsrBS / 32) * vb;
-    case FP_VAR_CSR_VECTOR: return yb + vb;
-    case FP_VAR_CSR_VECTOR_L2: return y_in_smem_l2(a) ? vb : 0;
+    case FP_VAR_CSR_VECTOR:
+    case FP_VAR_CSR_FLAT: return yb + vb;
+    case FP_VAR_CSR_VECTOR_L2:
+    case FP_VAR_CSR_FLAT_L2: return y_in_smem_l2(a) ? vb : 0;
     default: return 0;
   }
 }
@@ -94,7 +99,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: launch plan (variant=%d vs=%d) has no kernel", L.variant, L.vs);
   FP_REQUIRE(L.bs == kCsrBS, FP_ERR_UNSUPPORTED, "fp_csr: block size %d not supported", L.bs);
   FP_REQUIRE(L.grid >= 1, FP_ERR_INVALID_ARG, "fp_csr: grid must be >= 1");
-  const bool l2 = L.variant == FP_VAR_CSR_VECTOR_L2;
+  const bool l2 = L.variant == FP_VAR_CSR_VECTOR_L2 || L.variant == FP_VAR_CSR_FLAT_L2;
   const size_t smem = smem_for(a, L.variant);
   FP_REQUIRE(smem <= 227 * 1024, FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs %zu B shared memory (n too large)",
              L.variant, smem);

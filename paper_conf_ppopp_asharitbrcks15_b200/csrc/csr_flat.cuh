@@ -1,0 +1,162 @@
+// csr_flat.cuh -- "flat" CSR kernel for short rows (included by csr_kernels.cuh).
+//
+// The CSR-vector layout of Algorithm 2 (VS lanes per row) leaves lanes idle when rows
+// are short and ragged (C3: Binomial(1000, 0.01) rows -> ~60 % of the lanes of a VS = 8 warp
+// instruction carry a nonzero).  On sm_100a the scatter into the on-chip partial w costs per
+// instruction, not per useful lane, so idle lanes are paid for.  This kernel keeps the paper's
+// fusion (row dot -> v[r] scale -> scatter of the same row from registers) but maps the warp's
+// lanes onto CONSECUTIVE NONZEROS instead of onto rows:
+//   - a batch = up to 32 consecutive rows whose nonzeros fit in NB tiles of 32 (one coalesced
+//     load per tile, every lane busy); longer rows take a warp-per-row path;
+//   - each lane finds its nonzero's row by a 5-step shuffle binary search of the batch's
+//     rowptr (held one row per lane);
+//   - row dots: y gathered from shared memory, segmented shuffle reduction inside each tile,
+//     segment heads add into a per-warp 32-entry row-sum scratch (heads of one tile have
+//     distinct rows, so plain load-add-store suffices);
+//   - lane i then owns row i: q_i = v_i p_i (or the row epilogue), and every nonzero fetches
+//     its row's q by shuffle and scatters x q into the partial w (shared-memory atomicAdd in
+//     MODE_SHARED, red.global in MODE_L2) -- again with every lane busy.
+#pragma once
+
+namespace fp {
+
+template <typename T, int NB, int YM, int MODE, int BS>
+__global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
+  static_assert(MODE == MODE_SHARED || MODE == MODE_L2, "flat kernel: shared-atomic or L2 aggregation");
+  constexpr int NW = BS / 32;
+  constexpr int CAP = 32 * NB;  // nonzeros per batch
+  const int64_t* __restrict__ rowptr = a.rowptr;
+  const int32_t* __restrict__ colidx = a.colidx;
+  const T* __restrict__ val = (const T*)a.val;
+  const T* __restrict__ y = (const T*)a.y;
+  const T* __restrict__ v = (const T*)a.v;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t m = a.m, n = a.n;
+  constexpr bool HAS_Y = YM != 0;
+
+  // shared memory: [y_s: n (if staged)] [w_s: n (SHARED)] ; static: per-warp row sums
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ T rsum[NW][32];
+  T* y_s = reinterpret_cast<T*>(smem_raw);
+  const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
+  T* w_s = y_s + (ysm ? n : 0);
+  {
+    const int64_t nw_copies = MODE == MODE_SHARED ? 1 : 0;
+    for (int64_t j = threadIdx.x; j < nw_copies * n; j += BS) w_s[j] = T(0);
+    if (ysm)
+      for (int64_t j = threadIdx.x; j < n; j += BS) y_s[j] = y[j];
+    __syncthreads();
+  }
+  const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
+  auto Y = [&](int c) -> T { return ysm ? y_s[c] : __ldg(y + c); };
+  auto W_ADD = [&](int c, T val_) {
+    if constexpr (MODE == MODE_SHARED) atomicAdd(w_s + c, val_);
+    else fpd::red_add((T*)a.w + c, val_);
+  };
+
+  const int64_t gw = (int64_t)blockIdx.x * NW + warp, tw = (int64_t)gridDim.x * NW;
+  const int64_t total = a.nnz + kRowCost * m;
+  const int64_t r0 = warp_search_rows(rowptr, m, (total * gw) / tw, lane);
+  const int64_t r1 = warp_search_rows(rowptr, m, (total * (gw + 1)) / tw, lane);
+  double loss_acc = 0.0;
+
+  for (int64_t rb = r0; rb < r1;) {
+    // ---- batch rows [rb, rb + nrows): lane i holds rowptr[rb + i] (clamped at r1)
+    const int64_t ri = rb + lane < r1 ? rb + lane : r1;
+    const int64_t rp = __ldg(rowptr + ri);
+    const int64_t rp_end = __ldg(rowptr + (rb + 32 < r1 ? rb + 32 : r1));
+    const int64_t a0 = __shfl_sync(0xffffffffu, rp, 0);
+    int64_t nxt = __shfl_down_sync(0xffffffffu, rp, 1);
+    if (lane == 31) nxt = rp_end;
+    const bool fits = (rb + lane < r1) && (nxt - a0 <= CAP);
+    const int nrows = __popc(__ballot_sync(0xffffffffu, fits));  // rowptr monotone: a prefix
+
+    if (nrows == 0) {
+      // ---- a row longer than CAP: warp-per-row, dot pass then scatter pass (tail re-read)
+      const int64_t s0 = a0, L = __shfl_sync(0xffffffffu, nxt, 0) - a0;
+      T p = T(0);
+      if constexpr (HAS_Y) {
+        for (int64_t k = lane; k < L; k += 32) p = fma(__ldg(val + s0 + k), Y(__ldg(colidx + s0 + k)), p);
+        p = fpd::vector_allreduce<32>(p);
+      }
+      const T vr = v ? v[rb] : T(1);
+      T q;
+      if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr, true, rb, lane == 0, a.epi, loss_acc) * qscale;
+      else if constexpr (HAS_Y) q = p * vr * qscale;
+      else q = vr * qscale;
+      for (int64_t k = lane; k < L; k += 32) W_ADD(__ldg(colidx + s0 + k), __ldg(val + s0 + k) * q);
+      rb += 1;
+      continue;
+    }
+    const int64_t cnt = __shfl_sync(0xffffffffu, nxt, nrows - 1) - a0;   // nonzeros in the batch
+    const int rel = lane < nrows ? (int)(rp - a0) : 0x7fffffff;          // row start, batch-relative
+
+    // ---- first touch: NB coalesced tiles of (col, val), every lane busy
+    int cc[NB], rid[NB];
+    T xv[NB];
+#pragma unroll
+    for (int j = 0; j < NB; ++j) {
+      const int pos = j * 32 + lane;
+      const bool act = pos < cnt;
+      cc[j] = act ? fpd::ld_once(colidx + a0 + pos) : 0;
+      xv[j] = act ? fpd::ld_once(val + a0 + pos) : T(0);
+      // row of this nonzero: largest i < nrows with rel_i <= pos (5-step shuffle search)
+      int lo = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const int cand = lo + step;
+        const int rc = __shfl_sync(0xffffffffu, rel, cand & 31);
+        if (cand < nrows && rc <= pos) lo = cand;
+      }
+      rid[j] = lo;
+    }
+
+    T q = T(0);  // lane i: q of row rb + i
+    if constexpr (HAS_Y) {
+      rsum[warp][lane] = T(0);
+      __syncwarp();
+#pragma unroll
+      for (int j = 0; j < NB; ++j) {
+        const int pos = j * 32 + lane;
+        T s = pos < cnt ? xv[j] * Y(cc[j]) : T(0);  // Eq. (2) products
+        // segmented reduction toward the segment head (lanes of a row are contiguous)
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const T t = __shfl_down_sync(0xffffffffu, s, d);
+          const int r2 = __shfl_down_sync(0xffffffffu, rid[j], d);
+          if (lane + d < 32 && r2 == rid[j]) s += t;
+        }
+        const int rprev = __shfl_up_sync(0xffffffffu, rid[j], 1);
+        const bool head = pos < cnt && (lane == 0 || rprev != rid[j]);
+        if (head) rsum[warp][rid[j]] += s;  // heads of one tile hold distinct rows
+        __syncwarp();
+      }
+      const T p = rsum[warp][lane];
+      const int64_t row = rb + lane;
+      const bool ok = lane < nrows;
+      const T vr = ok ? (v ? v[row] : T(1)) : T(0);
+      if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr, ok, row, ok, a.epi, loss_acc) * qscale;
+      else q = ok ? p * vr * qscale : T(0);
+    } else {
+      const int64_t row = rb + lane;
+      q = lane < nrows ? (v ? v[row] : T(1)) * qscale : T(0);
+    }
+
+    // ---- second touch from registers: Eq. (3), every lane busy
+#pragma unroll
+    for (int j = 0; j < NB; ++j) {
+      const T qj = __shfl_sync(0xffffffffu, q, rid[j]);
+      if (j * 32 + lane < cnt) W_ADD(cc[j], xv[j] * qj);
+    }
+    rb += nrows;
+  }
+  if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
+
+  if constexpr (MODE == MODE_SHARED) {
+    __syncthreads();
+    fpd::grid_finalize<T, T>(w_s, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
+                             a.accumulate);
+  }
+}
+
+}  // namespace fp

@@ -296,6 +296,23 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
 constexpr int kCsrBS = 256;
 using CsrKFn = void (*)(const CsrKArgs);
 
+}  // namespace fp
+#include "csr_flat.cuh"
+namespace fp {
+
+// dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
+enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4 };
+
+template <typename T, int YM, int MODE>
+CsrKFn csr_pick_flat(int nb) {
+  switch (nb) {
+    case 2: return k_csr_flat<T, 2, YM, MODE, kCsrBS>;
+    case 4: return k_csr_flat<T, 4, YM, MODE, kCsrBS>;
+    case 8: return k_csr_flat<T, 8, YM, MODE, kCsrBS>;
+    default: return nullptr;
+  }
+}
+
 // (VS, K) -> kernel: a vector caches VS*K nonzeros of a row in registers; RPV row groups per
 // warp iteration (1 for VS <= 2, else 2).  K is fp_launch.tl for the CSR variants.
 template <typename T, int YM, int MODE>
@@ -315,6 +332,8 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case MODE_L2: return csr_pick_vs<T, YM, MODE_L2>(vs, k);
     case MODE_SHARED: return csr_pick_vs<T, YM, MODE_SHARED>(vs, k);
     case MODE_PRIVATE: return csr_pick_vs<T, YM, MODE_PRIVATE>(vs, k);
+    case DMODE_FLAT_SHARED: return csr_pick_flat<T, YM, MODE_SHARED>(k);
+    case DMODE_FLAT_L2: return csr_pick_flat<T, YM, MODE_L2>(k);
     default: return nullptr;
   }
 }

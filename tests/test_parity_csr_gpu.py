@@ -169,3 +169,20 @@ def test_csr_plan_c3_c4(cuda_dev):
     st.mean = 40.0
     L = fp.choose(True, st, fp.FP_F32, 0)
     assert (L.vs, L.variant) == (32, 4)
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("variant", [6, 7])
+@pytest.mark.parametrize("nb", [2, 4, 8])
+@pytest.mark.parametrize("lengths", [("uniform", 0, 70), ("powerlaw", 2.0, 3.0), ("binomial", 0.02)])
+def test_csr_flat_bitexact(cuda_dev, dt, variant, nb, lengths):
+    """Flat kernels (lanes on consecutive nonzeros, rows longer than 32*NB take the warp-per-
+    row path): integer twins bit-exact for every instance."""
+    m, n = 4000, 600
+    rp, ci, va, y, v, z = make_csr(m, n, dt, lengths, seed=nb + variant, kind="int_pm12")
+    L = fp.fp_launch()
+    L.variant, L.vs, L.tl, L.bs, L.grid = variant, 32, nb, 256, 59
+    for args in ((y, v, z, 1.0, 1.0), (None, v, None, -1.0, 0.0), (y, None, None, 2.0, 0.0)):
+        ref, _ = oracle.csr(m, n, rp, ci, va, *args)
+        w = gpu_csr(cuda_dev, rp, ci, va, n, *args, launch=L)
+        assert_bitexact(w, ref, f"flat variant={variant} nb={nb} {lengths}")
