@@ -12,6 +12,7 @@ int mode_of(int variant) {
     case FP_VAR_CSR_VECTOR_PRIVATE: return MODE_PRIVATE;
     case FP_VAR_CSR_FLAT: return DMODE_FLAT_SHARED;
     case FP_VAR_CSR_FLAT_L2: return DMODE_FLAT_L2;
+    case FP_VAR_CSR_FLAT_PRIVATE: return DMODE_FLAT_PRIVATE;
     default: return -1;
   }
 }
@@ -23,7 +24,7 @@ CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int mode = mode_of(L.variant);
   if (mode < 0) return nullptr;
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
-  const bool flat = L.variant == FP_VAR_CSR_FLAT || L.variant == FP_VAR_CSR_FLAT_L2;
+  const bool flat = L.variant >= FP_VAR_CSR_FLAT;
   const int k = L.tl > 0 ? L.tl : (flat ? 4 : default_k(L.vs));
   return a.dtype == FP_F64 ? csr_pick_f64(ym, mode, L.vs, k) : csr_pick_f32(ym, mode, L.vs, k);
 }
@@ -38,7 +39,8 @@ size_t smem_for(const PatternArgs& a, int variant) {
   const size_t vb = (size_t)a.n * dtype_size(a.dtype);
   const size_t yb = a.y ? vb : 0;
   switch (variant) {
-    case FP_VAR_CSR_VECTOR_PRIVATE: return yb + (size_t)(kCsrBS / 32) * vb;
+    case FP_VAR_CSR_VECTOR_PRIVATE:
+    case FP_VAR_CSR_FLAT_PRIVATE: return yb + (size_t)(kCsrBS / 32) * vb;
     case FP_VAR_CSR_VECTOR:
     case FP_VAR_CSR_FLAT: return yb + vb;
     case FP_VAR_CSR_VECTOR_L2:

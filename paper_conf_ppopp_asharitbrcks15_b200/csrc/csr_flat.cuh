@@ -22,7 +22,7 @@ namespace fp {
 
 template <typename T, int NB, int YM, int MODE, int BS>
 __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
-  static_assert(MODE == MODE_SHARED || MODE == MODE_L2, "flat kernel: shared-atomic or L2 aggregation");
+  static_assert(MODE == MODE_SHARED || MODE == MODE_L2 || MODE == MODE_PRIVATE, "flat kernel aggregation mode");
   constexpr int NW = BS / 32;
   constexpr int CAP = 32 * NB;  // nonzeros per batch
   const int64_t* __restrict__ rowptr = a.rowptr;
@@ -40,8 +40,9 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   T* y_s = reinterpret_cast<T*>(smem_raw);
   const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
   T* w_s = y_s + (ysm ? n : 0);
+  T* w_mine = MODE == MODE_PRIVATE ? w_s + (int64_t)warp * n : w_s;
   {
-    const int64_t nw_copies = MODE == MODE_SHARED ? 1 : 0;
+    const int64_t nw_copies = MODE == MODE_PRIVATE ? NW : (MODE == MODE_SHARED ? 1 : 0);
     for (int64_t j = threadIdx.x; j < nw_copies * n; j += BS) w_s[j] = T(0);
     if (ysm)
       for (int64_t j = threadIdx.x; j < n; j += BS) y_s[j] = y[j];
@@ -52,6 +53,25 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   auto W_ADD = [&](int c, T val_) {
     if constexpr (MODE == MODE_SHARED) atomicAdd(w_s + c, val_);
     else fpd::red_add((T*)a.w + c, val_);
+  };
+  // one row's entries spread over the active lanes (long-row path): distinct columns when the
+  // row is canonical; duplicates (R7) are serialised lane by lane
+  auto ROW_ADD = [&](int c, T val_, bool act) {
+    if constexpr (MODE == MODE_PRIVATE) {
+      const int cn = __shfl_down_sync(0xffffffffu, c, 1);
+      const bool nact = __shfl_down_sync(0xffffffffu, (int)act, 1) != 0;
+      if (!__any_sync(0xffffffffu, act && nact && lane < 31 && cn <= c)) {
+        if (act) w_mine[c] += val_;
+      } else {
+        for (int l = 0; l < 32; ++l) {
+          if (act && lane == l) w_mine[c] += val_;
+          __syncwarp();
+        }
+      }
+      __syncwarp();
+    } else {
+      if (act) W_ADD(c, val_);
+    }
   };
 
   const int64_t gw = (int64_t)blockIdx.x * NW + warp, tw = (int64_t)gridDim.x * NW;
@@ -84,7 +104,11 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
       if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr, true, rb, lane == 0, a.epi, loss_acc) * qscale;
       else if constexpr (HAS_Y) q = p * vr * qscale;
       else q = vr * qscale;
-      for (int64_t k = lane; k < L; k += 32) W_ADD(__ldg(colidx + s0 + k), __ldg(val + s0 + k) * q);
+      for (int64_t kb = 0; kb < L; kb += 32) {  // warp-uniform trip count
+        const int64_t k = kb + lane;
+        const bool act = k < L;
+        ROW_ADD(act ? __ldg(colidx + s0 + k) : 0, act ? __ldg(val + s0 + k) * q : T(0), act);
+      }
       rb += 1;
       continue;
     }
@@ -146,13 +170,46 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
 #pragma unroll
     for (int j = 0; j < NB; ++j) {
       const T qj = __shfl_sync(0xffffffffu, q, rid[j]);
-      if (j * 32 + lane < cnt) W_ADD(cc[j], xv[j] * qj);
+      const bool act = j * 32 + lane < cnt;
+      if constexpr (MODE == MODE_PRIVATE) {
+        // per-warp private partial, plain load-add-store: one round per row present in the
+        // tile (columns of one canonical row are distinct; different rows may collide)
+        if (j * 32 >= cnt) break;
+        const int last = (int)(cnt - 1 - j * 32) < 31 ? (int)(cnt - 1 - j * 32) : 31;
+        const int rf = __shfl_sync(0xffffffffu, rid[j], 0), rl = __shfl_sync(0xffffffffu, rid[j], last);
+        const int cn = __shfl_down_sync(0xffffffffu, cc[j], 1);
+        const int rn = __shfl_down_sync(0xffffffffu, rid[j], 1);
+        const bool dup = act && lane < last && rn == rid[j] && cn <= cc[j];  // non-canonical row (R7)
+        const T contrib = xv[j] * qj;
+        if (!__any_sync(0xffffffffu, dup)) {
+          for (int r = rf; r <= rl; ++r) {
+            if (act && rid[j] == r) w_mine[cc[j]] += contrib;
+            __syncwarp();
+          }
+        } else {
+          for (int l = 0; l <= last; ++l) {
+            if (lane == l) w_mine[cc[j]] += contrib;
+            __syncwarp();
+          }
+        }
+      } else {
+        if (act) W_ADD(cc[j], xv[j] * qj);
+      }
     }
     rb += nrows;
   }
   if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
 
-  if constexpr (MODE == MODE_SHARED) {
+  if constexpr (MODE == MODE_PRIVATE) {
+    __syncthreads();
+    for (int64_t j = threadIdx.x; j < n; j += BS) {  // fixed warp order: deterministic in the CTA
+      T s = w_s[j];
+#pragma unroll
+      for (int ww = 1; ww < NW; ++ww) s += w_s[(int64_t)ww * n + j];
+      w_s[j] = s;
+    }
+  }
+  if constexpr (MODE == MODE_SHARED || MODE == MODE_PRIVATE) {
     __syncthreads();
     fpd::grid_finalize<T, T>(w_s, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
                              a.accumulate);

@@ -301,7 +301,7 @@ using CsrKFn = void (*)(const CsrKArgs);
 namespace fp {
 
 // dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
-enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4 };
+enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5 };
 
 template <typename T, int YM, int MODE>
 CsrKFn csr_pick_flat(int nb) {
@@ -334,6 +334,7 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case MODE_PRIVATE: return csr_pick_vs<T, YM, MODE_PRIVATE>(vs, k);
     case DMODE_FLAT_SHARED: return csr_pick_flat<T, YM, MODE_SHARED>(k);
     case DMODE_FLAT_L2: return csr_pick_flat<T, YM, MODE_L2>(k);
+    case DMODE_FLAT_PRIVATE: return csr_pick_flat<T, YM, MODE_PRIVATE>(k);
     default: return nullptr;
   }
 }

@@ -172,7 +172,7 @@ def test_csr_plan_c3_c4(cuda_dev):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f32"])
-@pytest.mark.parametrize("variant", [6, 7])
+@pytest.mark.parametrize("variant", [6, 7, 8])
 @pytest.mark.parametrize("nb", [2, 4, 8])
 @pytest.mark.parametrize("lengths", [("uniform", 0, 70), ("powerlaw", 2.0, 3.0), ("binomial", 0.02)])
 def test_csr_flat_bitexact(cuda_dev, dt, variant, nb, lengths):
