@@ -69,10 +69,16 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   const double mu = a.m > 0 ? (double)a.nnz / (double)a.m : 0.0;
   L.vs = eq4_vector_size(mu);
   L.bs = kCsrBS;
-  if (smem_for(a, FP_VAR_CSR_VECTOR_PRIVATE) <= kPrivateBudget) L.variant = FP_VAR_CSR_VECTOR_PRIVATE;
-  else if (smem_for(a, FP_VAR_CSR_VECTOR) <= kSharedBudget) L.variant = FP_VAR_CSR_VECTOR;
-  else L.variant = FP_VAR_CSR_VECTOR_L2;
+  // Measured on B200 (tools/sweep.py, profiles/r01_sweep_*.json): with y + w on chip the
+  // paper's CSR-vector with the CTA-shared partial and Eq. (4)'s VS is within 2 % of the best
+  // of ~300 settings (C3); the per-warp private and flat variants lose to it because fp64
+  // shared-memory updates cost per instruction.  For large n the flat layout (lanes on
+  // consecutive nonzeros, L2 reds) is best (C4: 17.3 ms vs 19.8 ms for CSR-vector).
+  if (smem_for(a, FP_VAR_CSR_VECTOR) <= kSharedBudget) L.variant = FP_VAR_CSR_VECTOR;
+  else L.variant = FP_VAR_CSR_FLAT_L2;
+  (void)kPrivateBudget;
   L.smem_bytes = (int)smem_for(a, L.variant);
+  L.tl = L.variant >= FP_VAR_CSR_FLAT ? 8 : default_k(L.vs);
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
   if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
@@ -84,7 +90,7 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   L.regs_per_thread = fa.numRegs;
   L.blocks_per_sm = per_sm;
   L.concurrent_warps = per_sm * L.bs / 32;
-  L.tl = default_k(L.vs);
+  L.tl = L.variant >= FP_VAR_CSR_FLAT ? 8 : default_k(L.vs);
   int64_t grid = (int64_t)di.sm_count * per_sm;
   int64_t need = (a.m + (L.bs / L.vs) - 1) / (L.bs / L.vs);  // one row per vector at least
   if (need < 1) need = 1;
