@@ -189,9 +189,13 @@ def run_gpu(args):
     import paper_conf_ppopp_asharitbrcks15_b200 as fp
 
     comm = None
-    if world > 1:
+    if world > 1 or args.force_dist:
         import torch.distributed as dist
 
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29531")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
         dist.init_process_group("nccl", device_id=dev)
         comm = fp.Comm(device=local)
     name = args.config
@@ -258,7 +262,7 @@ def run_gpu(args):
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)
-    if world > 1:
+    if comm is not None:
         import torch.distributed as dist
 
         dist.barrier()
@@ -274,7 +278,7 @@ def run_gpu(args):
         ends[i].record(stream)
     t_end.record(stream)
     torch.cuda.synchronize()
-    if world > 1:
+    if comm is not None:
         dist.barrier()
     clk = clocks.stop()
     step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
@@ -468,6 +472,8 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-seconds", type=float, default=4.0)
     ap.add_argument("--cg-iters", type=int, default=20)
+    ap.add_argument("--force-dist", action="store_true",
+                    help="use the NCCL row-sharded path (fp_*_dist + allreduce) even with one rank")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":

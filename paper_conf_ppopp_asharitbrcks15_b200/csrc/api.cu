@@ -2,6 +2,10 @@
 // validation (every call), alias checks, the alpha == 0 / m == 0 path, plan + launch.
 #include <string.h>
 
+#include <array>
+#include <map>
+#include <mutex>
+
 #include "kernels.cuh"
 
 namespace fp {
@@ -71,6 +75,42 @@ static fp_status prepare_epilogue(const PatternArgs& a, cudaStream_t s) {
   return FP_OK;
 }
 
+// Plan cache: the chooser queries the occupancy API and kernel attributes (host calls of a few
+// microseconds); repeated calls with the same shape class reuse the plan.  The key holds
+// everything a plan depends on (format, device, sizes, dtype, alignment class, y/epilogue
+// mode, presence of y for the smem sizing).
+namespace {
+std::mutex g_plan_mu;
+std::map<std::array<int64_t, 10>, fp_launch> g_plans;
+
+std::array<int64_t, 10> plan_key(bool csr, const PatternArgs& a, int dev) {
+  const int64_t s = (int64_t)dtype_size(a.dtype);
+  const int64_t align = csr ? 0 : (((uintptr_t)a.X % 32 == 0 && (a.ld * s) % 32 == 0) ? 32 :
+                                   (((uintptr_t)a.X % 16 == 0 && (a.ld * s) % 16 == 0) ? 16 : s));
+  const int64_t ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
+  return {csr ? 1 : 0, dev, a.m, a.n, csr ? a.nnz : 0, (int64_t)a.dtype, align, ym, a.y ? 1 : 0, 0};
+}
+}  // namespace
+
+static fp_status cached_plan(bool csr, const PatternArgs& a, fp_launch* L) {
+  const int dev = current_device();
+  const auto key = plan_key(csr, a, dev);
+  {
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    auto it = g_plans.find(key);
+    if (it != g_plans.end()) {
+      *L = it->second;
+      return FP_OK;
+    }
+  }
+  fp_status st = csr ? plan_csr(a, dev, L) : plan_dense(a, dev, L);
+  if (st != FP_OK) return st;
+  std::lock_guard<std::mutex> lk(g_plan_mu);
+  if (g_plans.size() > 4096) g_plans.clear();
+  g_plans[key] = *L;
+  return FP_OK;
+}
+
 fp_status run_dense(const PatternArgs& a, const fp_launch* override_, cudaStream_t s) {
   fp_status st = check_dense(a);
   if (st == FP_OK) st = prepare_epilogue(a, s);
@@ -81,7 +121,7 @@ fp_status run_dense(const PatternArgs& a, const fp_launch* override_, cudaStream
   if (override_) {
     L = *override_;
   } else {
-    st = plan_dense(a, current_device(), &L);
+    st = cached_plan(false, a, &L);
     if (st != FP_OK) return st;
   }
   return launch_dense(a, L, s);
@@ -97,7 +137,7 @@ fp_status run_csr(const PatternArgs& a, const fp_launch* override_, cudaStream_t
   if (override_) {
     L = *override_;
   } else {
-    st = plan_csr(a, current_device(), &L);
+    st = cached_plan(true, a, &L);
     if (st != FP_OK) return st;
   }
   return launch_csr(a, L, s);
