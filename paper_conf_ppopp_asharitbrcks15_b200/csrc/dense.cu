@@ -108,7 +108,9 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
   L.blocks_per_sm = per_sm;
   L.concurrent_warps = per_sm * L.bs / 32;
   const int64_t vectors_per_cta = L.variant == FP_VAR_DENSE_CTA ? 1 : L.bs / L.vs;
-  const int64_t need_ctas = (a.m + vectors_per_cta - 1) / vectors_per_cta;
+  // rows a CTA consumes per iteration: vectors x RPV (rows in flight per vector)
+  const int64_t rpv = L.variant == FP_VAR_DENSE_CTA ? 1 : rpv_for(L.tl / (cb / s), cb);
+  const int64_t need_ctas = (a.m + vectors_per_cta * rpv - 1) / (vectors_per_cta * rpv);
   int64_t grid = (int64_t)di.sm_count * per_sm;
   if (need_ctas < grid) grid = need_ctas > 0 ? need_ctas : 1;
   L.grid = (int)grid;
