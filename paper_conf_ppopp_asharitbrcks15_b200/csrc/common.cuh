@@ -132,6 +132,18 @@ __device__ __forceinline__ double ld_once(const double* p) {
   return r;
 }
 
+// Gathers of y that should stay in L1 (y is re-read randomly; X streams past it).
+__device__ __forceinline__ float ld_keep(const float* p) {
+  float r;
+  asm("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ double ld_keep(const double* p) {
+  double r;
+  asm("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(r) : "l"(p));
+  return r;
+}
+
 // Fire-and-forget fp reduction into global memory (SASS REDG.E.ADD.F32/F64).
 __device__ __forceinline__ void red_add(float* p, float v) { atomicAdd(p, v); }
 __device__ __forceinline__ void red_add(double* p, double v) { atomicAdd(p, v); }

@@ -121,6 +121,9 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
              ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (l2 && y_in_smem_l2(a)) ? 1 : 0,
              {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}};
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // L2 path without y in shared memory: prefer the largest L1 so the random y gathers hit it
+  // (X itself streams with L1::no_allocate and never displaces y)
+  if (l2 && smem == 0) cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
   f<<<L.grid, L.bs, smem, s>>>(k);
   FP_CUDA(cudaGetLastError());
   return FP_OK;

@@ -49,7 +49,7 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
     __syncthreads();
   }
   const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
-  auto Y = [&](int c) -> T { return ysm ? y_s[c] : __ldg(y + c); };
+  auto Y = [&](int c) -> T { return ysm ? y_s[c] : fpd::ld_keep(y + c); };
   auto W_ADD = [&](int c, T val_) {
     if constexpr (MODE == MODE_SHARED) atomicAdd(w_s + c, val_);
     else fpd::red_add((T*)a.w + c, val_);

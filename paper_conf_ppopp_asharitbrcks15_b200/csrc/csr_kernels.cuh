@@ -136,7 +136,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   }
   // alpha: folded into q on the L2 path, applied once by the finaliser on the smem paths
   const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
-  auto Y = [&](int c) -> T { return ysm ? y_s[c] : __ldg(y + c); };
+  auto Y = [&](int c) -> T { return ysm ? y_s[c] : fpd::ld_keep(y + c); };
   auto W_ADD = [&](int c, T val_, bool act) {
     if constexpr (MODE == MODE_PRIVATE) {
       warp_private_add<VS>(w_mine, c, val_, act, lane);
