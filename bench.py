@@ -404,22 +404,17 @@ def run_e2e(args, cfg, inp, comm, world, rank, dev, x_bytes):
 
 
 # ------------------------------------------------------------------------------ CPU oracle
-def _oracle_sample(name, target_s):
-    """Bounded sample of config `name` for the oracle: leading rows of the same seeded matrix
-    (the generator is counter-based, so they are the matrix's actual first rows)."""
+def _oracle_sample(name, rows):
+    """The first `rows` rows of config `name` (the generator is counter-based, so they are the
+    matrix's actual first rows), with the matching slices of v and the full y, z."""
     cfg = synth.CONFIGS[name]
     seed = synth.config_seed(name)
     m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
-    # rows sized for ~target_s of oracle work at ~0.5-1 G entries/s on 16 cores
-    budget_entries = int(3e8 * target_s / 15)
+    rows = max(1, min(m, int(rows)))
     if cfg["fmt"] == "dense":
-        rows = min(m, max(1, budget_entries // n))
-        X = synth.dense(rows, n, dt, kind=cfg["xkind"], seed=seed)
-        data = dict(X=X)
+        data = dict(X=synth.dense(rows, n, dt, kind=cfg["xkind"], seed=seed))
         entries = rows * n
     else:
-        mean = {"C3": 10.0, "C4": 40.0}.get(name, 10.0)
-        rows = min(m, max(1, int(budget_entries / mean)))
         rp, ci, va = synth.csr(rows, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed)
         data = dict(rp=rp, ci=ci, va=va)
         entries = int(va.numel())
@@ -427,6 +422,22 @@ def _oracle_sample(name, target_s):
     v = synth.vector(rows, dt, kind="pos", seed=seed, stream=synth.S_V) if cfg["use_v"] else None
     z = synth.vector(n, dt, seed=seed, stream=synth.S_Z) if cfg["use_z"] else None
     return cfg, rows, entries, data, y, v, z
+
+
+def _calibrated_sample(name, target_s, threads):
+    """A sample sized for ~target_s seconds of oracle work per evaluation (capped at the whole
+    matrix): time a small leading block first, then scale the row count."""
+    cfg = synth.CONFIGS[name]
+    per_row = cfg["n"] if cfg["fmt"] == "dense" else {"C3": 10.0, "C4": 40.0}.get(name, 10.0)
+    rows0 = max(1, min(cfg["m"], int(2e7 / per_row)))
+    smp = _oracle_sample(name, rows0)
+    t0 = time.perf_counter()
+    _oracle_eval(*smp[:1], smp[1], *smp[3:], threads)
+    dt0 = max(time.perf_counter() - t0, 1e-4)
+    rows1 = min(cfg["m"], int(rows0 * target_s / dt0))
+    if rows1 > 1.3 * rows0:
+        smp = _oracle_sample(name, rows1)
+    return smp
 
 
 def _oracle_eval(cfg, rows, data, y, v, z, threads):
@@ -439,8 +450,8 @@ def _oracle_eval(cfg, rows, data, y, v, z, threads):
 
 
 def cpu_baseline(name, target_s=15.0):
-    cfg, rows, entries, data, y, v, z = _oracle_sample(name, target_s)
     threads = os.cpu_count() or 1
+    cfg, rows, entries, data, y, v, z = _calibrated_sample(name, target_s, threads)
     t0 = time.perf_counter()
     _oracle_eval(cfg, rows, data, y, v, z, threads)
     dt = time.perf_counter() - t0
@@ -456,8 +467,8 @@ def run_reference(args):
     if rank != 0:
         return
     name = args.config
-    cfg, rows, entries, data, y, v, z = _oracle_sample(name, args.ref_seconds)
     threads = os.cpu_count() or 1
+    cfg, rows, entries, data, y, v, z = _calibrated_sample(name, args.ref_seconds, threads)
     for _ in range(args.warmup):
         _oracle_eval(cfg, rows, data, y, v, z, threads)
     t0 = time.perf_counter()
@@ -466,7 +477,8 @@ def run_reference(args):
     dt = (time.perf_counter() - t0) / args.steps
     xb, _ = algorithmic_bytes(cfg, rows, entries)
     val = xb / dt / 1e9
-    sample = (f"first {rows:,} of {cfg['m']:,} rows of {name} per step (same generator); "
+    sample = (f"first {rows:,} of {cfg['m']:,} rows of {name} per step (same generator, whole matrix when the "
+              f"oracle finishes it within --ref-seconds); "
               f"GB/s of X streamed by the fp64 oracle")
     out = {"impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "GB/s", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True,
