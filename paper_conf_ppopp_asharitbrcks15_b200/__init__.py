@@ -26,7 +26,8 @@ LIB_PATH = os.path.join(_HERE, "libfusedpat.so")
 FP_F32, FP_F64 = 0, 1
 STATUS = {0: "FP_OK", 1: "FP_ERR_INVALID_ARG", 2: "FP_ERR_UNSUPPORTED", 3: "FP_ERR_ALIAS", 4: "FP_ERR_INVALID_CSR",
           5: "FP_ERR_CUDA", 6: "FP_ERR_NCCL", 7: "FP_ERR_NOMEM"}
-VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2", 5: "csr_vector_private"}
+VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2", 5: "csr_vector_private",
+            6: "csr_flat_smem", 7: "csr_flat_l2", 8: "csr_flat_private", 9: "dense_cluster"}
 
 
 class FusedPatError(RuntimeError):
@@ -51,7 +52,8 @@ class fp_device_profile(ctypes.Structure):
 class fp_launch(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int), ("vs", ctypes.c_int), ("bs", ctypes.c_int), ("tl", ctypes.c_int),
                 ("grid", ctypes.c_int), ("blocks_per_sm", ctypes.c_int), ("rows_per_vector", ctypes.c_int64),
-                ("smem_bytes", ctypes.c_int), ("regs_per_thread", ctypes.c_int), ("concurrent_warps", ctypes.c_int)]
+                ("smem_bytes", ctypes.c_int), ("regs_per_thread", ctypes.c_int), ("concurrent_warps", ctypes.c_int),
+                ("cluster", ctypes.c_int)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_}

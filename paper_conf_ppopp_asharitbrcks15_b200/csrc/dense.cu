@@ -80,16 +80,28 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
       L.bs = kBS;
     } else {
       nch = round_up_in((int)((chunks + kBSCta - 1) / kBSCta), cta_set, 7);
-      if (nch < 0 || nch * cb > 256) {
-        set_error("fp_dense: n=%lld exceeds the register-resident row limit (256 B per thread x %d threads); "
-                  "wide-n dense is not implemented (DESIGN.md NEXT-4)",
-                  (long long)a.n, kBSCta);
-        return FP_ERR_UNSUPPORTED;
+      if (nch > 0 && nch * cb <= 256) {
+        L.variant = FP_VAR_DENSE_CTA;
+        L.vs = kBSCta;
+        L.tl = nch * ce;
+        L.bs = kBSCta;
+      } else {
+        // a cluster of CS CTAs shares the row (VS = CS x BS), full 256-byte thread load
+        const int64_t per_cta = (int64_t)kBSCta * (256 / s);  // elements of a row per CTA
+        int cs = 2;
+        while (cs < 8 && (int64_t)cs * per_cta < a.n) cs <<= 1;
+        if ((int64_t)cs * per_cta < a.n) {
+          set_error("fp_dense: n=%lld exceeds the cluster-resident row limit (%lld elements = 8 CTAs x %d "
+                    "threads x 256 B); wider dense rows are not implemented (DESIGN.md NEXT-4)",
+                    (long long)a.n, (long long)(8 * per_cta), kBSCta);
+          return FP_ERR_UNSUPPORTED;
+        }
+        L.variant = FP_VAR_DENSE_CLUSTER;
+        L.vs = cs * kBSCta;
+        L.tl = 256 / s;
+        L.bs = kBSCta;
+        L.cluster = cs;
       }
-      L.variant = FP_VAR_DENSE_CTA;
-      L.vs = kBSCta;
-      L.tl = nch * ce;
-      L.bs = kBSCta;
     }
   }
   DenseKFn f = pick_any(a, L);
@@ -97,7 +109,8 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
     set_error("fp_dense: no kernel instantiation for vs=%d tl=%d (chunk %d B)", L.vs, L.tl, cb);
     return FP_ERR_UNSUPPORTED;
   }
-  L.smem_bytes = (int)(a.n * sizeof(double));
+  const bool clu = L.variant == FP_VAR_DENSE_CLUSTER;
+  L.smem_bytes = clu ? 0 : (int)(a.n * sizeof(double));
   if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, L.bs, L.smem_bytes);
@@ -107,12 +120,14 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
   L.regs_per_thread = fa.numRegs;
   L.blocks_per_sm = per_sm;
   L.concurrent_warps = per_sm * L.bs / 32;
-  const int64_t vectors_per_cta = L.variant == FP_VAR_DENSE_CTA ? 1 : L.bs / L.vs;
+  const int64_t vectors_per_cta = (L.variant == FP_VAR_DENSE_CTA || clu) ? 1 : L.bs / L.vs;
   // rows a CTA consumes per iteration: vectors x RPV (rows in flight per vector)
-  const int64_t rpv = L.variant == FP_VAR_DENSE_CTA ? 1 : rpv_for(L.tl / (cb / s), cb);
-  const int64_t need_ctas = (a.m + vectors_per_cta * rpv - 1) / (vectors_per_cta * rpv);
+  const int64_t rpv = (L.variant == FP_VAR_DENSE_CTA || clu) ? 1 : rpv_for(L.tl / (cb / s), cb);
+  int64_t need_ctas = (a.m + vectors_per_cta * rpv - 1) / (vectors_per_cta * rpv);
+  if (clu) need_ctas = a.m * L.cluster;  // a cluster of CS CTAs per row
   int64_t grid = (int64_t)di.sm_count * per_sm;
   if (need_ctas < grid) grid = need_ctas > 0 ? need_ctas : 1;
+  if (clu) grid = (grid / L.cluster > 0 ? grid / L.cluster : 1) * L.cluster;
   L.grid = (int)grid;
   L.rows_per_vector = (a.m + grid * vectors_per_cta - 1) / (grid * vectors_per_cta);
   *out = L;
@@ -131,13 +146,32 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
   DenseKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_dense: launch plan (variant=%d vs=%d tl=%d) has no kernel", L.variant, L.vs,
              L.tl);
-  FP_REQUIRE(L.bs == (L.variant == FP_VAR_DENSE_CTA ? kBSCta : kBS), FP_ERR_UNSUPPORTED,
+  const bool clu = L.variant == FP_VAR_DENSE_CLUSTER;
+  FP_REQUIRE(L.bs == ((L.variant == FP_VAR_DENSE_CTA || clu) ? kBSCta : kBS), FP_ERR_UNSUPPORTED,
              "fp_dense: block size %d not supported by the selected kernel", L.bs);
   FP_REQUIRE(L.grid >= 1, FP_ERR_INVALID_ARG, "fp_dense: grid must be >= 1");
+  const int cs = clu ? L.vs / kBSCta : 1;
+  FP_REQUIRE(!clu || (L.grid % cs == 0), FP_ERR_INVALID_ARG, "fp_dense: grid must be a multiple of the cluster size");
   Workspace* ws = workspace(s, (size_t)a.n, 0);
   if (!ws) return FP_ERR_NOMEM;
   DenseKArgs k{a.m, a.n, a.ld, a.X, a.y, a.v, a.z, a.alpha, a.beta, a.w, ws->acc, ws->counters, a.add_beta_z ? 1 : 0,
                a.accumulate ? 1 : 0, {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}};
+  if (clu) {  // thread-block cluster launch: CS CTAs share one row through DSMEM
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)L.grid);
+    cfg.blockDim = dim3((unsigned)L.bs);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)cs;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    FP_CUDA(cudaLaunchKernelEx(&cfg, f, k));
+    return FP_OK;
+  }
   const size_t smem = (size_t)a.n * sizeof(double);
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   f<<<L.grid, L.bs, smem, s>>>(k);

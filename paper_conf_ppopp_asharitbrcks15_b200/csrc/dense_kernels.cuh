@@ -290,9 +290,33 @@ DenseKFn pick_cta(int nch) {
   }
 }
 
+}  // namespace fp
+#include "dense_cluster.cuh"
+namespace fp {
+
+// cluster kernel: always the full 256-byte thread load (NCH = 256 / (E * sizeof(T)))
+template <typename T, int E, int YM>
+DenseKFn pick_cluster(int cs, int nch) {
+  constexpr int NCH = 256 / (E * (int)sizeof(T));
+  if (nch != NCH) return nullptr;
+  switch (cs) {
+    case 2: return k_dense_cluster<T, NCH, E, 2, YM, kBSCta>;
+    case 4: return k_dense_cluster<T, NCH, E, 4, YM, kBSCta>;
+    case 8: return k_dense_cluster<T, NCH, E, 8, YM, kBSCta>;
+    default: return nullptr;
+  }
+}
+
 template <typename T, int YM>
 DenseKFn pick_t(int variant, int chunk_bytes, int vs, int nch) {
   constexpr int E32 = 32 / (int)sizeof(T), E16 = 16 / (int)sizeof(T);
+  if (variant == FP_VAR_DENSE_CLUSTER) {
+    const int cs = vs / kBSCta;
+    if (chunk_bytes == 32) return pick_cluster<T, E32, YM>(cs, nch);
+    if (chunk_bytes == 16) return pick_cluster<T, E16, YM>(cs, nch);
+    if (chunk_bytes == (int)sizeof(T)) return pick_cluster<T, 1, YM>(cs, nch);
+    return nullptr;
+  }
   const bool cta = variant == FP_VAR_DENSE_CTA;
   if (variant != FP_VAR_DENSE_VECTOR && !cta) return nullptr;
   if (chunk_bytes == 32) return cta ? pick_cta<T, E32, YM>(nch) : pick_vector<T, E32, YM>(vs, nch);

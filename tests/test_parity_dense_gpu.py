@@ -177,3 +177,20 @@ def test_plan_reports(cuda_dev):
     st = fp.row_stats_dense(4_000_000, 1000)
     L = fp.choose(False, st, fp.FP_F64, 0)
     assert L.variant == 1 and L.vs == 32 and L.tl == 32
+
+
+@pytest.mark.parametrize("dt,m,n", [("f32", 500, 20000), ("f32", 97, 70001), ("f32", 64, 131072),
+                                    ("f64", 300, 10000), ("f64", 61, 40000), ("f64", 33, 65536)])
+def test_dense_cluster_variant(cuda_dev, dt, m, n):
+    """Rows wider than one CTA's registers: thread-block cluster of CS CTAs, the row's dot
+    reduced through DSMEM (NEXT-4 wide-n dense; the paper's fallback was two gemv)."""
+    X, y, v, z = make(m, n, dt, seed=n + m)
+    st = fp.row_stats_dense(m, n)
+    L = fp.choose(False, st, fp.FP_F32 if dt == "f32" else fp.FP_F64, 0)
+    assert L.variant == 9 and L.cluster in (2, 4, 8)
+    w, ref, mag = run_both(X, y, v, z, "full", cuda_dev)
+    assert_parity(w, ref, mag, DT[dt], f"cluster {dt} {m}x{n}")
+    Xi, yi, vi, zi = make(m, n, dt, seed=7, kind="int_pm12")
+    w, ref, _ = run_both(Xi, yi, vi, zi, "full", cuda_dev)
+    if dt == "f64":
+        assert_bitexact(w, ref, f"cluster twin {m}x{n}")
