@@ -129,8 +129,10 @@ def length_table(spec, n):
         p = float(spec[1])
         cdf = binom.cdf(np.arange(n + 1), n, p)
     elif kind == "powerlaw":
+        # optional 4th entry caps the length (min(cap, n)); the table then has cap+1 entries
         a, xmin = float(spec[1]), float(spec[2])
-        L = np.arange(n + 1, dtype=np.float64)
+        cap = min(n, int(spec[3])) if len(spec) > 3 else n
+        L = np.arange(cap + 1, dtype=np.float64)
         cdf = np.where(L + 1 > xmin, 1.0 - (xmin / (L + 1)) ** (a - 1), 0.0)
     else:
         raise ValueError(spec)
@@ -214,6 +216,15 @@ CONFIGS = {
                beta=1.0, use_v=True, use_z=True, xkind="uniform", desc="CSR fp32 50Mx100K power-law, full with v"),
     "C5": dict(fmt="dense", dtype="f64", m=4_000_000, n=1000, alpha=1.0, beta=1e-3, use_v=False, use_z=True,
                xkind="colscaled", desc="dense fp64 4Mx1000 CG iteration X^T(Xp)+eps p"),
+    # NEXT rows, not BASELINE.json configs:
+    # NEXT-2: KDD2010-shaped ultra-wide CSR (15.0M x 29.9M, 424M nnz at P:419-427): power-law rows of
+    # mean ~28, w and y (240 MB fp64) beyond L2 -> the flat L2/HBM-red path.
+    "K1": dict(fmt="csr", dtype="f64", m=15_009_374, n=29_890_095, lengths=("powerlaw", 2.5, 9.5, 1_000_000),
+               alpha=1.0, beta=1.0, use_v=True, use_z=True, xkind="uniform",
+               desc="CSR fp64 KDD-shaped 15Mx29.9M power-law rows (mean ~28), full with v"),
+    # NEXT-4: dense rows wider than one CTA's registers (thread-block cluster kernel)
+    "W1": dict(fmt="dense", dtype="f32", m=40_000, n=65_536, alpha=1.0, beta=0.0, use_v=False, use_z=False,
+               xkind="uniform", desc="dense fp32 40000x65536 wide rows, X^T(Xy)"),
 }
 
 
