@@ -154,7 +154,8 @@ def build_inputs(name, rank, world, dev):
         else:
             b = [0, m]
         r0, r1 = b[rank], b[rank + 1]
-        rp, ci, va = synth.csr(r1 - r0, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed, row0=r0, device=dev)
+        rp, ci, va = synth.csr(r1 - r0, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed, row0=r0, device=dev,
+                               col_skew=cfg.get("col_skew", 0))
         inp = dict(rowptr=rp, colidx=ci, val=va, m_local=r1 - r0, nnz_local=int(va.numel()), row0=r0)
     inp["y"] = synth.vector(n, dt, seed=seed, stream=synth.S_Y, device=dev)
     inp["v"] = synth.vector(inp["m_local"], dt, kind="pos", seed=seed, stream=synth.S_V, i0=inp["row0"],
@@ -415,7 +416,8 @@ def _oracle_sample(name, rows):
         data = dict(X=synth.dense(rows, n, dt, kind=cfg["xkind"], seed=seed))
         entries = rows * n
     else:
-        rp, ci, va = synth.csr(rows, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed)
+        rp, ci, va = synth.csr(rows, n, dt, cfg["lengths"], kind=cfg["xkind"], seed=seed,
+                               col_skew=cfg.get("col_skew", 0))
         data = dict(rp=rp, ci=ci, va=va)
         entries = int(va.numel())
     y = synth.vector(n, dt, seed=seed, stream=synth.S_Y)

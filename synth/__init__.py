@@ -39,7 +39,7 @@ def _host():
         lib.synth_vector.argtypes = [i64, i64, ci, ci, u64, u64, vp]
         lib.synth_row_lengths.argtypes = [i64, i64, vp, i64, u64, vp]
         lib.synth_rowptr.argtypes = [i64, vp, vp]
-        lib.synth_csr_fill.argtypes = [i64, i64, i64, i64, vp, ci, ci, u64, vp, vp]
+        lib.synth_csr_fill.argtypes = [i64, i64, i64, i64, vp, ci, ci, ci, u64, vp, vp]
         lib.synth_fnv1a.argtypes = [vp, i64]
         lib.synth_fnv1a.restype = u64
         _HOST = lib
@@ -57,7 +57,7 @@ def _cuda():
         lib.synth_vector_cuda.argtypes = [i64, i64, ci, ci, u64, u64, vp, vp]
         lib.synth_row_lengths_cuda.argtypes = [i64, i64, vp, i64, u64, vp, vp]
         lib.synth_rowptr_cuda.argtypes = [i64, vp, vp, vp, ctypes.POINTER(ctypes.c_size_t), vp]
-        lib.synth_csr_fill_cuda.argtypes = [i64, i64, i64, vp, ci, ci, u64, vp, vp, vp]
+        lib.synth_csr_fill_cuda.argtypes = [i64, i64, i64, vp, ci, ci, ci, u64, vp, vp, vp]
         _CUDA = lib
     return _CUDA
 
@@ -143,11 +143,12 @@ def length_table(spec, n):
     return thr
 
 
-def csr(m, n, dtype, lengths, kind="uniform", seed=BASE_SEED, row0=0, device="cpu"):
+def csr(m, n, dtype, lengths, kind="uniform", seed=BASE_SEED, row0=0, device="cpu", col_skew=0):
     """CSR (rowptr int64[m+1], colidx int32[nnz], val[nnz]) for rows [row0, row0+m) of the
     seeded matrix.  Columns are distinct and sorted (stratified-uniform, synth_core.h).
     A shard (row0 > 0) is bit-identical to the slice of the full matrix (its val/col hash index
-    is the GLOBAL nnz index, found from the row lengths of rows [0, row0))."""
+    is the GLOBAL nnz index, found from the row lengths of rows [0, row0)).
+    col_skew > 0 draws Zipf-like skewed columns (synth_core.h syn_column_skew, u^(2^col_skew))."""
     tdt, code = _tdt(dtype)
     thr = length_table(lengths, n)
     lmax = len(thr) - 1
@@ -177,7 +178,7 @@ def csr(m, n, dtype, lengths, kind="uniform", seed=BASE_SEED, row0=0, device="cp
         nnz = int(rowptr[-1].item())
         colidx = torch.empty(nnz, dtype=torch.int32, device=dev)
         val = torch.empty(nnz, dtype=tdt, device=dev)
-        _check(lib.synth_csr_fill_cuda(m, n, nnz0, ctypes.c_void_p(rowptr.data_ptr()), code, KINDS[kind], seed,
+        _check(lib.synth_csr_fill_cuda(m, n, nnz0, ctypes.c_void_p(rowptr.data_ptr()), code, KINDS[kind], col_skew, seed,
                                        ctypes.c_void_p(colidx.data_ptr()), ctypes.c_void_p(val.data_ptr()), s),
                "synth_csr_fill_cuda")
         return rowptr, colidx, val
@@ -190,7 +191,7 @@ def csr(m, n, dtype, lengths, kind="uniform", seed=BASE_SEED, row0=0, device="cp
     nnz = int(rowptr[-1])
     colidx = np.empty(nnz, np.int32)
     val = np.empty(nnz, np.float64 if code == F64 else np.float32)
-    _check(lib.synth_csr_fill(m, n, row0, nnz0, rowptr.ctypes.data_as(vp), code, KINDS[kind], seed,
+    _check(lib.synth_csr_fill(m, n, row0, nnz0, rowptr.ctypes.data_as(vp), code, KINDS[kind], col_skew, seed,
                               colidx.ctypes.data_as(vp), val.ctypes.data_as(vp)), "synth_csr_fill")
     return torch.from_numpy(rowptr), torch.from_numpy(colidx), torch.from_numpy(val)
 
@@ -220,8 +221,8 @@ CONFIGS = {
     # NEXT-2: KDD2010-shaped ultra-wide CSR (15.0M x 29.9M, 424M nnz at P:419-427): power-law rows of
     # mean ~28, w and y (240 MB fp64) beyond L2 -> the flat L2/HBM-red path.
     "K1": dict(fmt="csr", dtype="f64", m=15_009_374, n=29_890_095, lengths=("powerlaw", 2.5, 9.5, 1_000_000),
-               alpha=1.0, beta=1.0, use_v=True, use_z=True, xkind="uniform",
-               desc="CSR fp64 KDD-shaped 15Mx29.9M power-law rows (mean ~28), full with v"),
+               alpha=1.0, beta=1.0, use_v=True, use_z=True, xkind="uniform", col_skew=2,
+               desc="CSR fp64 KDD-shaped 15Mx29.9M power-law rows (mean ~28), Zipf-like columns (u^4), full with v"),
     # NEXT-4: dense rows wider than one CTA's registers (thread-block cluster kernel)
     "W1": dict(fmt="dense", dtype="f32", m=40_000, n=65_536, alpha=1.0, beta=0.0, use_v=False, use_z=False,
                xkind="uniform", desc="dense fp32 40000x65536 wide rows, X^T(Xy)"),

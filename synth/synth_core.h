@@ -104,4 +104,14 @@ SYNTH_HD int32_t syn_column(uint64_t h, int64_t k, int64_t L, int64_t n) {
   return (int32_t)(b0 + (int64_t)(h % (uint64_t)(b1 - b0)));
 }
 
+/* Skewed ("Zipf-like") variant: popularity decreasing with the column index.  The k-th of L
+   columns is k + floor((n - L) * g(u_k)), u_k = (k + frac(h)) / L in 32-bit fixed point and
+   g(u) = u^(2^skew_log2) (repeated squaring) -- strictly increasing in k, so sorted and
+   distinct; density of column c ~ c^(1/2^skew_log2 - 1).  Integer arithmetic only. */
+SYNTH_HD int32_t syn_column_skew(uint64_t h, int64_t k, int64_t L, int64_t n, int skew_log2) {
+  uint64_t u = (((uint64_t)k << 32) + (h >> 32)) / (uint64_t)L;  /* in [0, 2^32) */
+  for (int i = 0; i < skew_log2; ++i) u = (u * u) >> 32;
+  return (int32_t)(k + (int64_t)((((uint64_t)(n - L)) * u) >> 32));
+}
+
 #endif

@@ -43,8 +43,8 @@ __global__ void k_row_lengths(int64_t m, int64_t row0, const uint64_t* thr, int6
 
 /* one warp per row (heavy power-law rows reach 1e5 entries) */
 template <typename T>
-__global__ void k_csr_fill(int64_t m, int64_t n, int64_t nnz0, const int64_t* rowptr, int kind, uint64_t seed,
-                           int32_t* colidx, T* val) {
+__global__ void k_csr_fill(int64_t m, int64_t n, int64_t nnz0, const int64_t* rowptr, int kind, int col_skew,
+                           uint64_t seed, int32_t* colidx, T* val) {
   int lane = threadIdx.x & 31;
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -52,7 +52,8 @@ __global__ void k_csr_fill(int64_t m, int64_t n, int64_t nnz0, const int64_t* ro
     int64_t a = rowptr[r], L = rowptr[r + 1] - a;
     for (int64_t k = lane; k < L; k += 32) {
       uint64_t g = (uint64_t)(nnz0 + a + k);
-      int32_t c = syn_column(syn_hash(seed, SYN_S_COL, g), k, L, n);
+      uint64_t hc = syn_hash(seed, SYN_S_COL, g);
+      int32_t c = col_skew > 0 ? syn_column_skew(hc, k, L, n, col_skew) : syn_column(hc, k, L, n);
       colidx[a + k] = c;
       val[a + k] = syn_value<T>(syn_hash(seed, SYN_S_VAL, g), kind, syn_colscale_exp(seed, (uint64_t)c));
     }
@@ -108,13 +109,13 @@ int synth_rowptr_cuda(int64_t m, const int64_t* len, int64_t* rowptr, void* temp
   return cudaGetLastError() == cudaSuccess ? 0 : 2;
 }
 
-int synth_csr_fill_cuda(int64_t m, int64_t n, int64_t nnz0, const int64_t* rowptr, int dtype, int kind, uint64_t seed,
-                        int32_t* colidx, void* val, cudaStream_t s) {
+int synth_csr_fill_cuda(int64_t m, int64_t n, int64_t nnz0, const int64_t* rowptr, int dtype, int kind, int col_skew,
+                        uint64_t seed, int32_t* colidx, void* val, cudaStream_t s) {
   if (m < 0 || n < 0) return 1;
   if (m == 0) return 0;
   int g = grid_for(m * 32);
-  if (dtype == SYN_F64) k_csr_fill<double><<<g, 256, 0, s>>>(m, n, nnz0, rowptr, kind, seed, colidx, (double*)val);
-  else k_csr_fill<float><<<g, 256, 0, s>>>(m, n, nnz0, rowptr, kind, seed, colidx, (float*)val);
+  if (dtype == SYN_F64) k_csr_fill<double><<<g, 256, 0, s>>>(m, n, nnz0, rowptr, kind, col_skew, seed, colidx, (double*)val);
+  else k_csr_fill<float><<<g, 256, 0, s>>>(m, n, nnz0, rowptr, kind, col_skew, seed, colidx, (float*)val);
   return cudaGetLastError() == cudaSuccess ? 0 : 2;
 }
 

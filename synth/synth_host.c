@@ -70,7 +70,7 @@ int synth_rowptr(int64_t m, const int64_t* len, int64_t* rowptr) {
    of local entry k is nnz0 + k, so a row shard is bit-identical to the slice of the full
    matrix when nnz0 = global rowptr[row0]. */
 int synth_csr_fill(int64_t m, int64_t n, int64_t row0, int64_t nnz0, const int64_t* rowptr,
-                   int dtype, int kind, uint64_t seed, int32_t* colidx, void* val) {
+                   int dtype, int kind, int col_skew, uint64_t seed, int32_t* colidx, void* val) {
   if (m < 0 || n < 0) return 1;
 #pragma omp parallel for schedule(dynamic, 1024)
   for (int64_t r = 0; r < m; ++r) {
@@ -78,7 +78,8 @@ int synth_csr_fill(int64_t m, int64_t n, int64_t row0, int64_t nnz0, const int64
     (void)row0;
     for (int64_t k = 0; k < L; ++k) {
       uint64_t g = (uint64_t)(nnz0 + a + k);
-      int32_t c = syn_column(syn_hash(seed, SYN_S_COL, g), k, L, n);
+      uint64_t hc = syn_hash(seed, SYN_S_COL, g);
+      int32_t c = col_skew > 0 ? syn_column_skew(hc, k, L, n, col_skew) : syn_column(hc, k, L, n);
       colidx[a + k] = c;
       uint64_t h = syn_hash(seed, SYN_S_VAL, g);
       if (dtype == SYN_F64) ((double*)val)[a + k] = syn_value_f64(h, kind, syn_colscale_exp(seed, (uint64_t)c));

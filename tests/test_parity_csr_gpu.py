@@ -186,3 +186,24 @@ def test_csr_flat_bitexact(cuda_dev, dt, variant, nb, lengths):
         ref, _ = oracle.csr(m, n, rp, ci, va, *args)
         w = gpu_csr(cuda_dev, rp, ci, va, n, *args, launch=L)
         assert_bitexact(w, ref, f"flat variant={variant} nb={nb} {lengths}")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+def test_kdd_like_skewed_columns(cuda_dev, dt):
+    """NEXT-2 shape, scaled: power-law rows, Zipf-like column popularity over a wide n (the L2
+    path with hot columns contending on the same w entries); integer twin bit-exact in fp64."""
+    m, n = 60000, 2_000_000
+    rp, ci, va = synth.csr(m, n, dt, ("powerlaw", 2.5, 9.5, 20000), seed=21, col_skew=2)
+    y = synth.vector(n, dt, seed=21, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="pos", seed=21, stream=synth.S_V)
+    z = synth.vector(n, dt, seed=21, stream=synth.S_Z)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = gpu_csr(cuda_dev, rp, ci, va, n, y, v, z, 1.0, 1.0)
+    assert_parity(w, ref, mag, DT[dt], "kdd-like")
+    if dt == "f64":
+        rp, ci, va = synth.csr(m, n, dt, ("powerlaw", 2.5, 9.5, 20000), seed=22, col_skew=2, kind="int_pm12")
+        yi = synth.vector(n, dt, kind="int_small", seed=22, stream=synth.S_Y)
+        vi = synth.vector(m, dt, kind="int_pos", seed=22, stream=synth.S_V)
+        ref, _ = oracle.csr(m, n, rp, ci, va, yi, vi, None, 1.0, 0.0)
+        w = gpu_csr(cuda_dev, rp, ci, va, n, yi, vi, None, 1.0, 0.0)
+        assert_bitexact(w, ref, "kdd-like twin")

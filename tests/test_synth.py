@@ -65,3 +65,14 @@ def test_shard_equals_slice():
 def test_fnv_checksum_stable():
     x = synth.vector(1000, "f64", seed=1)
     assert synth.fnv1a(x) == synth.fnv1a(x.clone())
+
+
+def test_skewed_columns_sorted_distinct_and_skewed():
+    m, n = 5000, 1_000_000
+    rp, ci, _ = synth.csr(m, n, "f32", ("powerlaw", 2.5, 9.5, 100000), seed=3, col_skew=2)
+    rp, ci = rp.numpy(), ci.numpy()
+    for r in range(0, m, 97):
+        row = ci[rp[r]:rp[r + 1]]
+        assert np.all(np.diff(row) > 0) and row.min() >= 0 and row.max() < n
+    # popularity decreases with the column index: the first 1 % of columns take far more than 1 %
+    assert (ci < n // 100).mean() > 0.2
