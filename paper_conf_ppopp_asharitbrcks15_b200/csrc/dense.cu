@@ -86,21 +86,34 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
         L.tl = nch * ce;
         L.bs = kBSCta;
       } else {
-        // a cluster of CS CTAs shares the row (VS = CS x BS), full 256-byte thread load
-        const int64_t per_cta = (int64_t)kBSCta * (256 / s);  // elements of a row per CTA
-        int cs = 2;
-        while (cs < 8 && (int64_t)cs * per_cta < a.n) cs <<= 1;
-        if ((int64_t)cs * per_cta < a.n) {
-          set_error("fp_dense: n=%lld exceeds the cluster-resident row limit (%lld elements = 8 CTAs x %d "
-                    "threads x 256 B); wider dense rows are not implemented (DESIGN.md NEXT-4)",
-                    (long long)a.n, (long long)(8 * per_cta), kBSCta);
-          return FP_ERR_UNSUPPORTED;
+        // a cluster of CS CTAs shares the row (VS = CS x BS); 128-byte thread load when 8 CTAs
+        // cover the row with it (two resident CTAs per SM), else the full 256-byte load
+        const int64_t half_cta = (int64_t)kBSCta * (128 / s);
+        if ((int64_t)8 * half_cta >= a.n) {
+          int cs = 2;
+          while (cs < 8 && (int64_t)cs * half_cta < a.n) cs <<= 1;
+          L.variant = FP_VAR_DENSE_CLUSTER;
+          L.vs = cs * kBSCta;
+          L.tl = 128 / s;
+          L.bs = kBSCta;
+          L.cluster = cs;
         }
-        L.variant = FP_VAR_DENSE_CLUSTER;
-        L.vs = cs * kBSCta;
-        L.tl = 256 / s;
-        L.bs = kBSCta;
-        L.cluster = cs;
+        if (L.variant != FP_VAR_DENSE_CLUSTER) {
+          const int64_t per_cta = (int64_t)kBSCta * (256 / s);  // elements of a row per CTA
+          int cs = 2;
+          while (cs < 8 && (int64_t)cs * per_cta < a.n) cs <<= 1;
+          if ((int64_t)cs * per_cta < a.n) {
+            set_error("fp_dense: n=%lld exceeds the cluster-resident row limit (%lld elements = 8 CTAs x %d "
+                      "threads x 256 B); wider dense rows are not implemented (DESIGN.md NEXT-4)",
+                      (long long)a.n, (long long)(8 * per_cta), kBSCta);
+            return FP_ERR_UNSUPPORTED;
+          }
+          L.variant = FP_VAR_DENSE_CLUSTER;
+          L.vs = cs * kBSCta;
+          L.tl = 256 / s;
+          L.bs = kBSCta;
+          L.cluster = cs;
+        }
       }
     }
   }

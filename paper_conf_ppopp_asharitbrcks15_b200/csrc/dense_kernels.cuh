@@ -294,17 +294,29 @@ DenseKFn pick_cta(int nch) {
 #include "dense_cluster.cuh"
 namespace fp {
 
-// cluster kernel: always the full 256-byte thread load (NCH = 256 / (E * sizeof(T)))
+// cluster kernel: 256-byte thread load (NCH = 256 / (E * sizeof(T))) or 128-byte (NCH / 2,
+// fewer registers -> two clusters' CTAs resident per SM, hiding the per-row cluster barrier)
 template <typename T, int E, int YM>
 DenseKFn pick_cluster(int cs, int nch) {
   constexpr int NCH = 256 / (E * (int)sizeof(T));
-  if (nch != NCH) return nullptr;
-  switch (cs) {
-    case 2: return k_dense_cluster<T, NCH, E, 2, YM, kBSCta>;
-    case 4: return k_dense_cluster<T, NCH, E, 4, YM, kBSCta>;
-    case 8: return k_dense_cluster<T, NCH, E, 8, YM, kBSCta>;
-    default: return nullptr;
+  constexpr int NH = NCH / 2 > 0 ? NCH / 2 : 1;
+  if (nch == NCH) {
+    switch (cs) {
+      case 2: return k_dense_cluster<T, NCH, E, 2, YM, kBSCta>;
+      case 4: return k_dense_cluster<T, NCH, E, 4, YM, kBSCta>;
+      case 8: return k_dense_cluster<T, NCH, E, 8, YM, kBSCta>;
+      default: return nullptr;
+    }
   }
+  if (nch == NH) {
+    switch (cs) {
+      case 2: return k_dense_cluster<T, NH, E, 2, YM, kBSCta>;
+      case 4: return k_dense_cluster<T, NH, E, 4, YM, kBSCta>;
+      case 8: return k_dense_cluster<T, NH, E, 8, YM, kBSCta>;
+      default: return nullptr;
+    }
+  }
+  return nullptr;
 }
 
 template <typename T, int YM>
