@@ -1,0 +1,53 @@
+#!/usr/bin/env python
+"""Small-shape driver for compute-sanitizer (memcheck / racecheck / synccheck): every kernel
+family once -- dense vector / CTA / cluster, CSR vector (3 modes) and flat (3 modes), the row
+epilogues, CG and TRON drivers -- on tiny inputs.
+
+  compute-sanitizer --tool memcheck python tools/sanitize.py
+"""
+import os
+import sys
+
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import paper_conf_ppopp_asharitbrcks15_b200 as fp  # noqa: E402
+import synth  # noqa: E402
+
+
+def main():
+    dev = torch.device("cuda:0")
+    for dt in ("f64", "f32"):
+        for (m, n) in ((300, 33), (257, 128), (70, 3000), (9, 20000)):
+            X = synth.dense(m, n, dt, seed=1, device=dev)
+            y = synth.vector(n, dt, seed=1, device=dev)
+            v = synth.vector(m, dt, kind="pos", seed=1, stream=synth.S_V, device=dev)
+            z = synth.vector(n, dt, seed=1, stream=synth.S_Z, device=dev)
+            fp.dense(X, y, v, z, 0.5, 1.5)
+            fp.dense(X, None, v, None, 1.0, 0.0)
+            p = torch.empty(m, dtype=X.dtype, device=dev)
+            fp.dense_epi(X, y, v, None, 1.0, 0.0, fp.FP_EPI_LINEAR, row_out=p)
+        rp, ci, va = synth.csr(2000, 700, dt, ("powerlaw", 2.0, 3.0), seed=2, device=dev)
+        y = synth.vector(700, dt, seed=2, device=dev)
+        v = synth.vector(2000, dt, kind="pos", seed=2, stream=synth.S_V, device=dev)
+        z = synth.vector(700, dt, seed=2, stream=synth.S_Z, device=dev)
+        for var, vs, tl in ((3, 8, 2), (4, 32, 4), (5, 8, 2), (6, 32, 4), (7, 32, 8), (8, 32, 2)):
+            L = fp.fp_launch()
+            L.variant, L.vs, L.tl, L.bs, L.grid = var, vs, tl, 256, 13
+            fp.csr(rp, ci, va, 700, y, v, z, 1.0, 1.0, launch=L)
+        lab = torch.where(synth.vector(2000, dt, seed=3, device=dev) > 0, 1.0, -1.0).to(va.dtype)
+        D = torch.empty(2000, dtype=va.dtype, device=dev)
+        loss = torch.zeros(1, dtype=torch.float64, device=dev)
+        fp.csr_epi(rp, ci, va, 700, y, lab, y, 1.0, 1.0, fp.FP_EPI_LOGISTIC, c=1.0, row_out=D, scalar_out=loss)
+        Xc = synth.dense(500, 40, dt, seed=4, device=dev)
+        b = synth.vector(500, dt, seed=4, device=dev)
+        fp.cg_linreg_dense(Xc, b, max_iter=3, tol=0.0)
+        fp.logreg_tron_dense(Xc, torch.where(b > 0, 1.0, -1.0).to(b.dtype), max_iter=2)
+    torch.cuda.synchronize()
+    print("sanitize driver ok")
+
+
+if __name__ == "__main__":
+    main()
