@@ -21,10 +21,11 @@ int mode_of(int variant) {
 int default_k(int vs) { return (vs == 8 || vs == 16) ? 2 : (vs == 32 ? 4 : 4); }
 
 CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
-  const int mode = mode_of(L.variant);
+  int mode = mode_of(L.variant);
+  if (L.variant == FP_VAR_CSR_OWNER) mode = a.n <= 4 * kCsrBS ? DMODE_OWNER4 : (a.n <= 8 * kCsrBS ? DMODE_OWNER8 : -1);
   if (mode < 0) return nullptr;
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
-  const bool flat = L.variant >= FP_VAR_CSR_FLAT;
+  const bool flat = L.variant >= FP_VAR_CSR_FLAT && L.variant <= FP_VAR_CSR_FLAT_PRIVATE;
   const int k = L.tl > 0 ? L.tl : (flat ? 4 : default_k(L.vs));
   return a.dtype == FP_F64 ? csr_pick_f64(ym, mode, L.vs, k) : csr_pick_f32(ym, mode, L.vs, k);
 }
@@ -41,12 +42,25 @@ size_t smem_for(const PatternArgs& a, int variant) {
   switch (variant) {
     case FP_VAR_CSR_VECTOR_PRIVATE:
     case FP_VAR_CSR_FLAT_PRIVATE: return yb + (size_t)(kCsrBS / 32) * vb;
+    case FP_VAR_CSR_OWNER:  // y + spill partial + queues (values, 1-byte hi, counters)
+      return yb + vb + (size_t)kOwnerQ * kCsrBS * (dtype_size(a.dtype) + 1) + (size_t)kCsrBS * 4;
     case FP_VAR_CSR_VECTOR:
     case FP_VAR_CSR_FLAT: return yb + vb;
     case FP_VAR_CSR_VECTOR_L2:
     case FP_VAR_CSR_FLAT_L2: return y_in_smem_l2(a) ? vb : 0;
     default: return 0;
   }
+}
+
+// owner-computes: row-group iterations per phase so that one phase fills the queues to about
+// half (BS * kOwnerQ / 2 entries per CTA) at the mean row length
+int phase_iters_for(const PatternArgs& a, const fp_launch& L) {
+  if (L.variant != FP_VAR_CSR_OWNER) return 0;
+  const double mu = a.m > 0 ? (double)a.nnz / (double)a.m : 1.0;
+  const int rpv = 2;
+  const double per_iter = (double)(kCsrBS / 32) * (32 / (L.vs > 0 ? L.vs : 32)) * rpv * (mu > 1.0 ? mu : 1.0);
+  int pi = (int)((kCsrBS * kOwnerQ / 2) / per_iter);
+  return pi < 1 ? 1 : pi;
 }
 
 }  // namespace
@@ -119,7 +133,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   }
   CsrKArgs k{a.m, a.n, a.nnz, a.rowptr, a.colidx, a.val, a.y, a.v, a.z, a.alpha, a.beta, a.w,
              ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (l2 && y_in_smem_l2(a)) ? 1 : 0,
-             {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}};
+             {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}, phase_iters_for(a, L)};
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // L2 path without y in shared memory: prefer the largest L1 so the random y gathers hit it
   // (X itself streams with L1::no_allocate and never displaces y)

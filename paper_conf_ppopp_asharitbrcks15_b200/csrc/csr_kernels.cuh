@@ -45,6 +45,7 @@ struct CsrKArgs {
   int accumulate;
   int y_in_smem;  // MODE_L2 only: stage y in shared memory (n*s bytes) for the gathers
   fpd::RowEpi epi;
+  int phase_iters;  // owner-computes kernel: row-group iterations between queue drains
 };
 
 enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2 };
@@ -298,10 +299,20 @@ using CsrKFn = void (*)(const CsrKArgs);
 
 }  // namespace fp
 #include "csr_flat.cuh"
+#include "csr_owner.cuh"
 namespace fp {
 
+template <typename T, int YM, int NPT>
+CsrKFn csr_pick_owner_n(int vs, int k) {
+#define FP_CSR_OW(VS_, K_, RPV_) \
+  if (vs == VS_ && k == K_) return k_csr_owner<T, VS_, K_, RPV_, YM, NPT, kCsrBS>;
+  FP_CSR_OW(4, 4, 2) FP_CSR_OW(8, 2, 2) FP_CSR_OW(16, 2, 2) FP_CSR_OW(32, 4, 2)
+#undef FP_CSR_OW
+  return nullptr;
+}
+
 // dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
-enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5 };
+enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5, DMODE_OWNER4 = 6, DMODE_OWNER8 = 7 };
 
 template <typename T, int YM, int MODE>
 CsrKFn csr_pick_flat(int nb) {
@@ -335,6 +346,8 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case DMODE_FLAT_SHARED: return csr_pick_flat<T, YM, MODE_SHARED>(k);
     case DMODE_FLAT_L2: return csr_pick_flat<T, YM, MODE_L2>(k);
     case DMODE_FLAT_PRIVATE: return csr_pick_flat<T, YM, MODE_PRIVATE>(k);
+    case DMODE_OWNER4: return csr_pick_owner_n<T, YM, 4>(vs, k);
+    case DMODE_OWNER8: return csr_pick_owner_n<T, YM, 8>(vs, k);
     default: return nullptr;
   }
 }

@@ -207,3 +207,20 @@ def test_kdd_like_skewed_columns(cuda_dev, dt):
         ref, _ = oracle.csr(m, n, rp, ci, va, yi, vi, None, 1.0, 0.0)
         w = gpu_csr(cuda_dev, rp, ci, va, n, yi, vi, None, 1.0, 0.0)
         assert_bitexact(w, ref, "kdd-like twin")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("vs,k", [(4, 4), (8, 2), (16, 2), (32, 4)])
+@pytest.mark.parametrize("n", [700, 2000])
+def test_csr_owner_bitexact(cuda_dev, dt, vs, k, n):
+    """Owner-computes aggregation (variant 10): queues, drains, spills -- integer twins exact,
+    including heavy rows (power-law) that overflow the queues into the CAS spill partial."""
+    m = 6000
+    for lengths in (("binomial", 0.01), ("powerlaw", 2.0, 4.0)):
+        rp, ci, va, y, v, z = make_csr(m, n, dt, lengths, seed=vs + n, kind="int_pm12")
+        L = fp.fp_launch()
+        L.variant, L.vs, L.tl, L.bs, L.grid = 10, vs, k, 256, 23
+        for args in ((y, v, z, 1.0, 1.0), (None, v, None, -1.0, 0.0)):
+            ref, _ = oracle.csr(m, n, rp, ci, va, *args)
+            w = gpu_csr(cuda_dev, rp, ci, va, n, *args, launch=L)
+            assert_bitexact(w, ref, f"owner vs={vs} k={k} n={n} {lengths}")

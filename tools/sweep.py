@@ -72,6 +72,8 @@ def main():
         space = [(var, vs, k) for var in (3, 4, 5) for vs, k in
                  [(1, 2), (1, 4), (2, 2), (2, 4), (4, 2), (4, 4), (8, 1), (8, 2), (16, 1), (16, 2), (32, 2), (32, 4)]]
         space += [(var, 32, nb) for var in (6, 7, 8) for nb in (2, 4, 8)]   # flat kernels: k = NB tiles
+        if cfg["n"] <= 2048:
+            space += [(10, vs, k) for vs, k in ((4, 4), (8, 2), (16, 2), (32, 4))]   # owner-computes
     else:
         space = [(base.variant, base.vs, base.tl)]
     rows = []
