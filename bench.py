@@ -492,13 +492,65 @@ def run_reference(args):
     print(json.dumps(out), flush=True)
 
 
+def run_unfused(args):
+    """--impl unfused: the multi-kernel library chain the paper compares against (P:81-109,
+    P:417): cuBLAS gemv X y, elementwise v, cuBLAS gemv X^T q (+ beta z) for dense; cuSPARSE SpMV
+    X y and X^T q (torch sparse CSR, transpose via a CSC view) for CSR -- two passes over X.
+    A second GPU reference (north_star), NOT the product path."""
+    world, rank, local = dist_info()
+    if world > 1 and rank != 0:
+        return
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    name = args.config
+    cfg, inp = build_inputs(name, 0, 1, dev)
+    alpha, beta, n = cfg["alpha"], cfg["beta"], cfg["n"]
+    if cfg["fmt"] == "dense":
+        X = inp["X"]
+
+        def step():
+            p = torch.mv(X, inp["y"])
+            if inp["v"] is not None:
+                p = p * inp["v"]
+            w = torch.mv(X.t(), p)
+            w = alpha * w + (beta * inp["z"] if beta != 0.0 else 0.0)
+            return w
+    else:
+        A = torch.sparse_csr_tensor(inp["rowptr"], inp["colidx"], inp["val"], size=(cfg["m"], n))
+        At = A.t()  # CSC view of X: X^T q is a transposed SpMV
+
+        def step():
+            p = torch.mv(A, inp["y"])
+            if inp["v"] is not None:
+                p = p * inp["v"]
+            w = torch.mv(At, p)
+            return alpha * w + (beta * inp["z"] if beta != 0.0 else 0.0)
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record()
+    for _ in range(args.steps):
+        step()
+    e.record()
+    torch.cuda.synchronize()
+    ms = s.elapsed_time(e) / args.steps
+    x_bytes, _ = algorithmic_bytes(cfg, cfg["m"], inp["nnz_local"])
+    out = {"impl": "unfused", "metric": METRIC, "value": round(x_bytes / ms / 1e6, 2), "unit": "GB/s", "n_gpus": 1,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
+           "config": {"workload": f"{name}: {cfg['desc']}", "m": cfg["m"], "n": n,
+                      "chain": "torch.mv (cuBLAS gemv / cuSPARSE SpMV) x2 + elementwise"}}
+    print(json.dumps(out), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="C2", choices=sorted(synth.CONFIGS))
-    ap.add_argument("--impl", default="fusedpat", choices=["fusedpat", "reference"])
+    ap.add_argument("--impl", default="fusedpat", choices=["fusedpat", "reference", "unfused"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -514,6 +566,8 @@ def main():
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
         run_reference(args)
+    elif args.impl == "unfused":
+        run_unfused(args)
     else:
         run_gpu(args)
 
