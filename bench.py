@@ -516,7 +516,14 @@ def run_unfused(args):
             w = alpha * w + (beta * inp["z"] if beta != 0.0 else 0.0)
             return w
     else:
-        A = torch.sparse_csr_tensor(inp["rowptr"], inp["colidx"], inp["val"], size=(cfg["m"], n))
+        # torch/cuSPARSE need one index dtype: int32 when nnz fits (C3, C4), else int64 columns
+        if inp["nnz_local"] < 2**31 - 1:
+            crow, col = inp["rowptr"].to(torch.int32), inp["colidx"]
+        else:
+            crow, col = inp["rowptr"], inp["colidx"].to(torch.int64)
+        del inp["rowptr"]
+        torch.cuda.empty_cache()
+        A = torch.sparse_csr_tensor(crow, col, inp["val"], size=(cfg["m"], n))
         At = A.t()  # CSC view of X: X^T q is a transposed SpMV
 
         def step():
