@@ -206,6 +206,7 @@ def run_gpu(args):
     stream = torch.cuda.current_stream(dev)
     n = cfg["n"]
 
+    plan = None
     if name == "C5":
         iters = args.cg_iters
 
@@ -221,6 +222,8 @@ def run_gpu(args):
                 fp.dense(inp["X"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
             else:
                 fp.dense_dist(comm, inp["X"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
+        plan = fp.choose(False, fp.row_stats_dense(inp["m_local"], n),
+                         fp.FP_F64 if cfg["dtype"] == "f64" else fp.FP_F32, local)
         launches_per_step = 1
         passes_per_step = 1
     else:
@@ -342,7 +345,10 @@ def run_gpu(args):
                        "z": cfg["use_z"], "parallelism": f"row-sharded x{world}, one NCCL allreduce of w",
                        "l2": ("flushed (256 MiB memset) between timed steps" if flush is not None else
                               f"inputs larger than L2 (X = {x_bytes / 1e9:.2f} GB >> 126 MB)"),
-                       "passes_per_step": passes_per_step, "cuda_graph": graphed},
+                       "passes_per_step": passes_per_step, "cuda_graph": graphed,
+                       "plan": None if plan is None else {
+                           k: int(getattr(plan, k)) for k in ("variant", "vs", "tl", "bs", "grid", "cluster",
+                                                              "blocks_per_sm", "smem_bytes", "regs_per_thread")}},
             "evals_per_s": round(evals_per_s * (1 if name != "C5" else 1), 3),
             "pct_hbm_peak": round(100 * value / world / peak, 2),
             "x_bytes_per_eval": x_bytes, "algorithmic_bytes_per_eval": alg_bytes,

@@ -1,5 +1,9 @@
 // dense.cu -- B200 plan and launch of the fused dense kernels (dense_kernels.cuh), and the
 // beta*z / zero-fill kernel shared by the alpha == 0 path and the CSR L2 path.
+#include <stdlib.h>
+
+#include <algorithm>
+
 #include "dense_kernels.cuh"
 
 namespace fp {
@@ -31,6 +35,47 @@ int chunk_bytes_for(const PatternArgs& a) {
   return (int)s;
 }
 
+// Bulk-copy (TMA) ring for the cluster kernel: on unless FP_CLUSTER_TMA=0 (A/B measurement).
+bool cluster_tma_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("FP_CLUSTER_TMA");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
+// The cluster plan runs the bulk-copy ring kernel for 16/32-byte-aligned rows and thread slices
+// of at most 128 bytes; 256-byte slices (rows up to 2x wider) and unaligned rows run the
+// register kernel.
+bool uses_tma(const PatternArgs& a, const fp_launch& L, int cb) {
+  return L.variant == FP_VAR_DENSE_CLUSTER && cb >= 16 && cluster_tma_enabled() &&
+         L.tl * (int)dtype_size(a.dtype) <= 128;
+}
+
+// Ring depth of the TMA cluster kernel: 3 slices (two rows in flight beyond the one being
+// consumed; 3 x 32 KB -> two CTAs per SM).  FP_CLUSTER_RING=2..8 overrides (measurement),
+// clamped to the 227 KB opt-in limit.
+int cluster_ring_depth(const PatternArgs& a, const fp_launch& L) {
+  const int slice = L.tl * (int)dtype_size(a.dtype) * L.bs;
+  int d = 3;
+  static const int env = [] {
+    const char* e = getenv("FP_CLUSTER_RING");
+    return e ? atoi(e) : 0;
+  }();
+  if (env >= 2 && env <= 8) d = env;
+  while (d > 2 && d * slice > 220 * 1024) --d;
+  return d;
+}
+
+// dynamic shared memory of a plan: the fp64 w row (vector/CTA kernels), the D-row ring of the
+// TMA cluster kernel (D x TL elements x BS threads), 0 for the register-only cluster kernel
+int dense_smem_bytes(const PatternArgs& a, const fp_launch& L) {
+  const int cb = chunk_bytes_for(a);
+  if (L.variant != FP_VAR_DENSE_CLUSTER) return (int)(a.n * sizeof(double));
+  if (!uses_tma(a, L, cb)) return 0;
+  return cluster_ring_depth(a, L) * L.tl * (int)dtype_size(a.dtype) * L.bs;
+}
+
 DenseKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int cb = chunk_bytes_for(a);
   const int ce = cb / (int)dtype_size(a.dtype);
@@ -38,7 +83,39 @@ DenseKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   const int nch = L.tl / ce;
   // 0: no y (Table 1 row 1); 1: Eq. (1) fast path; 2: Eq. (1) + row epilogue (outputs / logistic)
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
-  return a.dtype == FP_F64 ? dense_pick_f64(ym, L.variant, cb, L.vs, nch) : dense_pick_f32(ym, L.variant, cb, L.vs, nch);
+  const int tma = uses_tma(a, L, cb) ? 1 : 0;
+  return a.dtype == FP_F64 ? dense_pick_f64(ym, L.variant, cb, L.vs, nch, tma)
+                           : dense_pick_f32(ym, L.variant, cb, L.vs, nch, tma);
+}
+
+
+// Clusters of plan C that can be co-resident on the device (0 if the kernel is missing or the
+// query fails).
+int cluster_capacity(const PatternArgs& a, const fp_launch& C) {
+  DenseKFn f = pick_any(a, C);
+  if (!f) return 0;
+  const int dsm = dense_smem_bytes(a, C);
+  if (dsm > 48 * 1024 && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)(C.cluster * 64));
+  cfg.blockDim = dim3((unsigned)C.bs);
+  cfg.dynamicSmemBytes = (size_t)dsm;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)C.cluster;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, (const void*)f, &cfg) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
 }
 
 int round_up_in(int need, const int* set, int cnt) {
@@ -86,33 +163,60 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
         L.tl = nch * ce;
         L.bs = kBSCta;
       } else {
-        // a cluster of CS CTAs shares the row (VS = CS x BS); 128-byte thread load when 8 CTAs
-        // cover the row with it (two resident CTAs per SM), else the full 256-byte load
-        const int64_t half_cta = (int64_t)kBSCta * (128 / s);
-        if ((int64_t)8 * half_cta >= a.n) {
-          int cs = 2;
-          while (cs < 8 && (int64_t)cs * half_cta < a.n) cs <<= 1;
-          L.variant = FP_VAR_DENSE_CLUSTER;
-          L.vs = cs * kBSCta;
-          L.tl = 128 / s;
-          L.bs = kBSCta;
-          L.cluster = cs;
+        // a cluster of CS CTAs (BS = 256 each) shares the row (VS = CS x BS).  Candidates in
+        // preference order, each with the smallest CS in {2,4,8} covering n: bulk-copy ring
+        // kernel with 128- / 64-byte thread slices (16-byte-aligned rows), register kernel with
+        // 256-byte, then (rows not aligned, or ring disabled) 128-byte slices.  The one keeping
+        // the most SMs streaming wins (co-resident clusters x CS / CTAs per SM, occupancy API:
+        // an 8-CTA cluster must fit one GPC, so only 15 fit 148 SMs at one CTA per SM); ties
+        // keep the earlier.
+        const bool ring = cb >= 16 && cluster_tma_enabled();
+        struct Cand { int tb; };
+        Cand cands[4];
+        int nc = 0;
+        if (ring) {
+          cands[nc++] = {128};
+          cands[nc++] = {64};
+          cands[nc++] = {256};
+        } else {
+          cands[nc++] = {256};
+          cands[nc++] = {128};
         }
-        if (L.variant != FP_VAR_DENSE_CLUSTER) {
-          const int64_t per_cta = (int64_t)kBSCta * (256 / s);  // elements of a row per CTA
+        int best_sms = -1;
+        static const int force_tb = [] {  // FP_CLUSTER_TB=<bytes per thread>: pin (measurement)
+          const char* e = getenv("FP_CLUSTER_TB");
+          return e ? atoi(e) : 0;
+        }();
+        for (int ci = 0; ci < nc; ++ci) {
+          const int tb = cands[ci].tb;
+          if (force_tb && tb != force_tb) continue;
+          const int64_t per_cta = (int64_t)kBSCta * (tb / s);
           int cs = 2;
           while (cs < 8 && (int64_t)cs * per_cta < a.n) cs <<= 1;
-          if ((int64_t)cs * per_cta < a.n) {
-            set_error("fp_dense: n=%lld exceeds the cluster-resident row limit (%lld elements = 8 CTAs x %d "
-                      "threads x 256 B); wider dense rows are not implemented (DESIGN.md NEXT-4)",
-                      (long long)a.n, (long long)(8 * per_cta), kBSCta);
-            return FP_ERR_UNSUPPORTED;
+          if ((int64_t)cs * per_cta < a.n) continue;
+          fp_launch C{};
+          C.variant = FP_VAR_DENSE_CLUSTER;
+          C.vs = cs * kBSCta;
+          C.tl = tb / s;
+          C.bs = kBSCta;
+          C.cluster = cs;
+          const int clusters = cluster_capacity(a, C);
+          DenseKFn fc = pick_any(a, C);
+          int bps = 1;
+          if (fc) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fc, C.bs, dense_smem_bytes(a, C));
+          if (bps < 1) bps = 1;
+          const int sms = std::min((clusters * cs + bps - 1) / bps, di.sm_count);  // SMs streaming
+          if (clusters > 0 && sms > best_sms) {
+            best_sms = sms;
+            L = C;
           }
-          L.variant = FP_VAR_DENSE_CLUSTER;
-          L.vs = cs * kBSCta;
-          L.tl = 256 / s;
-          L.bs = kBSCta;
-          L.cluster = cs;
+        }
+        if (L.variant != FP_VAR_DENSE_CLUSTER) {
+          const int64_t per_cta = (int64_t)kBSCta * (256 / s);
+          set_error("fp_dense: n=%lld exceeds the cluster-resident row limit (%lld elements = 8 CTAs x %d "
+                    "threads x 256 B); wider dense rows are not implemented (DESIGN.md NEXT-4)",
+                    (long long)a.n, (long long)(8 * per_cta), kBSCta);
+          return FP_ERR_UNSUPPORTED;
         }
       }
     }
@@ -123,7 +227,7 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
     return FP_ERR_UNSUPPORTED;
   }
   const bool clu = L.variant == FP_VAR_DENSE_CLUSTER;
-  L.smem_bytes = clu ? 0 : (int)(a.n * sizeof(double));
+  L.smem_bytes = dense_smem_bytes(a, L);
   if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, L.bs, L.smem_bytes);
@@ -140,7 +244,12 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
   if (clu) need_ctas = a.m * L.cluster;  // a cluster of CS CTAs per row
   int64_t grid = (int64_t)di.sm_count * per_sm;
   if (need_ctas < grid) grid = need_ctas > 0 ? need_ctas : 1;
-  if (clu) grid = (grid / L.cluster > 0 ? grid / L.cluster : 1) * L.cluster;
+  if (clu) {  // co-resident clusters only: a second wave would double the time of the first
+    int64_t nc = cluster_capacity(a, L);
+    if (nc < 1) nc = 1;
+    if (nc > a.m) nc = a.m > 0 ? a.m : 1;
+    grid = nc * L.cluster;
+  }
   L.grid = (int)grid;
   L.rows_per_vector = (a.m + grid * vectors_per_cta - 1) / (grid * vectors_per_cta);
   *out = L;
@@ -160,10 +269,13 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_dense: launch plan (variant=%d vs=%d tl=%d) has no kernel", L.variant, L.vs,
              L.tl);
   const bool clu = L.variant == FP_VAR_DENSE_CLUSTER;
-  FP_REQUIRE(L.bs == ((L.variant == FP_VAR_DENSE_CTA || clu) ? kBSCta : kBS), FP_ERR_UNSUPPORTED,
+  const int want_bs = (clu || L.variant == FP_VAR_DENSE_CTA) ? kBSCta : kBS;
+  FP_REQUIRE(L.bs == want_bs, FP_ERR_UNSUPPORTED,
              "fp_dense: block size %d not supported by the selected kernel", L.bs);
   FP_REQUIRE(L.grid >= 1, FP_ERR_INVALID_ARG, "fp_dense: grid must be >= 1");
-  const int cs = clu ? L.vs / kBSCta : 1;
+  const int cs = clu ? L.vs / L.bs : 1;
+  FP_REQUIRE(!clu || ((cs == 2 || cs == 4 || cs == 8) && L.vs == cs * L.bs), FP_ERR_INVALID_ARG,
+             "fp_dense: cluster plan needs vs = CS x bs with CS in {2,4,8}");
   FP_REQUIRE(!clu || (L.grid % cs == 0), FP_ERR_INVALID_ARG, "fp_dense: grid must be a multiple of the cluster size");
   Workspace* ws = workspace(s, (size_t)a.n, 0);
   if (!ws) return FP_ERR_NOMEM;
@@ -173,7 +285,9 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)L.grid);
     cfg.blockDim = dim3((unsigned)L.bs);
-    cfg.dynamicSmemBytes = 0;
+    const int dsm = dense_smem_bytes(a, L);
+    if (dsm > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm));
+    cfg.dynamicSmemBytes = (size_t)dsm;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;

@@ -3,11 +3,11 @@
 
 namespace fp {
 // ym: 0 = no y (Table 1 row 1), 1 = Eq. (1), 2 = Eq. (1) with a row epilogue
-DenseKFn dense_pick_f64(int ym, int variant, int chunk_bytes, int vs, int nch) {
+DenseKFn dense_pick_f64(int ym, int variant, int chunk_bytes, int vs, int nch, int tma) {
   switch (ym) {
-    case 0: return pick_t<double, 0>(variant, chunk_bytes, vs, nch);
-    case 1: return pick_t<double, 1>(variant, chunk_bytes, vs, nch);
-    case 2: return pick_t<double, 2>(variant, chunk_bytes, vs, nch);
+    case 0: return pick_t<double, 0>(variant, chunk_bytes, vs, nch, tma);
+    case 1: return pick_t<double, 1>(variant, chunk_bytes, vs, nch, tma);
+    case 2: return pick_t<double, 2>(variant, chunk_bytes, vs, nch, tma);
     default: return nullptr;
   }
 }

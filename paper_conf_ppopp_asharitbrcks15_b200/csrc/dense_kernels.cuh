@@ -296,37 +296,57 @@ namespace fp {
 
 // cluster kernel: 256-byte thread load (NCH = 256 / (E * sizeof(T))) or 128-byte (NCH / 2,
 // fewer registers -> two clusters' CTAs resident per SM, hiding the per-row cluster barrier)
-template <typename T, int E, int YM>
-DenseKFn pick_cluster(int cs, int nch) {
-  constexpr int NCH = 256 / (E * (int)sizeof(T));
-  constexpr int NH = NCH / 2 > 0 ? NCH / 2 : 1;
-  if (nch == NCH) {
-    switch (cs) {
-      case 2: return k_dense_cluster<T, NCH, E, 2, YM, kBSCta>;
-      case 4: return k_dense_cluster<T, NCH, E, 4, YM, kBSCta>;
-      case 8: return k_dense_cluster<T, NCH, E, 8, YM, kBSCta>;
-      default: return nullptr;
-    }
+
+template <typename T, int NCH, int E, int YM>
+DenseKFn cluster_reg_k(int cs) {
+  switch (cs) {
+    case 2: return k_dense_cluster<T, NCH, E, 2, YM, kBSCta>;
+    case 4: return k_dense_cluster<T, NCH, E, 4, YM, kBSCta>;
+    case 8: return k_dense_cluster<T, NCH, E, 8, YM, kBSCta>;
+    default: return nullptr;
   }
-  if (nch == NH) {
+}
+
+template <typename T, int NCH, int E, int YM>
+DenseKFn cluster_tma_k(int cs) {
+  if constexpr (E * sizeof(T) >= 16) {
     switch (cs) {
-      case 2: return k_dense_cluster<T, NH, E, 2, YM, kBSCta>;
-      case 4: return k_dense_cluster<T, NH, E, 4, YM, kBSCta>;
-      case 8: return k_dense_cluster<T, NH, E, 8, YM, kBSCta>;
+      case 2: return k_dense_cluster_tma<T, NCH, E, 2, YM, kBSCta>;
+      case 4: return k_dense_cluster_tma<T, NCH, E, 4, YM, kBSCta>;
+      case 8: return k_dense_cluster_tma<T, NCH, E, 8, YM, kBSCta>;
       default: return nullptr;
     }
   }
   return nullptr;
 }
 
+// cluster kernels.  Register kernel (BS = 256): 256- or 128-byte thread slices.  Bulk-copy
+// ring kernel (BS = 256, 16/32-byte chunks only): 128- or 64-byte thread slices.
+template <typename T, int E, int YM>
+DenseKFn pick_cluster(int cs, int nch, int tma) {
+  if (tma) {
+    constexpr int NF = 128 / (E * (int)sizeof(T)), NHf = 64 / (E * (int)sizeof(T));
+    if constexpr (NHf >= 1) {
+      if (nch == NF) return cluster_tma_k<T, NF, E, YM>(cs);
+      if (nch == NHf) return cluster_tma_k<T, NHf, E, YM>(cs);
+    }
+    return nullptr;
+  }
+  constexpr int NCH = 256 / (E * (int)sizeof(T));
+  constexpr int NH = NCH / 2 > 0 ? NCH / 2 : 1;
+  if (nch == NCH) return cluster_reg_k<T, NCH, E, YM>(cs);
+  if (nch == NH) return cluster_reg_k<T, NH, E, YM>(cs);
+  return nullptr;
+}
+
 template <typename T, int YM>
-DenseKFn pick_t(int variant, int chunk_bytes, int vs, int nch) {
+DenseKFn pick_t(int variant, int chunk_bytes, int vs, int nch, int tma) {
   constexpr int E32 = 32 / (int)sizeof(T), E16 = 16 / (int)sizeof(T);
   if (variant == FP_VAR_DENSE_CLUSTER) {
     const int cs = vs / kBSCta;
-    if (chunk_bytes == 32) return pick_cluster<T, E32, YM>(cs, nch);
-    if (chunk_bytes == 16) return pick_cluster<T, E16, YM>(cs, nch);
-    if (chunk_bytes == (int)sizeof(T)) return pick_cluster<T, 1, YM>(cs, nch);
+    if (chunk_bytes == 32) return pick_cluster<T, E32, YM>(cs, nch, tma);
+    if (chunk_bytes == 16) return pick_cluster<T, E16, YM>(cs, nch, tma);
+    if (chunk_bytes == (int)sizeof(T)) return pick_cluster<T, 1, YM>(cs, nch, 0);
     return nullptr;
   }
   const bool cta = variant == FP_VAR_DENSE_CTA;
@@ -338,7 +358,7 @@ DenseKFn pick_t(int variant, int chunk_bytes, int vs, int nch) {
 }
 
 // defined in dense_f32.cu / dense_f64.cu (separate translation units: parallel build)
-DenseKFn dense_pick_f32(int ym, int variant, int chunk_bytes, int vs, int nch);
-DenseKFn dense_pick_f64(int ym, int variant, int chunk_bytes, int vs, int nch);
+DenseKFn dense_pick_f32(int ym, int variant, int chunk_bytes, int vs, int nch, int tma);
+DenseKFn dense_pick_f64(int ym, int variant, int chunk_bytes, int vs, int nch, int tma);
 
 }  // namespace fp

@@ -21,7 +21,7 @@ def labels_for(Xd, seed):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f32"])
-@pytest.mark.parametrize("m,n", [(5000, 64), (3001, 128), (2000, 1000)])
+@pytest.mark.parametrize("m,n", [(5000, 64), (3001, 128), (2000, 1000), (300, 20000)])
 def test_logistic_epilogue_dense(cuda_dev, dt, m, n):
     X = synth.dense(m, n, dt, seed=m)
     y = torch.from_numpy(labels_for(X.double().numpy(), m)).to(DT[dt])

@@ -194,3 +194,52 @@ def test_dense_cluster_variant(cuda_dev, dt, m, n):
     w, ref, _ = run_both(Xi, yi, vi, zi, "full", cuda_dev)
     if dt == "f64":
         assert_bitexact(w, ref, f"cluster twin {m}x{n}")
+
+
+@pytest.mark.parametrize("dt,ldpad", [("f32", 0), ("f32", 4), ("f32", 1), ("f64", 2), ("f64", 0)])
+@pytest.mark.parametrize("inst", ["xty", "xtvxy", "full"])
+def test_dense_cluster_instances_ld(cuda_dev, dt, ldpad, inst):
+    """Cluster variant over Table-1 instances (incl. row 1, no y: YM=0) and padded row strides:
+    ld = n+4 fp32 / n+2 fp64 keeps 16-byte rows (bulk-copy ring), ld = n+1 fp32 falls back to
+    scalar loads (register-only cluster kernel)."""
+    m, n = 203, 30001 if dt == "f32" else 17003
+    X, y, v, z = make(m, n, dt, seed=ldpad + 11, ld=n + ldpad if ldpad else None)
+    st = fp.row_stats_dense(m, n)
+    L = fp.choose(False, st, fp.FP_F32 if dt == "f32" else fp.FP_F64, 0)
+    assert L.variant == 9
+    w, ref, mag = run_both(X, y, v, z, inst, cuda_dev, n=n)
+    assert_parity(w, ref, mag, DT[dt], f"cluster {dt} ld+{ldpad} {inst}")
+
+
+def test_dense_cluster_register_kernel(cuda_dev, tmp_path):
+    """The register-only cluster kernel (FP_CLUSTER_TMA=0: per-row cluster barrier, x held in
+    registers; the path taken for rows that are not 16-byte aligned) on 16-byte-aligned rows,
+    in a subprocess because the switch is read once per process; parity against the oracle
+    like the default bulk-copy ring kernel."""
+    import os
+    import subprocess
+    import sys
+    m, n = 150, 40000
+    script = tmp_path / "regk.py"
+    script.write_text(
+        "import sys, torch, synth, paper_conf_ppopp_asharitbrcks15_b200 as fp\n"
+        f"m, n = {m}, {n}\n"
+        "X = synth.dense(m, n, 'f32', seed=5).cuda()\n"
+        "y = synth.vector(n, 'f32', seed=5, stream=synth.S_Y).cuda()\n"
+        "v = synth.vector(m, 'f32', kind='pos', seed=5, stream=synth.S_V).cuda()\n"
+        "L = fp.choose(False, fp.row_stats_dense(m, n), fp.FP_F32, 0)\n"
+        "assert L.variant == 9 and L.tl * 4 == 256, L.as_dict()\n"
+        "w = fp.dense(X, y, v, None, 1.0, 0.0)\n"
+        "torch.save(w.cpu(), sys.argv[1])\n")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, FP_CLUSTER_TMA="0", PYTHONPATH=root)
+    out = tmp_path / "w.pt"
+    subprocess.run([sys.executable, str(script), str(out)], check=True, env=env, cwd=root, timeout=300)
+    w = torch.load(out)
+    X = synth.dense(m, n, "f32", seed=5)
+    y = synth.vector(n, "f32", seed=5, stream=synth.S_Y)
+    v = synth.vector(m, "f32", kind="pos", seed=5, stream=synth.S_V)
+    ref, mag = oracle.dense(X, y, v, None, 1.0, 0.0)
+    assert_parity(w, ref, mag, torch.float32, "cluster register kernel")
+    L = fp.choose(False, fp.row_stats_dense(m, n), fp.FP_F32, 0)
+    assert L.tl * 4 <= 128  # default process: the bulk-copy ring kernel
