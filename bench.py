@@ -238,7 +238,17 @@ def run_gpu(args):
         st.m, st.n, st.nnz = inp["m_local"], n, inp["nnz_local"]
         st.mean = st.nnz / max(1, st.m)
         plan = fp.choose(True, st, fp.FP_F64 if cfg["dtype"] == "f64" else fp.FP_F32, local)
-        launches_per_step = 1 if plan.variant == 3 else 2
+        if args.launch:  # explicit plan (profiling / sweeps): variant,vs,k,grid
+            var, vs, k, g = (int(t) for t in args.launch.split(","))
+            plan = fp.fp_launch()
+            plan.variant, plan.vs, plan.tl, plan.bs, plan.grid = var, vs, k, 256, g
+            forced = plan
+
+            def step():
+                fp.csr(inp["rowptr"], inp["colidx"], inp["val"], n, inp["y"], inp["v"], inp["z"], alpha, beta,
+                       w=inp["w"], launch=forced)
+        # the L2 variants write beta*z (k_scale_z) before the main kernel
+        launches_per_step = 2 if plan.variant in (4, 7) else 1
         passes_per_step = 1
 
     flush = None
@@ -573,6 +583,7 @@ def main():
     ap.add_argument("--graph", dest="graph", action="store_true", default=True,
                     help="replay each step from a captured CUDA graph (default)")
     ap.add_argument("--no-graph", dest="graph", action="store_false")
+    ap.add_argument("--launch", default=None, help="CSR only: force the plan 'variant,vs,k,grid' (profiling)")
     ap.add_argument("--force-dist", action="store_true",
                     help="use the NCCL row-sharded path (fp_*_dist + allreduce) even with one rank")
     args = ap.parse_args()

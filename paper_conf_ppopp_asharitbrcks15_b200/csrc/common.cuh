@@ -208,6 +208,15 @@ struct Vec16<double> {
 };
 
 // Gathers of y that should stay in L1 (y is re-read randomly; X streams past it).
+// cp.async.bulk.prefetch.L2: one instruction pulls a contiguous byte range into L2 (TMA unit;
+// no registers, no completion to wait for).  The range is widened to 16-byte alignment.
+__device__ __forceinline__ void prefetch_l2(const void* p, size_t bytes) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~(uintptr_t)15;
+  const uintptr_t e = (reinterpret_cast<uintptr_t>(p) + bytes + 15) & ~(uintptr_t)15;
+  if (e > a)
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((unsigned)(e - a)) : "memory");
+}
+
 __device__ __forceinline__ float ld_keep(const float* p) {
   float r;
   asm("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(r) : "l"(p));

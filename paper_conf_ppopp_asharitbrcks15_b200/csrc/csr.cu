@@ -1,9 +1,15 @@
 // csr.cu -- B200 plan and launch of the fused CSR kernels (csr_kernels.cuh).
+#include <cstdlib>
+
 #include "csr_kernels.cuh"
 
 namespace fp {
 
 namespace {
+
+bool is_flat(int variant) {
+  return (variant >= FP_VAR_CSR_FLAT && variant <= FP_VAR_CSR_FLAT_PRIVATE) || variant == FP_VAR_CSR_FLAT_FIXED;
+}
 
 int mode_of(int variant) {
   switch (variant) {
@@ -13,6 +19,8 @@ int mode_of(int variant) {
     case FP_VAR_CSR_FLAT: return DMODE_FLAT_SHARED;
     case FP_VAR_CSR_FLAT_L2: return DMODE_FLAT_L2;
     case FP_VAR_CSR_FLAT_PRIVATE: return DMODE_FLAT_PRIVATE;
+    case FP_VAR_CSR_VECTOR_FIXED: return MODE_FIXED;
+    case FP_VAR_CSR_FLAT_FIXED: return DMODE_FLAT_FIXED;
     default: return -1;
   }
 }
@@ -25,7 +33,7 @@ CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   if (L.variant == FP_VAR_CSR_OWNER) mode = a.n <= 4 * kCsrBS ? DMODE_OWNER4 : (a.n <= 8 * kCsrBS ? DMODE_OWNER8 : -1);
   if (mode < 0) return nullptr;
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
-  const bool flat = L.variant >= FP_VAR_CSR_FLAT && L.variant <= FP_VAR_CSR_FLAT_PRIVATE;
+  const bool flat = is_flat(L.variant);
   const int k = L.tl > 0 ? L.tl : (flat ? 4 : default_k(L.vs));
   return a.dtype == FP_F64 ? csr_pick_f64(ym, mode, L.vs, k) : csr_pick_f32(ym, mode, L.vs, k);
 }
@@ -46,6 +54,8 @@ size_t smem_for(const PatternArgs& a, int variant) {
       return yb + vb + (size_t)kOwnerQ * kCsrBS * (dtype_size(a.dtype) + 1) + (size_t)kCsrBS * 4;
     case FP_VAR_CSR_VECTOR:
     case FP_VAR_CSR_FLAT: return yb + vb;
+    case FP_VAR_CSR_VECTOR_FIXED:  // y (16-byte aligned) + fp64 spill + two 32-bit limbs per column
+    case FP_VAR_CSR_FLAT_FIXED: return (size_t)(a.y ? fix_y_bytes(a.n, (int)dtype_size(a.dtype)) : 0) + (size_t)a.n * 16;
     case FP_VAR_CSR_VECTOR_L2:
     case FP_VAR_CSR_FLAT_L2: return y_in_smem_l2(a) ? vb : 0;
     default: return 0;
@@ -62,6 +72,7 @@ int phase_iters_for(const PatternArgs& a, const fp_launch& L) {
   int pi = (int)((kCsrBS * kOwnerQ / 2) / per_iter);
   return pi < 1 ? 1 : pi;
 }
+
 
 }  // namespace
 
@@ -88,11 +99,14 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   // of ~300 settings (C3); the per-warp private and flat variants lose to it because fp64
   // shared-memory updates cost per instruction.  For large n the flat layout (lanes on
   // consecutive nonzeros, L2 reds) is best (C4: 17.3 ms vs 19.8 ms for CSR-vector).
+  // The fixed-point partial (variant 11: native int32 shared atomics instead of the fp64 CAS
+  // loop) measured no faster on C3 (1.28 vs 1.25-1.27 ms): the scatter is not what bounds this
+  // kernel (ncu: issue-latency bound, 4 warp instructions per nonzero), so the paper's layout stays.
   if (smem_for(a, FP_VAR_CSR_VECTOR) <= kSharedBudget) L.variant = FP_VAR_CSR_VECTOR;
   else L.variant = FP_VAR_CSR_FLAT_L2;
   (void)kPrivateBudget;
   L.smem_bytes = (int)smem_for(a, L.variant);
-  L.tl = L.variant >= FP_VAR_CSR_FLAT ? 8 : default_k(L.vs);
+  L.tl = is_flat(L.variant) ? 8 : default_k(L.vs);
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
   if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
@@ -104,7 +118,6 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   L.regs_per_thread = fa.numRegs;
   L.blocks_per_sm = per_sm;
   L.concurrent_warps = per_sm * L.bs / 32;
-  L.tl = L.variant >= FP_VAR_CSR_FLAT ? 8 : default_k(L.vs);
   int64_t grid = (int64_t)di.sm_count * per_sm;
   int64_t need = (a.m + (L.bs / L.vs) - 1) / (L.bs / L.vs);  // one row per vector at least
   if (need < 1) need = 1;
@@ -120,7 +133,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: launch plan (variant=%d vs=%d) has no kernel", L.variant, L.vs);
   FP_REQUIRE(L.bs == kCsrBS, FP_ERR_UNSUPPORTED, "fp_csr: block size %d not supported", L.bs);
-  FP_REQUIRE(L.grid >= 1, FP_ERR_INVALID_ARG, "fp_csr: grid must be >= 1");
+  FP_REQUIRE(L.grid >= 0, FP_ERR_INVALID_ARG, "fp_csr: grid must be >= 0 (0 = one resident wave)");
   const bool l2 = L.variant == FP_VAR_CSR_VECTOR_L2 || L.variant == FP_VAR_CSR_FLAT_L2;
   const size_t smem = smem_for(a, L.variant);
   FP_REQUIRE(smem <= 227 * 1024, FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs %zu B shared memory (n too large)",
@@ -138,7 +151,13 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   // L2 path without y in shared memory: prefer the largest L1 so the random y gathers hit it
   // (X itself streams with L1::no_allocate and never displaces y)
   if (l2 && smem == 0) cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
-  f<<<L.grid, L.bs, smem, s>>>(k);
+  int grid = L.grid;
+  if (grid == 0) {  // one full resident wave: SMs x occupancy of this kernel
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, L.bs, (int)smem);
+    grid = device_info(current_device()).sm_count * (per_sm > 0 ? per_sm : 1);
+  }
+  f<<<grid, L.bs, smem, s>>>(k);
   FP_CUDA(cudaGetLastError());
   return FP_OK;
 }

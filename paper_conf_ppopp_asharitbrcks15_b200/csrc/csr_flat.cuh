@@ -22,7 +22,8 @@ namespace fp {
 
 template <typename T, int NB, int YM, int MODE, int BS>
 __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
-  static_assert(MODE == MODE_SHARED || MODE == MODE_L2 || MODE == MODE_PRIVATE, "flat kernel aggregation mode");
+  static_assert(MODE == MODE_SHARED || MODE == MODE_L2 || MODE == MODE_PRIVATE || MODE == MODE_FIXED,
+                "flat kernel aggregation mode");
   constexpr int NW = BS / 32;
   constexpr int CAP = 32 * NB;  // nonzeros per batch
   const int64_t* __restrict__ rowptr = a.rowptr;
@@ -41,9 +42,13 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
   T* w_s = y_s + (ysm ? n : 0);
   T* w_mine = MODE == MODE_PRIVATE ? w_s + (int64_t)warp * n : w_s;
+  __shared__ int fix_e;
+  const fpd::FixAcc FA = fix_layout(smem_raw + (ysm ? fix_y_bytes(n, sizeof(T)) : 0), n, &fix_e);
+  fpd::FixScale FS;
   {
     const int64_t nw_copies = MODE == MODE_PRIVATE ? NW : (MODE == MODE_SHARED ? 1 : 0);
     for (int64_t j = threadIdx.x; j < nw_copies * n; j += BS) w_s[j] = T(0);
+    if constexpr (MODE == MODE_FIXED) fpd::fix_init<BS>(FA, n);
     if (ysm)
       for (int64_t j = threadIdx.x; j < n; j += BS) y_s[j] = y[j];
     __syncthreads();
@@ -52,7 +57,18 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   auto Y = [&](int c) -> T { return ysm ? y_s[c] : fpd::ld_keep(y + c); };
   auto W_ADD = [&](int c, T val_) {
     if constexpr (MODE == MODE_SHARED) atomicAdd(w_s + c, val_);
+    else if constexpr (MODE == MODE_FIXED) fpd::fix_add(FA, FS, c, val_);
     else fpd::red_add((T*)a.w + c, val_);
+  };
+  // MODE_FIXED: until the CTA's scale is set, every warp offers its batch's largest |term|
+  auto FIX_SET = [&](T term, bool act) {
+    if constexpr (MODE == MODE_FIXED) {
+      if (FS.e == fpd::kFixUnset) {
+        double at, tm = 0.0;
+        if (act && fpd::fix_finite_abs((double)term, at)) tm = at;
+        fpd::fix_try_set(FA, FS, tm);
+      }
+    }
   };
   // one row's entries spread over the active lanes (long-row path): distinct columns when the
   // row is canonical; duplicates (R7) are serialised lane by lane
@@ -107,7 +123,9 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
       for (int64_t kb = 0; kb < L; kb += 32) {  // warp-uniform trip count
         const int64_t k = kb + lane;
         const bool act = k < L;
-        ROW_ADD(act ? __ldg(colidx + s0 + k) : 0, act ? __ldg(val + s0 + k) * q : T(0), act);
+        const T term = act ? __ldg(val + s0 + k) * q : T(0);
+        FIX_SET(term, act);
+        ROW_ADD(act ? __ldg(colidx + s0 + k) : 0, term, act);
       }
       rb += 1;
       continue;
@@ -167,6 +185,18 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
     }
 
     // ---- second touch from registers: Eq. (3), every lane busy
+    if constexpr (MODE == MODE_FIXED) {
+      if (FS.e == fpd::kFixUnset) {
+        double tm = 0.0;
+#pragma unroll
+        for (int j = 0; j < NB; ++j) {
+          double at;
+          const T qj = __shfl_sync(0xffffffffu, q, rid[j]);
+          if (j * 32 + lane < cnt && fpd::fix_finite_abs((double)(xv[j] * qj), at)) tm = fmax(tm, at);
+        }
+        fpd::fix_try_set(FA, FS, tm);
+      }
+    }
 #pragma unroll
     for (int j = 0; j < NB; ++j) {
       const T qj = __shfl_sync(0xffffffffu, q, rid[j]);
@@ -213,6 +243,12 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
     __syncthreads();
     fpd::grid_finalize<T, T>(w_s, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
                              a.accumulate);
+  } else if constexpr (MODE == MODE_FIXED) {
+    __syncthreads();
+    fpd::fix_to_double<BS>(FA, n);
+    __syncthreads();
+    fpd::grid_finalize<T, double>(FA.sp, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
+                                  a.accumulate);
   }
 }
 

@@ -25,6 +25,7 @@
 //     Small-n modes finish with the fp64 grid accumulator + last-CTA finalize (aggregate.cuh).
 #pragma once
 #include "aggregate.cuh"
+#include "fixacc.cuh"
 #include "kernels.cuh"
 
 namespace fp {
@@ -48,7 +49,18 @@ struct CsrKArgs {
   int phase_iters;  // owner-computes kernel: row-group iterations between queue drains
 };
 
-enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2 };
+enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2, MODE_FIXED = 8 };
+
+// shared-memory layout of the MODE_FIXED partial behind y_s (fixacc.cuh): [sp: n f64][lo: n u32][hi: n u32]
+__device__ __forceinline__ fpd::FixAcc fix_layout(unsigned char* base, int64_t n, int* e) {
+  fpd::FixAcc A;
+  A.sp = reinterpret_cast<double*>(base);
+  A.lo = reinterpret_cast<uint32_t*>(A.sp + n);
+  A.hi = reinterpret_cast<int32_t*>(A.lo + n);
+  A.e = e;
+  return A;
+}
+__host__ __device__ constexpr int64_t fix_y_bytes(int64_t n, int s) { return (n * s + 15) / 16 * 16; }
 
 constexpr int64_t kRowCost = 4;  // a row costs about as much as 4 nonzeros (rowptr, v, reduce)
 
@@ -128,12 +140,16 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
   T* w_s = y_s + (ysm ? n : 0);
   T* w_mine = MODE == MODE_PRIVATE ? w_s + (int64_t)warp * n : w_s;
+  __shared__ int fix_e;
+  const fpd::FixAcc FA = fix_layout(smem_raw + (ysm ? fix_y_bytes(n, sizeof(T)) : 0), n, &fix_e);
+  fpd::FixScale FS;
   {
     const int64_t nw_copies = MODE == MODE_PRIVATE ? NW : (MODE == MODE_SHARED ? 1 : 0);
     for (int64_t j = threadIdx.x; j < nw_copies * n; j += BS) w_s[j] = T(0);
+    if constexpr (MODE == MODE_FIXED) fpd::fix_init<BS>(FA, n);
     if (ysm)
       for (int64_t j = threadIdx.x; j < n; j += BS) y_s[j] = y[j];
-    if (nw_copies > 0 || ysm) __syncthreads();
+    if (nw_copies > 0 || ysm || MODE == MODE_FIXED) __syncthreads();
   }
   // alpha: folded into q on the L2 path, applied once by the finaliser on the smem paths
   const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
@@ -143,6 +159,8 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
       warp_private_add<VS>(w_mine, c, val_, act, lane);
     } else if constexpr (MODE == MODE_SHARED) {
       if (act) atomicAdd(w_s + c, val_);
+    } else if constexpr (MODE == MODE_FIXED) {
+      if (act) fpd::fix_add(FA, FS, c, val_);
     } else {
       if (act) fpd::red_add((T*)a.w + c, val_);
     }
@@ -250,6 +268,19 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
     }
 
     // ---- second touch from registers: Eq. (3) / Alg. 2 l.13-14
+    if constexpr (MODE == MODE_FIXED) {
+      if (FS.e == fpd::kFixUnset) {  // warp-uniform; until the CTA's fixed-point scale is set
+        double tmax = 0.0;
+#pragma unroll
+        for (int i = 0; i < RPV; ++i)
+#pragma unroll
+          for (int k = 0; k < K; ++k) {
+            double at;
+            if (lid + k * VS < len[i] && fpd::fix_finite_abs((double)(xv[i][k] * q[i]), at)) tmax = fmax(tmax, at);
+          }
+        fpd::fix_try_set(FA, FS, tmax);
+      }
+    }
 #pragma unroll
     for (int i = 0; i < RPV; ++i)
 #pragma unroll
@@ -290,6 +321,12 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
     __syncthreads();
     fpd::grid_finalize<T, T>(w_s, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
                              a.accumulate);
+  } else if constexpr (MODE == MODE_FIXED) {
+    __syncthreads();
+    fpd::fix_to_double<BS>(FA, n);
+    __syncthreads();
+    fpd::grid_finalize<T, double>(FA.sp, n, a.acc, a.counter, a.alpha, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
+                                  a.accumulate);
   }
 }
 
@@ -312,7 +349,8 @@ CsrKFn csr_pick_owner_n(int vs, int k) {
 }
 
 // dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
-enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5, DMODE_OWNER4 = 6, DMODE_OWNER8 = 7 };
+enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5, DMODE_OWNER4 = 6, DMODE_OWNER8 = 7,
+       DMODE_FLAT_FIXED = 9 };
 
 template <typename T, int YM, int MODE>
 CsrKFn csr_pick_flat(int nb) {
@@ -343,6 +381,8 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case MODE_L2: return csr_pick_vs<T, YM, MODE_L2>(vs, k);
     case MODE_SHARED: return csr_pick_vs<T, YM, MODE_SHARED>(vs, k);
     case MODE_PRIVATE: return csr_pick_vs<T, YM, MODE_PRIVATE>(vs, k);
+    case MODE_FIXED: return csr_pick_vs<T, YM, MODE_FIXED>(vs, k);
+    case DMODE_FLAT_FIXED: return csr_pick_flat<T, YM, MODE_FIXED>(k);
     case DMODE_FLAT_SHARED: return csr_pick_flat<T, YM, MODE_SHARED>(k);
     case DMODE_FLAT_L2: return csr_pick_flat<T, YM, MODE_L2>(k);
     case DMODE_FLAT_PRIVATE: return csr_pick_flat<T, YM, MODE_PRIVATE>(k);

@@ -62,7 +62,7 @@ def test_csr_instances(cuda_dev, dt, m, n, lengths, inst):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f32"])
-@pytest.mark.parametrize("variant", [3, 4, 5])
+@pytest.mark.parametrize("variant", [3, 4, 5, 11])
 @pytest.mark.parametrize("vs", [1, 2, 4, 8, 16, 32])
 def test_csr_every_vs_and_variant_bitexact(cuda_dev, dt, variant, vs):
     """fp_csr_ex with every VS of Eq. (4) and both aggregation variants: integer twins
@@ -172,7 +172,7 @@ def test_csr_plan_c3_c4(cuda_dev):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f32"])
-@pytest.mark.parametrize("variant", [6, 7, 8])
+@pytest.mark.parametrize("variant", [6, 7, 8, 12])
 @pytest.mark.parametrize("nb", [2, 4, 8])
 @pytest.mark.parametrize("lengths", [("uniform", 0, 70), ("powerlaw", 2.0, 3.0), ("binomial", 0.02)])
 def test_csr_flat_bitexact(cuda_dev, dt, variant, nb, lengths):
@@ -224,3 +224,44 @@ def test_csr_owner_bitexact(cuda_dev, dt, vs, k, n):
             ref, _ = oracle.csr(m, n, rp, ci, va, *args)
             w = gpu_csr(cuda_dev, rp, ci, va, n, *args, launch=L)
             assert_bitexact(w, ref, f"owner vs={vs} k={k} n={n} {lengths}")
+
+
+def _single_column(m, v_of_row, dt):
+    rp = torch.arange(m + 1, dtype=torch.int64)
+    ci = torch.zeros(m, dtype=torch.int32)
+    va = torch.ones(m, dtype=DT[dt])
+    v = torch.tensor([v_of_row(r) for r in range(m)], dtype=DT[dt])
+    return rp, ci, va, torch.ones(1, dtype=DT[dt]), v
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("variant,vs,tl", [(11, 1, 2), (11, 8, 2), (12, 32, 4)])
+def test_fixed_point_limb_moves_and_spill_bitexact(cuda_dev, dt, variant, vs, tl):
+    """Fixed-point partial (fixacc.cuh) on one CTA and one column: the first rows set the cap
+    exponent from terms of 1 (cap 2^7); then 40k terms of 63 push the high limb past 2^29
+    (value-preserving moves into the fp64 spill) and terms of 1000 exceed the cap (spill
+    path).  Integers: the sum is exact, so w must equal the oracle bit for bit."""
+    m = 60000  # one CTA of 8 warps: warp w owns rows [7500 w, 7500 (w + 1)); each starts with 256 rows of 1
+    rp, ci, va, y, v = _single_column(m, lambda r: 1.0 if r % 7500 < 256 else (1000.0 if r % 97 == 0 else 63.0), dt)
+    ref, _ = oracle.csr(m, 1, rp, ci, va, y, v, None, 1.0, 0.0)
+    L = fp.fp_launch()
+    L.variant, L.vs, L.tl, L.bs, L.grid = variant, vs, tl, 256, 1
+    w = gpu_csr(cuda_dev, rp, ci, va, 1, y, v, None, 1.0, 0.0, launch=L)
+    assert_bitexact(w, ref, f"fixed moves variant={variant}")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("variant", [11, 12])
+def test_fixed_point_wide_dynamic_range(cuda_dev, dt, variant):
+    """Rows scaled by 2^k, k uniform in [-40, 40] (terms spanning ~2^160): the fixed-point
+    partial keeps the stated normwise tolerance (small terms round to the CTA's grid, large
+    ones spill to fp64; DESIGN reading R21)."""
+    m, n = 30000, 800
+    rp, ci, va, y, v, z = make_csr(m, n, dt, ("binomial", 0.01), seed=41)
+    k = torch.from_numpy(np.random.default_rng(41).integers(-40, 41, m)).double()
+    v = (v.double() * torch.pow(2.0, k)).to(DT[dt])
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    L = fp.fp_launch()
+    L.variant, L.vs, L.tl, L.bs, L.grid = variant, 8 if variant == 11 else 32, 2 if variant == 11 else 4, 256, 148
+    w = gpu_csr(cuda_dev, rp, ci, va, n, y, v, z, 1.0, 1.0, launch=L)
+    assert_parity(w, ref, mag, DT[dt], f"fixed wide range variant={variant}")

@@ -43,6 +43,8 @@ def main():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--variants", default=None, help="comma-separated subset of variants to sweep")
+    ap.add_argument("--grids", default="148,296,444,592,888,1184,2368")
     args = ap.parse_args()
     dev = torch.device("cuda:0")
     cfg, inp = bench.build_inputs(args.config, 0, 1, dev)
@@ -67,15 +69,18 @@ def main():
     ref = inp["w"].double().cpu().numpy().copy()
     t_base = time_call(lambda: run(base), args.reps)
 
-    grids = [148, 296, 444, 592, 888, 1184, 2368]
+    grids = [int(g) for g in args.grids.split(",")]
     if csr:
-        space = [(var, vs, k) for var in (3, 4, 5) for vs, k in
+        space = [(var, vs, k) for var in (3, 4, 5, 11) for vs, k in
                  [(1, 2), (1, 4), (2, 2), (2, 4), (4, 2), (4, 4), (8, 1), (8, 2), (16, 1), (16, 2), (32, 2), (32, 4)]]
-        space += [(var, 32, nb) for var in (6, 7, 8) for nb in (2, 4, 8)]   # flat kernels: k = NB tiles
+        space += [(var, 32, nb) for var in (6, 7, 8, 12) for nb in (2, 4, 8)]   # flat kernels: k = NB tiles
         if cfg["n"] <= 2048:
             space += [(10, vs, k) for vs, k in ((4, 4), (8, 2), (16, 2), (32, 4))]   # owner-computes
     else:
         space = [(base.variant, base.vs, base.tl)]
+    if args.variants:
+        keep = {int(v) for v in args.variants.split(",")}
+        space = [s for s in space if s[0] in keep]
     rows = []
     for (var, vs, k), g in itertools.product(space, grids):
         L = fp.fp_launch()
