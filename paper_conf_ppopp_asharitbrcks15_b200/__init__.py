@@ -27,7 +27,8 @@ FP_F32, FP_F64 = 0, 1
 STATUS = {0: "FP_OK", 1: "FP_ERR_INVALID_ARG", 2: "FP_ERR_UNSUPPORTED", 3: "FP_ERR_ALIAS", 4: "FP_ERR_INVALID_CSR",
           5: "FP_ERR_CUDA", 6: "FP_ERR_NCCL", 7: "FP_ERR_NOMEM"}
 VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2", 5: "csr_vector_private",
-            6: "csr_flat_smem", 7: "csr_flat_l2", 8: "csr_flat_private", 9: "dense_cluster", 10: "csr_owner"}
+            6: "csr_flat_smem", 7: "csr_flat_l2", 8: "csr_flat_private", 9: "dense_cluster", 10: "csr_owner",
+            11: "csr_vector_fixed", 12: "csr_flat_fixed", 13: "csr_colsplit_cluster"}
 
 
 class FusedPatError(RuntimeError):
@@ -81,6 +82,10 @@ _SIGS = {
     "fp_choose_paper": (_int, [_int, _P(fp_row_stats), _int, _P(fp_device_profile), _int, _int, _int, _P(fp_launch)]),
     "fp_choose": (_int, [_int, _P(fp_row_stats), _int, _int, _P(fp_launch)]),
     "fp_csr_validate": (_int, [_i64, _i64, _i64, _vp, _vp, _vp]),
+    "fp_csr_plan_create": (_int, [_i64, _i64, _i64, _vp, _vp, _int, _P(fp_launch), _P(_vp), _vp]),
+    "fp_csr_plan_exec": (_int, [_vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _vp]),
+    "fp_csr_plan_launch": (_int, [_vp, _P(fp_launch)]),
+    "fp_csr_plan_destroy": (_int, [_vp]),
     "fp_dense_host": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_csr_host": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_release_workspace": (_int, []),
@@ -227,6 +232,54 @@ def csr(rowptr, colidx, val, n, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=N
     else:
         _call("fp_csr_ex", *args, ctypes.byref(launch), s)
     return w
+
+
+class CsrPlan:
+    """fp_csr_plan: the once-per-matrix analysis of a CSR structure (launch parameters and, for
+    wide n, the column split of the cluster kernel).  Keeps rowptr/colidx alive; the structure
+    must not change while the plan is used.  ``plan(val, y, v, z, alpha, beta, w)`` evaluates
+    Eq. (1) on the plan's matrix."""
+
+    def __init__(self, rowptr, colidx, n, dtype, launch=None, stream=None):
+        _require_cuda(rowptr, colidx)
+        if rowptr.dtype != torch.int64 or colidx.dtype != torch.int32:
+            raise TypeError("rowptr must be int64 and colidx int32")
+        self.rowptr, self.colidx, self.n = rowptr, colidx, int(n)
+        self.m, self.nnz = rowptr.shape[0] - 1, colidx.shape[0]
+        self.dtype = dtype
+        self._h = ctypes.c_void_p()
+        fdt = FP_F64 if dtype == torch.float64 else FP_F32
+        _call("fp_csr_plan_create", self.m, self.n, self.nnz, _ptr(rowptr), _ptr(colidx), fdt,
+              None if launch is None else ctypes.byref(launch), ctypes.byref(self._h), _stream(rowptr.device, stream))
+
+    @property
+    def launch(self):
+        L = fp_launch()
+        _call("fp_csr_plan_launch", self._h, ctypes.byref(L))
+        return L
+
+    def __call__(self, val, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
+        _require_cuda(val, y, v, z, w)
+        if val.dtype != self.dtype or val.shape[0] != self.nnz:
+            raise ValueError(f"val must be {self.dtype}[{self.nnz}]")
+        y, v, z = _vec(y, self.n, val.dtype, "y"), _vec(v, self.m, val.dtype, "v"), _vec(z, self.n, val.dtype, "z")
+        if w is None:
+            w = torch.empty(self.n, dtype=val.dtype, device=val.device)
+        _vec(w, self.n, val.dtype, "w")
+        _call("fp_csr_plan_exec", self._h, _ptr(val), _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w),
+              _stream(val.device, stream))
+        return w
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib().fp_csr_plan_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def dense_host(X, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, device=0):

@@ -37,6 +37,32 @@ __device__ __forceinline__ void grid_finalize(const S* __restrict__ sw, int64_t 
   if (threadIdx.x == 0) *counter = 0ull;
 }
 
+// Same, for a CTA whose partial covers only columns [off, off + len) of w (column-split
+// cluster kernel): the last CTA of the grid still finalises all n columns.
+template <typename T, typename S>
+__device__ __forceinline__ void grid_finalize_window(const S* __restrict__ sw, int64_t off, int64_t len, int64_t n,
+                                                     double* acc, unsigned long long* counter, double alpha,
+                                                     double beta, const T* z, T* w, bool add_beta_z,
+                                                     bool accumulate) {
+  for (int64_t j = threadIdx.x; j < len; j += blockDim.x) atomicAdd(acc + off + j, (double)sw[j]);
+  __threadfence();
+  __syncthreads();
+  __shared__ int s_last_w;
+  if (threadIdx.x == 0) s_last_w = (atomicAdd(counter, 1ull) == (unsigned long long)gridDim.x - 1ull);
+  __syncthreads();
+  if (!s_last_w) return;
+  __threadfence();
+  for (int64_t j = threadIdx.x; j < n; j += blockDim.x) {
+    double s = __ldcg(acc + j);
+    acc[j] = 0.0;
+    double r = alpha * s;
+    if (add_beta_z && beta != 0.0) r += beta * (double)z[j];
+    if (accumulate) r += (double)w[j];
+    w[j] = (T)r;
+  }
+  if (threadIdx.x == 0) *counter = 0ull;
+}
+
 }  // namespace fpd
 
 namespace fpd {

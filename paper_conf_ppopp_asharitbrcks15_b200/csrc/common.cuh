@@ -217,6 +217,18 @@ __device__ __forceinline__ void prefetch_l2(const void* p, size_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((unsigned)(e - a)) : "memory");
 }
 
+// one shared-memory compare-and-swap of a float / double (returns the previous value)
+__device__ __forceinline__ float cas_shared(float* p, float cmp, float val) {
+  return __int_as_float(atomicCAS(reinterpret_cast<int*>(p), __float_as_int(cmp), __float_as_int(val)));
+}
+__device__ __forceinline__ double cas_shared(double* p, double cmp, double val) {
+  return __longlong_as_double((long long)atomicCAS(reinterpret_cast<unsigned long long*>(p),
+                                                   (unsigned long long)__double_as_longlong(cmp),
+                                                   (unsigned long long)__double_as_longlong(val)));
+}
+__device__ __forceinline__ bool same_bits(float a, float b) { return __float_as_int(a) == __float_as_int(b); }
+__device__ __forceinline__ bool same_bits(double a, double b) { return __double_as_longlong(a) == __double_as_longlong(b); }
+
 __device__ __forceinline__ float ld_keep(const float* p) {
   float r;
   asm("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(r) : "l"(p));

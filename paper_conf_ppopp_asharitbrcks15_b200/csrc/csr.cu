@@ -1,4 +1,5 @@
 // csr.cu -- B200 plan and launch of the fused CSR kernels (csr_kernels.cuh).
+#include <algorithm>
 #include <cstdlib>
 
 #include "csr_kernels.cuh"
@@ -129,7 +130,118 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   return FP_OK;
 }
 
+namespace {
+int ym_of(const PatternArgs& a) { return !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2); }
+
+SplitKFn pick_split(const PatternArgs& a, int cs, int nb) {
+  return a.dtype == FP_F64 ? csr_pick_colsplit_f64(ym_of(a), cs, nb) : csr_pick_colsplit_f32(ym_of(a), cs, nb);
+}
+
+// register tiles per warp batch: 16 when the mean block segment of a 32-row batch exceeds 8 tiles
+int split_nb(const PatternArgs& a, int cs) {
+  const double seg = a.m > 0 ? 32.0 * (double)a.nnz / (double)a.m / cs : 0.0;
+  return seg > 0.8 * 8 * 32 ? 16 : 8;
+}
+
+cudaLaunchConfig_t split_config(const PatternArgs& a, const CsrSplit& sp, int grid, cudaLaunchAttribute* attr,
+                                cudaStream_t s) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3((unsigned)kSplitBS);
+  cfg.dynamicSmemBytes = colsplit_smem(a.dtype, sp.cs, sp.width, a.y != nullptr);
+  cfg.stream = s;
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)sp.cs;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cfg;
+}
+
+// co-resident clusters of the split kernel (0 if it does not fit)
+int split_capacity(const PatternArgs& a, const CsrSplit& sp, int nb) {
+  SplitKFn f = pick_split(a, sp.cs, nb);
+  if (!f) return 0;
+  const size_t smem = colsplit_smem(a.dtype, sp.cs, sp.width, a.y != nullptr);
+  if (smem > 227 * 1024) return 0;
+  if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  cudaLaunchAttribute attr[1];
+  cudaLaunchConfig_t cfg = split_config(a, sp, sp.cs * 64, attr, 0);
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, (const void*)f, &cfg) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
+}
+}  // namespace
+
+// Column-split plan (FP_VAR_CSR_COLSPLIT): the smallest cluster (2, 4, 8 CTAs, one per SM)
+// whose column blocks of y and w fit one CTA's shared memory; equal-width column blocks.
+bool plan_colsplit(const PatternArgs& a, int device, int cs_force, CsrSplit* sp, fp_launch* L) {
+  (void)device;
+  if (a.n < 2 || a.n > INT32_MAX) return false;
+  for (int cs = 2; cs <= kSplitMaxCS; cs *= 2) {
+    if (cs_force && cs != cs_force) continue;
+    CsrSplit t;
+    t.cs = cs;
+    for (int k = 0; k <= cs; ++k) t.cb[k] = (int)((a.n * k) / cs);
+    t.width = 0;
+    for (int k = 0; k < cs; ++k) t.width = std::max(t.width, t.cb[k + 1] - t.cb[k]);
+    if (colsplit_smem(a.dtype, cs, t.width, a.y != nullptr) > 227 * 1024) continue;
+    const int nb = split_nb(a, cs);
+    const int nc = split_capacity(a, t, nb);
+    if (nc < 1) continue;
+    *sp = t;
+    fp_launch o{};
+    o.variant = FP_VAR_CSR_COLSPLIT;
+    o.vs = 32;
+    o.bs = kSplitBS;
+    o.tl = nb;
+    o.cluster = cs;
+    o.grid = nc * cs;
+    o.blocks_per_sm = 1;
+    o.concurrent_warps = kSplitBS / 32;
+    o.smem_bytes = (int)colsplit_smem(a.dtype, cs, t.width, a.y != nullptr);
+    cudaFuncAttributes fa{};
+    if (cudaFuncGetAttributes(&fa, (const void*)pick_split(a, cs, nb)) == cudaSuccess) o.regs_per_thread = fa.numRegs;
+    const int64_t vectors = (int64_t)o.grid / cs * (kSplitBS / 32);
+    o.rows_per_vector = vectors > 0 ? (a.m + vectors - 1) / vectors : 0;
+    *L = o;
+    return true;
+  }
+  return false;
+}
+
 fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
+  if (L.variant == FP_VAR_CSR_COLSPLIT) {
+    FP_REQUIRE(a.split && a.split->soff && a.split->cs == L.cluster, FP_ERR_UNSUPPORTED,
+               "fp_csr: variant %d (column split) runs from a CSR plan (fp_csr_plan_create)", L.variant);
+    const CsrSplit& sp = *a.split;
+    SplitKFn f = pick_split(a, sp.cs, L.tl);
+    FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no column-split kernel for cluster %d, %d tiles", sp.cs, L.tl);
+    FP_REQUIRE(L.grid >= sp.cs && L.grid % sp.cs == 0, FP_ERR_INVALID_ARG, "fp_csr: split grid must be k x %d",
+               sp.cs);
+    Workspace* ws = workspace(s, (size_t)a.n, 0);
+    if (!ws) return FP_ERR_NOMEM;
+    SplitKArgs k{};
+    k.k = CsrKArgs{a.m, a.n, a.nnz, a.rowptr, a.colidx, a.val, a.y, a.v, a.z, a.alpha, a.beta, a.w,
+                   ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, 0,
+                   {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}, 0};
+    k.soff = sp.soff;
+    for (int i = 0; i <= kSplitMaxCS; ++i) k.cb[i] = sp.cb[i];
+    k.width = sp.width;
+    const size_t smem = colsplit_smem(a.dtype, sp.cs, sp.width, a.y != nullptr);
+    FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    cudaLaunchAttribute attr[1];
+    cudaLaunchConfig_t cfg = split_config(a, sp, L.grid, attr, s);
+    FP_CUDA(cudaLaunchKernelEx(&cfg, f, k));
+    return FP_OK;
+  }
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: launch plan (variant=%d vs=%d) has no kernel", L.variant, L.vs);
   FP_REQUIRE(L.bs == kCsrBS, FP_ERR_UNSUPPORTED, "fp_csr: block size %d not supported", L.bs);

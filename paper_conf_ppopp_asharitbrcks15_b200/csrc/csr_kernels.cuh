@@ -335,9 +335,43 @@ constexpr int kCsrBS = 256;
 using CsrKFn = void (*)(const CsrKArgs);
 
 }  // namespace fp
+#include "csr_colsplit.cuh"
 #include "csr_flat.cuh"
 #include "csr_owner.cuh"
 namespace fp {
+
+// column-split cluster kernels (csr_colsplit.cuh): 512 threads, NB in {8, 16} register tiles
+constexpr int kSplitBS = 512;
+using SplitKFn = void (*)(const SplitKArgs);
+
+template <typename T, int YM, int NB>
+SplitKFn csr_pick_colsplit_y(int cs) {
+  switch (cs) {
+    case 2: return k_csr_colsplit<T, 2, NB, YM, kSplitBS>;
+    case 4: return k_csr_colsplit<T, 4, NB, YM, kSplitBS>;
+    case 8: return k_csr_colsplit<T, 8, NB, YM, kSplitBS>;
+    default: return nullptr;
+  }
+}
+template <typename T, int NB>
+SplitKFn csr_pick_colsplit_nb(int ym, int cs) {
+  switch (ym) {
+    case 0: return csr_pick_colsplit_y<T, 0, NB>(cs);
+    case 1: return csr_pick_colsplit_y<T, 1, NB>(cs);
+    case 2: return csr_pick_colsplit_y<T, 2, NB>(cs);
+    default: return nullptr;
+  }
+}
+template <typename T>
+SplitKFn csr_pick_colsplit_t(int ym, int cs, int nb) {
+  return nb == 8 ? csr_pick_colsplit_nb<T, 8>(ym, cs) : (nb == 16 ? csr_pick_colsplit_nb<T, 16>(ym, cs) : nullptr);
+}
+SplitKFn csr_pick_colsplit_f32(int ym, int cs, int nb);  // csr_split_f32.cu
+SplitKFn csr_pick_colsplit_f64(int ym, int cs, int nb);  // csr_split_f64.cu
+inline size_t colsplit_smem(fp_dtype dt, int cs, int width, bool has_y) {
+  const size_t s = dt == FP_F64 ? 8 : 4;
+  return (size_t)(kSplitBS / 32) * (2 * cs + 1) * 32 * s + (size_t)width * s * (has_y ? 2 : 1);
+}
 
 template <typename T, int YM, int NPT>
 CsrKFn csr_pick_owner_n(int vs, int k) {
@@ -368,8 +402,9 @@ template <typename T, int YM, int MODE>
 CsrKFn csr_pick_vs(int vs, int k) {
 #define FP_CSR_K(VS_, K_, RPV_) \
   if (vs == VS_ && k == K_) return k_csr_vector<T, VS_, K_, RPV_, YM, MODE, kCsrBS>;
-  FP_CSR_K(1, 2, 1) FP_CSR_K(1, 4, 1) FP_CSR_K(2, 2, 1) FP_CSR_K(2, 4, 1)
-  FP_CSR_K(4, 2, 2) FP_CSR_K(4, 4, 2) FP_CSR_K(8, 1, 2) FP_CSR_K(8, 2, 2)
+  FP_CSR_K(1, 2, 1) FP_CSR_K(1, 4, 1) FP_CSR_K(1, 12, 1) FP_CSR_K(1, 16, 1) FP_CSR_K(2, 2, 1) FP_CSR_K(2, 4, 1)
+  FP_CSR_K(2, 8, 1) FP_CSR_K(4, 4, 1)
+  FP_CSR_K(4, 2, 2) FP_CSR_K(8, 1, 2) FP_CSR_K(8, 2, 2)
   FP_CSR_K(16, 1, 2) FP_CSR_K(16, 2, 2) FP_CSR_K(32, 2, 2) FP_CSR_K(32, 4, 2)
 #undef FP_CSR_K
   return nullptr;

@@ -4,6 +4,17 @@
 
 namespace fp {
 
+constexpr int kSplitMaxCS = 8;
+
+// What a CSR plan precomputes for the column-split cluster kernel (csr_colsplit.cuh); soff is
+// device memory owned by the plan (fp_csr_plan).
+struct CsrSplit {
+  const int32_t* soff = nullptr;  // [(cs-1)][m]: entries of row r with column < cb[k+1]
+  int cs = 0;                     // CTAs per cluster = column blocks
+  int cb[kSplitMaxCS + 1] = {};   // column block bounds, cb[0] = 0, cb[cs] = n
+  int width = 0;                  // max_k cb[k+1] - cb[k]
+};
+
 struct PatternArgs {
   int64_t m = 0, n = 0;
   // dense
@@ -32,6 +43,8 @@ struct PatternArgs {
   double epi_c = 1.0;
   void* row_out = nullptr;
   double* scalar_out = nullptr;
+  // column split of a CSR plan (FP_VAR_CSR_COLSPLIT only)
+  const CsrSplit* split = nullptr;
 };
 
 // Dense chooser (B200 plan): fills vs, tl, bs, grid, variant ... for the kernels in dense.cu.
@@ -40,6 +53,16 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
 
 fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out);
 fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s);
+// Column-split cluster plan for a CSR matrix whose y / w blocks fit shared memory: fills
+// L (variant FP_VAR_CSR_COLSPLIT) and the host part of sp (cs, cb, width); cs_force = 0 picks
+// the smallest cluster that fits.  Returns false if no cluster size fits.
+bool plan_colsplit(const PatternArgs& a, int device, int cs_force, CsrSplit* sp, fp_launch* L);
+
+// api.cu: validation + alpha == 0 path + plan + launch of one pattern evaluation
+fp_status run_csr(const PatternArgs& a, const fp_launch* override_, cudaStream_t s);
+PatternArgs csr_args(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                     const void* val, const void* y, const void* v, const void* z, double alpha, double beta, void* w,
+                     fp_dtype dtype);
 
 // w = beta*z (or 0): the alpha == 0 / m == 0 path, and the pre-initialisation of the L2 path.
 fp_status launch_scale_z(int64_t n, const void* z, double beta, void* w, fp_dtype dt, cudaStream_t s);
