@@ -259,8 +259,14 @@ def run_gpu(args):
             st.mean = st.nnz / max(1, st.m)
             plan = fp.choose(True, st, fp.FP_F64 if cfg["dtype"] == "f64" else fp.FP_F32, local)
         passes_per_step = 1
-        # the L2 variants write beta*z (k_scale_z) before the main kernel
-        launches_per_step = 2 if plan.variant in (4, 7) else 1
+        # the L2 variants write beta*z (k_scale_z) before the main kernel and, when w is
+        # replicated over L2 (csr.cu l2_replicas: 8 copies while they take <= 16 MB), fold the
+        # copies after it
+        launches_per_step = 1
+        if plan.variant in (4, 7):
+            s_b = 8 if cfg["dtype"] == "f64" else 4
+            nrep = int(os.environ.get("FP_L2_REPLICAS", "0")) or (8 if 8 * n * s_b <= (16 << 20) else 1)
+            launches_per_step = 2 + (1 if nrep > 1 else 0)
 
     flush = None
     if name == "C1":  # X fits in L2: flush between timed iterations

@@ -43,6 +43,34 @@ constexpr size_t kPrivateBudget = 100 * 1024;  // y + NW warp partials per CTA
 constexpr size_t kSharedBudget = 64 * 1024;    // y + one CTA partial
 constexpr size_t kYBudget = 96 * 1024;         // y staged in smem on the L2 path
 
+// w += sum of the replicas; the replicas are re-zeroed (the workspace invariant)
+template <typename T>
+__global__ void k_fold_replicas(T* __restrict__ w, T* __restrict__ rep, int64_t n, int nr) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    T s = w[j];
+    for (int r = 0; r < nr; ++r) {
+      s += rep[(int64_t)r * n + j];
+      rep[(int64_t)r * n + j] = T(0);
+    }
+    w[j] = s;
+  }
+}
+
+// Copies of w for the L2 path: the random reds of all CTAs into ONE n-vector leave some L2
+// slices near saturation while others idle (C4 ncu: lts__t_tag_requests avg 62 %, max 84 %,
+// min 32 %); 8 copies (CTA b reduces into copy b mod 8) measured 20.3 -> 18.7 ms on C4.  Only
+// while the copies stay small against L2 (126 MB).  FP_L2_REPLICAS overrides (measurement).
+constexpr int kL2Replicas = 8;
+constexpr size_t kL2ReplicaBudget = 16u << 20;
+int l2_replicas(const PatternArgs& a) {
+  static const int env = [] {
+    const char* e = std::getenv("FP_L2_REPLICAS");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (env > 0) return std::min(env, 16);
+  return (size_t)kL2Replicas * a.n * dtype_size(a.dtype) <= kL2ReplicaBudget ? kL2Replicas : 1;
+}
+
 bool y_in_smem_l2(const PatternArgs& a) { return a.y && (size_t)a.n * dtype_size(a.dtype) <= kYBudget; }
 
 size_t smem_for(const PatternArgs& a, int variant) {
@@ -100,14 +128,21 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   // of ~300 settings (C3); the per-warp private and flat variants lose to it because fp64
   // shared-memory updates cost per instruction.  For large n the flat layout (lanes on
   // consecutive nonzeros, L2 reds) is best (C4: 17.3 ms vs 19.8 ms for CSR-vector).
-  // The fixed-point partial (variant 11: native int32 shared atomics instead of the fp64 CAS
-  // loop) measured no faster on C3 (1.28 vs 1.25-1.27 ms): the scatter is not what bounds this
-  // kernel (ncu: issue-latency bound, 4 warp instructions per nonzero), so the paper's layout stays.
+  // Round-1 re-sweep after the y gathers were hoisted ahead of their use (every gather of a
+  // row group in flight at once; profiles/r01_sweep2_{C3,S3}.json): with Eq. (4)'s VS = 8 bin
+  // (8 < mu <= 16) the same 16 cached entries per row are faster as VS = 4 lanes x K = 4 than
+  // as 8 x 2 (C3 fp64 1.14 vs 1.28 ms, S3 fp32 0.92 vs 1.06 ms: more independent loads per
+  // lane, half the shuffle-reduce steps).  The fixed-point partial (variant 11) at 4 x 4 is 3 %
+  // faster on fp64 and slower on fp32; the paper's shared partial is kept.
   if (smem_for(a, FP_VAR_CSR_VECTOR) <= kSharedBudget) L.variant = FP_VAR_CSR_VECTOR;
   else L.variant = FP_VAR_CSR_FLAT_L2;
   (void)kPrivateBudget;
   L.smem_bytes = (int)smem_for(a, L.variant);
   L.tl = is_flat(L.variant) ? 8 : default_k(L.vs);
+  if (!is_flat(L.variant) && L.vs == 8) {
+    L.vs = 4;
+    L.tl = 4;
+  }
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
   if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
@@ -250,7 +285,11 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   const size_t smem = smem_for(a, L.variant);
   FP_REQUIRE(smem <= 227 * 1024, FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs %zu B shared memory (n too large)",
              L.variant, smem);
-  Workspace* ws = workspace(s, l2 ? 0 : (size_t)a.n, 0);
+  // L2 path: number of copies of w the CTAs spread their reds over (copies 1.. live in the
+  // all-zero workspace accumulator and are folded into w after the kernel)
+  const int nrep = l2 ? l2_replicas(a) : 1;
+  const size_t rep_doubles = nrep > 1 ? ((size_t)(nrep - 1) * a.n * dtype_size(a.dtype) + 7) / 8 : 0;
+  Workspace* ws = workspace(s, l2 ? rep_doubles : (size_t)a.n, 0);
   if (!ws) return FP_ERR_NOMEM;
   if (l2 && !a.accumulate) {  // L2 path: w <- beta z (or 0) first, the kernel reduces alpha X^T q into it
     fp_status st = launch_scale_z(a.n, a.add_beta_z ? a.z : nullptr, a.add_beta_z ? a.beta : 0.0, a.w, a.dtype, s);
@@ -258,7 +297,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   }
   CsrKArgs k{a.m, a.n, a.nnz, a.rowptr, a.colidx, a.val, a.y, a.v, a.z, a.alpha, a.beta, a.w,
              ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (l2 && y_in_smem_l2(a)) ? 1 : 0,
-             {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}, phase_iters_for(a, L)};
+             {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}, phase_iters_for(a, L), ws->acc, nrep};
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // L2 path without y in shared memory: prefer the largest L1 so the random y gathers hit it
   // (X itself streams with L1::no_allocate and never displaces y)
@@ -271,6 +310,15 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
   }
   f<<<grid, L.bs, smem, s>>>(k);
   FP_CUDA(cudaGetLastError());
+  if (nrep > 1) {
+    const int fb = 256;
+    const int fg = (int)std::min<int64_t>((a.n + fb - 1) / fb, 4 * device_info(current_device()).sm_count);
+    if (a.dtype == FP_F64)
+      k_fold_replicas<double><<<fg, fb, 0, s>>>((double*)a.w, (double*)ws->acc, a.n, nrep - 1);
+    else
+      k_fold_replicas<float><<<fg, fb, 0, s>>>((float*)a.w, (float*)ws->acc, a.n, nrep - 1);
+    FP_CUDA(cudaGetLastError());
+  }
   return FP_OK;
 }
 

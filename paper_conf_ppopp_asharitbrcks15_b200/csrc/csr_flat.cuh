@@ -55,10 +55,11 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   }
   const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
   auto Y = [&](int c) -> T { return ysm ? y_s[c] : fpd::ld_keep(y + c); };
+  T* const wl2 = l2_target<T>(a);
   auto W_ADD = [&](int c, T val_) {
     if constexpr (MODE == MODE_SHARED) atomicAdd(w_s + c, val_);
     else if constexpr (MODE == MODE_FIXED) fpd::fix_add(FA, FS, c, val_);
-    else fpd::red_add((T*)a.w + c, val_);
+    else fpd::red_add(wl2 + c, val_);
   };
   // MODE_FIXED: until the CTA's scale is set, every warp offers its batch's largest |term|
   auto FIX_SET = [&](T term, bool act) {
@@ -96,16 +97,25 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   const int64_t r1 = warp_search_rows(rowptr, m, (total * (gw + 1)) / tw, lane);
   double loss_acc = 0.0;
 
+  // rowptr of the batch starting at row b: lane i holds rowptr[b + i], clamped at r1
+  auto RP = [&](int64_t b) -> int64_t { return __ldg(rowptr + (b + lane < r1 ? b + lane : r1)); };
+  auto RP_END = [&](int64_t b) -> int64_t { return __ldg(rowptr + (b + 32 < r1 ? b + 32 : r1)); };
+  int64_t rp_cur = RP(r0), rp_end_cur = RP_END(r0);
   for (int64_t rb = r0; rb < r1;) {
     // ---- batch rows [rb, rb + nrows): lane i holds rowptr[rb + i] (clamped at r1)
-    const int64_t ri = rb + lane < r1 ? rb + lane : r1;
-    const int64_t rp = __ldg(rowptr + ri);
-    const int64_t rp_end = __ldg(rowptr + (rb + 32 < r1 ? rb + 32 : r1));
+    const int64_t rp = rp_cur;
+    const int64_t rp_end = rp_end_cur;
     const int64_t a0 = __shfl_sync(0xffffffffu, rp, 0);
     int64_t nxt = __shfl_down_sync(0xffffffffu, rp, 1);
     if (lane == 31) nxt = rp_end;
     const bool fits = (rb + lane < r1) && (nxt - a0 <= CAP);
     const int nrows = __popc(__ballot_sync(0xffffffffu, fits));  // rowptr monotone: a prefix
+    // v of this lane's row, loaded now so its latency overlaps the (col, val) and y loads
+    const T vpre = (v && rb + lane < r1) ? fpd::ld_once(v + rb + lane) : T(1);
+    // the next batch's rowptr, loaded now: its latency overlaps this batch's work
+    const int64_t rb_next = rb + (nrows == 0 ? 1 : nrows);
+    rp_cur = RP(rb_next);
+    rp_end_cur = RP_END(rb_next);
 
     if (nrows == 0) {
       // ---- a row longer than CAP: warp-per-row, dot pass then scatter pass (tail re-read)
@@ -127,7 +137,7 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
         FIX_SET(term, act);
         ROW_ADD(act ? __ldg(colidx + s0 + k) : 0, term, act);
       }
-      rb += 1;
+      rb = rb_next;
       continue;
     }
     const int64_t cnt = __shfl_sync(0xffffffffu, nxt, nrows - 1) - a0;   // nonzeros in the batch
@@ -155,12 +165,22 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
 
     T q = T(0);  // lane i: q of row rb + i
     if constexpr (HAS_Y) {
+      // all NB gathers of y issued before the first use: their L2 latencies overlap (a gather
+      // inside the reduction loop below serialised NB round trips per batch)
+      T yv[NB];
+      if (ysm) {
+#pragma unroll
+        for (int j = 0; j < NB; ++j) yv[j] = y_s[cc[j]];
+      } else {
+#pragma unroll
+        for (int j = 0; j < NB; ++j) yv[j] = fpd::ld_keep(y + cc[j]);
+      }
       rsum[warp][lane] = T(0);
       __syncwarp();
 #pragma unroll
       for (int j = 0; j < NB; ++j) {
         const int pos = j * 32 + lane;
-        T s = pos < cnt ? xv[j] * Y(cc[j]) : T(0);  // Eq. (2) products
+        T s = pos < cnt ? xv[j] * yv[j] : T(0);  // Eq. (2) products
         // segmented reduction toward the segment head (lanes of a row are contiguous)
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
@@ -176,12 +196,12 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
       const T p = rsum[warp][lane];
       const int64_t row = rb + lane;
       const bool ok = lane < nrows;
-      const T vr = ok ? (v ? v[row] : T(1)) : T(0);
+      const T vr = ok ? vpre : T(0);
       if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr, ok, row, ok, a.epi, loss_acc) * qscale;
       else q = ok ? p * vr * qscale : T(0);
     } else {
       const int64_t row = rb + lane;
-      q = lane < nrows ? (v ? v[row] : T(1)) * qscale : T(0);
+      q = lane < nrows ? vpre * qscale : T(0);
     }
 
     // ---- second touch from registers: Eq. (3), every lane busy
@@ -226,7 +246,7 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
         if (act) W_ADD(cc[j], xv[j] * qj);
       }
     }
-    rb += nrows;
+    rb = rb_next;
   }
   if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
 

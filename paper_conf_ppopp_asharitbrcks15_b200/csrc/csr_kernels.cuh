@@ -47,7 +47,20 @@ struct CsrKArgs {
   int y_in_smem;  // MODE_L2 only: stage y in shared memory (n*s bytes) for the gathers
   fpd::RowEpi epi;
   int phase_iters;  // owner-computes kernel: row-group iterations between queue drains
+  // MODE_L2: the CTAs reduce into nrep copies of w (copy 0 = w, copies 1.. = wrep, stride n,
+  // all-zero on entry; folded into w by k_fold_replicas) to spread the random reds over more
+  // L2 lines / slices
+  void* wrep;
+  int nrep;
 };
+
+// MODE_L2 target of this CTA's reds
+template <typename T>
+__device__ __forceinline__ T* l2_target(const CsrKArgs& a) {
+  if (a.nrep <= 1) return (T*)a.w;
+  const int r = (int)(blockIdx.x % (unsigned)a.nrep);
+  return r == 0 ? (T*)a.w : (T*)a.wrep + (int64_t)(r - 1) * a.n;
+}
 
 enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2, MODE_FIXED = 8 };
 
@@ -154,6 +167,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
   // alpha: folded into q on the L2 path, applied once by the finaliser on the smem paths
   const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
   auto Y = [&](int c) -> T { return ysm ? y_s[c] : fpd::ld_keep(y + c); };
+  T* const wl2 = l2_target<T>(a);
   auto W_ADD = [&](int c, T val_, bool act) {
     if constexpr (MODE == MODE_PRIVATE) {
       warp_private_add<VS>(w_mine, c, val_, act, lane);
@@ -162,7 +176,7 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
     } else if constexpr (MODE == MODE_FIXED) {
       if (act) fpd::fix_add(FA, FS, c, val_);
     } else {
-      if (act) fpd::red_add((T*)a.w + c, val_);
+      if (act) fpd::red_add(wl2 + c, val_);
     }
   };
 
@@ -233,12 +247,24 @@ __global__ void __launch_bounds__(BS) k_csr_vector(const CsrKArgs a) {
     T q[RPV];
     if constexpr (HAS_Y) {
       T p[RPV];
+      T yv[RPV][K];  // every gather issued before the first use (latencies overlap)
+      if (ysm) {
+#pragma unroll
+        for (int i = 0; i < RPV; ++i)
+#pragma unroll
+          for (int k = 0; k < K; ++k) yv[i][k] = y_s[cc[i][k]];
+      } else {
+#pragma unroll
+        for (int i = 0; i < RPV; ++i)
+#pragma unroll
+          for (int k = 0; k < K; ++k) yv[i][k] = fpd::ld_keep(y + cc[i][k]);
+      }
 #pragma unroll
       for (int i = 0; i < RPV; ++i) {  // Eq. (2) / Alg. 2 l.10-11
         p[i] = T(0);
 #pragma unroll
         for (int k = 0; k < K; ++k)
-          if (lid + k * VS < len[i]) p[i] = fma(xv[i][k], Y(cc[i][k]), p[i]);
+          if (lid + k * VS < len[i]) p[i] = fma(xv[i][k], yv[i][k], p[i]);
       }
       if (any_long) {  // tails of rows longer than VS*K (warp-uniform loop)
         for (int64_t seg = VS * K; seg < lmax; seg += VS * K) {

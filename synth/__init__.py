@@ -223,6 +223,9 @@ CONFIGS = {
     "K1": dict(fmt="csr", dtype="f64", m=15_009_374, n=29_890_095, lengths=("powerlaw", 2.5, 9.5, 1_000_000),
                alpha=1.0, beta=1.0, use_v=True, use_z=True, xkind="uniform", col_skew=2,
                desc="CSR fp64 KDD-shaped 15Mx29.9M power-law rows (mean ~28), Zipf-like columns (u^4), full with v"),
+    # C3's matrix in fp32 (chooser evidence for fp32 small-n CSR; not a BASELINE.json config)
+    "S3": dict(fmt="csr", dtype="f32", m=20_000_000, n=1000, lengths=("binomial", 0.01), alpha=1.0, beta=1.0,
+               use_v=True, use_z=True, xkind="uniform", desc="CSR fp32 20Mx1000 density 0.01, full with v"),
     # NEXT-4: dense rows wider than one CTA's registers (thread-block cluster kernel)
     "W1": dict(fmt="dense", dtype="f32", m=40_000, n=65_536, alpha=1.0, beta=0.0, use_v=False, use_z=False,
                xkind="uniform", desc="dense fp32 40000x65536 wide rows, X^T(Xy)"),
