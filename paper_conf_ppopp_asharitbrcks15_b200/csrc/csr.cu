@@ -22,6 +22,8 @@ int mode_of(int variant) {
     case FP_VAR_CSR_FLAT_PRIVATE: return DMODE_FLAT_PRIVATE;
     case FP_VAR_CSR_VECTOR_FIXED: return MODE_FIXED;
     case FP_VAR_CSR_FLAT_FIXED: return DMODE_FLAT_FIXED;
+    case FP_VAR_CSR_STREAM: return DMODE_STREAM_SHARED;
+    case FP_VAR_CSR_STREAM_FIXED: return DMODE_STREAM_FIXED;
     default: return -1;
   }
 }
@@ -87,6 +89,13 @@ size_t smem_for(const PatternArgs& a, int variant) {
     case FP_VAR_CSR_FLAT_FIXED: return (size_t)(a.y ? fix_y_bytes(a.n, (int)dtype_size(a.dtype)) : 0) + (size_t)a.n * 16;
     case FP_VAR_CSR_VECTOR_L2:
     case FP_VAR_CSR_FLAT_L2: return y_in_smem_l2(a) ? vb : 0;
+    case FP_VAR_CSR_STREAM:  // y (16-byte padded) + partial + two stages per warp
+    case FP_VAR_CSR_STREAM_FIXED: {
+      const size_t s = dtype_size(a.dtype);
+      const size_t part = variant == FP_VAR_CSR_STREAM_FIXED ? (size_t)a.n * 16 : (vb + 15) / 16 * 16;
+      const size_t stage = s == 8 ? (size_t)stream_stage_bytes<double>() : (size_t)stream_stage_bytes<float>();
+      return (a.y ? (size_t)fix_y_bytes(a.n, (int)s) : 0) + part + (size_t)(kCsrBS / 32) * 2 * stage;
+    }
     default: return 0;
   }
 }
@@ -252,7 +261,19 @@ bool plan_colsplit(const PatternArgs& a, int device, int cs_force, CsrSplit* sp,
   return false;
 }
 
-fp_status launch_csr(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
+// The stream variants copy colidx / val in 16-byte chunks and have no row epilogue; otherwise
+// the same (VS, K) runs as plain CSR-vector with the same partial (identical arithmetic).
+fp_launch stream_fallback(const PatternArgs& a, const fp_launch& L) {
+  fp_launch o = L;
+  if (L.variant != FP_VAR_CSR_STREAM && L.variant != FP_VAR_CSR_STREAM_FIXED) return o;
+  const bool aligned = ((uintptr_t)a.colidx % 16 == 0) && ((uintptr_t)a.val % 16 == 0);
+  const bool epi = a.y && !(a.epi_kind == 0 && !a.row_out);
+  if (!aligned || epi) o.variant = L.variant == FP_VAR_CSR_STREAM ? FP_VAR_CSR_VECTOR : FP_VAR_CSR_VECTOR_FIXED;
+  return o;
+}
+
+fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s) {
+  const fp_launch L = stream_fallback(a, L_in);
   if (L.variant == FP_VAR_CSR_COLSPLIT) {
     FP_REQUIRE(a.split && a.split->soff && a.split->cs == L.cluster, FP_ERR_UNSUPPORTED,
                "fp_csr: variant %d (column split) runs from a CSR plan (fp_csr_plan_create)", L.variant);

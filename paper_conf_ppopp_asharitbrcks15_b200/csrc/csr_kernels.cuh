@@ -364,6 +364,7 @@ using CsrKFn = void (*)(const CsrKArgs);
 #include "csr_colsplit.cuh"
 #include "csr_flat.cuh"
 #include "csr_owner.cuh"
+#include "csr_stream.cuh"
 namespace fp {
 
 // column-split cluster kernels (csr_colsplit.cuh): 512 threads, NB in {8, 16} register tiles
@@ -410,7 +411,21 @@ CsrKFn csr_pick_owner_n(int vs, int k) {
 
 // dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
 enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5, DMODE_OWNER4 = 6, DMODE_OWNER8 = 7,
-       DMODE_FLAT_FIXED = 9 };
+       DMODE_FLAT_FIXED = 9, DMODE_STREAM_SHARED = 10, DMODE_STREAM_FIXED = 11 };
+
+// stream kernels (csr_stream.cuh): (VS, K) as for CSR-vector; no row epilogues (YM 2)
+template <typename T, int YM, int MODE>
+CsrKFn csr_pick_stream(int vs, int k) {
+  if constexpr (YM == 2) {
+    return nullptr;
+  } else {
+#define FP_CSR_S(VS_, K_) \
+  if (vs == VS_ && k == K_) return k_csr_stream<T, VS_, K_, YM, MODE, kCsrBS>;
+    FP_CSR_S(2, 4) FP_CSR_S(4, 4) FP_CSR_S(8, 2) FP_CSR_S(16, 2) FP_CSR_S(32, 4)
+#undef FP_CSR_S
+    return nullptr;
+  }
+}
 
 template <typename T, int YM, int MODE>
 CsrKFn csr_pick_flat(int nb) {
@@ -449,6 +464,8 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case DMODE_FLAT_PRIVATE: return csr_pick_flat<T, YM, MODE_PRIVATE>(k);
     case DMODE_OWNER4: return csr_pick_owner_n<T, YM, 4>(vs, k);
     case DMODE_OWNER8: return csr_pick_owner_n<T, YM, 8>(vs, k);
+    case DMODE_STREAM_SHARED: return csr_pick_stream<T, YM, MODE_SHARED>(vs, k);
+    case DMODE_STREAM_FIXED: return csr_pick_stream<T, YM, MODE_FIXED>(vs, k);
     default: return nullptr;
   }
 }

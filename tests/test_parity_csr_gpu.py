@@ -267,3 +267,57 @@ def test_fixed_point_wide_dynamic_range(cuda_dev, dt, variant):
     L.variant, L.vs, L.tl, L.bs, L.grid = variant, 8 if variant == 11 else 32, 2 if variant == 11 else 4, 256, 148
     w = gpu_csr(cuda_dev, rp, ci, va, n, y, v, z, 1.0, 1.0, launch=L)
     assert_parity(w, ref, mag, DT[dt], f"fixed wide range variant={variant}")
+
+
+STREAM_VSK = [(2, 4), (4, 4), (8, 2), (16, 2), (32, 4)]
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("variant", [14, 15])
+@pytest.mark.parametrize("vsk", STREAM_VSK)
+@pytest.mark.parametrize("lengths", [("uniform", 0, 70), ("powerlaw", 2.5, 13.64), ("binomial", 0.01)])
+def test_csr_stream_bitexact(cuda_dev, dt, variant, vsk, lengths):
+    """Stream variants (csr_stream.cuh: cp.async two-stage row stream): batches that overflow
+    the stage (rows read from global), rows longer than VS*K, empty rows, an nnz that is not a
+    multiple of the 16-byte chunk (zero-filled tail), warps with no rows -- integer twins must
+    equal the oracle bit for bit, with and without y."""
+    m, n = 7001, 1000
+    rp, ci, va, y, v, z = make_csr(m, n, dt, lengths, seed=vsk[0] * 10 + vsk[1], kind="int_pm12")
+    vs, k = vsk
+    for yy, grid in ((y, 37), (None, 148), (y, 1)):
+        ref, _ = oracle.csr(m, n, rp, ci, va, yy, v, z, 1.0, 1.0)
+        L = fp.fp_launch()
+        L.variant, L.vs, L.tl, L.bs, L.grid = variant, vs, k, 256, grid
+        w = gpu_csr(cuda_dev, rp, ci, va, n, yy, v, z, 1.0, 1.0, launch=L)
+        assert_bitexact(w, ref, f"stream variant={variant} vs={vs} k={k} y={yy is not None} grid={grid}")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+def test_csr_stream_misaligned_falls_back(cuda_dev, dt):
+    """colidx / val not 16-byte aligned: variant 14 runs as variant 3 (same result)."""
+    m, n = 2000, 300
+    rp, ci, va, y, v, z = make_csr(m, n, dt, ("binomial", 0.05), seed=3, kind="int_pm12")
+    nnz = int(rp[-1])
+    ci2 = torch.cat([torch.zeros(1, dtype=ci.dtype), ci])
+    va2 = torch.cat([torch.zeros(1, dtype=va.dtype), va])
+    ref, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    dev = cuda_dev
+    ci_d, va_d = ci2.to(dev)[1:], va2.to(dev)[1:]
+    assert ci_d.data_ptr() % 16 != 0 and ci_d.numel() == nnz
+    L = fp.fp_launch()
+    L.variant, L.vs, L.tl, L.bs, L.grid = 14, 4, 4, 256, 64
+    w = fp.csr(rp.to(dev), ci_d, va_d, n, y.to(dev), v.to(dev), z.to(dev), 1.0, 1.0, launch=L)
+    assert_bitexact(w.cpu(), ref, "misaligned stream fallback")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("variant", [14, 15])
+def test_csr_stream_float_parity(cuda_dev, dt, variant):
+    """Full-precision C3-shaped inputs (scaled down): normwise tolerance of north_star."""
+    m, n = 200_000, 1000
+    rp, ci, va, y, v, z = make_csr(m, n, dt, ("binomial", 0.01), seed=9)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 0.75, -1.25)
+    L = fp.fp_launch()
+    L.variant, L.vs, L.tl, L.bs, L.grid = variant, 4, 4, 256, 0
+    w = gpu_csr(cuda_dev, rp, ci, va, n, y, v, z, 0.75, -1.25, launch=L)
+    assert_parity(w, ref, mag, DT[dt], f"stream float variant={variant}")
