@@ -77,19 +77,24 @@ struct Tron {
   cudaStream_t s;
   int64_t n, m;
   double* scal = nullptr;  // device scratch: [0..1] dots, [2] loss
-  std::vector<void*> bufs;
+  // vectors are carved from the per-stream library workspace (allocated once and reused; no
+  // per-solve cudaMallocAsync / cudaFreeAsync -- see drivers.cu cg_typed)
+  char* cursor = nullptr;
+  size_t left = 0;
+  static size_t bytes_for(int64_t len) { return ((size_t)(len > 0 ? len : 1) * sizeof(T) + 255) / 256 * 256; }
 
   T* alloc(int64_t len, fp_status* st) {
-    void* p = nullptr;
-    if (cudaMallocAsync(&p, (size_t)(len > 0 ? len : 1) * sizeof(T), s) != cudaSuccess) *st = FP_ERR_NOMEM;
-    bufs.push_back(p);
-    return (T*)p;
+    const size_t b = bytes_for(len);
+    if (b > left) {
+      *st = FP_ERR_NOMEM;
+      return nullptr;
+    }
+    T* p = (T*)cursor;
+    cursor += b;
+    left -= b;
+    return p;
   }
-  ~Tron() {
-    for (void* p : bufs) cudaFreeAsync(p, s);
-    if (scal) cudaFreeAsync(scal, s);
-    cudaStreamSynchronize(s);
-  }
+  ~Tron() { cudaStreamSynchronize(s); }
   fp_status fused(fp::PatternArgs a) {
     if (comm) a.add_beta_z = fp_comm_rank(comm) == 0;
     fp_status st = csr ? fp::run_csr(a, nullptr, s) : fp::run_dense(a, nullptr, s);
@@ -142,7 +147,14 @@ fp_status tron_typed(fp::PatternArgs base, bool csr, const void* labels, double 
   const double eta0 = 1e-4, eta1 = 0.25, eta2 = 0.75, sigma1 = 0.25, sigma2 = 0.5, sigma3 = 4.0;
   Tron<T> t{base, csr, labels, C, comm, s, base.n, base.m};
   fp_status st = FP_OK;
-  FP_CUDA(cudaMallocAsync((void**)&t.scal, 4 * sizeof(double), s));
+  {
+    const size_t need = 256 + 7 * Tron<T>::bytes_for(base.n) + 2 * Tron<T>::bytes_for(base.m);
+    fp::Workspace* ws = fp::workspace(s, 0, need);
+    if (!ws) return FP_ERR_NOMEM;
+    t.scal = (double*)ws->scratch;
+    t.cursor = (char*)ws->scratch + 256;
+    t.left = need - 256;
+  }
   const int64_t n = base.n, m = base.m;
   T* w = (T*)w_out;
   T *g = t.alloc(n, &st), *sv = t.alloc(n, &st), *r = t.alloc(n, &st), *d = t.alloc(n, &st), *Hd = t.alloc(n, &st);
