@@ -235,6 +235,8 @@ def run_gpu(args):
             forced.variant, forced.vs, forced.tl, forced.bs, forced.grid = var, vs, k, 256, g
             if var == 13:
                 forced.cluster = k
+            if var == 16:
+                forced.bs = 1024
         # the once-per-matrix analysis (fp_csr_plan_create: launch parameters, column split) is
         # outside the timed region, like the paper's amortised transpose; timed here
         torch.cuda.synchronize()
@@ -263,7 +265,7 @@ def run_gpu(args):
         # replicated over L2 (csr.cu l2_replicas: 8 copies while they take <= 16 MB), fold the
         # copies after it
         launches_per_step = 1
-        if plan.variant in (4, 7):
+        if plan.variant in (4, 7, 16):
             s_b = 8 if cfg["dtype"] == "f64" else 4
             nrep = int(os.environ.get("FP_L2_REPLICAS", "0")) or (8 if 8 * n * s_b <= (16 << 20) else 1)
             launches_per_step = 2 + (1 if nrep > 1 else 0)

@@ -29,7 +29,7 @@ STATUS = {0: "FP_OK", 1: "FP_ERR_INVALID_ARG", 2: "FP_ERR_UNSUPPORTED", 3: "FP_E
 VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2", 5: "csr_vector_private",
             6: "csr_flat_smem", 7: "csr_flat_l2", 8: "csr_flat_private", 9: "dense_cluster", 10: "csr_owner",
             11: "csr_vector_fixed", 12: "csr_flat_fixed", 13: "csr_colsplit_cluster",
-            14: "csr_stream_smem", 15: "csr_stream_fixed"}
+            14: "csr_stream_smem", 15: "csr_stream_fixed", 16: "csr_flat_l2_wide"}
 
 
 class FusedPatError(RuntimeError):

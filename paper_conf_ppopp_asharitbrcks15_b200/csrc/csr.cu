@@ -9,7 +9,8 @@ namespace fp {
 namespace {
 
 bool is_flat(int variant) {
-  return (variant >= FP_VAR_CSR_FLAT && variant <= FP_VAR_CSR_FLAT_PRIVATE) || variant == FP_VAR_CSR_FLAT_FIXED;
+  return (variant >= FP_VAR_CSR_FLAT && variant <= FP_VAR_CSR_FLAT_PRIVATE) || variant == FP_VAR_CSR_FLAT_FIXED ||
+         variant == FP_VAR_CSR_FLAT_L2_WIDE;
 }
 
 int mode_of(int variant) {
@@ -24,6 +25,7 @@ int mode_of(int variant) {
     case FP_VAR_CSR_FLAT_FIXED: return DMODE_FLAT_FIXED;
     case FP_VAR_CSR_STREAM: return DMODE_STREAM_SHARED;
     case FP_VAR_CSR_STREAM_FIXED: return DMODE_STREAM_FIXED;
+    case FP_VAR_CSR_FLAT_L2_WIDE: return DMODE_FLAT_L2_WIDE;
     default: return -1;
   }
 }
@@ -75,6 +77,20 @@ int l2_replicas(const PatternArgs& a) {
 
 bool y_in_smem_l2(const PatternArgs& a) { return a.y && (size_t)a.n * dtype_size(a.dtype) <= kYBudget; }
 
+// variant 16: shared memory of the 1024-thread CTA left for a y prefix: 227 KB minus the
+// static per-warp row sums (32 warps x 32 x s) and a little slack
+int64_t wide_y_entries(const PatternArgs& a) {
+  if (!a.y) return 0;
+  const size_t budget = 227 * 1024 - (size_t)(kWideBS / 32) * 32 * dtype_size(a.dtype) - 512;
+  const int64_t cap = (int64_t)(budget / dtype_size(a.dtype)) / 4 * 4;
+  return a.n < cap ? a.n : cap;
+}
+// entries of y the L2-path kernels stage in shared memory (CsrKArgs::y_in_smem)
+int l2_y_entries(const PatternArgs& a, int variant) {
+  if (variant == FP_VAR_CSR_FLAT_L2_WIDE) return (int)wide_y_entries(a);
+  return y_in_smem_l2(a) ? (int)a.n : 0;
+}
+
 size_t smem_for(const PatternArgs& a, int variant) {
   const size_t vb = (size_t)a.n * dtype_size(a.dtype);
   const size_t yb = a.y ? vb : 0;
@@ -89,6 +105,7 @@ size_t smem_for(const PatternArgs& a, int variant) {
     case FP_VAR_CSR_FLAT_FIXED: return (size_t)(a.y ? fix_y_bytes(a.n, (int)dtype_size(a.dtype)) : 0) + (size_t)a.n * 16;
     case FP_VAR_CSR_VECTOR_L2:
     case FP_VAR_CSR_FLAT_L2: return y_in_smem_l2(a) ? vb : 0;
+    case FP_VAR_CSR_FLAT_L2_WIDE: return (size_t)wide_y_entries(a) * dtype_size(a.dtype);
     case FP_VAR_CSR_STREAM:  // y (16-byte padded) + partial + two stages per warp
     case FP_VAR_CSR_STREAM_FIXED: {
       const size_t s = dtype_size(a.dtype);
@@ -151,6 +168,19 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   if (!is_flat(L.variant) && L.vs == 8) {
     L.vs = 4;
     L.tl = 4;
+  }
+  // Wide y on the L2 path: one 1024-thread CTA per SM with a y prefix in shared memory takes
+  // that share of the gathers off the L2 request stream, the bound of this path (C4: 18.5 ->
+  // 17.2 ms with 56 % of y staged).  Only when the prefix is a sizeable share of y; the
+  // decision depends on (n, dtype) only, so a CSR plan made without y picks the same.
+  if (L.variant == FP_VAR_CSR_FLAT_L2) {
+    PatternArgs ay = a;
+    ay.y = reinterpret_cast<const void*>(uintptr_t(256));
+    if (4 * wide_y_entries(ay) >= a.n) {
+      L.variant = FP_VAR_CSR_FLAT_L2_WIDE;
+      L.bs = kWideBS;
+      L.smem_bytes = (int)smem_for(a, L.variant);
+    }
   }
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
@@ -300,9 +330,12 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s
   }
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: launch plan (variant=%d vs=%d) has no kernel", L.variant, L.vs);
-  FP_REQUIRE(L.bs == kCsrBS, FP_ERR_UNSUPPORTED, "fp_csr: block size %d not supported", L.bs);
+  const int bs_need = L.variant == FP_VAR_CSR_FLAT_L2_WIDE ? kWideBS : kCsrBS;
+  FP_REQUIRE(L.bs == bs_need, FP_ERR_UNSUPPORTED, "fp_csr: block size %d not supported (variant %d runs %d)", L.bs,
+             L.variant, bs_need);
   FP_REQUIRE(L.grid >= 0, FP_ERR_INVALID_ARG, "fp_csr: grid must be >= 0 (0 = one resident wave)");
-  const bool l2 = L.variant == FP_VAR_CSR_VECTOR_L2 || L.variant == FP_VAR_CSR_FLAT_L2;
+  const bool l2 = L.variant == FP_VAR_CSR_VECTOR_L2 || L.variant == FP_VAR_CSR_FLAT_L2 ||
+                  L.variant == FP_VAR_CSR_FLAT_L2_WIDE;
   const size_t smem = smem_for(a, L.variant);
   FP_REQUIRE(smem <= 227 * 1024, FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs %zu B shared memory (n too large)",
              L.variant, smem);
@@ -317,7 +350,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s
     if (st != FP_OK) return st;
   }
   CsrKArgs k{a.m, a.n, a.nnz, a.rowptr, a.colidx, a.val, a.y, a.v, a.z, a.alpha, a.beta, a.w,
-             ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (l2 && y_in_smem_l2(a)) ? 1 : 0,
+             ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, l2 ? l2_y_entries(a, L.variant) : 0,
              {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}, phase_iters_for(a, L), ws->acc, nrep};
   if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // L2 path without y in shared memory: prefer the largest L1 so the random y gathers hit it

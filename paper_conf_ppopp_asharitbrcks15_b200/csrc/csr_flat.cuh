@@ -39,7 +39,14 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ T rsum[NW][32];
   T* y_s = reinterpret_cast<T*>(smem_raw);
-  const bool ysm = HAS_Y && (MODE != MODE_L2 || a.y_in_smem);
+  // y entries staged in shared memory: all of y on the smem-partial paths; on the L2 path the
+  // leading a.y_in_smem columns (all of y when it fits, a prefix for the 1024-thread variant 16)
+  // (a partial prefix only in the 1024-thread instantiation: the extra branch costs registers)
+  constexpr bool PARTIAL_Y = BS == 1024 && MODE == MODE_L2;
+  const int64_t ny_s = !HAS_Y ? 0
+                              : (MODE != MODE_L2 ? n
+                                                 : (a.y_in_smem >= n ? n : (PARTIAL_Y ? (int64_t)a.y_in_smem : 0)));
+  const bool ysm = ny_s == n && HAS_Y;
   T* w_s = y_s + (ysm ? n : 0);
   T* w_mine = MODE == MODE_PRIVATE ? w_s + (int64_t)warp * n : w_s;
   __shared__ int fix_e;
@@ -49,12 +56,14 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
     const int64_t nw_copies = MODE == MODE_PRIVATE ? NW : (MODE == MODE_SHARED ? 1 : 0);
     for (int64_t j = threadIdx.x; j < nw_copies * n; j += BS) w_s[j] = T(0);
     if constexpr (MODE == MODE_FIXED) fpd::fix_init<BS>(FA, n);
-    if (ysm)
-      for (int64_t j = threadIdx.x; j < n; j += BS) y_s[j] = y[j];
+    for (int64_t j = threadIdx.x; j < ny_s; j += BS) y_s[j] = y[j];
     __syncthreads();
   }
   const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
-  auto Y = [&](int c) -> T { return ysm ? y_s[c] : fpd::ld_keep(y + c); };
+  auto Y = [&](int c) -> T {
+    if constexpr (PARTIAL_Y) return ysm ? y_s[c] : (c < ny_s ? y_s[c] : fpd::ld_keep(y + c));
+    else return ysm ? y_s[c] : fpd::ld_keep(y + c);
+  };
   T* const wl2 = l2_target<T>(a);
   auto W_ADD = [&](int c, T val_) {
     if constexpr (MODE == MODE_SHARED) atomicAdd(w_s + c, val_);
@@ -165,22 +174,31 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
 
     T q = T(0);  // lane i: q of row rb + i
     if constexpr (HAS_Y) {
-      // all NB gathers of y issued before the first use: their L2 latencies overlap (a gather
-      // inside the reduction loop below serialised NB round trips per batch)
-      T yv[NB];
-      if (ysm) {
+      // fp32: all NB gathers of y issued before the first use (their latencies overlap; 8 more
+      // registers, still 64).  fp64: gathered inside the reduction loop -- hoisting costs 16
+      // registers there (64 -> 91, half the resident CTAs) and made K1 slower (45.7 -> 59 ms).
+      constexpr bool HOIST = sizeof(T) == 4;
+      T yv[HOIST ? NB : 1];
+      if constexpr (HOIST) {
+        if (ysm) {
 #pragma unroll
-        for (int j = 0; j < NB; ++j) yv[j] = y_s[cc[j]];
-      } else {
+          for (int j = 0; j < NB; ++j) yv[j] = y_s[cc[j]];
+        } else if (PARTIAL_Y && ny_s > 0) {
 #pragma unroll
-        for (int j = 0; j < NB; ++j) yv[j] = fpd::ld_keep(y + cc[j]);
+          for (int j = 0; j < NB; ++j) yv[j] = cc[j] < ny_s ? y_s[cc[j]] : fpd::ld_keep(y + cc[j]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < NB; ++j) yv[j] = fpd::ld_keep(y + cc[j]);
+        }
       }
       rsum[warp][lane] = T(0);
       __syncwarp();
 #pragma unroll
       for (int j = 0; j < NB; ++j) {
         const int pos = j * 32 + lane;
-        T s = pos < cnt ? xv[j] * yv[j] : T(0);  // Eq. (2) products
+        T s;  // Eq. (2) products
+        if constexpr (HOIST) s = pos < cnt ? xv[j] * yv[j] : T(0);
+        else s = pos < cnt ? xv[j] * Y(cc[j]) : T(0);
         // segmented reduction toward the segment head (lanes of a row are contiguous)
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {

@@ -44,7 +44,8 @@ struct CsrKArgs {
   unsigned long long* counter;
   int add_beta_z;
   int accumulate;
-  int y_in_smem;  // MODE_L2 only: stage y in shared memory (n*s bytes) for the gathers
+  int y_in_smem;  // MODE_L2 only: number of leading y entries staged in shared memory (0: none;
+                  // >= n: all -- the only case the CSR-vector kernel accepts)
   fpd::RowEpi epi;
   int phase_iters;  // owner-computes kernel: row-group iterations between queue drains
   // MODE_L2: the CTAs reduce into nrep copies of w (copy 0 = w, copies 1.. = wrep, stride n,
@@ -411,7 +412,8 @@ CsrKFn csr_pick_owner_n(int vs, int k) {
 
 // dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
 enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5, DMODE_OWNER4 = 6, DMODE_OWNER8 = 7,
-       DMODE_FLAT_FIXED = 9, DMODE_STREAM_SHARED = 10, DMODE_STREAM_FIXED = 11 };
+       DMODE_FLAT_FIXED = 9, DMODE_STREAM_SHARED = 10, DMODE_STREAM_FIXED = 11, DMODE_FLAT_L2_WIDE = 12 };
+constexpr int kWideBS = 1024;  // variant 16: one 1024-thread CTA per SM, a y prefix in shared memory
 
 // stream kernels (csr_stream.cuh): (VS, K) as for CSR-vector; no row epilogues (YM 2)
 template <typename T, int YM, int MODE>
@@ -466,6 +468,7 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case DMODE_OWNER8: return csr_pick_owner_n<T, YM, 8>(vs, k);
     case DMODE_STREAM_SHARED: return csr_pick_stream<T, YM, MODE_SHARED>(vs, k);
     case DMODE_STREAM_FIXED: return csr_pick_stream<T, YM, MODE_FIXED>(vs, k);
+    case DMODE_FLAT_L2_WIDE: return k == 8 ? k_csr_flat<T, 8, YM, MODE_L2, kWideBS> : nullptr;
     default: return nullptr;
   }
 }

@@ -48,14 +48,15 @@ def run_plan(dev, rp, ci, va, n, args, launch=None):
 
 @pytest.mark.parametrize("dt", ["f32", "f64"])
 def test_c4_shape_chooser_plan(cuda_dev, dt):
-    """C4 shape scaled to the oracle (power-law rows, n = 1e5): the chooser's plan (flat + L2)
+    """C4 shape scaled to the oracle (power-law rows, n = 1e5): the chooser's plan (flat + L2,
+    1024-thread CTAs with a y prefix in shared memory)
     and, for fp32, the forced column split (y and w blocks of 25K columns in 4 CTAs; fp64 at
     this n does not fit a cluster) -- both within the north_star tolerance."""
     m, n = 20000, 100000
     rp, ci, va, y, v, z = make(m, n, dt, ("powerlaw", 2.5, 13.64), seed=404)
     ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
     P, w = run_plan(cuda_dev, rp, ci, va, n, (y, v, z, 1.0, 1.0))
-    assert P.launch.variant == 7
+    assert P.launch.variant == 16 and P.launch.bs == 1024
     assert_parity(w, ref, mag, DT[dt], "C4-shape chooser plan")
     if dt == "f32":
         P, w = run_plan(cuda_dev, rp, ci, va, n, (y, v, z, 1.0, 1.0), launch=forced(4))

@@ -170,7 +170,8 @@ def test_csr_plan_c3_c4(cuda_dev):
     st.m, st.n, st.nnz = 50_000_000, 100_000, 2_000_000_000
     st.mean = 40.0
     L = fp.choose(True, st, fp.FP_F32, 0)
-    assert L.variant == 7 and L.tl == 8   # flat layout, L2 reds (large n)
+    # flat layout, L2 reds (large n), as one 1024-thread CTA per SM with 56 % of y in smem
+    assert L.variant == 16 and L.tl == 8 and L.bs == 1024
 
 
 @pytest.mark.parametrize("dt", ["f64", "f32"])
@@ -321,3 +322,19 @@ def test_csr_stream_float_parity(cuda_dev, dt, variant):
     L.variant, L.vs, L.tl, L.bs, L.grid = variant, 4, 4, 256, 0
     w = gpu_csr(cuda_dev, rp, ci, va, n, y, v, z, 0.75, -1.25, launch=L)
     assert_parity(w, ref, mag, DT[dt], f"stream float variant={variant}")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("n", [1000, 60_000, 120_000])
+def test_csr_flat_l2_wide_bitexact(cuda_dev, dt, n):
+    """Variant 16 (1024-thread flat CTA, reds into L2, a y prefix of ~220 KB in shared memory):
+    y fully staged (n = 1000), partly staged (fp32 n = 60K fits, fp64 does not; n = 120K
+    splits both) -- integer twins bit-exact, with and without y."""
+    m = 20_000
+    rp, ci, va, y, v, z = make_csr(m, n, dt, ("powerlaw", 2.5, 13.64), seed=n % 97, kind="int_pm12")
+    for yy in (y, None):
+        ref, _ = oracle.csr(m, n, rp, ci, va, yy, v, z, 1.0, -1.0)
+        L = fp.fp_launch()
+        L.variant, L.vs, L.tl, L.bs, L.grid = 16, 32, 8, 1024, 0
+        w = gpu_csr(cuda_dev, rp, ci, va, n, yy, v, z, 1.0, -1.0, launch=L)
+        assert_bitexact(w, ref, f"wide flat n={n} y={yy is not None}")
