@@ -42,8 +42,17 @@ struct DenseKArgs {
 
 // Warp-granular vector kernel: VS in {1,2,4,8,16,32} lanes per row, NCH chunks of E
 // elements per lane (thread load TL = NCH*E), RPV rows per vector per iteration.
+#ifndef FP_DENSE_PF
+#define FP_DENSE_PF 0
+#endif
+#ifndef FP_DENSE_MINB
+#define FP_DENSE_MINB 1
+#endif
+#ifndef FP_DENSE_RPV32
+#define FP_DENSE_RPV32 4
+#endif
 template <typename T, int VS, int NCH, int E, int RPV, int YM, int BS>
-__global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
+__global__ void __launch_bounds__(BS, FP_DENSE_MINB) k_dense_vector(const DenseKArgs a) {
   constexpr int VPW = 32 / VS;       // vectors per warp
   constexpr int NW = BS / 32;        // warps per CTA
   constexpr int RPW = VPW * RPV;     // rows per warp iteration
@@ -67,10 +76,8 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
 
   const int64_t nwarps = (int64_t)gridDim.x * NW;
   double loss_acc = 0.0;  // logistic epilogue only
-  for (int64_t base = ((int64_t)blockIdx.x * NW + warp) * RPW; base < m; base += nwarps * RPW) {
-    T x[RPV][NCH][E];
-    T vr[RPV];
-    bool okr[RPV];
+  // rows [base + vid*RPV, +RPV) of this vector: x into registers (first and only HBM touch)
+  auto LOAD = [&](int64_t base, T (&x)[RPV][NCH][E], T (&vr)[RPV], bool (&okr)[RPV]) {
 #pragma unroll
     for (int i = 0; i < RPV; ++i) {
       const int64_t row = base + vid * RPV + i;
@@ -92,6 +99,26 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
         }
       }
     }
+  };
+  // PF: the next iteration's rows are loaded before this iteration's are reduced (the loads
+  // stay in flight through the shuffles).  Build switch for measurement only: on C2 it is
+  // slower at every occupancy tried (RPV 2 + PF: 0.726 ms at 3 CTAs/SM, 0.794 ms at 2, 0.96 ms
+  // at 4 with spills; RPV 4 + PF: 0.872 ms at 1) than the default (RPV 4, no PF: 0.717 ms).
+  // FP_DENSE_MINB / FP_DENSE_RPV32 are the matching occupancy / rows-in-flight switches.
+  constexpr bool PF = FP_DENSE_PF != 0;
+  T x[RPV][NCH][E], xn[PF ? RPV : 1][NCH][E];
+  T vr[RPV], vrn[PF ? RPV : 1];
+  bool okr[RPV], okrn[PF ? RPV : 1];
+  const int64_t base0 = ((int64_t)blockIdx.x * NW + warp) * RPW;
+  if constexpr (PF) {
+    if (base0 < m) LOAD(base0, x, vr, okr);
+  }
+  for (int64_t base = base0; base < m; base += nwarps * RPW) {
+    if constexpr (PF) {
+      if (base + nwarps * RPW < m) LOAD(base + nwarps * RPW, xn, vrn, okrn);
+    } else {
+      LOAD(base, x, vr, okr);
+    }
 #pragma unroll
     for (int i = 0; i < RPV; ++i) {
       T q;
@@ -112,6 +139,17 @@ __global__ void __launch_bounds__(BS) k_dense_vector(const DenseKArgs a) {
       for (int k = 0; k < NCH; ++k)  // Eq. (3): l_w += X[r,:]^T q, same registers
 #pragma unroll
         for (int e = 0; e < E; ++e) lw[k][e] = fma(x[i][k][e], q, lw[k][e]);
+    }
+    if constexpr (PF) {
+#pragma unroll
+      for (int i = 0; i < RPV; ++i) {
+        vr[i] = vrn[i];
+        okr[i] = okrn[i];
+#pragma unroll
+        for (int k = 0; k < NCH; ++k)
+#pragma unroll
+          for (int e = 0; e < E; ++e) x[i][k][e] = xn[i][k][e];
+      }
     }
   }
 
@@ -234,7 +272,7 @@ constexpr int kBS = 256;     // vector-kernel block size
 constexpr int kBSCta = 256;  // CTA-kernel block size
 using DenseKFn = void (*)(const DenseKArgs);
 
-constexpr int rpv_for(int nch, int eb) { return nch * eb <= 32 ? 4 : (nch * eb <= 64 ? 2 : 1); }
+constexpr int rpv_for(int nch, int eb) { return nch * eb <= 32 ? FP_DENSE_RPV32 : (nch * eb <= 64 ? 2 : 1); }
 
 template <typename T, int VS, int NCH, int E, int YM>
 DenseKFn vec_k() {
