@@ -51,3 +51,14 @@ for vs in (4, 8, 16, 32):
             print(f"vs={vs} tl={tl} grid={grid}: {ms:.4f} ms  rel {rel:.1e}")
         except fp.FusedPatError as e:
             print(f"vs={vs} tl={tl} grid={grid}: {str(e)[:70]}")
+for tl in (4, 8, 16, 32):
+    for grid in (148, 296, 592, 888, 1184):
+        L = fp.fp_launch()
+        L.variant, L.vs, L.tl, L.bs, L.grid = 2, 256, tl, 256, grid
+        try:
+            ms = t(L)
+            w = inp["w"].double().cpu().numpy()
+            rel = np.linalg.norm(w - ref) / np.linalg.norm(ref)
+            print(f"CTA variant tl={tl} grid={grid}: {ms:.4f} ms  rel {rel:.1e}")
+        except fp.FusedPatError as e:
+            print(f"CTA variant tl={tl} grid={grid}: {str(e)[:70]}")
