@@ -1,7 +1,9 @@
 #!/usr/bin/env python
 """Small-shape driver for compute-sanitizer (memcheck / racecheck / synccheck): every kernel
-family once -- dense vector / CTA / cluster, CSR vector (3 modes) and flat (3 modes), the row
-epilogues, CG and TRON drivers -- on tiny inputs.
+family once -- dense vector / CTA / cluster, CSR vector (shared / L2 / private / owner /
+fixed-point / cp.async stream), flat (shared / L2 / private / fixed / 1024-thread with a y
+prefix), the L2-replica fold, the column-split plan, the row epilogues, CG and TRON drivers --
+on tiny inputs.
 
   compute-sanitizer --tool memcheck python tools/sanitize.py
 """
@@ -33,10 +35,23 @@ def main():
         y = synth.vector(700, dt, seed=2, device=dev)
         v = synth.vector(2000, dt, kind="pos", seed=2, stream=synth.S_V, device=dev)
         z = synth.vector(700, dt, seed=2, stream=synth.S_Z, device=dev)
-        for var, vs, tl in ((3, 8, 2), (4, 32, 4), (5, 8, 2), (6, 32, 4), (7, 32, 8), (8, 32, 2)):
+        for var, vs, tl in ((3, 8, 2), (3, 4, 4), (4, 32, 4), (5, 8, 2), (6, 32, 4), (7, 32, 8), (8, 32, 2),
+                            (10, 8, 2), (11, 4, 4), (12, 32, 4), (14, 4, 4), (15, 4, 4), (16, 32, 8)):
             L = fp.fp_launch()
-            L.variant, L.vs, L.tl, L.bs, L.grid = var, vs, tl, 256, 13
-            fp.csr(rp, ci, va, 700, y, v, z, 1.0, 1.0, launch=L)
+            L.variant, L.vs, L.tl, L.bs, L.grid = var, vs, tl, 1024 if var == 16 else 256, 13
+            fp.csr(rp, ci, va, 700, y, v, z, 1.0, 1.0, launch=L)  # 4/7/16: w replicated over L2, folded
+        # variant 16 with a partial y prefix in shared memory (n beyond the ~56K / 28K staged)
+        nw = 60000 if dt == "f32" else 30000
+        rpw, ciw, vaw = synth.csr(500, nw, dt, ("powerlaw", 2.0, 3.0), seed=5, device=dev)
+        yw = synth.vector(nw, dt, seed=5, device=dev)
+        L = fp.fp_launch()
+        L.variant, L.vs, L.tl, L.bs, L.grid = 16, 32, 8, 1024, 7
+        fp.csr(rpw, ciw, vaw, nw, yw, None, yw, 1.0, 1.0, launch=L)
+        # CSR plan with the column split of variant 13 (cluster of 2)
+        F = fp.fp_launch()
+        F.variant, F.cluster = 13, 2
+        P = fp.CsrPlan(rp, ci, 700, va.dtype, launch=F)
+        P(va, y, v, z, 1.0, 1.0)
         lab = torch.where(synth.vector(2000, dt, seed=3, device=dev) > 0, 1.0, -1.0).to(va.dtype)
         D = torch.empty(2000, dtype=va.dtype, device=dev)
         loss = torch.zeros(1, dtype=torch.float64, device=dev)
