@@ -1,6 +1,17 @@
-// csr_f64.cu -- double instantiations of the CSR kernels (csr_kernels.cuh).
+// csr_f64.cu -- double dispatch of the CSR kernels (csr_kernels.cuh); the instantiations live in
+// csr_f64_y{0,1,2}.cu, one translation unit per y mode so that they compile in parallel.
 #include "csr_kernels.cuh"
 
 namespace fp {
-CsrKFn csr_pick_f64(int ym, int mode, int vs, int k) { return csr_pick_t<double>(ym, mode, vs, k); }
+CsrKFn csr_pick_f64_y0(int mode, int vs, int k);
+CsrKFn csr_pick_f64_y1(int mode, int vs, int k);
+CsrKFn csr_pick_f64_y2(int mode, int vs, int k);
+CsrKFn csr_pick_f64(int ym, int mode, int vs, int k) {
+  switch (ym) {
+    case 0: return csr_pick_f64_y0(mode, vs, k);
+    case 1: return csr_pick_f64_y1(mode, vs, k);
+    case 2: return csr_pick_f64_y2(mode, vs, k);
+    default: return nullptr;
+  }
+}
 }  // namespace fp

@@ -213,12 +213,12 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
       }
       const T p = rsum[warp][lane];
       const int64_t row = rb + lane;
+      (void)row;
       const bool ok = lane < nrows;
       const T vr = ok ? vpre : T(0);
       if constexpr (YM == 2) q = fpd::row_epilogue<T>(p, vr, ok, row, ok, a.epi, loss_acc) * qscale;
       else q = ok ? p * vr * qscale : T(0);
     } else {
-      const int64_t row = rb + lane;
       q = lane < nrows ? vpre * qscale : T(0);
     }
 

@@ -109,6 +109,9 @@ __global__ void __launch_bounds__(BS, FP_DENSE_MINB) k_dense_vector(const DenseK
   T x[RPV][NCH][E], xn[PF ? RPV : 1][NCH][E];
   T vr[RPV], vrn[PF ? RPV : 1];
   bool okr[RPV], okrn[PF ? RPV : 1];
+  (void)xn;
+  (void)vrn;
+  (void)okrn;
   const int64_t base0 = ((int64_t)blockIdx.x * NW + warp) * RPW;
   if constexpr (PF) {
     if (base0 < m) LOAD(base0, x, vr, okr);
