@@ -40,6 +40,9 @@ FALLBACK_HBM_GBS = 6650.0
 
 
 # ------------------------------------------------------------------------------ helpers
+READ_CEILING_GBS = 7371.0  # measured pure HBM read stream, best setting (profiles/r01_read_ceiling.md)
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -352,6 +355,10 @@ def run_gpu(args):
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": traffic_for(name),
             "peak_source": peak_src,
+            # the copy peak counts read + write bytes of b.copy_(a); a read-only stream goes
+            # further on this part (tools/microbench/read_bw.cu, profiles/r01_read_ceiling.md)
+            "read_ceiling_gbs": READ_CEILING_GBS,
+            "frac_of_read_ceiling": round(achieved / READ_CEILING_GBS, 4),
             "note": ("achieved = algorithmic bytes of one fp_* call (SURVEY 8(d): X once + rowptr + v + y + z + w) "
                      "/ mean CUDA-event duration of that call on its launch stream")}
 
