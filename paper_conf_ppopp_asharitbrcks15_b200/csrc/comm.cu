@@ -81,7 +81,9 @@ int fp_comm_size(const fp_comm* comm) { return comm ? comm->size : -1; }
 fp_status fp_allreduce(fp_comm* comm, void* buf, int64_t n, fp_dtype dtype, fp_stream stream) {
   FP_REQUIRE(comm && fp::valid_dtype(dtype) && n >= 0 && (n == 0 || buf), FP_ERR_INVALID_ARG,
              "fp_allreduce: bad arguments");
-  if (n == 0 || comm->size == 1) return FP_OK;
+  // no short cut for one rank: the collective runs (a copy in place) so that every *_dist call
+  // exercises the same NCCL path at any world size
+  if (n == 0) return FP_OK;
   FP_NCCL(ncclAllReduce(buf, buf, (size_t)n, dtype == FP_F64 ? ncclFloat64 : ncclFloat32, ncclSum, comm->nccl,
                         (cudaStream_t)stream));
   return FP_OK;

@@ -4,6 +4,7 @@
 
 #include <map>
 #include <mutex>
+#include <set>
 #include <utility>
 #include <vector>
 
@@ -59,70 +60,160 @@ const DeviceInfo& device_info(int ordinal) {
 }
 
 // ---------------------------------------------------------------------------- workspace
+// Keyed by (device, stream, capture id).  A call made while `s` is being captured into a CUDA
+// graph gets a workspace of its own (capture id != 0) that is never regrown or freed while the
+// library is loaded: the graph keeps the pointers baked into its kernel nodes, and two graphs
+// -- or a graph and direct calls on the capture stream -- never share accumulators/tickets.
+// Buffers replaced by a larger allocation are retired (freed only by release_all_workspaces),
+// so a pointer handed to a launch another host thread has not enqueued yet stays valid.
 namespace {
 std::mutex g_ws_mu;
-std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+struct WsKey {
+  int dev;
+  cudaStream_t s;
+  unsigned long long cap;
+  bool operator<(const WsKey& o) const {
+    if (dev != o.dev) return dev < o.dev;
+    if (s != o.s) return s < o.s;
+    return cap < o.cap;
+  }
+};
+std::map<WsKey, Workspace*> g_ws;
+std::vector<std::pair<int, void*>> g_retired;  // (device, pointer)
+std::map<int, cudaStream_t> g_init_stream;     // per device: zero-fills outside any capture
+
+unsigned long long capture_id(cudaStream_t s) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  unsigned long long id = 0;
+  if (cudaStreamGetCaptureInfo(s, &st, &id) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return st == cudaStreamCaptureStatusActive ? id : 0;
+}
+
+// cudaMalloc + zero fill that is legal while another stream of this thread is capturing
+// (relaxed capture mode for the allocation; the fill runs on a private stream and is waited
+// for, so it is never recorded into the graph)
+cudaError_t alloc_zeroed(void** p, size_t bytes, bool zero, int dev) {
+  cudaStreamCaptureMode mode = cudaStreamCaptureModeRelaxed;
+  cudaThreadExchangeStreamCaptureMode(&mode);
+  cudaError_t e = cudaMalloc(p, bytes);
+  if (e == cudaSuccess && zero) {
+    cudaStream_t& is = g_init_stream[dev];
+    if (!is) e = cudaStreamCreateWithFlags(&is, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaMemsetAsync(*p, 0, bytes, is);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(is);
+  }
+  cudaThreadExchangeStreamCaptureMode(&mode);
+  return e;
+}
+
+Workspace* get_ws(cudaStream_t s, int dev) {
+  Workspace*& ws = g_ws[WsKey{dev, s, capture_id(s)}];
+  if (!ws) ws = new Workspace();
+  return ws;
+}
+
+void retire(int dev, void* p) {
+  if (p) g_retired.emplace_back(dev, p);
+}
 }  // namespace
 
 Workspace* workspace(cudaStream_t s, size_t acc_elems, size_t scratch_bytes) {
   int dev = current_device();
   std::lock_guard<std::mutex> lk(g_ws_mu);
-  Workspace*& ws = g_ws[{dev, s}];
-  if (!ws) ws = new Workspace();
+  Workspace* ws = get_ws(s, dev);
   if (!ws->counters) {
-    if (cudaMalloc(&ws->counters, 4 * sizeof(unsigned long long)) != cudaSuccess) {
+    if (alloc_zeroed((void**)&ws->counters, 4 * sizeof(unsigned long long), true, dev) != cudaSuccess) {
+      ws->counters = nullptr;
       set_error("workspace: cudaMalloc(counters) failed");
       return nullptr;
     }
-    cudaMemsetAsync(ws->counters, 0, 4 * sizeof(unsigned long long), s);
   }
   if (acc_elems > ws->acc_cap) {
-    size_t cap = acc_elems < 4096 ? 4096 : acc_elems;
+    size_t cap = acc_elems < 4096 ? 4096 : acc_elems + acc_elems / 2;
     double* p = nullptr;
-    if (cudaMalloc(&p, cap * sizeof(double)) != cudaSuccess) {
+    if (alloc_zeroed((void**)&p, cap * sizeof(double), true, dev) != cudaSuccess) {
       set_error("workspace: cudaMalloc(acc, %zu doubles) failed", cap);
       return nullptr;
     }
-    cudaMemsetAsync(p, 0, cap * sizeof(double), s);
-    if (ws->acc) {
-      cudaStreamSynchronize(s);   // previous launches on s may still use the old buffer
-      cudaFree(ws->acc);
-    }
+    retire(dev, ws->acc);
     ws->acc = p;
     ws->acc_cap = cap;
   }
   if (scratch_bytes > ws->scratch_cap) {
     void* p = nullptr;
-    if (cudaMalloc(&p, scratch_bytes) != cudaSuccess) {
-      set_error("workspace: cudaMalloc(scratch, %zu B) failed", scratch_bytes);
+    const size_t cap = scratch_bytes + scratch_bytes / 2;
+    if (alloc_zeroed(&p, cap, false, dev) != cudaSuccess) {
+      set_error("workspace: cudaMalloc(scratch, %zu B) failed", cap);
       return nullptr;
     }
-    if (ws->scratch) {
-      cudaStreamSynchronize(s);
-      cudaFree(ws->scratch);
-    }
+    retire(dev, ws->scratch);
     ws->scratch = p;
-    ws->scratch_cap = scratch_bytes;
+    ws->scratch_cap = cap;
   }
   return ws;
+}
+
+void* workspace_buffer(cudaStream_t s, int slot, size_t bytes, bool zero) {
+  int dev = current_device();
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  Workspace* ws = get_ws(s, dev);
+  if (slot < 0 || slot >= kWsSlots) return nullptr;
+  if (bytes > ws->buf_cap[slot]) {
+    void* p = nullptr;
+    const size_t cap = bytes + bytes / 8;
+    if (alloc_zeroed(&p, cap, zero, dev) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("workspace: cudaMalloc(%zu B) failed", cap);
+      return nullptr;
+    }
+    retire(dev, ws->buf[slot]);
+    ws->buf[slot] = p;
+    ws->buf_cap[slot] = cap;
+  }
+  return ws->buf[slot];
 }
 
 void release_all_workspaces() {
   std::lock_guard<std::mutex> lk(g_ws_mu);
   int prev = current_device();
   for (auto& kv : g_ws) {
-    cudaSetDevice(kv.first.first);
+    cudaSetDevice(kv.first.dev);
     cudaDeviceSynchronize();
     Workspace* ws = kv.second;
     if (ws) {
       cudaFree(ws->acc);
       cudaFree(ws->counters);
       cudaFree(ws->scratch);
+      for (int i = 0; i < kWsSlots; ++i) cudaFree(ws->buf[i]);
       delete ws;
     }
   }
   g_ws.clear();
+  for (auto& r : g_retired) {
+    cudaSetDevice(r.first);
+    cudaDeviceSynchronize();
+    cudaFree(r.second);
+  }
+  g_retired.clear();
   cudaSetDevice(prev);
+}
+
+// The dynamic shared-memory cap of a kernel is raised once to the per-block maximum instead of
+// per call to the call's size: a concurrent call with a smaller size can no longer lower it
+// between another thread's set and launch.  (The cap does not change occupancy; the launch's
+// actual size does.)
+void set_max_dynamic_smem(const void* f) {
+  static std::mutex mu;
+  static std::set<const void*> done;
+  std::lock_guard<std::mutex> lk(mu);
+  if (done.count(f)) return;
+  const int dev = current_device();
+  const int cap = (int)device_info(dev).smem_optin_per_block;
+  if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, cap) == cudaSuccess) done.insert(f);
+  else cudaGetLastError();
 }
 
 }  // namespace fp

@@ -45,17 +45,27 @@ int current_device();
 // One per (device, stream).  acc: fp64 grid accumulator, ALWAYS all-zero between launches
 // (the finalising CTA re-zeroes what it consumed).  counters: [0] CTA-done ticket,
 // [1] dynamic row-chunk counter; both reset to 0 by the finalising CTA.
+// Extra per-workspace buffers (workspace_buffer slots).
+enum { kWsBins = 0, kWsBinsZero = 1, kWsSlots = 4 };
 struct Workspace {
   double* acc = nullptr;
   size_t acc_cap = 0;          // elements
   unsigned long long* counters = nullptr;
   void* scratch = nullptr;     // general device scratch (row stats, CG scalars)
   size_t scratch_cap = 0;      // bytes
+  void* buf[kWsSlots] = {};    // kWsBins: variant-17 messages; kWsBinsZero: its all-zero vectors
+  size_t buf_cap[kWsSlots] = {};
 };
-// Returns nullptr (and sets the error) on allocation failure.  Growing reallocates, which
-// synchronises the device; steady-state calls never allocate.
+// Returns nullptr (and sets the error) on allocation failure.  Growing allocates a larger
+// buffer and retires the old one (freed by release_all_workspaces); steady-state calls never
+// allocate.  Calls made while the stream is being captured get their own workspace.
 Workspace* workspace(cudaStream_t s, size_t acc_elems, size_t scratch_bytes);
+// Slot `slot` of the (device, stream[, capture]) workspace with at least `bytes`; a new
+// allocation is zero-filled when `zero` (callers that need an all-zero invariant keep it).
+void* workspace_buffer(cudaStream_t s, int slot, size_t bytes, bool zero);
 void release_all_workspaces();
+// cudaFuncAttributeMaxDynamicSharedMemorySize = the device's per-block maximum, once per kernel
+void set_max_dynamic_smem(const void* f);
 
 // ---------------------------------------------------------------------------- helpers
 inline size_t dtype_size(fp_dtype t) { return t == FP_F64 ? 8 : 4; }

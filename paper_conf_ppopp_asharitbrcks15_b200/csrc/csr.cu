@@ -10,7 +10,7 @@ namespace {
 
 bool is_flat(int variant) {
   return (variant >= FP_VAR_CSR_FLAT && variant <= FP_VAR_CSR_FLAT_PRIVATE) || variant == FP_VAR_CSR_FLAT_FIXED ||
-         variant == FP_VAR_CSR_FLAT_L2_WIDE;
+         variant == FP_VAR_CSR_FLAT_L2_WIDE || variant == FP_VAR_CSR_BINNED;
 }
 
 int mode_of(int variant) {
@@ -35,6 +35,10 @@ int default_k(int vs) { return (vs == 8 || vs == 16) ? 2 : (vs == 32 ? 4 : 4); }
 
 CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   int mode = mode_of(L.variant);
+  if (L.variant == FP_VAR_CSR_BINNED) {
+    const int nb = L.cluster > 0 ? L.cluster : binned_nbin(a.n);
+    mode = nb == 1 ? DMODE_BIN1 : (nb == 2 ? DMODE_BIN2 : (nb == 4 ? DMODE_BIN4 : -1));
+  }
   if (L.variant == FP_VAR_CSR_OWNER) mode = a.n <= 4 * kCsrBS ? DMODE_OWNER4 : (a.n <= 8 * kCsrBS ? DMODE_OWNER8 : -1);
   if (mode < 0) return nullptr;
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
@@ -46,6 +50,7 @@ CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
 constexpr size_t kPrivateBudget = 100 * 1024;  // y + NW warp partials per CTA
 constexpr size_t kSharedBudget = 64 * 1024;    // y + one CTA partial
 constexpr size_t kYBudget = 96 * 1024;         // y staged in smem on the L2 path
+constexpr int64_t kBinMinNnz = 1 << 24;         // variant 17 only from 16M nonzeros
 
 // w += sum of the replicas; the replicas are re-zeroed (the workspace invariant)
 template <typename T>
@@ -105,7 +110,8 @@ size_t smem_for(const PatternArgs& a, int variant) {
     case FP_VAR_CSR_FLAT_FIXED: return (size_t)(a.y ? fix_y_bytes(a.n, (int)dtype_size(a.dtype)) : 0) + (size_t)a.n * 16;
     case FP_VAR_CSR_VECTOR_L2:
     case FP_VAR_CSR_FLAT_L2: return y_in_smem_l2(a) ? vb : 0;
-    case FP_VAR_CSR_FLAT_L2_WIDE: return (size_t)wide_y_entries(a) * dtype_size(a.dtype);
+    case FP_VAR_CSR_FLAT_L2_WIDE:
+    case FP_VAR_CSR_BINNED: return (size_t)wide_y_entries(a) * dtype_size(a.dtype);
     case FP_VAR_CSR_STREAM:  // y (16-byte padded) + partial + two stages per warp
     case FP_VAR_CSR_STREAM_FIXED: {
       const size_t s = dtype_size(a.dtype);
@@ -182,9 +188,37 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
       L.smem_bytes = (int)smem_for(a, L.variant);
     }
   }
+  // Binned scatter (variant 17, csr_binned.cu): for fp32 and n up to 4 column blocks of one
+  // SM's shared memory, when the matrix is large enough that the ~4 extra launches and the
+  // message round trip (6 B per nonzero written and read) are repaid by removing the per-lane
+  // global reds, and the message workspace fits in free device memory with 1 GB to spare.
+  // FP_NO_BINNED=1 keeps variant 16 (A/B measurement).
+  if (L.variant == FP_VAR_CSR_FLAT_L2_WIDE && a.dtype == FP_F32 && binned_nbin(a.n) > 0 && a.nnz >= kBinMinNnz &&
+      !std::getenv("FP_NO_BINNED")) {
+    const int nb = binned_nbin(a.n);
+    size_t fr = 0, tot = 0;
+    const size_t need = binned_ws_bytes(a.n, a.nnz, nb, di.sm_count, di.sm_count);
+    if (cudaMemGetInfo(&fr, &tot) == cudaSuccess && need + (1ull << 30) <= fr) {
+      L.variant = FP_VAR_CSR_BINNED;
+      L.cluster = nb;
+    } else {
+      cudaGetLastError();
+    }
+  }
   CsrKFn f = pick_any(a, L);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
-  if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
+  set_max_dynamic_smem((const void*)f);
+  if (L.variant == FP_VAR_CSR_BINNED) {  // one producer CTA per SM (the plan of variant 16)
+    cudaFuncAttributes fa{};
+    cudaFuncGetAttributes(&fa, f);
+    L.regs_per_thread = fa.numRegs;
+    L.blocks_per_sm = 1;
+    L.concurrent_warps = L.bs / 32;
+    L.grid = di.sm_count;
+    L.rows_per_vector = (a.m + (int64_t)L.grid * 32 - 1) / ((int64_t)L.grid * 32);
+    *out = L;
+    return FP_OK;
+  }
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, L.bs, L.smem_bytes);
   if (per_sm < 1) per_sm = 1;
@@ -239,10 +273,7 @@ int split_capacity(const PatternArgs& a, const CsrSplit& sp, int nb) {
   if (!f) return 0;
   const size_t smem = colsplit_smem(a.dtype, sp.cs, sp.width, a.y != nullptr);
   if (smem > 227 * 1024) return 0;
-  if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
-    cudaGetLastError();
-    return 0;
-  }
+  set_max_dynamic_smem((const void*)f);
   cudaLaunchAttribute attr[1];
   cudaLaunchConfig_t cfg = split_config(a, sp, sp.cs * 64, attr, 0);
   int n = 0;
@@ -304,6 +335,7 @@ fp_launch stream_fallback(const PatternArgs& a, const fp_launch& L) {
 
 fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s) {
   const fp_launch L = stream_fallback(a, L_in);
+  if (L.variant == FP_VAR_CSR_BINNED) return launch_binned(a, L, wide_y_entries(a), s);
   if (L.variant == FP_VAR_CSR_COLSPLIT) {
     FP_REQUIRE(a.split && a.split->soff && a.split->cs == L.cluster, FP_ERR_UNSUPPORTED,
                "fp_csr: variant %d (column split) runs from a CSR plan (fp_csr_plan_create)", L.variant);
@@ -322,7 +354,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s
     for (int i = 0; i <= kSplitMaxCS; ++i) k.cb[i] = sp.cb[i];
     k.width = sp.width;
     const size_t smem = colsplit_smem(a.dtype, sp.cs, sp.width, a.y != nullptr);
-    FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    set_max_dynamic_smem((const void*)f);
     cudaLaunchAttribute attr[1];
     cudaLaunchConfig_t cfg = split_config(a, sp, L.grid, attr, s);
     FP_CUDA(cudaLaunchKernelEx(&cfg, f, k));
@@ -352,7 +384,7 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s
   CsrKArgs k{a.m, a.n, a.nnz, a.rowptr, a.colidx, a.val, a.y, a.v, a.z, a.alpha, a.beta, a.w,
              ws->acc, ws->counters, a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, l2 ? l2_y_entries(a, L.variant) : 0,
              {a.epi_kind, a.epi_c, a.row_out, a.scalar_out}, phase_iters_for(a, L), ws->acc, nrep};
-  if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  set_max_dynamic_smem((const void*)f);
   // L2 path without y in shared memory: prefer the largest L1 so the random y gathers hit it
   // (X itself streams with L1::no_allocate and never displaces y)
   if (l2 && smem == 0) cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, 0);

@@ -95,10 +95,8 @@ int cluster_capacity(const PatternArgs& a, const fp_launch& C) {
   DenseKFn f = pick_any(a, C);
   if (!f) return 0;
   const int dsm = dense_smem_bytes(a, C);
-  if (dsm > 48 * 1024 && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm) != cudaSuccess) {
-    cudaGetLastError();
-    return 0;
-  }
+  if (dsm > (int)device_info(current_device()).smem_optin_per_block) return 0;
+  set_max_dynamic_smem((const void*)f);
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)(C.cluster * 64));
   cfg.blockDim = dim3((unsigned)C.bs);
@@ -228,7 +226,7 @@ fp_status plan_dense(const PatternArgs& a, int device, fp_launch* out) {
   }
   const bool clu = L.variant == FP_VAR_DENSE_CLUSTER;
   L.smem_bytes = dense_smem_bytes(a, L);
-  if (L.smem_bytes > 48 * 1024) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem_bytes);
+  set_max_dynamic_smem((const void*)f);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, L.bs, L.smem_bytes);
   if (per_sm < 1) per_sm = 1;
@@ -286,7 +284,7 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
     cfg.gridDim = dim3((unsigned)L.grid);
     cfg.blockDim = dim3((unsigned)L.bs);
     const int dsm = dense_smem_bytes(a, L);
-    if (dsm > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm));
+    set_max_dynamic_smem((const void*)f);
     cfg.dynamicSmemBytes = (size_t)dsm;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
@@ -300,7 +298,7 @@ fp_status launch_dense(const PatternArgs& a, const fp_launch& L, cudaStream_t s)
     return FP_OK;
   }
   const size_t smem = (size_t)a.n * sizeof(double);
-  if (smem > 48 * 1024) FP_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  set_max_dynamic_smem((const void*)f);
   f<<<L.grid, L.bs, smem, s>>>(k);
   FP_CUDA(cudaGetLastError());
   return FP_OK;

@@ -64,6 +64,11 @@ PatternArgs csr_args(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, c
                      const void* val, const void* y, const void* v, const void* z, double alpha, double beta, void* w,
                      fp_dtype dtype);
 
+// Variant 17 (csr_binned.cu): binned producer + fixed-point consumer + exact finalize.
+fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_prefix, cudaStream_t s);
+int binned_nbin(int64_t n);     // 1, 2 or 4 column blocks; 0 if n is too wide
+size_t binned_ws_bytes(int64_t n, int64_t nnz, int nbin, int producer_grid, int consumers);
+
 // w = beta*z (or 0): the alpha == 0 / m == 0 path, and the pre-initialisation of the L2 path.
 fp_status launch_scale_z(int64_t n, const void* z, double beta, void* w, fp_dtype dt, cudaStream_t s);
 

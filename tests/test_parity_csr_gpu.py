@@ -170,8 +170,9 @@ def test_csr_plan_c3_c4(cuda_dev):
     st.m, st.n, st.nnz = 50_000_000, 100_000, 2_000_000_000
     st.mean = 40.0
     L = fp.choose(True, st, fp.FP_F32, 0)
-    # flat layout, L2 reds (large n), as one 1024-thread CTA per SM with 56 % of y in smem
-    assert L.variant == 16 and L.tl == 8 and L.bs == 1024
+    # flat producer (one 1024-thread CTA per SM, 56 % of y in smem) writing column-block bins
+    # that a fixed-point shared-memory consumer reduces (variant 17, 2 bins of 50K columns)
+    assert L.variant == 17 and L.tl == 8 and L.bs == 1024 and L.cluster == 2
 
 
 @pytest.mark.parametrize("dt", ["f64", "f32"])
