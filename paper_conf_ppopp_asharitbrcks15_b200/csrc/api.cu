@@ -1,5 +1,7 @@
-// api.cu -- the C ABI entry points of fusedpat.h for the single-GPU pattern: argument
-// validation (every call), alias checks, the alpha == 0 / m == 0 path, plan + launch.
+// api.cu -- the C ABI entry points of fusedpat.h for the single-GPU pattern: argument checks
+// on every call (pointers, sizes, dtype, aliasing -- NOT the CSR structure, which
+// fp_csr_validate / fp_csr_plan_create check once per matrix), the alpha == 0 / m == 0 path,
+// plan + launch.
 #include <string.h>
 
 #include <array>

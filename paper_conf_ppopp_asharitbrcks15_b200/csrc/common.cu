@@ -211,7 +211,13 @@ void set_max_dynamic_smem(const void* f) {
   std::lock_guard<std::mutex> lk(mu);
   if (done.count(f)) return;
   const int dev = current_device();
-  const int cap = (int)device_info(dev).smem_optin_per_block;
+  cudaFuncAttributes fa{};
+  if (cudaFuncGetAttributes(&fa, f) != cudaSuccess) {
+    cudaGetLastError();
+    return;
+  }
+  // static + dynamic shared memory of a block must stay within the opt-in limit
+  const int cap = (int)device_info(dev).smem_optin_per_block - (int)fa.sharedSizeBytes;
   if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, cap) == cudaSuccess) done.insert(f);
   else cudaGetLastError();
 }

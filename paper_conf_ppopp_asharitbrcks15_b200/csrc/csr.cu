@@ -35,10 +35,6 @@ int default_k(int vs) { return (vs == 8 || vs == 16) ? 2 : (vs == 32 ? 4 : 4); }
 
 CsrKFn pick_any(const PatternArgs& a, const fp_launch& L) {
   int mode = mode_of(L.variant);
-  if (L.variant == FP_VAR_CSR_BINNED) {
-    const int nb = L.cluster > 0 ? L.cluster : binned_nbin(a.n);
-    mode = nb == 1 ? DMODE_BIN1 : (nb == 2 ? DMODE_BIN2 : (nb == 4 ? DMODE_BIN4 : -1));
-  }
   if (L.variant == FP_VAR_CSR_OWNER) mode = a.n <= 4 * kCsrBS ? DMODE_OWNER4 : (a.n <= 8 * kCsrBS ? DMODE_OWNER8 : -1);
   if (mode < 0) return nullptr;
   const int ym = !a.y ? 0 : ((a.epi_kind == 0 && !a.row_out) ? 1 : 2);
@@ -194,7 +190,7 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
   // global reds, and the message workspace fits in free device memory with 1 GB to spare.
   // FP_NO_BINNED=1 keeps variant 16 (A/B measurement).
   if (L.variant == FP_VAR_CSR_FLAT_L2_WIDE && a.dtype == FP_F32 && binned_nbin(a.n) > 0 && a.nnz >= kBinMinNnz &&
-      !std::getenv("FP_NO_BINNED")) {
+      a.epi_kind == 0 && !a.row_out && !std::getenv("FP_NO_BINNED")) {
     const int nb = binned_nbin(a.n);
     size_t fr = 0, tot = 0;
     const size_t need = binned_ws_bytes(a.n, a.nnz, nb, di.sm_count, di.sm_count);
@@ -205,13 +201,8 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
       cudaGetLastError();
     }
   }
-  CsrKFn f = pick_any(a, L);
-  FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
-  set_max_dynamic_smem((const void*)f);
-  if (L.variant == FP_VAR_CSR_BINNED) {  // one producer CTA per SM (the plan of variant 16)
-    cudaFuncAttributes fa{};
-    cudaFuncGetAttributes(&fa, f);
-    L.regs_per_thread = fa.numRegs;
+  if (L.variant == FP_VAR_CSR_BINNED) {  // one producer CTA of 1024 threads per SM
+    L.regs_per_thread = binned_producer_regs(a.y != nullptr);
     L.blocks_per_sm = 1;
     L.concurrent_warps = L.bs / 32;
     L.grid = di.sm_count;
@@ -219,6 +210,9 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
     *out = L;
     return FP_OK;
   }
+  CsrKFn f = pick_any(a, L);
+  FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr: no kernel for vs=%d", L.vs);
+  set_max_dynamic_smem((const void*)f);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, L.bs, L.smem_bytes);
   if (per_sm < 1) per_sm = 1;

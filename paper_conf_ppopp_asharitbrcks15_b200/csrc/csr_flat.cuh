@@ -22,13 +22,8 @@ namespace fp {
 
 template <typename T, int NB, int YM, int MODE, int BS>
 __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
-  static_assert(MODE == MODE_SHARED || MODE == MODE_L2 || MODE == MODE_PRIVATE || MODE == MODE_FIXED ||
-                    is_bin_mode(MODE),
+  static_assert(MODE == MODE_SHARED || MODE == MODE_L2 || MODE == MODE_PRIVATE || MODE == MODE_FIXED,
                 "flat kernel aggregation mode");
-  static_assert(!is_bin_mode(MODE) || sizeof(T) == 4, "binned messages are fp32");
-  // global-target modes: alpha folded into q, y staged as a prefix (variant 16 / 17)
-  constexpr bool GLOBAL_W = MODE == MODE_L2 || is_bin_mode(MODE);
-  constexpr int NBIN = is_bin_mode(MODE) ? 1 << (MODE - MODE_BIN1) : 1;
   constexpr int NW = BS / 32;
   constexpr int CAP = 32 * NB;  // nonzeros per batch
   const int64_t* __restrict__ rowptr = a.rowptr;
@@ -47,9 +42,9 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   // y entries staged in shared memory: all of y on the smem-partial paths; on the L2 path the
   // leading a.y_in_smem columns (all of y when it fits, a prefix for the 1024-thread variant 16)
   // (a partial prefix only in the 1024-thread instantiation: the extra branch costs registers)
-  constexpr bool PARTIAL_Y = BS == 1024 && GLOBAL_W;
+  constexpr bool PARTIAL_Y = BS == 1024 && MODE == MODE_L2;
   const int64_t ny_s = !HAS_Y ? 0
-                              : (!GLOBAL_W ? n
+                              : (MODE != MODE_L2 ? n
                                                  : (a.y_in_smem >= n ? n : (PARTIAL_Y ? (int64_t)a.y_in_smem : 0)));
   const bool ysm = ny_s == n && HAS_Y;
   T* w_s = y_s + (ysm ? n : 0);
@@ -64,7 +59,7 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
     for (int64_t j = threadIdx.x; j < ny_s; j += BS) y_s[j] = y[j];
     __syncthreads();
   }
-  const T qscale = GLOBAL_W ? (T)a.alpha : T(1);
+  const T qscale = MODE == MODE_L2 ? (T)a.alpha : T(1);
   auto Y = [&](int c) -> T {
     if constexpr (PARTIAL_Y) return ysm ? y_s[c] : (c < ny_s ? y_s[c] : fpd::ld_keep(y + c));
     else return ysm ? y_s[c] : fpd::ld_keep(y + c);
@@ -87,57 +82,8 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   };
   // one row's entries spread over the active lanes (long-row path): distinct columns when the
   // row is canonical; duplicates (R7) are serialised lane by lane
-  // ---- MODE_BIN*: message writer.  Warp-uniform state per bin: the open chunk cur[b] and its
-  // fill; new chunks come from the warp's own region (next), so no global atomics.  Called by
-  // all 32 lanes with one candidate term each.
-  int64_t cur[NBIN];
-  int fil[NBIN];
-  int64_t next = 0, wbase = 0;
-  float tmax = 0.f;  // largest finite |term| of this lane
-  auto BIN_APPEND = [&](int c, T t, bool act) {
-    if constexpr (is_bin_mode(MODE)) {
-      int b = 0;
-      if constexpr (NBIN > 1) {
-        b = __float2int_rz((float)c * a.inv_bw);
-        b += (b + 1) * a.bw <= c;
-        b -= b * a.bw > c;
-        b = b < NBIN - 1 ? b : NBIN - 1;
-      }
-      const int cl = c - b * a.bw;
-      if (act) {
-        const float at = fabsf((float)t);
-        if (at <= 3.402823466e38f) tmax = fmaxf(tmax, at);  // finite only (NaN fails the compare)
-      }
-      unsigned lt;
-      asm("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
-#pragma unroll
-      for (int k = 0; k < NBIN; ++k) {
-        const unsigned mk = __ballot_sync(0xffffffffu, act && b == k);
-        if (mk == 0) continue;
-        const int cnt = __popc(mk);
-        const int f = fil[k];
-        if (act && b == k) {
-          const int slot = f + __popc(mk & lt);
-          const int64_t chunk = slot < kBinCH ? cur[k] : next;
-          const int64_t pos = chunk * kBinCH + (slot < kBinCH ? slot : slot - kBinCH);
-          a.bcol[pos] = (uint16_t)cl;
-          a.bval[pos] = (float)t;
-        }
-        if (f + cnt >= kBinCH) {  // chunk full: publish it, open the next one of the region
-          if (lane == 0) a.bdir[cur[k]] = ((uint32_t)k << 16) | (uint32_t)kBinCH;
-          cur[k] = next;
-          ++next;
-          fil[k] = f + cnt - kBinCH;
-        } else {
-          fil[k] = f + cnt;
-        }
-      }
-    }
-  };
   auto ROW_ADD = [&](int c, T val_, bool act) {
-    if constexpr (is_bin_mode(MODE)) {
-      BIN_APPEND(c, val_, act);
-    } else if constexpr (MODE == MODE_PRIVATE) {
+    if constexpr (MODE == MODE_PRIVATE) {
       const int cn = __shfl_down_sync(0xffffffffu, c, 1);
       const bool nact = __shfl_down_sync(0xffffffffu, (int)act, 1) != 0;
       if (!__any_sync(0xffffffffu, act && nact && lane < 31 && cn <= c)) {
@@ -159,18 +105,6 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
   const int64_t r0 = warp_search_rows(rowptr, m, (total * gw) / tw, lane);
   const int64_t r1 = warp_search_rows(rowptr, m, (total * (gw + 1)) / tw, lane);
   double loss_acc = 0.0;
-  if constexpr (is_bin_mode(MODE)) {
-    // region of warp gw: chunks [floor(nz0 / CH) + gw (NBIN + 1), ...) -- never overlaps the
-    // next warp's (it uses < entries/CH + NBIN chunks, see csr_binned.cu)
-    const int64_t nz0 = __ldg(rowptr + r0) - __ldg(rowptr);
-    wbase = nz0 / kBinCH + gw * (NBIN + 1);
-    next = wbase;
-#pragma unroll
-    for (int k = 0; k < NBIN; ++k) {
-      cur[k] = next++;
-      fil[k] = 0;
-    }
-  }
 
   // rowptr of the batch starting at row b: lane i holds rowptr[b + i], clamped at r1
   auto RP = [&](int64_t b) -> int64_t { return __ldg(rowptr + (b + lane < r1 ? b + lane : r1)); };
@@ -326,8 +260,6 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
             __syncwarp();
           }
         }
-      } else if constexpr (is_bin_mode(MODE)) {
-        BIN_APPEND(cc[j], xv[j] * qj, act);
       } else {
         if (act) W_ADD(cc[j], xv[j] * qj);
       }
@@ -335,16 +267,6 @@ __global__ void __launch_bounds__(BS) k_csr_flat(const CsrKArgs a) {
     rb = rb_next;
   }
   if constexpr (YM == 2) fpd::flush_loss(a.epi, loss_acc);
-  if constexpr (is_bin_mode(MODE)) {
-    // publish the open chunks (possibly empty) and the region size; the warp's largest |term|
-#pragma unroll
-    for (int k = 0; k < NBIN; ++k)
-      if (lane == k) a.bdir[cur[k]] = ((uint32_t)k << 16) | (uint32_t)fil[k];
-    if (lane == 0) a.wbase[gw] = wbase, a.wcount[gw] = (int32_t)(next - wbase);
-#pragma unroll
-    for (int d = 16; d > 0; d >>= 1) tmax = fmaxf(tmax, __shfl_xor_sync(0xffffffffu, tmax, d));
-    if (lane == 0 && tmax > 0.f) atomicMax(a.gmax, __float_as_uint(tmax));
-  }
 
   if constexpr (MODE == MODE_PRIVATE) {
     __syncthreads();

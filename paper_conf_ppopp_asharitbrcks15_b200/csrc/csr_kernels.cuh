@@ -53,18 +53,6 @@ struct CsrKArgs {
   // L2 lines / slices
   void* wrep;
   int nrep;
-  // MODE_BIN* (variant 17, csr_binned.cuh): the producer appends every term alpha*x*q to the
-  // bin of its column block as a message (16-bit column within the block, fp32 value) in
-  // chunks of kBinCH; warp gw owns chunks [wbase[gw], wbase[gw] + wcount[gw]) and records
-  // each chunk's (bin << 16 | count) in bdir; gmax collects the largest finite |term| (bits)
-  uint16_t* bcol = nullptr;
-  float* bval = nullptr;
-  uint32_t* bdir = nullptr;
-  int64_t* wbase = nullptr;
-  int32_t* wcount = nullptr;
-  unsigned* gmax = nullptr;
-  int bw = 0;          // columns per bin
-  float inv_bw = 0.f;  // 1 / bw (bin of a column by multiply + correction)
 };
 
 // MODE_L2 target of this CTA's reds
@@ -75,10 +63,7 @@ __device__ __forceinline__ T* l2_target(const CsrKArgs& a) {
   return r == 0 ? (T*)a.w : (T*)a.wrep + (int64_t)(r - 1) * a.n;
 }
 
-enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2, MODE_FIXED = 8,
-       MODE_BIN1 = 16, MODE_BIN2 = 17, MODE_BIN4 = 18 };  // MODE_BINk: k = 1 << (MODE - 16) bins
-__host__ __device__ constexpr bool is_bin_mode(int mode) { return mode >= MODE_BIN1 && mode <= MODE_BIN4; }
-constexpr int kBinCH = 256;  // messages per chunk
+enum { MODE_L2 = 0, MODE_SHARED = 1, MODE_PRIVATE = 2, MODE_FIXED = 8 };
 
 // shared-memory layout of the MODE_FIXED partial behind y_s (fixacc.cuh): [sp: n f64][lo: n u32][hi: n u32]
 __device__ __forceinline__ fpd::FixAcc fix_layout(unsigned char* base, int64_t n, int* e) {
@@ -427,8 +412,7 @@ CsrKFn csr_pick_owner_n(int vs, int k) {
 
 // dispatch modes of the flat kernel (aggregation as MODE_SHARED / MODE_L2); k = NB tiles
 enum { DMODE_FLAT_SHARED = 3, DMODE_FLAT_L2 = 4, DMODE_FLAT_PRIVATE = 5, DMODE_OWNER4 = 6, DMODE_OWNER8 = 7,
-       DMODE_FLAT_FIXED = 9, DMODE_STREAM_SHARED = 10, DMODE_STREAM_FIXED = 11, DMODE_FLAT_L2_WIDE = 12,
-       DMODE_BIN1 = 13, DMODE_BIN2 = 14, DMODE_BIN4 = 15 };
+       DMODE_FLAT_FIXED = 9, DMODE_STREAM_SHARED = 10, DMODE_STREAM_FIXED = 11, DMODE_FLAT_L2_WIDE = 12 };
 constexpr int kWideBS = 1024;  // variant 16: one 1024-thread CTA per SM, a y prefix in shared memory
 
 // stream kernels (csr_stream.cuh): (VS, K) as for CSR-vector; no row epilogues (YM 2)
@@ -485,17 +469,6 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
     case DMODE_STREAM_SHARED: return csr_pick_stream<T, YM, MODE_SHARED>(vs, k);
     case DMODE_STREAM_FIXED: return csr_pick_stream<T, YM, MODE_FIXED>(vs, k);
     case DMODE_FLAT_L2_WIDE: return k == 8 ? k_csr_flat<T, 8, YM, MODE_L2, kWideBS> : nullptr;
-    case DMODE_BIN1:
-    case DMODE_BIN2:
-    case DMODE_BIN4:  // variant 17 producer (fp32 messages only)
-      if constexpr (sizeof(T) == 4) {
-        if (k != 8) return nullptr;
-        return mode == DMODE_BIN1 ? k_csr_flat<T, 8, YM, MODE_BIN1, kWideBS>
-                                  : (mode == DMODE_BIN2 ? k_csr_flat<T, 8, YM, MODE_BIN2, kWideBS>
-                                                        : k_csr_flat<T, 8, YM, MODE_BIN4, kWideBS>);
-      } else {
-        return nullptr;
-      }
     default: return nullptr;
   }
 }

@@ -58,6 +58,12 @@ fp_status fp_csr_plan_create(int64_t m, int64_t n, int64_t nnz, const int64_t* r
   FP_REQUIRE(m == 0 || rowptr, FP_ERR_INVALID_ARG, "fp_csr_plan_create: rowptr is NULL");
   FP_REQUIRE(nnz == 0 || colidx, FP_ERR_INVALID_ARG, "fp_csr_plan_create: colidx is NULL");
   cudaStream_t s = (cudaStream_t)stream;
+  // the once-per-matrix structure check (rowptr[0] == 0, monotone, rowptr[m] == nnz, 0 <= col
+  // < n): the hot path trusts the plan's matrix, so an invalid one is refused here
+  if (m > 0) {
+    fp_status vs = fp_csr_validate(m, n, nnz, rowptr, colidx, stream);
+    if (vs != FP_OK) return vs;
+  }
   fp_csr_plan* p = new (std::nothrow) fp_csr_plan;
   FP_REQUIRE(p, FP_ERR_NOMEM, "fp_csr_plan_create: out of host memory");
   p->m = m;

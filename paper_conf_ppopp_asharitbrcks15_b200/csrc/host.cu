@@ -157,7 +157,9 @@ fp_status fp_dense_host(int64_t m, int64_t n, const void* X, int64_t ld, const v
   for (int64_t k = 0; st == FP_OK && alpha != 0.0 && k < nchunks; ++k) {
     const int b = (int)(k & 1);
     const int64_t r0 = k * rows_per_chunk, mc = (m - r0) < rows_per_chunk ? (m - r0) : rows_per_chunk;
-    Piece pc[2] = {{(const char*)X + (size_t)r0 * row_b, (size_t)mc * row_b, xoff},
+    // the chunk's last row is copied as n elements, not ld: X may end right after it (its
+    // extent is (m-1)*ld + n elements, check_dense), and padded columns are never read (R9)
+    Piece pc[2] = {{(const char*)X + (size_t)r0 * row_b, (size_t)(mc - 1) * row_b + (size_t)n * s, xoff},
                    {v ? (const char*)v + (size_t)r0 * s : nullptr, v ? (size_t)mc * s : 0, voff}};
     st = stage(*S, b, pc, 2, pinned);
     if (st != FP_OK) break;

@@ -66,7 +66,8 @@ PatternArgs csr_args(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, c
 
 // Variant 17 (csr_binned.cu): binned producer + fixed-point consumer + exact finalize.
 fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_prefix, cudaStream_t s);
-int binned_nbin(int64_t n);     // 1, 2 or 4 column blocks; 0 if n is too wide
+int binned_nbin(int64_t n);     // 1 or 2 column blocks; 0 if n is too wide
+int binned_producer_regs(bool has_y);
 size_t binned_ws_bytes(int64_t n, int64_t nnz, int nbin, int producer_grid, int consumers);
 
 // w = beta*z (or 0): the alpha == 0 / m == 0 path, and the pre-initialisation of the L2 path.

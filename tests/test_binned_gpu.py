@@ -3,7 +3,7 @@
 The large-n CSR path of SURVEY 8 rows a7/a10: the scatter of Eq. (3) (Alg. 2 l.13-14, P:220-
 221) goes through column-block bins and a shared-memory fixed-point reduction instead of
 per-nonzero global atomics.  Checked here, at sizes the oracle finishes in seconds:
-* integer twins bit-exact for 1, 2 and 4 bins, every instance (with/without y, v, beta*z),
+* integer twins bit-exact for 1 and 2 column blocks, every instance (with/without y, v, beta*z),
   forced producer grids, rows longer than the 256-nonzero batch (warp-per-row path);
 * the int32 wrap carried into hi[] (columns hit by thousands of same-sign maximal terms);
 * U[-1,1) fp32 data within the north_star 2e-5 normwise tolerance;
@@ -45,8 +45,7 @@ def run(dev, rp, ci, va, n, y, v, z, alpha, beta, L):
     return w
 
 
-@pytest.mark.parametrize("n,nbin", [(1000, 1), (40_000, 1), (40_000, 2), (40_000, 4), (100_000, 2),
-                                    (120_000, 4), (220_000, 4)])
+@pytest.mark.parametrize("n,nbin", [(1000, 1), (40_000, 1), (40_000, 2), (100_000, 2), (113_000, 2)])
 @pytest.mark.parametrize("lengths", [("powerlaw", 2.5, 13.64), ("binomial", 0.01), ("uniform", 0, 600)])
 def test_binned_integer_twin_bitexact(cuda_dev, n, nbin, lengths):
     m = 30_000 if lengths[0] != "binomial" else 8_000
@@ -93,7 +92,7 @@ def test_binned_int32_wrap_carries(cuda_dev):
     assert_bitexact(w, ref, "binned wraps")
 
 
-@pytest.mark.parametrize("n,nbin", [(100_000, 2), (200_000, 4), (30_000, 1)])
+@pytest.mark.parametrize("n,nbin", [(100_000, 2), (60_000, 2), (30_000, 1)])
 def test_binned_float_parity(cuda_dev, n, nbin):
     m = 40_000
     rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=7, kind="uniform")
@@ -113,6 +112,19 @@ def test_binned_nonfinite_propagates(cuda_dev):
     ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
     w = run(cuda_dev, rp, ci, va, n, y, v, z, 1.0, 1.0, launch(2))
     assert_parity(w, ref, mag, torch.float32, "binned non-finite")
+
+
+def test_binned_refuses_what_it_cannot_do(cuda_dev):
+    """fp64, a row epilogue, or n beyond two blocks of one SM's shared memory: FP_ERR_UNSUPPORTED
+    through an explicit plan (the chooser never picks variant 17 there)."""
+    m, n = 2000, 150_000
+    rp, ci, va, y, v, z = make(m, n, ("uniform", 0, 20), seed=3, kind="uniform")
+    with pytest.raises(fp.FusedPatError):
+        run(cuda_dev, rp, ci, va, n, y, v, z, 1.0, 1.0, launch(2))
+    rp, ci, va = synth.csr(m, 5000, "f64", ("uniform", 0, 20), seed=3)
+    y = synth.vector(5000, "f64", seed=3)
+    with pytest.raises(fp.FusedPatError):
+        run(cuda_dev, rp, ci, va, 5000, y, None, None, 1.0, 0.0, launch(1))
 
 
 def test_binned_chosen_for_c4_shape(cuda_dev):
