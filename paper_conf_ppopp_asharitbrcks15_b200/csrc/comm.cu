@@ -7,13 +7,32 @@
 #include <nccl.h>
 #include <string.h>
 
+#include <algorithm>
+#include <vector>
+
 #include "kernels.cuh"
 
+constexpr int kMaxPeers = 8;  // one NVSwitch node
+
+// Peer (P2P) exchange state.  Every rank owns a symmetric buffer [D0: cap][D1: cap][flags:
+// kMaxPeers x u64] mapped into every other rank (CUDA IPC across processes, plain pointers in a
+// single-process group).  Call e writes its partial into D[e & 1] of its own buffer, publishes
+// epoch e into flags[rank] of every rank, waits until its own flags[k] >= e for all k, then
+// every rank sums D_k[e & 1] over k in rank order (identical bits on every rank).  Reuse of
+// D[e & 1] at call e + 2 is safe: passing call e + 1's barrier means every peer finished
+// reading call e.
 struct fp_comm {
   ncclComm_t nccl = nullptr;
   int rank = 0;
   int size = 1;
   int device = 0;
+  int mode = FP_COMM_NCCL;
+  size_t cap = 0;                             // bytes of one D buffer
+  unsigned char* sym = nullptr;               // own symmetric buffer
+  unsigned char* peer[kMaxPeers] = {};        // every rank's buffer (peer[rank] == sym)
+  bool ipc_mapped[kMaxPeers] = {};            // opened with cudaIpcOpenMemHandle
+  uint64_t epoch = 0;
+  unsigned* timeout_flag = nullptr;           // device: set if a barrier gave up waiting
 };
 
 namespace fp {
@@ -30,6 +49,142 @@ static fp_status nccl_fail(ncclResult_t r, const char* what) {
   return FP_ERR_NCCL;
 }
 }  // namespace fp
+
+namespace {
+fp_status peer_begin(fp_comm* c, size_t bytes, cudaStream_t s, void** D);
+fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double beta, void* w, cudaStream_t s);
+
+// Peer-mode pattern: the local pass writes this rank's partial alpha X_r^T(v_r (.) X_r y)
+// straight into its symmetric D buffer (no beta z), then the exchange sums the ranks' D in
+// rank order and adds beta z once: every rank ends with the same bits.
+fp_status dist_peer(fp::PatternArgs a, bool csr, fp_comm* comm, cudaStream_t s) {
+  if (a.n == 0) return FP_OK;
+  void* D = nullptr;
+  fp_status st = peer_begin(comm, (size_t)a.n * fp::dtype_size(a.dtype), s, &D);
+  if (st != FP_OK) return st;
+  void* w = a.w;
+  const void* z = a.z;
+  const double beta = a.beta;
+  a.w = D;
+  a.add_beta_z = false;
+  st = csr ? fp::run_csr(a, nullptr, s) : fp::run_dense(a, nullptr, s);
+  if (st != FP_OK) return st;
+  return peer_finish(comm, a.n, a.dtype, beta != 0.0 ? z : nullptr, beta, w, s);
+}
+}  // namespace
+
+namespace {
+
+struct PeerTab {
+  unsigned char* p[kMaxPeers];
+  size_t cap;
+  int P, rank;
+  uint64_t epoch;
+  unsigned* timeout_flag;
+};
+
+__device__ __forceinline__ uint64_t* flags_of(unsigned char* buf, size_t cap) {
+  return reinterpret_cast<uint64_t*>(buf + 2 * cap);
+}
+
+// Publish this rank's arrival (epoch) into every rank's flags[rank], then wait until every
+// rank has arrived here.  One warp; release/acquire at system scope (the flags and the D
+// buffers are read over NVLink).  Gives up after ~20 s (sets *timeout_flag) rather than hang.
+__global__ void k_peer_barrier(const PeerTab t) {
+  const int lane = threadIdx.x;
+  __threadfence_system();
+  if (lane < t.P) {
+    uint64_t* f = flags_of(t.p[lane], t.cap) + t.rank;
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(t.epoch) : "memory");
+  }
+  if (lane < t.P) {
+    const uint64_t* f = flags_of(t.p[t.rank], t.cap) + lane;
+    uint64_t t0, now, v;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    while (true) {
+      asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(f) : "memory");
+      if (v >= t.epoch) break;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+      if (now - t0 > 20000000000ull) {
+        atomicExch(t.timeout_flag, 1u);
+        break;
+      }
+      __nanosleep(100);
+    }
+  }
+  __syncwarp();
+}
+
+// w[j] = sum_k D_k[j] (rank order, fp64 accumulation) + beta z[j]: the same bits on every rank
+template <typename T>
+__global__ void k_peer_sum(const PeerTab t, int64_t n, const T* __restrict__ z, double beta, T* w) {
+  const size_t off = (t.epoch & 1) * t.cap;
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+#pragma unroll 1
+    for (int k = 0; k < t.P; ++k) s += (double)reinterpret_cast<const T*>(t.p[k] + off)[j];
+    if (z && beta != 0.0) s += beta * (double)z[j];
+    w[j] = (T)s;
+  }
+}
+
+PeerTab peer_tab(const fp_comm* c) {
+  PeerTab t{};
+  for (int k = 0; k < c->size; ++k) t.p[k] = c->peer[k];
+  t.cap = c->cap;
+  t.P = c->size;
+  t.rank = c->rank;
+  t.epoch = c->epoch;
+  t.timeout_flag = c->timeout_flag;
+  return t;
+}
+
+bool capturing(cudaStream_t s) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &st) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return st != cudaStreamCaptureStatusNone;
+}
+
+// Start call e: returns this rank's D[e & 1] (where the local partial goes).
+fp_status peer_begin(fp_comm* c, size_t bytes, cudaStream_t s, void** D) {
+  FP_REQUIRE(bytes <= c->cap, FP_ERR_INVALID_ARG, "peer exchange: %zu B exceed the %zu B enabled", bytes, c->cap);
+  FP_REQUIRE(!capturing(s), FP_ERR_UNSUPPORTED,
+             "peer exchange: not capturable in a CUDA graph (its epoch advances per call); use NCCL mode");
+  c->epoch += 1;
+  *D = c->sym + (c->epoch & 1) * c->cap;
+  return FP_OK;
+}
+
+// Finish call e: barrier, then w = sum_k D_k + beta z.
+fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double beta, void* w, cudaStream_t s) {
+  const PeerTab t = peer_tab(c);
+  k_peer_barrier<<<1, 32, 0, s>>>(t);
+  FP_CUDA(cudaGetLastError());
+  const int grid = (int)std::min<int64_t>((n + 255) / 256, 4 * fp::device_info(c->device).sm_count);
+  if (n > 0) {
+    if (dt == FP_F64) k_peer_sum<double><<<grid, 256, 0, s>>>(t, n, (const double*)z, beta, (double*)w);
+    else k_peer_sum<float><<<grid, 256, 0, s>>>(t, n, (const float*)z, beta, (float*)w);
+    FP_CUDA(cudaGetLastError());
+  }
+  return FP_OK;
+}
+
+fp_status alloc_sym(fp_comm* c, size_t cap) {
+  const size_t bytes = 2 * cap + kMaxPeers * sizeof(uint64_t);
+  FP_CUDA(cudaSetDevice(c->device));
+  FP_CUDA(cudaMalloc((void**)&c->sym, bytes));
+  FP_CUDA(cudaMemset(c->sym, 0, bytes));
+  FP_CUDA(cudaMalloc((void**)&c->timeout_flag, sizeof(unsigned)));
+  FP_CUDA(cudaMemset(c->timeout_flag, 0, sizeof(unsigned)));
+  c->cap = cap;
+  c->peer[c->rank] = c->sym;
+  return FP_OK;
+}
+
+}  // namespace
 
 #define FP_NCCL(call)                                      \
   do {                                                     \
@@ -69,6 +224,12 @@ fp_status fp_comm_init(fp_comm** comm, int nranks, int rank, const unsigned char
 
 fp_status fp_comm_destroy(fp_comm* comm) {
   if (!comm) return FP_OK;
+  cudaSetDevice(comm->device);
+  cudaDeviceSynchronize();
+  for (int k = 0; k < kMaxPeers; ++k)
+    if (comm->ipc_mapped[k]) cudaIpcCloseMemHandle(comm->peer[k]);
+  if (comm->sym) cudaFree(comm->sym);
+  if (comm->timeout_flag) cudaFree(comm->timeout_flag);
   ncclResult_t r = comm->nccl ? ncclCommDestroy(comm->nccl) : ncclSuccess;
   delete comm;
   if (r != ncclSuccess) return fp::nccl_fail(r, "ncclCommDestroy");
@@ -84,6 +245,16 @@ fp_status fp_allreduce(fp_comm* comm, void* buf, int64_t n, fp_dtype dtype, fp_s
   // no short cut for one rank: the collective runs (a copy in place) so that every *_dist call
   // exercises the same NCCL path at any world size
   if (n == 0) return FP_OK;
+  if (comm->mode == FP_COMM_PEER) {
+    cudaStream_t s = (cudaStream_t)stream;
+    void* D = nullptr;
+    const size_t bytes = (size_t)n * fp::dtype_size(dtype);
+    fp_status st = peer_begin(comm, bytes, s, &D);
+    if (st != FP_OK) return st;
+    FP_CUDA(cudaMemcpyAsync(D, buf, bytes, cudaMemcpyDeviceToDevice, s));
+    return peer_finish(comm, n, dtype, nullptr, 0.0, buf, s);
+  }
+  FP_REQUIRE(comm->nccl, FP_ERR_INVALID_ARG, "fp_allreduce: communicator has no NCCL backend (local group)");
   FP_NCCL(ncclAllReduce(buf, buf, (size_t)n, dtype == FP_F64 ? ncclFloat64 : ncclFloat32, ncclSum, comm->nccl,
                         (cudaStream_t)stream));
   return FP_OK;
@@ -116,12 +287,98 @@ fp_status fp_shard_rows_csr(int64_t m, const int64_t* rowptr, int nranks, int64_
   return FP_OK;
 }
 
+// --------------------------------------------------------------------- peer mode setup
+// Collective: every rank allocates its symmetric buffer, exports a CUDA IPC handle, the
+// handles are all-gathered through NCCL, and every rank maps every peer's buffer.
+fp_status fp_comm_enable_peer(fp_comm* comm, int64_t max_bytes, fp_stream stream) {
+  FP_REQUIRE(comm && max_bytes > 0, FP_ERR_INVALID_ARG, "fp_comm_enable_peer: bad arguments");
+  FP_REQUIRE(comm->size <= kMaxPeers, FP_ERR_UNSUPPORTED, "fp_comm_enable_peer: at most %d ranks", kMaxPeers);
+  if (comm->sym) {
+    FP_REQUIRE((size_t)max_bytes <= comm->cap, FP_ERR_INVALID_ARG, "fp_comm_enable_peer: already enabled smaller");
+    comm->mode = FP_COMM_PEER;
+    return FP_OK;
+  }
+  FP_REQUIRE(comm->nccl, FP_ERR_INVALID_ARG, "fp_comm_enable_peer: needs an NCCL communicator");
+  const size_t cap = ((size_t)max_bytes + 255) / 256 * 256;
+  fp_status st = alloc_sym(comm, cap);
+  if (st != FP_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaIpcMemHandle_t mine;
+  FP_CUDA(cudaIpcGetMemHandle(&mine, comm->sym));
+  unsigned char* dh = nullptr;
+  FP_CUDA(cudaMalloc((void**)&dh, (size_t)comm->size * sizeof(cudaIpcMemHandle_t)));
+  FP_CUDA(cudaMemcpyAsync(dh + (size_t)comm->rank * sizeof(mine), &mine, sizeof(mine), cudaMemcpyHostToDevice, s));
+  ncclResult_t r = ncclAllGather(dh + (size_t)comm->rank * sizeof(mine), dh, sizeof(mine), ncclUint8, comm->nccl, s);
+  if (r != ncclSuccess) {
+    cudaFree(dh);
+    return fp::nccl_fail(r, "ncclAllGather(ipc handles)");
+  }
+  std::vector<cudaIpcMemHandle_t> all(comm->size);
+  FP_CUDA(cudaMemcpyAsync(all.data(), dh, (size_t)comm->size * sizeof(mine), cudaMemcpyDeviceToHost, s));
+  FP_CUDA(cudaStreamSynchronize(s));
+  cudaFree(dh);
+  for (int k = 0; k < comm->size; ++k) {
+    if (k == comm->rank) continue;
+    void* p = nullptr;
+    FP_CUDA(cudaIpcOpenMemHandle(&p, all[k], cudaIpcMemLazyEnablePeerAccess));
+    comm->peer[k] = (unsigned char*)p;
+    comm->ipc_mapped[k] = true;
+  }
+  comm->mode = FP_COMM_PEER;
+  return FP_OK;
+}
+
+fp_status fp_comm_set_mode(fp_comm* comm, int mode) {
+  FP_REQUIRE(comm && (mode == FP_COMM_NCCL || mode == FP_COMM_PEER), FP_ERR_INVALID_ARG,
+             "fp_comm_set_mode: bad arguments");
+  FP_REQUIRE(mode != FP_COMM_PEER || comm->sym, FP_ERR_INVALID_ARG, "fp_comm_set_mode: peer mode not enabled");
+  FP_REQUIRE(mode != FP_COMM_NCCL || comm->nccl, FP_ERR_INVALID_ARG, "fp_comm_set_mode: no NCCL backend");
+  comm->mode = mode;
+  return FP_OK;
+}
+
+int fp_comm_mode(const fp_comm* comm) { return comm ? comm->mode : -1; }
+
+// Single-process group of `nranks` communicators on ONE device whose symmetric buffers are
+// plain device allocations (no IPC, no NCCL): the peer exchange exactly as across GPUs, for
+// tests and for replicas sharing a GPU.  Ranks must be driven concurrently (one host thread or
+// one stream per rank): a rank's barrier waits for the others.
+fp_status fp_comm_init_local_group(int nranks, int device, int64_t max_bytes, fp_comm** comms) {
+  FP_REQUIRE(comms && nranks >= 1 && nranks <= kMaxPeers && max_bytes > 0, FP_ERR_INVALID_ARG,
+             "fp_comm_init_local_group: bad arguments (1 <= nranks <= %d)", kMaxPeers);
+  const size_t cap = ((size_t)max_bytes + 255) / 256 * 256;
+  for (int r = 0; r < nranks; ++r) {
+    comms[r] = new fp_comm();
+    comms[r]->rank = r;
+    comms[r]->size = nranks;
+    comms[r]->device = device;
+    comms[r]->mode = FP_COMM_PEER;
+    fp_status st = alloc_sym(comms[r], cap);
+    if (st != FP_OK) {
+      for (int k = 0; k <= r; ++k) fp_comm_destroy(comms[k]);
+      return st;
+    }
+  }
+  for (int r = 0; r < nranks; ++r)
+    for (int k = 0; k < nranks; ++k) comms[r]->peer[k] = comms[k]->sym;
+  return FP_OK;
+}
+
+// 1 if a peer barrier of this communicator ever timed out (its results are then invalid).
+int fp_comm_timed_out(const fp_comm* comm) {
+  if (!comm || !comm->timeout_flag) return 0;
+  unsigned h = 0;
+  if (cudaMemcpy(&h, comm->timeout_flag, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
+  return h ? 1 : 0;
+}
+
 // --------------------------------------------------------------------- distributed pattern
 fp_status fp_dense_dist(int64_t m_local, int64_t n, const void* X, int64_t ld, const void* y, const void* v,
                         const void* z, double alpha, double beta, void* w, fp_dtype dtype, fp_comm* comm,
                         fp_stream stream) {
   FP_REQUIRE(comm, FP_ERR_INVALID_ARG, "fp_dense_dist: comm is NULL");
   fp::PatternArgs a = fp::dense_args(m_local, n, X, ld, y, v, z, alpha, beta, w, dtype);
+  if (comm->mode == FP_COMM_PEER) return dist_peer(a, false, comm, (cudaStream_t)stream);
   a.add_beta_z = comm->rank == 0;
   fp_status st = fp::run_dense(a, nullptr, (cudaStream_t)stream);
   if (st != FP_OK) return st;
@@ -133,6 +390,7 @@ fp_status fp_csr_dist(int64_t m_local, int64_t n, int64_t nnz_local, const int64
                       void* w, fp_dtype dtype, fp_comm* comm, fp_stream stream) {
   FP_REQUIRE(comm, FP_ERR_INVALID_ARG, "fp_csr_dist: comm is NULL");
   fp::PatternArgs a = fp::csr_args(m_local, n, nnz_local, rowptr, colidx, val, y, v, z, alpha, beta, w, dtype);
+  if (comm->mode == FP_COMM_PEER) return dist_peer(a, true, comm, (cudaStream_t)stream);
   a.add_beta_z = comm->rank == 0;
   fp_status st = fp::run_csr(a, nullptr, (cudaStream_t)stream);
   if (st != FP_OK) return st;

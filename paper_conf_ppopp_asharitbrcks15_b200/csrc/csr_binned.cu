@@ -15,9 +15,9 @@
 //    column block (16 bits).  Two column blocks: warp gw owns the message slots of its own
 //    nonzero range [nz0, nz1); block-0 messages fill it upward from nz0, block-1 messages
 //    downward from nz1 -- plain coalesced stores, no allocation, no atomics.  Rows up to
-//    kLT nonzeros go in "flat" batches (lanes on consecutive nonzeros, a segmented reduction
-//    steered by a per-tile head bitmask); longer rows go warp-per-row in kNB-tile segments
-//    (every load of a segment in flight at once).
+//    kLT nonzeros go in "flat" batches (4 consecutive nonzeros per lane from 128-bit loads, a
+//    two-level segmented reduction steered by a head bitmask); longer rows go warp-per-row in
+//    steps of 256 nonzeros (every load of a step in flight at once).
 //  k_bin_consume -- one 1024-thread CTA per SM holds one column block of w in shared memory
 //    as 32-bit fixed point and adds its block's messages with native shared atomics.
 //  k_bin_finalize -- sums the consumers' partials exactly in int64 and writes
@@ -41,8 +41,7 @@ namespace {
 
 constexpr int kProdBS = 1024;
 constexpr int kConsBS = 1024;
-constexpr int kNB = 8;            // register tiles of 32 nonzeros per batch / segment
-constexpr int kCAP = 32 * kNB;    // nonzeros per flat batch
+constexpr int kNT = 2;            // super-tiles of 128 nonzeros (4 per lane) per batch
 constexpr int kLT = 128;          // rows longer than this go warp-per-row
 
 struct BinPArgs {
@@ -55,6 +54,7 @@ struct BinPArgs {
   float alpha;
   int ny_s;          // leading y entries staged in shared memory
   int bw;            // block-0 width (columns >= bw are block 1; bw >= n: one block)
+  int mis;           // (address of colidx / 4) mod 4 -- the same for val (checked on launch)
   uint16_t* bcol;    // [nnz] message column within its block
   float* bval;       // [nnz] message value
   int64_t* wsplit;   // [warps][3]: nz0, split (first block-1 slot), nz1
@@ -91,13 +91,42 @@ __device__ __forceinline__ int bin_exponent(const unsigned* gmax) {
   return e;
 }
 
-template <int YM>
+// 16-byte read-once loads of 4 consecutive colidx / val entries (index aligned to 4 in memory)
+__device__ __forceinline__ void ld4(const int32_t* pc, const float* pv, int (&c)[4], float (&x)[4]) {
+  asm("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+      : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3])
+      : "l"(pc));
+  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+      : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3])
+      : "l"(pv));
+}
+
+// The producer.  Nonzeros are handled 4 per lane: a "super-tile" is 128 consecutive nonzeros
+// starting at a 16-byte-aligned index, lane l holding entries 4l..4l+3 (two 128-bit loads);
+// a batch spans kNT super-tiles.  Row boundaries inside a batch are a 256-bit head mask in
+// shared memory (bit p set where a non-empty row starts at batch position p).  The row dot is
+// a two-level segmented sum: in-lane over the lane's 4 products, then across lanes over the
+// lanes' leading partial sums (a shuffle reduction bounded by the next lane holding a head).
+// predicated message store (no branch around it)
+__device__ __forceinline__ void st_msg(uint16_t* pc, float* pv, int c, float t, bool on) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "@p st.global.u16 [%0], %2;\n\t"
+      "@p st.global.f32 [%1], %3;\n\t}"
+      ::"l"(pc), "l"(pv), "h"((unsigned short)c), "f"(t), "r"((int)on)
+      : "memory");
+}
+
+template <int YM, int NBIN>
 __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
   constexpr int NW = kProdBS / 32;
+  constexpr int NT = kNT;
+  constexpr int SPAN = 128 * NT;                // nonzero positions of a batch
   extern __shared__ __align__(16) float y_s[];
-  __shared__ float rs[NW][32];          // per-warp row sums, compressed (non-empty) row order
-  __shared__ unsigned hmw[NW][kNB];     // per-warp head masks of the batch's tiles
-  __shared__ unsigned char cmap[NW][32];  // compressed row -> lane of the batch
+  __shared__ float rs[NW][32];                  // per-warp row sums, compressed (non-empty) row order
+  __shared__ unsigned hmw[NW][SPAN / 32];       // per-warp head masks
+  __shared__ unsigned char cmap[NW][32];        // compressed row -> lane of the batch
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t* __restrict__ rowptr = a.rowptr;
   const int32_t* __restrict__ colidx = a.colidx;
@@ -107,6 +136,7 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
   for (int j = threadIdx.x; j < ny_s; j += kProdBS) y_s[j] = y[j];
   __syncthreads();
   auto Y = [&](int c) -> float { return c < ny_s ? y_s[c] : fpd::ld_keep(y + c); };
+  const int mis = a.mis;
 
   const int64_t m = a.m;
   const int64_t gw = (int64_t)blockIdx.x * NW + warp, tw = (int64_t)gridDim.x * NW;
@@ -115,30 +145,64 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
   const int64_t r1 = warp_search_rows(rowptr, m, (total * (gw + 1)) / tw, lane);
   const int64_t base0 = __ldg(rowptr);
   const int64_t nz0 = __ldg(rowptr + r0) - base0, nz1 = __ldg(rowptr + r1) - base0;
-  int64_t up = nz0, dn = nz1;  // next block-0 slot (upward), one past the last free block-1 slot
+  // message slots of this warp: [nz0, nz1); offsets relative to nz0 (< 2^31, checked on launch)
+  uint16_t* const bcol = a.bcol + nz0;
+  float* const bval = a.bval + nz0;
+  int up = 0, dn = (int)(nz1 - nz0);  // next block-0 slot (upward), one past the last free block-1 slot
   float tmax = 0.f;
-  const unsigned lt = lanemask_lt(), le = lanemask_le();
+  const unsigned lt = lanemask_lt();
   const int bw = a.bw;
   const float alpha = a.alpha;
 
-  // one tile of terms (lane: column c, term t, active) -> message slots of the warp
-  auto EMIT = [&](int c, float t, bool act) {
-    const float at = fabsf(t);
-    tmax = fmaxf(tmax, at <= 3.402823466e38f ? at : 0.f);
-    const bool b1 = act && c >= bw;
-    const unsigned m1 = __ballot_sync(0xffffffffu, b1);
-    const unsigned m0 = __ballot_sync(0xffffffffu, act) & ~m1;
-    if (act) {
-      const int64_t idx = b1 ? dn - 1 - __popc(m1 & lt) : up + __popc(m0 & lt);
-      a.bcol[idx] = (uint16_t)(b1 ? c - bw : c);
-      a.bval[idx] = t;
+  // The scatter of one super-tile: lane l's 4 terms (columns c, values t, active bits act),
+  // one entry index per step: the step's block-0 lanes take consecutive slots upward from
+  // `up`, its block-1 lanes consecutive slots downward from `dn` -- every store instruction
+  // covers consecutive slots.  Branch-free: predicated stores, 32-bit slot arithmetic.
+  auto EMIT4 = [&](const int (&c)[4], const float (&t)[4], unsigned act) {
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      tmax = fmaxf(tmax, fabsf(t[e]));  // inactive terms are 0; NaN is ignored, Inf kept
+      const bool on = (act >> e) & 1u;
+      unsigned idx;
+      int cl = c[e];
+      if constexpr (NBIN == 2) {
+        const bool b1 = on && c[e] >= bw;
+        const unsigned m1 = __ballot_sync(0xffffffffu, b1);
+        const unsigned m0 = __ballot_sync(0xffffffffu, on) & ~m1;
+        const unsigned i0 = (unsigned)up + __popc(m0 & lt), i1 = (unsigned)dn - 1u - __popc(m1 & lt);
+        idx = b1 ? i1 : i0;
+        cl = b1 ? c[e] - bw : c[e];
+        up += __popc(m0);
+        dn -= __popc(m1);
+      } else {
+        const unsigned m0 = __ballot_sync(0xffffffffu, on);
+        idx = (unsigned)up + __popc(m0 & lt);
+        up += __popc(m0);
+      }
+      st_msg(bcol + idx, bval + idx, cl, t[e], on);
     }
-    up += __popc(m0);
-    dn -= __popc(m1);
   };
 
   auto RP = [&](int64_t b) -> int64_t { return __ldg(rowptr + (b + lane < r1 ? b + lane : r1)); };
   auto RP_END = [&](int64_t b) -> int64_t { return __ldg(rowptr + (b + 32 < r1 ? b + 32 : r1)); };
+  // 4 entries at aligned index g = A + o (o = 4 * lane + 128 * t): loaded when any is before
+  // `hi`; active = inside [lo, hi) (positions relative to A, 32-bit)
+  auto LOAD4 = [&](int64_t A, int o, int lo, int hi, int (&c)[4], float (&x)[4]) -> unsigned {
+    unsigned act = 0;
+    if (o < hi) {
+      ld4(colidx + A + o, val + A + o, c, x);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const bool in = o + e >= lo && o + e < hi;
+        act |= (unsigned)in << e;
+        if (!in) c[e] = 0, x[e] = 0.f;
+      }
+    } else {
+#pragma unroll
+      for (int e = 0; e < 4; ++e) c[e] = 0, x[e] = 0.f;
+    }
+    return act;
+  };
   int64_t rp_cur = RP(r0), rp_end_cur = RP_END(r0);
   for (int64_t rb = r0; rb < r1;) {
     const int64_t rp = rp_cur, rp_end = rp_end_cur;
@@ -147,122 +211,158 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
     if (lane == 31) nxt = rp_end;
     const bool inr = rb + lane < r1;
     const int64_t len = inr ? nxt - rp : 0;
-    // a flat batch: the leading run of rows with <= kLT nonzeros whose total fits kCAP
-    const bool ok = inr && len <= kLT && nxt - a0 <= kCAP;
+    const int64_t A = a0 - ((a0 + mis) & 3);  // aligned start (colidx + A is 16-byte aligned)
+    // a flat batch: the leading run of rows with <= kLT nonzeros within SPAN positions of A
+    const bool ok = inr && len <= kLT && nxt - A <= SPAN;
     const int nrows = __ffs(~__ballot_sync(0xffffffffu, ok)) - 1;  // leading ones (-1 if all 32 ok)
     const int nr = nrows < 0 ? 32 : nrows;
     const float vpre = (a.v && inr) ? fpd::ld_once(a.v + rb + lane) : 1.f;
     const int64_t rb_next = rb + (nr == 0 ? 1 : nr);
     rp_cur = RP(rb_next);
     rp_end_cur = RP_END(rb_next);
+    const int lo = (int)(a0 - A);  // 0..3
+    // the next flat batch's colidx / val (at most SPAN entries from where this one ends) on
+    // their way into L2 while this batch is processed
+    {
+      const int64_t nstart = __shfl_sync(0xffffffffu, nxt, (nr == 0 ? 1 : nr) - 1);
+      const int64_t rem = base0 + a.nnz - nstart;  // never past the arrays' end
+      if (lane == 0 && rem > 0) {
+        const size_t bytes = (size_t)(rem < SPAN ? rem : SPAN) * 4;
+        fpd::prefetch_l2(colidx + nstart, bytes);
+        fpd::prefetch_l2(val + nstart, bytes);
+      }
+    }
 
     if (nr == 0) {
-      // ---- row rb is long: warp-per-row in segments of kNB tiles, loads of a segment in flight
-      // together; the first segment stays in registers for the scatter, the rest is re-read
-      // (L2-resident after the dot pass; the paper's "likely a cache hit")
-      const int64_t s0 = a0;
+      // ---- row rb is long: warp-per-row, SPAN positions per step with every load of a step in
+      // flight together; the first step stays in registers for the scatter, the rest is re-read
+      // (just read, so L2-resident: the paper's "likely a cache hit")
       const int64_t L = __shfl_sync(0xffffffffu, len, 0);
-      int cc[kNB];
-      float xv[kNB];
+      const int64_t endA = L + lo;  // end relative to A (may exceed 2^31 only for n > 2^31)
+      const int hi0 = (int)(endA < SPAN ? endA : SPAN);
+      int cc[NT][4];
+      float xv[NT][4];
+      unsigned act[NT];
+#pragma unroll
+      for (int t = 0; t < NT; ++t) act[t] = LOAD4(A, 128 * t + 4 * lane, lo, hi0, cc[t], xv[t]);
       float acc = 0.f;
-#pragma unroll
-      for (int j = 0; j < kNB; ++j) {
-        const int64_t k = j * 32 + lane;
-        cc[j] = k < L ? fpd::ld_once(colidx + s0 + k) : 0;
-        xv[j] = k < L ? fpd::ld_once(val + s0 + k) : 0.f;
-      }
       if constexpr (YM != 0) {
-        float yv[kNB];
 #pragma unroll
-        for (int j = 0; j < kNB; ++j) yv[j] = Y(cc[j]);
+        for (int t = 0; t < NT; ++t)
 #pragma unroll
-        for (int j = 0; j < kNB; ++j) acc = fmaf(xv[j], yv[j], acc);
-        for (int64_t seg = kCAP; seg < L; seg += kCAP) {
-          int c2[kNB];
-          float x2[kNB], y2[kNB];
+          for (int e = 0; e < 4; ++e) acc = fmaf(xv[t][e], Y(cc[t][e]), acc);
+        for (int64_t s0 = SPAN; s0 < endA; s0 += SPAN) {
+          const int64_t As = A + s0;
+          const int his = (int)(endA - s0 < SPAN ? endA - s0 : SPAN);
 #pragma unroll
-          for (int j = 0; j < kNB; ++j) {
-            const int64_t k = seg + j * 32 + lane;
-            c2[j] = k < L ? __ldg(colidx + s0 + k) : 0;
-            x2[j] = k < L ? __ldg(val + s0 + k) : 0.f;
+          for (int t = 0; t < NT; ++t) {
+            int c2[4];
+            float x2[4];
+            LOAD4(As, 128 * t + 4 * lane, 0, his, c2, x2);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc = fmaf(x2[e], Y(c2[e]), acc);
           }
-#pragma unroll
-          for (int j = 0; j < kNB; ++j) y2[j] = Y(c2[j]);
-#pragma unroll
-          for (int j = 0; j < kNB; ++j) acc = fmaf(x2[j], y2[j], acc);
         }
         acc = fpd::vector_allreduce<32>(acc);
       }
       const float vr = __shfl_sync(0xffffffffu, vpre, 0);
       const float q = (YM != 0 ? acc * vr : vr) * alpha;
 #pragma unroll
-      for (int j = 0; j < kNB; ++j) EMIT(cc[j], xv[j] * q, j * 32 + lane < L);
-      for (int64_t seg = kCAP; seg < L; seg += 32) {
-        const int64_t k = seg + lane;
-        const bool act = k < L;
-        const int c = act ? __ldg(colidx + s0 + k) : 0;
-        const float x = act ? __ldg(val + s0 + k) : 0.f;
-        EMIT(c, x * q, act);
+      for (int t = 0; t < NT; ++t) {
+        float tv[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) tv[e] = xv[t][e] * q;
+        EMIT4(cc[t], tv, act[t]);
+      }
+      for (int64_t s0 = SPAN; s0 < endA; s0 += 128) {
+        const int his = (int)(endA - s0 < 128 ? endA - s0 : 128);
+        int c2[4];
+        float x2[4];
+        const unsigned a2 = LOAD4(A + s0, 4 * lane, 0, his, c2, x2);
+        float tv[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) tv[e] = x2[e] * q;
+        EMIT4(c2, tv, a2);
       }
       rb = rb_next;
       continue;
     }
 
-    // ---- flat batch of rows [rb, rb + nr): lanes on consecutive nonzeros
-    const int cnt = (int)(__shfl_sync(0xffffffffu, nxt, nr - 1) - a0);
+    // ---- flat batch of rows [rb, rb + nr) within positions [A, A + SPAN)
+    const int hi = (int)(__shfl_sync(0xffffffffu, nxt, nr - 1) - A);
     const bool ne = lane < nr && len > 0;
     const unsigned nem = __ballot_sync(0xffffffffu, ne);
-    const int rel = (int)(rp - a0);
-    if (lane < kNB) hmw[warp][lane] = 0u;
+    const int rel = (int)(rp - A);
+    if (lane < SPAN / 32) hmw[warp][lane] = 0u;
     __syncwarp();
     if (ne) {
       atomicOr(&hmw[warp][rel >> 5], 1u << (rel & 31));
       cmap[warp][__popc(nem & lt)] = (unsigned char)lane;
     }
-    int cc[kNB];
-    float xv[kNB];
+    int cc[NT][4];
+    float xv[NT][4];
+    unsigned act[NT];
 #pragma unroll
-    for (int j = 0; j < kNB; ++j) {
-      const int pos = j * 32 + lane;
-      cc[j] = pos < cnt ? fpd::ld_once(colidx + a0 + pos) : 0;
-      xv[j] = pos < cnt ? fpd::ld_once(val + a0 + pos) : 0.f;
-    }
+    for (int t = 0; t < NT; ++t) act[t] = LOAD4(A, 128 * t + 4 * lane, lo, hi, cc[t], xv[t]);
     rs[warp][lane] = 0.f;
     __syncwarp();
-    unsigned hm[kNB];
+    // head bits of this lane's 4 positions per super-tile, and the compressed row index of the
+    // lane's first position (heads strictly before it, minus one)
+    const unsigned hword = lane < SPAN / 32 ? hmw[warp][lane] : 0u;
+    int pre = __popc(hword);
 #pragma unroll
-    for (int j = 0; j < kNB; ++j) hm[j] = hmw[warp][j];
-    // compressed row index of every nonzero: heads at or before it, minus one
-    int rid[kNB];
-    {
-      int base = 0;
+    for (int d = 1; d < SPAN / 32; d <<= 1) {
+      const int t2 = __shfl_up_sync(0xffffffffu, pre, d);
+      if (lane >= d) pre += t2;
+    }
+    pre -= __popc(hword);  // exclusive prefix of head counts over the mask words
+    unsigned hb[NT];
+    int rbase[NT];
 #pragma unroll
-      for (int j = 0; j < kNB; ++j) {
-        rid[j] = base - 1 + __popc(hm[j] & le);
-        base += __popc(hm[j]);
-      }
+    for (int t = 0; t < NT; ++t) {
+      const int wi = 4 * t + (lane >> 3);
+      const unsigned hw = __shfl_sync(0xffffffffu, hword, wi);
+      const int sh = (lane & 7) * 4;
+      hb[t] = (hw >> sh) & 0xFu;
+      rbase[t] = __shfl_sync(0xffffffffu, pre, wi) + __popc(hw & ((1u << sh) - 1u)) - 1;
     }
     if constexpr (YM != 0) {
-      float yv[kNB];
 #pragma unroll
-      for (int j = 0; j < kNB; ++j) yv[j] = Y(cc[j]);
+      for (int t = 0; t < NT; ++t) {
+        float sv[4];
 #pragma unroll
-      for (int j = 0; j < kNB; ++j) {
-        if (j * 32 >= cnt) break;
-        float s = xv[j] * yv[j];  // Eq. (2) products (0 on inactive lanes)
-        // segmented suffix sums toward each segment's first lane: lane l adds lane l+d while
-        // l+d is in its segment (no head in (l, l+d], and inside the tile)
-        const unsigned after = (hm[j] >> lane) >> 1;
-        const int dist = after ? __ffs(after) : 32 - lane;
+        for (int e = 0; e < 4; ++e) sv[e] = xv[t][e] * Y(cc[t][e]);  // Eq. (2) products
+        // in-lane: P = sum before the first head, complete segments flushed, the last one kept
+        float sum = 0.f, P = 0.f;
+        int rid = rbase[t];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          if ((hb[t] >> e) & 1u) {
+            if (rid == rbase[t]) P = sum;
+            else rs[warp][rid] += sum;  // a row entirely inside this lane
+            sum = 0.f;
+            ++rid;
+          }
+          sum += sv[e];
+        }
+        if (!hb[t]) P = sum;
+        // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a head
+        const unsigned H = __ballot_sync(0xffffffffu, hb[t] != 0u);
+        const unsigned hl = H >> lane;
+        const int dist = hl ? __ffs(hl) : 32 - lane;
+        float r = P;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
-          const float t = __shfl_down_sync(0xffffffffu, s, d);
-          if (d < dist) s += t;
+          const float t2 = __shfl_down_sync(0xffffffffu, r, d);
+          if (d < dist) r += t2;
         }
-        const bool head = j * 32 + lane < cnt && (lane == 0 || ((hm[j] >> lane) & 1u));
-        if (head) rs[warp][rid[j]] += s;  // heads of one tile hold distinct rows
+        float rn = __shfl_down_sync(0xffffffffu, r, 1);
+        if (lane == 31) rn = 0.f;  // continues in the next super-tile: its lane 0 adds it
+        if (hb[t]) rs[warp][rid] += sum + rn;           // the lane's last row: its suffix + what follows
+        if (lane == 0 && !(hb[t] & 1u) && rbase[t] >= 0)  // the row running in from the previous tile
+          rs[warp][rbase[t]] += r;
+        __syncwarp();
       }
-      __syncwarp();
     }
     // lane k owns the k-th non-empty row of the batch: q = alpha v p
     float q = 0.f;
@@ -273,16 +373,22 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       if (lane < nne) q = (YM != 0 ? rs[warp][lane] * vr : vr) * alpha;
     }
 #pragma unroll
-    for (int j = 0; j < kNB; ++j) {
-      if (j * 32 >= cnt) break;
-      const float qj = __shfl_sync(0xffffffffu, q, rid[j] & 31);
-      EMIT(cc[j], xv[j] * qj, j * 32 + lane < cnt);
+    for (int t = 0; t < NT; ++t) {
+      if (128 * t >= hi) break;
+      int rid = rbase[t];
+      float tv[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        rid += (hb[t] >> e) & 1u;
+        tv[e] = xv[t][e] * __shfl_sync(0xffffffffu, q, rid & 31);
+      }
+      EMIT4(cc[t], tv, act[t]);
     }
     rb = rb_next;
   }
   if (lane == 0) {
     a.wsplit[3 * gw] = nz0;
-    a.wsplit[3 * gw + 1] = up;  // == dn: every slot of [nz0, nz1) written
+    a.wsplit[3 * gw + 1] = nz0 + up;  // == nz0 + dn: every slot of [nz0, nz1) written
     a.wsplit[3 * gw + 2] = nz1;
   }
 #pragma unroll
@@ -299,13 +405,15 @@ __global__ void __launch_bounds__(kConsBS, 1) k_bin_consume(const BinCArgs a) {
   const int cid = (int)(blockIdx.x / (unsigned)a.nbin);
   const int ncons = ((int)gridDim.x - b + a.nbin - 1) / a.nbin;
   const int64_t pw0 = a.pw * cid / ncons, pw1 = a.pw * (cid + 1) / ncons;
-  const int ex = 26 - bin_exponent(a.gmax);
+  // an infinite term (gmax = +Inf) leaves no finite scale: then every term goes to the spill
+  const bool allspill = *a.gmax == 0x7f800000u;
+  const int ex = allspill ? 0 : 26 - bin_exponent(a.gmax);
   const bool fscale = ex >= -125 && ex <= 127;  // 2^ex representable as float (the usual case)
   const float sf = fscale ? ldexpf(1.f, ex) : 0.f;
   const double sd = ldexp(1.0, ex);
   const int64_t col0 = (int64_t)b * a.bw;
   auto ADD = [&](int cl, float t) {
-    if (!(fabsf(t) <= 3.402823466e38f)) {  // Inf / NaN: IEEE propagation through the spill
+    if (allspill || !(fabsf(t) <= 3.402823466e38f)) {  // Inf / NaN: IEEE propagation through the spill
       atomicAdd(a.spill + col0 + cl, t);
       return;
     }
@@ -315,21 +423,35 @@ __global__ void __launch_bounds__(kConsBS, 1) k_bin_consume(const BinCArgs a) {
     if ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0)  // signed wrap: carry into hi
       atomicAdd(a.hi + col0 + cl, qi > 0 ? 1 : -1);
   };
-  constexpr int U = 4;  // loads in flight per lane
+  // each lane takes 8 consecutive messages per step (a 16-byte column load and a 32-byte value
+  // load at 8-aligned indices), two steps in flight
   for (int64_t p = pw0 + warp; p < pw1; p += kConsBS / 32) {
     const int64_t lo = a.wsplit[3 * p + b], hi = a.wsplit[3 * p + b + 1];
-    for (int64_t i0 = lo; i0 < hi; i0 += 32 * U) {
-      int c[U];
-      float t[U];
+    for (int64_t g0 = (lo & ~int64_t(7)) + 8 * lane; g0 < hi; g0 += 2 * 256) {
+      uint4 cv[2];
+      float tv[2][8];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int64_t i = i0 + u * 32 + lane;
-        c[u] = i < hi ? (int)__ldcs(a.bcol + i) : 0;
-        t[u] = i < hi ? __ldcs(a.bval + i) : 0.f;
+      for (int u = 0; u < 2; ++u) {
+        const int64_t g = g0 + u * 256;
+        if (g < hi) {
+          asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+              : "=r"(cv[u].x), "=r"(cv[u].y), "=r"(cv[u].z), "=r"(cv[u].w)
+              : "l"(a.bcol + g));
+          asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+              : "=f"(tv[u][0]), "=f"(tv[u][1]), "=f"(tv[u][2]), "=f"(tv[u][3]), "=f"(tv[u][4]), "=f"(tv[u][5]),
+                "=f"(tv[u][6]), "=f"(tv[u][7])
+              : "l"(a.bval + g));
+        }
       }
 #pragma unroll
-      for (int u = 0; u < U; ++u)
-        if (i0 + u * 32 + lane < hi) ADD(c[u], t[u]);
+      for (int u = 0; u < 2; ++u) {
+        const int64_t g = g0 + u * 256;
+        if (g >= hi) continue;
+        const uint32_t cw[4] = {cv[u].x, cv[u].y, cv[u].z, cv[u].w};
+#pragma unroll
+        for (int e = 0; e < 8; ++e)
+          if (g + e >= lo && g + e < hi) ADD((int)((cw[e >> 1] >> (16 * (e & 1))) & 0xffffu), tv[u][e]);
+      }
     }
   }
   __syncthreads();
@@ -341,7 +463,7 @@ template <typename T>
 __global__ void k_bin_finalize(int64_t n, int bw, int nbin, int ncons, const int32_t* __restrict__ part,
                                int32_t* __restrict__ hi, float* __restrict__ spill, const unsigned* __restrict__ gmax,
                                const T* __restrict__ z, double beta, int add_beta_z, int accumulate, T* w) {
-  const double quantum = ldexp(1.0, bin_exponent(gmax) - 26);
+  const double quantum = *gmax == 0x7f800000u ? 0.0 : ldexp(1.0, bin_exponent(gmax) - 26);
   for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
     const int b = (int)(j / bw);
     const int c = (int)(j - (int64_t)b * bw);
@@ -386,8 +508,15 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
   const int bw = (int)((a.n + nbin - 1) / nbin);
   FP_REQUIRE(bw <= binned_max_bw(), FP_ERR_UNSUPPORTED, "fp_csr: n = %lld too wide for %d column blocks",
              (long long)a.n, nbin);
+  const int mis = (int)(((uintptr_t)a.colidx >> 2) & 3);
+  FP_REQUIRE(((uintptr_t)a.colidx & 3) == 0 && ((uintptr_t)a.val & 3) == 0 &&
+                 (int)(((uintptr_t)a.val >> 2) & 3) == mis,
+             FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs colidx and val with the same 16-byte misalignment",
+             L.variant);
   const int sms = device_info(current_device()).sm_count;
   const int grid = L.grid > 0 ? L.grid : sms;
+  FP_REQUIRE(a.nnz / ((int64_t)grid * (kProdBS / 32)) + a.n < INT32_MAX, FP_ERR_UNSUPPORTED,
+             "fp_csr: variant %d: too many nonzeros per producer warp (grid %d)", L.variant, grid);
   const int ncons = std::max(sms, nbin);
   const int64_t pw = (int64_t)grid * (kProdBS / 32);
   // workspace: [bcol][bval][wsplit][part][gmax]; hi and spill live in a second buffer that is
@@ -412,8 +541,19 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
   k.y = (const float*)a.y;
   k.v = (const float*)a.v;
   k.alpha = (float)a.alpha;
-  k.ny_s = a.y ? (int)y_prefix : 0;
+  // y prefix: what the opt-in shared memory leaves beside the producer's static arrays
+  (void)y_prefix;
+  const void* f = a.y ? (nbin == 2 ? (const void*)k_bin_produce<1, 2> : (const void*)k_bin_produce<1, 1>)
+                      : (nbin == 2 ? (const void*)k_bin_produce<0, 2> : (const void*)k_bin_produce<0, 1>);
+  {
+    cudaFuncAttributes fa{};
+    FP_CUDA(cudaFuncGetAttributes(&fa, f));
+    const int64_t room = ((int64_t)device_info(current_device()).smem_optin_per_block - (int64_t)fa.sharedSizeBytes -
+                          256) / 4 / 4 * 4;
+    k.ny_s = a.y ? (int)std::min<int64_t>(a.n, room) : 0;
+  }
   k.bw = nbin == 2 ? bw : INT32_MAX;
+  k.mis = mis;
   k.bcol = (uint16_t*)take((size_t)a.nnz * 2);
   k.bval = (float*)take((size_t)a.nnz * 4);
   k.wsplit = (int64_t*)take((size_t)pw * 24);
@@ -422,11 +562,10 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
   int32_t* hi = (int32_t*)zbase;
   float* spill = (float*)(zbase + al((size_t)a.n * 4));
   FP_CUDA(cudaMemsetAsync(k.gmax, 0, 16, s));
-  const void* f = a.y ? (const void*)k_bin_produce<1> : (const void*)k_bin_produce<0>;
   set_max_dynamic_smem(f);
   const size_t psmem = (size_t)k.ny_s * 4;
-  if (a.y) k_bin_produce<1><<<grid, kProdBS, psmem, s>>>(k);
-  else k_bin_produce<0><<<grid, kProdBS, psmem, s>>>(k);
+  void* args[] = {&k};
+  FP_CUDA(cudaLaunchKernel(f, dim3(grid), dim3(kProdBS), args, psmem, s));
   FP_CUDA(cudaGetLastError());
   BinCArgs c{k.bcol, k.bval, k.wsplit, k.gmax, part, hi, spill, bw, nbin, pw};
   set_max_dynamic_smem((const void*)k_bin_consume);
@@ -443,7 +582,7 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
 // register count of the producer (plan reports)
 int binned_producer_regs(bool has_y) {
   cudaFuncAttributes fa{};
-  if (cudaFuncGetAttributes(&fa, has_y ? (const void*)k_bin_produce<1> : (const void*)k_bin_produce<0>) !=
+  if (cudaFuncGetAttributes(&fa, has_y ? (const void*)k_bin_produce<1, 2> : (const void*)k_bin_produce<0, 2>) !=
       cudaSuccess) {
     cudaGetLastError();
     return 0;
