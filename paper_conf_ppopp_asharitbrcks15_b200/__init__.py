@@ -96,6 +96,11 @@ _SIGS = {
     "fp_comm_rank": (_int, [_vp]),
     "fp_comm_size": (_int, [_vp]),
     "fp_allreduce": (_int, [_vp, _vp, _i64, _int, _vp]),
+    "fp_comm_enable_peer": (_int, [_vp, _i64, _vp]),
+    "fp_comm_set_mode": (_int, [_vp, _int]),
+    "fp_comm_mode": (_int, [_vp]),
+    "fp_comm_init_local_group": (_int, [_int, _int, _i64, _vp]),
+    "fp_comm_timed_out": (_int, [_vp]),
     "fp_shard_rows_dense": (_int, [_i64, _int, _vp]),
     "fp_shard_rows_csr": (_int, [_i64, _vp, _int, _vp]),
     "fp_dense_dist": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _vp, _vp]),
@@ -148,7 +153,8 @@ def _call(name, *args):
 def _make_raw(name):
     def f(*args):
         r = getattr(lib(), name)(*args)
-        if _SIGS[name][0] is _int and name not in ("fp_comm_rank", "fp_comm_size"):
+        if _SIGS[name][0] is _int and name not in ("fp_comm_rank", "fp_comm_size", "fp_comm_mode",
+                                                    "fp_comm_timed_out"):
             _check(r, name)
         return r
     f.__name__ = name
@@ -401,6 +407,43 @@ class Comm:
     def allreduce(self, t, stream=None):
         _call("fp_allreduce", self.handle, _ptr(t), t.numel(), _dt(t), _stream(t.device, stream))
         return t
+
+    def enable_peer(self, max_bytes, stream=None):
+        """Collective: switch this communicator to the fused peer-memory exchange
+        (FP_COMM_PEER, include/fusedpat.h) for vectors of up to max_bytes."""
+        _call("fp_comm_enable_peer", self.handle, int(max_bytes), _stream(torch.device("cuda", self.device), stream))
+
+    def set_mode(self, mode):
+        _call("fp_comm_set_mode", self.handle, int(mode))
+
+    @property
+    def mode(self):
+        return lib().fp_comm_mode(self.handle)
+
+
+FP_COMM_NCCL, FP_COMM_PEER = 0, 1
+
+
+class LocalGroup:
+    """fp_comm_init_local_group: `nranks` peer-exchange communicators on ONE device (a single
+    process, no NCCL) -- the same fused exchange as across GPUs, between plain allocations.
+    Drive the ranks concurrently (one host thread per rank): each rank's barrier waits for all."""
+
+    def __init__(self, nranks, device=0, max_bytes=1 << 22):
+        arr = (ctypes.c_void_p * nranks)()
+        _call("fp_comm_init_local_group", int(nranks), int(device), int(max_bytes), ctypes.cast(arr, ctypes.c_void_p))
+        self.comms = []
+        for r in range(nranks):
+            c = Comm.__new__(Comm)
+            c.rank, c.size, c.device, c.handle = r, nranks, int(device), ctypes.c_void_p(arr[r])
+            self.comms.append(c)
+
+    def timed_out(self):
+        return any(lib().fp_comm_timed_out(c.handle) == 1 for c in self.comms)
+
+    def close(self):
+        for c in self.comms:
+            c.close()
 
 
 def dense_dist(comm, X_local, y=None, v_local=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
