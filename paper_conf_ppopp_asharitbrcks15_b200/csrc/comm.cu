@@ -8,11 +8,38 @@
 #include <string.h>
 
 #include <algorithm>
+#include <chrono>
+#include <condition_variable>
+#include <memory>
+#include <mutex>
 #include <vector>
 
 #include "kernels.cuh"
 
 constexpr int kMaxPeers = 8;  // one NVSwitch node
+
+// Host rendezvous of a single-process local group.  A device allocation is an implicit
+// synchronisation point between streams: a rank allocating its workspace on its first call
+// would wait for another rank's barrier kernel, which waits for the allocating rank -- so the
+// ranks of one process meet on the host before any of them launches its barrier kernel (by
+// then every rank has finished allocating).  Not needed across processes.
+struct LocalSync {
+  std::mutex mu;
+  std::condition_variable cv;
+  int P = 1, count = 0;
+  uint64_t gen = 0;
+  bool arrive_and_wait() {
+    std::unique_lock<std::mutex> lk(mu);
+    const uint64_t g = gen;
+    if (++count == P) {
+      count = 0;
+      ++gen;
+      cv.notify_all();
+      return true;
+    }
+    return cv.wait_for(lk, std::chrono::seconds(30), [&] { return gen != g; });
+  }
+};
 
 // Peer (P2P) exchange state.  Every rank owns a symmetric buffer [D0: cap][D1: cap][flags:
 // kMaxPeers x u64] mapped into every other rank (CUDA IPC across processes, plain pointers in a
@@ -33,6 +60,7 @@ struct fp_comm {
   bool ipc_mapped[kMaxPeers] = {};            // opened with cudaIpcOpenMemHandle
   uint64_t epoch = 0;
   unsigned* timeout_flag = nullptr;           // device: set if a barrier gave up waiting
+  std::shared_ptr<LocalSync> lsync;           // local groups only
 };
 
 namespace fp {
@@ -128,6 +156,15 @@ __global__ void k_peer_sum(const PeerTab t, int64_t n, const T* __restrict__ z, 
   }
 }
 
+__global__ void k_copy_bytes(unsigned char* __restrict__ d, const unsigned char* __restrict__ s, size_t bytes) {
+  const size_t n16 = ((uintptr_t)d % 16 == 0 && (uintptr_t)s % 16 == 0) ? bytes / 16 : 0;
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += (size_t)gridDim.x * blockDim.x)
+    reinterpret_cast<uint4*>(d)[i] = reinterpret_cast<const uint4*>(s)[i];
+  for (size_t i = n16 * 16 + (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < bytes;
+       i += (size_t)gridDim.x * blockDim.x)
+    d[i] = s[i];
+}
+
 PeerTab peer_tab(const fp_comm* c) {
   PeerTab t{};
   for (int k = 0; k < c->size; ++k) t.p[k] = c->peer[k];
@@ -160,6 +197,7 @@ fp_status peer_begin(fp_comm* c, size_t bytes, cudaStream_t s, void** D) {
 
 // Finish call e: barrier, then w = sum_k D_k + beta z.
 fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double beta, void* w, cudaStream_t s) {
+  if (c->lsync) FP_REQUIRE(c->lsync->arrive_and_wait(), FP_ERR_CUDA, "local group: ranks did not meet within 30 s");
   const PeerTab t = peer_tab(c);
   k_peer_barrier<<<1, 32, 0, s>>>(t);
   FP_CUDA(cudaGetLastError());
@@ -251,7 +289,10 @@ fp_status fp_allreduce(fp_comm* comm, void* buf, int64_t n, fp_dtype dtype, fp_s
     const size_t bytes = (size_t)n * fp::dtype_size(dtype);
     fp_status st = peer_begin(comm, bytes, s, &D);
     if (st != FP_OK) return st;
-    FP_CUDA(cudaMemcpyAsync(D, buf, bytes, cudaMemcpyDeviceToDevice, s));
+    // a kernel, not cudaMemcpyAsync: a same-device copy may serialise against other streams
+    const int grid = (int)std::min<int64_t>(((int64_t)bytes / 16 + 255) / 256 + 1, 1024);
+    k_copy_bytes<<<grid, 256, 0, s>>>((unsigned char*)D, (const unsigned char*)buf, bytes);
+    FP_CUDA(cudaGetLastError());
     return peer_finish(comm, n, dtype, nullptr, 0.0, buf, s);
   }
   FP_REQUIRE(comm->nccl, FP_ERR_INVALID_ARG, "fp_allreduce: communicator has no NCCL backend (local group)");
@@ -359,8 +400,12 @@ fp_status fp_comm_init_local_group(int nranks, int device, int64_t max_bytes, fp
       return st;
     }
   }
-  for (int r = 0; r < nranks; ++r)
+  auto sync = std::make_shared<LocalSync>();
+  sync->P = nranks;
+  for (int r = 0; r < nranks; ++r) {
     for (int k = 0; k < nranks; ++k) comms[r]->peer[k] = comms[k]->sym;
+    comms[r]->lsync = sync;
+  }
   return FP_OK;
 }
 
