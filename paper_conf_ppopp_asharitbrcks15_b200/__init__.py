@@ -97,6 +97,7 @@ _SIGS = {
     "fp_comm_size": (_int, [_vp]),
     "fp_allreduce": (_int, [_vp, _vp, _i64, _int, _vp]),
     "fp_comm_enable_peer": (_int, [_vp, _i64, _vp]),
+    "fp_comm_enable_nvls": (_int, [_vp, _i64, _vp]),
     "fp_comm_set_mode": (_int, [_vp, _int]),
     "fp_comm_mode": (_int, [_vp]),
     "fp_comm_init_local_group": (_int, [_int, _int, _i64, _vp]),
@@ -413,6 +414,10 @@ class Comm:
         (FP_COMM_PEER, include/fusedpat.h) for vectors of up to max_bytes."""
         _call("fp_comm_enable_peer", self.handle, int(max_bytes), _stream(torch.device("cuda", self.device), stream))
 
+    def enable_nvls(self, max_bytes, stream=None):
+        """Collective: switch to the NVSwitch multicast exchange (FP_COMM_NVLS)."""
+        _call("fp_comm_enable_nvls", self.handle, int(max_bytes), _stream(torch.device("cuda", self.device), stream))
+
     def set_mode(self, mode):
         _call("fp_comm_set_mode", self.handle, int(mode))
 
@@ -421,7 +426,7 @@ class Comm:
         return lib().fp_comm_mode(self.handle)
 
 
-FP_COMM_NCCL, FP_COMM_PEER = 0, 1
+FP_COMM_NCCL, FP_COMM_PEER, FP_COMM_NVLS = 0, 1, 2
 
 
 class LocalGroup:

@@ -4,6 +4,7 @@
 // Eq. (1) is a sum over rows of X[r,:]^T (v[r] X[r,:] y) (Eq. 2/3), so a row
 // partition needs exactly one exchange: the n-vector sum of per-rank partials.  beta*z is
 // added on rank 0 only (reading R18).  The paper is single-GPU; this layer is new.
+#include <cuda.h>
 #include <nccl.h>
 #include <string.h>
 
@@ -61,6 +62,13 @@ struct fp_comm {
   uint64_t epoch = 0;
   unsigned* timeout_flag = nullptr;           // device: set if a barrier gave up waiting
   std::shared_ptr<LocalSync> lsync;           // local groups only
+  // NVLS (FP_COMM_NVLS): one multicast object over all ranks' physical buffers (same layout
+  // as sym); uc = this rank's unicast mapping, mc = the multicast mapping
+  CUmemGenericAllocationHandle mc_handle = 0, ph_handle = 0;
+  unsigned char* uc = nullptr;
+  unsigned char* mc = nullptr;
+  size_t mc_size = 0;
+  bool nvls = false;
 };
 
 namespace fp {
@@ -165,6 +173,49 @@ __global__ void k_copy_bytes(unsigned char* __restrict__ d, const unsigned char*
     d[i] = s[i];
 }
 
+// NVLS barrier: one multimem red increments the epoch counter in EVERY rank's copy (release,
+// system scope); then wait until the local copy reaches P * epoch (acquire).
+__global__ void k_nvls_barrier(unsigned long long* mc_cnt, const unsigned long long* uc_cnt, unsigned long long target,
+                               unsigned* timeout_flag) {
+  if (threadIdx.x != 0) return;
+  __threadfence_system();
+  asm volatile("multimem.red.release.sys.global.add.u64 [%0], %1;" ::"l"(mc_cnt), "l"(1ull) : "memory");
+  uint64_t t0, now;
+  unsigned long long v;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  while (true) {
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(uc_cnt) : "memory");
+    if (v >= target) break;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+    if (now - t0 > 20000000000ull) {
+      atomicExch(timeout_flag, 1u);
+      break;
+    }
+    __nanosleep(100);
+  }
+}
+
+// w[j] = (in-switch sum over ranks of D[j]) + beta z[j]: multimem.ld_reduce on the multicast
+// address returns the sum of every rank's copy in one load
+__device__ __forceinline__ double ld_reduce(const double* p) {
+  double v;
+  asm volatile("multimem.ld_reduce.relaxed.sys.global.add.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ float ld_reduce(const float* p) {
+  float v;
+  asm volatile("multimem.ld_reduce.relaxed.sys.global.add.f32 %0, [%1];" : "=f"(v) : "l"(p) : "memory");
+  return v;
+}
+template <typename T>
+__global__ void k_nvls_sum(const T* mcD, int64_t n, const T* __restrict__ z, double beta, T* w) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    double s = (double)ld_reduce(mcD + j);
+    if (z && beta != 0.0) s += beta * (double)z[j];
+    w[j] = (T)s;
+  }
+}
+
 PeerTab peer_tab(const fp_comm* c) {
   PeerTab t{};
   for (int k = 0; k < c->size; ++k) t.p[k] = c->peer[k];
@@ -191,13 +242,30 @@ fp_status peer_begin(fp_comm* c, size_t bytes, cudaStream_t s, void** D) {
   FP_REQUIRE(!capturing(s), FP_ERR_UNSUPPORTED,
              "peer exchange: not capturable in a CUDA graph (its epoch advances per call); use NCCL mode");
   c->epoch += 1;
-  *D = c->sym + (c->epoch & 1) * c->cap;
+  *D = (c->nvls ? c->uc : c->sym) + (c->epoch & 1) * c->cap;
   return FP_OK;
 }
 
 // Finish call e: barrier, then w = sum_k D_k + beta z.
 fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double beta, void* w, cudaStream_t s) {
   if (c->lsync) FP_REQUIRE(c->lsync->arrive_and_wait(), FP_ERR_CUDA, "local group: ranks did not meet within 30 s");
+  if (c->nvls) {
+    unsigned long long* cnt_off = (unsigned long long*)(2 * c->cap);
+    k_nvls_barrier<<<1, 32, 0, s>>>((unsigned long long*)(c->mc + (size_t)cnt_off),
+                                    (const unsigned long long*)(c->uc + (size_t)cnt_off),
+                                    (unsigned long long)c->size * c->epoch, c->timeout_flag);
+    FP_CUDA(cudaGetLastError());
+    const int grid = (int)std::min<int64_t>((n + 255) / 256, 4 * fp::device_info(c->device).sm_count);
+    const size_t off = (c->epoch & 1) * c->cap;
+    if (n > 0) {
+      if (dt == FP_F64)
+        k_nvls_sum<double><<<grid, 256, 0, s>>>((const double*)(c->mc + off), n, (const double*)z, beta, (double*)w);
+      else
+        k_nvls_sum<float><<<grid, 256, 0, s>>>((const float*)(c->mc + off), n, (const float*)z, beta, (float*)w);
+      FP_CUDA(cudaGetLastError());
+    }
+    return FP_OK;
+  }
   const PeerTab t = peer_tab(c);
   k_peer_barrier<<<1, 32, 0, s>>>(t);
   FP_CUDA(cudaGetLastError());
@@ -210,7 +278,20 @@ fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double 
   return FP_OK;
 }
 
+// Load the exchange kernels now (lazy module loading would load them at their first launch,
+// and a load synchronises the device: in a single-process group a rank could then wait, before
+// launching its barrier kernel, for another rank's barrier kernel that waits for it).
+void preload_exchange_kernels() {
+  cudaFuncAttributes fa;
+  const void* ks[] = {(const void*)k_peer_barrier, (const void*)k_peer_sum<float>, (const void*)k_peer_sum<double>,
+                      (const void*)k_copy_bytes, (const void*)k_nvls_barrier, (const void*)k_nvls_sum<float>,
+                      (const void*)k_nvls_sum<double>};
+  for (const void* k : ks)
+    if (cudaFuncGetAttributes(&fa, k) != cudaSuccess) cudaGetLastError();
+}
+
 fp_status alloc_sym(fp_comm* c, size_t cap) {
+  preload_exchange_kernels();
   const size_t bytes = 2 * cap + kMaxPeers * sizeof(uint64_t);
   FP_CUDA(cudaSetDevice(c->device));
   FP_CUDA(cudaMalloc((void**)&c->sym, bytes));
@@ -220,6 +301,164 @@ fp_status alloc_sym(fp_comm* c, size_t cap) {
   c->cap = cap;
   c->peer[c->rank] = c->sym;
   return FP_OK;
+}
+
+// ---- CUDA driver entry points for NVLS (no link-time dependency on libcuda)
+template <typename F>
+bool drv(const char* name, F*& f) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  f = reinterpret_cast<F*>(p);
+  return true;
+}
+
+#define FP_CU(call)                                                              \
+  do {                                                                           \
+    CUresult r_ = (call);                                                        \
+    if (r_ != CUDA_SUCCESS) {                                                    \
+      fp::set_error("NVLS: %s failed (CUresult %d)", #call, (int)r_);            \
+      return FP_ERR_CUDA;                                                        \
+    }                                                                            \
+  } while (0)
+
+struct Drv {
+  decltype(&cuMulticastCreate) mcCreate = nullptr;
+  decltype(&cuMulticastAddDevice) mcAdd = nullptr;
+  decltype(&cuMulticastBindMem) mcBind = nullptr;
+  decltype(&cuMulticastUnbind) mcUnbind = nullptr;
+  decltype(&cuMulticastGetGranularity) mcGran = nullptr;
+  decltype(&cuMemCreate) memCreate = nullptr;
+  decltype(&cuMemRelease) memRelease = nullptr;
+  decltype(&cuMemAddressReserve) vaReserve = nullptr;
+  decltype(&cuMemAddressFree) vaFree = nullptr;
+  decltype(&cuMemMap) memMap = nullptr;
+  decltype(&cuMemUnmap) memUnmap = nullptr;
+  decltype(&cuMemSetAccess) memSetAccess = nullptr;
+  decltype(&cuMemGetAllocationGranularity) memGran = nullptr;
+  decltype(&cuMemExportToShareableHandle) memExport = nullptr;
+  decltype(&cuMemImportFromShareableHandle) memImport = nullptr;
+  bool ok = false;
+};
+const Drv& driver() {
+  static Drv d = [] {
+    Drv x;
+    x.ok = drv("cuMulticastCreate", x.mcCreate) && drv("cuMulticastAddDevice", x.mcAdd) &&
+           drv("cuMulticastBindMem", x.mcBind) && drv("cuMulticastUnbind", x.mcUnbind) &&
+           drv("cuMulticastGetGranularity", x.mcGran) && drv("cuMemCreate", x.memCreate) &&
+           drv("cuMemRelease", x.memRelease) && drv("cuMemAddressReserve", x.vaReserve) &&
+           drv("cuMemAddressFree", x.vaFree) && drv("cuMemMap", x.memMap) && drv("cuMemUnmap", x.memUnmap) &&
+           drv("cuMemSetAccess", x.memSetAccess) && drv("cuMemGetAllocationGranularity", x.memGran) &&
+           drv("cuMemExportToShareableHandle", x.memExport) &&
+           drv("cuMemImportFromShareableHandle", x.memImport);
+    return x;
+  }();
+  return d;
+}
+
+fp_status nccl_barrier(fp_comm* c, cudaStream_t s) {
+  float* d = nullptr;
+  FP_CUDA(cudaMalloc((void**)&d, sizeof(float)));
+  ncclResult_t r = ncclAllReduce(d, d, 1, ncclFloat32, ncclSum, c->nccl, s);
+  cudaStreamSynchronize(s);
+  cudaFree(d);
+  if (r != ncclSuccess) return fp::nccl_fail(r, "ncclAllReduce(barrier)");
+  return FP_OK;
+}
+
+fp_status nvls_setup(fp_comm* c, size_t cap, cudaStream_t s) {
+  const Drv& D = driver();
+  FP_REQUIRE(D.ok, FP_ERR_UNSUPPORTED, "NVLS: CUDA driver multicast entry points unavailable");
+  int mcsup = 0;
+  cudaDeviceGetAttribute(&mcsup, (cudaDeviceAttr)CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, c->device);
+  FP_REQUIRE(mcsup, FP_ERR_UNSUPPORTED, "NVLS: device %d does not support multicast", c->device);
+  CUmulticastObjectProp mp{};
+  mp.numDevices = (unsigned)c->size;
+  mp.handleTypes = CU_MEM_HANDLE_TYPE_FABRIC;
+  const size_t want = 2 * cap + 256;
+  mp.size = want;
+  size_t gmc = 0, gph = 0;
+  FP_CU(D.mcGran(&gmc, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED));
+  CUmemAllocationProp pp{};
+  pp.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  pp.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  pp.location.id = c->device;
+  FP_CU(D.memGran(&gph, &pp, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED));
+  const size_t g = gmc > gph ? gmc : gph;
+  const size_t size = (want + g - 1) / g * g;
+  mp.size = size;
+  // the multicast object: created on rank 0, imported elsewhere through a fabric handle
+  unsigned char* dh = nullptr;
+  if (c->size > 1) FP_CUDA(cudaMalloc((void**)&dh, sizeof(CUmemFabricHandle)));
+  if (c->rank == 0) {
+    // fabric handles (what the other ranks import); a POSIX-fd type for a single rank if the
+    // fabric type is refused
+    CUresult cr = D.mcCreate(&c->mc_handle, &mp);
+    if (cr != CUDA_SUCCESS && c->size == 1) {
+      mp.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+      cr = D.mcCreate(&c->mc_handle, &mp);
+    }
+    FP_CU(cr);
+    if (c->size > 1) {
+      CUmemFabricHandle fh;
+      FP_CU(D.memExport(&fh, c->mc_handle, CU_MEM_HANDLE_TYPE_FABRIC, 0));
+      FP_CUDA(cudaMemcpy(dh, &fh, sizeof(fh), cudaMemcpyHostToDevice));
+    }
+  }
+  if (c->size > 1) {
+    ncclResult_t r = ncclBroadcast(dh, dh, sizeof(CUmemFabricHandle), ncclUint8, 0, c->nccl, s);
+    if (r != ncclSuccess) return fp::nccl_fail(r, "ncclBroadcast(fabric handle)");
+    CUmemFabricHandle fh;
+    FP_CUDA(cudaMemcpyAsync(&fh, dh, sizeof(fh), cudaMemcpyDeviceToHost, s));
+    FP_CUDA(cudaStreamSynchronize(s));
+    cudaFree(dh);
+    if (c->rank != 0) FP_CU(D.memImport(&c->mc_handle, &fh, CU_MEM_HANDLE_TYPE_FABRIC));
+  }
+  CUdevice dev = (CUdevice)c->device;
+  FP_CU(D.mcAdd(c->mc_handle, dev));
+  if (c->size > 1) {
+    fp_status st = nccl_barrier(c, s);  // every device added before any binds
+    if (st != FP_OK) return st;
+  }
+  FP_CU(D.memCreate(&c->ph_handle, size, &pp, 0));
+  FP_CU(D.mcBind(c->mc_handle, 0, c->ph_handle, 0, size, 0));
+  CUdeviceptr uva = 0, mva = 0;
+  FP_CU(D.vaReserve(&uva, size, g, 0, 0));
+  FP_CU(D.memMap(uva, size, 0, c->ph_handle, 0));
+  FP_CU(D.vaReserve(&mva, size, g, 0, 0));
+  FP_CU(D.memMap(mva, size, 0, c->mc_handle, 0));
+  CUmemAccessDesc ad{};
+  ad.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ad.location.id = c->device;
+  ad.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  FP_CU(D.memSetAccess(uva, size, &ad, 1));
+  FP_CU(D.memSetAccess(mva, size, &ad, 1));
+  c->uc = (unsigned char*)uva;
+  c->mc = (unsigned char*)mva;
+  c->mc_size = size;
+  c->cap = cap;
+  c->nvls = true;
+  FP_CUDA(cudaMemset(c->uc, 0, size));
+  FP_CUDA(cudaDeviceSynchronize());
+  if (c->size > 1) return nccl_barrier(c, s);  // every copy zeroed before any red lands
+  return FP_OK;
+}
+
+void nvls_release(fp_comm* c) {
+  const Drv& D = driver();
+  if (!D.ok) return;
+  cudaDeviceSynchronize();
+  if (c->mc) D.memUnmap((CUdeviceptr)c->mc, c->mc_size), D.vaFree((CUdeviceptr)c->mc, c->mc_size);
+  if (c->uc) D.memUnmap((CUdeviceptr)c->uc, c->mc_size), D.vaFree((CUdeviceptr)c->uc, c->mc_size);
+  if (c->mc_handle && c->ph_handle) D.mcUnbind(c->mc_handle, (CUdevice)c->device, 0, c->mc_size);
+  if (c->ph_handle) D.memRelease(c->ph_handle);
+  if (c->mc_handle) D.memRelease(c->mc_handle);
+  c->mc = c->uc = nullptr;
+  c->mc_handle = c->ph_handle = 0;
+  c->nvls = false;
 }
 
 }  // namespace
@@ -268,6 +507,7 @@ fp_status fp_comm_destroy(fp_comm* comm) {
     if (comm->ipc_mapped[k]) cudaIpcCloseMemHandle(comm->peer[k]);
   if (comm->sym) cudaFree(comm->sym);
   if (comm->timeout_flag) cudaFree(comm->timeout_flag);
+  if (comm->nvls) nvls_release(comm);
   ncclResult_t r = comm->nccl ? ncclCommDestroy(comm->nccl) : ncclSuccess;
   delete comm;
   if (r != ncclSuccess) return fp::nccl_fail(r, "ncclCommDestroy");
@@ -283,7 +523,7 @@ fp_status fp_allreduce(fp_comm* comm, void* buf, int64_t n, fp_dtype dtype, fp_s
   // no short cut for one rank: the collective runs (a copy in place) so that every *_dist call
   // exercises the same NCCL path at any world size
   if (n == 0) return FP_OK;
-  if (comm->mode == FP_COMM_PEER) {
+  if (comm->mode == FP_COMM_PEER || comm->mode == FP_COMM_NVLS) {
     cudaStream_t s = (cudaStream_t)stream;
     void* D = nullptr;
     const size_t bytes = (size_t)n * fp::dtype_size(dtype);
@@ -369,10 +609,37 @@ fp_status fp_comm_enable_peer(fp_comm* comm, int64_t max_bytes, fp_stream stream
   return FP_OK;
 }
 
+// NVLS: one multicast object (CUDA driver API, resolved at run time) over every rank's buffer.
+// Rank 0 creates it and exports a fabric handle, broadcast through NCCL; every rank adds its
+// device, binds a physical allocation and maps both the unicast and the multicast range.
+fp_status fp_comm_enable_nvls(fp_comm* comm, int64_t max_bytes, fp_stream stream) {
+  FP_REQUIRE(comm && max_bytes > 0, FP_ERR_INVALID_ARG, "fp_comm_enable_nvls: bad arguments");
+  if (comm->nvls) {
+    FP_REQUIRE((size_t)max_bytes <= comm->cap, FP_ERR_INVALID_ARG, "fp_comm_enable_nvls: already enabled smaller");
+    comm->mode = FP_COMM_NVLS;
+    return FP_OK;
+  }
+  FP_REQUIRE(!comm->sym, FP_ERR_UNSUPPORTED, "fp_comm_enable_nvls: peer mode already enabled on this communicator");
+  FP_REQUIRE(comm->nccl, FP_ERR_INVALID_ARG, "fp_comm_enable_nvls: needs an NCCL communicator");
+  FP_CUDA(cudaSetDevice(comm->device));
+  preload_exchange_kernels();
+  cudaStream_t s = (cudaStream_t)stream;
+  fp_status st = nvls_setup(comm, ((size_t)max_bytes + 255) / 256 * 256, s);
+  if (st != FP_OK) {
+    nvls_release(comm);
+    return st;
+  }
+  FP_CUDA(cudaMalloc((void**)&comm->timeout_flag, sizeof(unsigned)));
+  FP_CUDA(cudaMemset(comm->timeout_flag, 0, sizeof(unsigned)));
+  comm->mode = FP_COMM_NVLS;
+  return FP_OK;
+}
+
 fp_status fp_comm_set_mode(fp_comm* comm, int mode) {
-  FP_REQUIRE(comm && (mode == FP_COMM_NCCL || mode == FP_COMM_PEER), FP_ERR_INVALID_ARG,
+  FP_REQUIRE(comm && (mode == FP_COMM_NCCL || mode == FP_COMM_PEER || mode == FP_COMM_NVLS), FP_ERR_INVALID_ARG,
              "fp_comm_set_mode: bad arguments");
   FP_REQUIRE(mode != FP_COMM_PEER || comm->sym, FP_ERR_INVALID_ARG, "fp_comm_set_mode: peer mode not enabled");
+  FP_REQUIRE(mode != FP_COMM_NVLS || comm->nvls, FP_ERR_INVALID_ARG, "fp_comm_set_mode: NVLS not enabled");
   FP_REQUIRE(mode != FP_COMM_NCCL || comm->nccl, FP_ERR_INVALID_ARG, "fp_comm_set_mode: no NCCL backend");
   comm->mode = mode;
   return FP_OK;
@@ -423,7 +690,7 @@ fp_status fp_dense_dist(int64_t m_local, int64_t n, const void* X, int64_t ld, c
                         fp_stream stream) {
   FP_REQUIRE(comm, FP_ERR_INVALID_ARG, "fp_dense_dist: comm is NULL");
   fp::PatternArgs a = fp::dense_args(m_local, n, X, ld, y, v, z, alpha, beta, w, dtype);
-  if (comm->mode == FP_COMM_PEER) return dist_peer(a, false, comm, (cudaStream_t)stream);
+  if (comm->mode != FP_COMM_NCCL) return dist_peer(a, false, comm, (cudaStream_t)stream);
   a.add_beta_z = comm->rank == 0;
   fp_status st = fp::run_dense(a, nullptr, (cudaStream_t)stream);
   if (st != FP_OK) return st;
@@ -435,7 +702,7 @@ fp_status fp_csr_dist(int64_t m_local, int64_t n, int64_t nnz_local, const int64
                       void* w, fp_dtype dtype, fp_comm* comm, fp_stream stream) {
   FP_REQUIRE(comm, FP_ERR_INVALID_ARG, "fp_csr_dist: comm is NULL");
   fp::PatternArgs a = fp::csr_args(m_local, n, nnz_local, rowptr, colidx, val, y, v, z, alpha, beta, w, dtype);
-  if (comm->mode == FP_COMM_PEER) return dist_peer(a, true, comm, (cudaStream_t)stream);
+  if (comm->mode != FP_COMM_NCCL) return dist_peer(a, true, comm, (cudaStream_t)stream);
   a.add_beta_z = comm->rank == 0;
   fp_status st = fp::run_csr(a, nullptr, (cudaStream_t)stream);
   if (st != FP_OK) return st;

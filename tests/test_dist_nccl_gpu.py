@@ -72,6 +72,55 @@ def test_nccl_allreduce_runs_one_rank(cuda_dev):
     assert n_ar >= 2, "NCCL logged no AllReduce launch:\n" + out[-4000:]
 
 
+def test_nvls_one_rank(cuda_dev):
+    """FP_COMM_NVLS on a one-rank communicator: the multicast object, the multimem.red
+    barrier and the multimem.ld_reduce sum run on the hardware (with one device the switch
+    sums one copy); integer twins bit-exact, three calls (both buffer parities), allreduce."""
+    import ctypes
+
+    import oracle
+    import paper_conf_ppopp_asharitbrcks15_b200 as fp
+    import synth
+    from _util import assert_bitexact
+
+    uid = (ctypes.c_ubyte * 128)()
+    fp.fp_comm_get_unique_id(ctypes.cast(uid, ctypes.c_void_p))
+    h = ctypes.c_void_p()
+    fp.fp_comm_init(ctypes.byref(h), 1, 0, ctypes.cast(uid, ctypes.c_void_p), 0)
+    c = fp.Comm.__new__(fp.Comm)
+    c.rank, c.size, c.device, c.handle = 0, 1, 0, h
+    try:
+        try:
+            c.enable_nvls(1 << 20)
+        except fp.FusedPatError as e:
+            pytest.skip(f"no NVLS here: {e}")
+        assert c.mode == fp.FP_COMM_NVLS
+        n = 3000
+        rp, ci, va = synth.csr(40_000, n, "f32", ("powerlaw", 2.5, 13.64), kind="int_pm12", seed=31)
+        y = synth.vector(n, "f32", kind="int_small", seed=31, stream=synth.S_Y)
+        z = synth.vector(n, "f32", kind="int_small", seed=31, stream=synth.S_Z)
+        v = synth.vector(40_000, "f32", kind="int_pos", seed=31, stream=synth.S_V)
+        ref, _ = oracle.csr(40_000, n, rp, ci, va, y, v, z, 1.0, 3.0)
+        d = cuda_dev
+        for _ in range(3):
+            w = fp.csr_dist(c, rp.to(d), ci.to(d), va.to(d), n, y.to(d), v.to(d), z.to(d), 1.0, 3.0)
+            torch.cuda.synchronize()
+            assert_bitexact(w, ref, "nvls csr_dist")
+        X = synth.dense(5000, 64, "f64", kind="int_pm12", seed=32)
+        y2 = synth.vector(64, "f64", kind="int_small", seed=32)
+        ref, _ = oracle.dense(X, y2, None, None, 2.0, 0.0)
+        w = fp.dense_dist(c, X.to(d), y2.to(d), None, None, 2.0, 0.0)
+        torch.cuda.synchronize()
+        assert_bitexact(w, ref, "nvls dense_dist")
+        t = torch.arange(1000, dtype=torch.float64, device=d)
+        c.allreduce(t)
+        torch.cuda.synchronize()
+        assert torch.equal(t.cpu(), torch.arange(1000, dtype=torch.float64))
+        assert fp.lib().fp_comm_timed_out(h) == 0
+    finally:
+        fp.fp_comm_destroy(h)
+
+
 def _worker(rank, world, port, q):
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -118,6 +167,33 @@ def _worker(rank, world, port, q):
             torch.cuda.synchronize()
             assert_bitexact(w, full, f"csr_dist {dt} rank {rank}")
             msgs.append(f"csr-int-{dt}")
+
+        # ---- the same exchange over peer memory (CUDA IPC) and over NVLS multicast
+        mm, nn = 60000, 20000
+        rp, ci, va = synth.csr(mm, nn, "f32", ("powerlaw", 2.5, 13.64), kind="int_pm12", seed=12)
+        yy = synth.vector(nn, "f32", kind="int_small", seed=12, stream=synth.S_Y)
+        zz = synth.vector(nn, "f32", kind="int_small", seed=12, stream=synth.S_Z)
+        vv = synth.vector(mm, "f32", kind="int_pos", seed=12, stream=synth.S_V)
+        full, _ = oracle.csr(mm, nn, rp, ci, va, yy, vv, zz, 1.0, 1.0)
+        bb = fp.shard_rows_csr(rp, world)
+        lrp, lci, lva, lv = (t.contiguous().to(dev) for t in fp.shard_slice_csr(rp, ci, va, vv, bb, rank))
+        for mode, enable in ((fp.FP_COMM_PEER, comm.enable_peer), (fp.FP_COMM_NVLS, comm.enable_nvls)):
+            cm = fp.Comm(device=rank)  # a fresh communicator per mode
+            try:
+                try:
+                    (cm.enable_peer if mode == fp.FP_COMM_PEER else cm.enable_nvls)(nn * 8)
+                except fp.FusedPatError:
+                    if mode == fp.FP_COMM_NVLS:
+                        msgs.append("nvls-unsupported")
+                        continue
+                    raise
+                for _ in range(3):
+                    w = fp.csr_dist(cm, lrp, lci, lva, nn, yy.to(dev), lv, zz.to(dev), 1.0, 1.0)
+                    torch.cuda.synchronize()
+                    assert_bitexact(w, full, f"csr_dist mode {mode} rank {rank}")
+                msgs.append(f"mode-{mode}")
+            finally:
+                cm.close()
 
         # ---- CSR fp32 U[-1,1): north_star tolerance
         mm, nn = 80000, 3000
