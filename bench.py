@@ -38,12 +38,12 @@ sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402
 
+COLS = "strat"  # --cols
 METRIC = "fused-pattern GB/s of X streamed and % of B200 HBM peak; evals/s at 1/2/4/8 GPU"
 FALLBACK_HBM_GBS = 6650.0
 
 
 # ------------------------------------------------------------------------------ helpers
-READ_CEILING_GBS = 7371.0  # measured pure HBM read stream, best setting (profiles/r01_read_ceiling.md)
 
 
 def peaks():
@@ -54,15 +54,58 @@ def peaks():
     return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def traffic_for(config):
-    """dram__bytes_read.sum + dram__bytes_write.sum per launch of the dominant kernel, from the
-    committed ncu --set full capture summary (profiles/), or None."""
+def traffic_for(config, variant):
+    """dram__bytes_read.sum + dram__bytes_write.sum of one step (every kernel of the fp_* call),
+    from the committed ncu --set full captures (profiles/ncu_traffic.json, tools/ncu_summary.py).
+    ncu cannot run inside the timed region, so this is the capture of the same build and plan
+    variant; a capture of another variant is reported as stale (value None)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
+        return None, "no capture"
+    e = json.load(open(p)).get(config)
+    if e is None:
+        return None, "no capture"
+    src = f"ncu --set full capture {e.get('round', '?')} ({e.get('file', '?')})"
+    if e.get("variant") is not None and variant is not None and int(e["variant"]) != int(variant):
+        return None, f"stale: {src} is of plan variant {e['variant']}, this run uses {variant}"
+    return e.get("dram_bytes_per_step", e.get("dram_bytes_per_launch")), src
+
+
+def second_ceiling(cfg, plan, nnz, kern_ms, dev):
+    """SURVEY 8(d) C4 'second ceiling': the random on-chip accesses of the CSR paths (y gathers
+    that miss the shared-memory copy of y, w updates) at the rates the device sustains, measured
+    live by fp_probe_rates in this run.  floor_ms = the time those accesses alone need;
+    frac = floor_ms / the measured step.  Uniform columns assumed for the prefix hit share."""
+    import paper_conf_ppopp_asharitbrcks15_b200 as fp
+
+    if cfg["fmt"] != "csr" or plan is None:
         return None
-    d = json.load(open(p))
-    e = d.get(config)
-    return None if e is None else e.get("dram_bytes_per_launch")
+    n = cfg["n"]
+    s = 8 if cfg["dtype"] == "f64" else 4
+    r = fp.probe_rates(min(n, 1 << 30), smem_elems=min(max(n, 1), 25600), device=dev.index)
+    v = int(plan.variant)
+    ops, floor = {}, 0.0
+    if v in (3, 5, 6, 8):  # y and the partial w in shared memory
+        ops = {"smem_gathers": nnz, "smem_fp_atomics": nnz}
+        floor = nnz / r["gather_smem_f64"] + nnz / r["atom_smem_f64"]
+        what = "y gathers from shared memory + shared-memory fp atomics (a CAS loop) per nonzero"
+    elif v in (4, 7, 16, 17):
+        prefix = min(n, int(plan.smem_bytes) // s) if v in (16, 17) else 0
+        g = int(nnz * (1.0 - prefix / n))
+        if v == 17:
+            ops = {"l2_gathers": g, "smem_int_atomics": nnz}
+            floor = g / r["gather_l2"] + nnz / r["atom_smem_u32"]
+            what = ("producer: y gathers beyond the shared-memory prefix (L1/L2); consumer: one native "
+                    "int32 shared atomic per nonzero")
+        else:
+            ops = {"l2_gathers": g, "l2_reds": nnz}
+            floor = g / r["gather_l2"] + nnz / r["red_l2"]
+            what = "y gathers beyond the shared-memory prefix + one fp red.global per nonzero (L1/L2)"
+    else:
+        return None
+    return {"what": what, "ops_per_step": ops, "rates_ops_per_s": {k: round(x / 1e9, 2) for k, x in r.items()},
+            "rates_unit": "G ops/s (fp_probe_rates, live)", "floor_ms": round(floor * 1e3, 4),
+            "frac": round(floor * 1e3 / kern_ms, 4)}
 
 
 class ClockSampler:
@@ -140,7 +183,9 @@ def algorithmic_bytes(cfg, m, nnz):
 def build_inputs(name, rank, world, dev):
     """This rank's row shard of config `name`, generated in HBM (bit-identical to the slice of
     the full matrix, synth/ is counter-based)."""
-    cfg = synth.CONFIGS[name]
+    cfg = dict(synth.CONFIGS[name])
+    if COLS == "iid" and cfg["fmt"] == "csr" and cfg.get("col_skew", 0) == 0:
+        cfg["col_skew"] = -1
     seed = synth.config_seed(name)
     m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
     import paper_conf_ppopp_asharitbrcks15_b200 as fp
@@ -357,15 +402,22 @@ def run_gpu(args):
     value = x_bytes * passes_per_step * evals_per_s / 1e9
     peak, peak_src = peaks()
     achieved = alg_local * passes_per_step / (kern_ms / 1e3) / 1e9   # per-GPU kernel bytes / kernel time
+    variant = None if plan is None else int(plan.variant)
+    traffic, traffic_src = traffic_for(name, variant)
+    sc = None if world > 1 else second_ceiling(cfg, plan, nnz_all or 0, kern_ms, dev)
+    frac = achieved / peak
+    # what binds: HBM when the step runs near the copy peak; else the random on-chip accesses
+    # when they alone account for most of the step; else latency / issue (profiles/)
+    binding = ("hbm" if frac >= 0.8 else
+               ("on-chip random access (second_ceiling)" if sc and sc["frac"] >= 0.5 else
+                "latency / instruction issue (see profiles/ and DESIGN.md section 5)"))
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic_for(name),
-            "peak_source": peak_src,
-            # the copy peak counts read + write bytes of b.copy_(a); a read-only stream goes
-            # further on this part (tools/microbench/read_bw.cu, profiles/r01_read_ceiling.md)
-            "read_ceiling_gbs": READ_CEILING_GBS,
-            "frac_of_read_ceiling": round(achieved / READ_CEILING_GBS, 4),
-            "note": ("achieved = algorithmic bytes of one fp_* call (SURVEY 8(d): X once + rowptr + v + y + z + w) "
-                     "/ mean CUDA-event duration of that call on its launch stream")}
+            "frac": round(frac, 4), "traffic": traffic, "traffic_source": traffic_src,
+            "peak_source": peak_src, "binding": binding, "second_ceiling": sc,
+            "note": ("bound = the roofline axis (the path moves ~1 flop per byte: memory); achieved = algorithmic "
+                     "bytes of one fp_* call (SURVEY 8(d): X once + rowptr + v + y + z + w) / mean CUDA-event "
+                     "duration of that call (all its kernels) on its launch stream; binding = what the "
+                     "measurements say limits it")}
 
     e2e = None
     if not args.no_e2e and name != "C5":
@@ -382,7 +434,10 @@ def run_gpu(args):
             "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"],
             "data": "synthetic (counter-based seeded generator synth/, generated in HBM)",
             "config": {"workload": f"{name}: {cfg['desc']}", "m": cfg["m"], "n": cfg["n"],
-                       "format": cfg["fmt"], "nnz": nnz_all, "alpha": alpha, "beta": beta, "v": cfg["use_v"],
+                       "format": cfg["fmt"], "nnz": nnz_all,
+                       "columns": (None if cfg["fmt"] != "csr" else
+                                   {0: "stratified-uniform distinct, sorted", -1: "i.i.d. uniform (unsorted)"}.get(
+                                       cfg.get("col_skew", 0), f"Zipf-like u^(2^{cfg.get('col_skew')})")), "alpha": alpha, "beta": beta, "v": cfg["use_v"],
                        "z": cfg["use_z"], "parallelism": f"row-sharded x{world}, one NCCL allreduce of w",
                        "l2": ("flushed (256 MiB memset) between timed steps" if flush is not None else
                               f"inputs larger than L2 (X = {x_bytes / 1e9:.2f} GB >> 126 MB)"),
@@ -610,6 +665,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--cols", default="strat", choices=["strat", "iid"],
+                    help="CSR column pattern: stratified-uniform distinct (default) or i.i.d. uniform")
     ap.add_argument("--ref-seconds", type=float, default=4.0)
     ap.add_argument("--cg-iters", type=int, default=20)
     ap.add_argument("--graph", dest="graph", action="store_true", default=True,
@@ -620,6 +677,8 @@ def main():
                     help="use the NCCL row-sharded path (fp_*_dist + allreduce) even with one rank")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    global COLS
+    COLS = args.cols
     if args.impl == "reference":
         run_reference(args)
     elif args.impl == "unfused":

@@ -90,6 +90,7 @@ _SIGS = {
     "fp_dense_host": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_csr_host": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_release_workspace": (_int, []),
+    "fp_probe_rates": (_int, [_i64, _i64, _vp, _vp]),
     "fp_comm_get_unique_id": (_int, [_vp]),
     "fp_comm_init": (_int, [_P(_vp), _int, _int, _vp, _int]),
     "fp_comm_destroy": (_int, [_vp]),
@@ -427,6 +428,15 @@ class Comm:
 
 
 FP_COMM_NCCL, FP_COMM_PEER, FP_COMM_NVLS = 0, 1, 2
+
+
+def probe_rates(n, smem_elems=1000, device=None):
+    """fp_probe_rates: live random-access throughputs (ops/s) -- gather_l2, red_l2, atom_smem_u32,
+    atom_smem_f64, gather_smem_f64 (include/fusedpat.h)."""
+    r = (ctypes.c_double * 5)()
+    dev = torch.device("cuda", torch.cuda.current_device() if device is None else device)
+    _call("fp_probe_rates", int(n), int(smem_elems), ctypes.cast(r, ctypes.c_void_p), _stream(dev, None))
+    return dict(zip(("gather_l2", "red_l2", "atom_smem_u32", "atom_smem_f64", "gather_smem_f64"), list(r)))
 
 
 class LocalGroup:

@@ -148,7 +148,8 @@ def csr(m, n, dtype, lengths, kind="uniform", seed=BASE_SEED, row0=0, device="cp
     seeded matrix.  Columns are distinct and sorted (stratified-uniform, synth_core.h).
     A shard (row0 > 0) is bit-identical to the slice of the full matrix (its val/col hash index
     is the GLOBAL nnz index, found from the row lengths of rows [0, row0)).
-    col_skew > 0 draws Zipf-like skewed columns (synth_core.h syn_column_skew, u^(2^col_skew))."""
+    col_skew > 0 draws Zipf-like skewed columns (synth_core.h syn_column_skew, u^(2^col_skew));
+    col_skew < 0 draws i.i.d. uniform columns (unsorted, repeats possible: syn_column_iid)."""
     tdt, code = _tdt(dtype)
     thr = length_table(lengths, n)
     lmax = len(thr) - 1

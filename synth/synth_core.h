@@ -114,4 +114,9 @@ SYNTH_HD int32_t syn_column_skew(uint64_t h, int64_t k, int64_t L, int64_t n, in
   return (int32_t)(k + (int64_t)((((uint64_t)(n - L)) * u) >> 32));
 }
 
+/* i.i.d. uniform columns (col_skew < 0): column k of a row is uniform on [0, n) independently
+   of the others -- unsorted, repeats possible (summed, reading R7).  The un-stratified
+   pattern for measuring the kernels on truly random column positions. */
+SYNTH_HD int32_t syn_column_iid(uint64_t h, int64_t n) { return (int32_t)(h % (uint64_t)n); }
+
 #endif

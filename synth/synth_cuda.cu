@@ -53,7 +53,8 @@ __global__ void k_csr_fill(int64_t m, int64_t n, int64_t nnz0, const int64_t* ro
     for (int64_t k = lane; k < L; k += 32) {
       uint64_t g = (uint64_t)(nnz0 + a + k);
       uint64_t hc = syn_hash(seed, SYN_S_COL, g);
-      int32_t c = col_skew > 0 ? syn_column_skew(hc, k, L, n, col_skew) : syn_column(hc, k, L, n);
+      int32_t c = col_skew > 0 ? syn_column_skew(hc, k, L, n, col_skew)
+                                 : (col_skew < 0 ? syn_column_iid(hc, n) : syn_column(hc, k, L, n));
       colidx[a + k] = c;
       val[a + k] = syn_value<T>(syn_hash(seed, SYN_S_VAL, g), kind, syn_colscale_exp(seed, (uint64_t)c));
     }

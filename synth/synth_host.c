@@ -79,7 +79,8 @@ int synth_csr_fill(int64_t m, int64_t n, int64_t row0, int64_t nnz0, const int64
     for (int64_t k = 0; k < L; ++k) {
       uint64_t g = (uint64_t)(nnz0 + a + k);
       uint64_t hc = syn_hash(seed, SYN_S_COL, g);
-      int32_t c = col_skew > 0 ? syn_column_skew(hc, k, L, n, col_skew) : syn_column(hc, k, L, n);
+      int32_t c = col_skew > 0 ? syn_column_skew(hc, k, L, n, col_skew)
+                                 : (col_skew < 0 ? syn_column_iid(hc, n) : syn_column(hc, k, L, n));
       colidx[a + k] = c;
       uint64_t h = syn_hash(seed, SYN_S_VAL, g);
       if (dtype == SYN_F64) ((double*)val)[a + k] = syn_value_f64(h, kind, syn_colscale_exp(seed, (uint64_t)c));
