@@ -4,6 +4,10 @@ NVCC     ?= nvcc
 CC       := gcc
 ARCH     := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC --expt-relaxed-constexpr
+# FP_EXPERIMENTAL=1 also builds the measured-but-never-chosen CSR variants 10, 12, 14, 15
+ifeq ($(FP_EXPERIMENTAL),1)
+NVFLAGS  += -DFP_EXPERIMENTAL_VARIANTS
+endif
 CFLAGS   := -O2 -fPIC -shared -fopenmp -ffp-contract=off -std=c11 -Wall
 PKG      := paper_conf_ppopp_asharitbrcks15_b200
 CSRC     := $(PKG)/csrc

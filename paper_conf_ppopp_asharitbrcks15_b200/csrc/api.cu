@@ -180,7 +180,11 @@ const char* fp_status_string(fp_status s) {
   return "FP_ERR_UNKNOWN";
 }
 
-const char* fp_version(void) { return "0.1.0 sm_100a"; }
+#ifdef FP_EXPERIMENTAL_VARIANTS
+const char* fp_version(void) { return "0.2.0 sm_100a +experimental"; }
+#else
+const char* fp_version(void) { return "0.2.0 sm_100a"; }
+#endif
 
 fp_status fp_dense(int64_t m, int64_t n, const void* X, int64_t ld, const void* y, const void* v, const void* z,
                    double alpha, double beta, void* w, fp_dtype dtype, fp_stream stream) {

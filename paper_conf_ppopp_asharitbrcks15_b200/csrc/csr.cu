@@ -201,6 +201,24 @@ fp_status plan_csr(const PatternArgs& a, int device, fp_launch* out) {
       cudaGetLastError();
     }
   }
+  // fp64, y + w on chip, short rows: the flat-4 kernel with the fixed-point CTA partial
+  // (variant 18) -- the best of 936 settings on C3 (profiles/r02_sweep_C3.json), 3.5 % ahead of
+  // the CSR-vector / shared-partial plan; for fp32 the CSR-vector plan stays best (S3 sweep)
+  if (L.variant == FP_VAR_CSR_VECTOR && a.dtype == FP_F64 && mu <= 32.0 && a.epi_kind == 0 && !a.row_out &&
+      flat4_fixed_smem(a.n, a.dtype, true) <= kSharedBudget && !std::getenv("FP_NO_FLAT4")) {
+    L.variant = FP_VAR_CSR_FLAT4_FIXED;
+    L.vs = 32;
+    L.tl = 8;
+    L.bs = 256;
+    const int occ = flat4_fixed_blocks_per_sm(a.n, a.dtype, true);
+    L.blocks_per_sm = occ > 0 ? occ : 1;
+    L.concurrent_warps = L.blocks_per_sm * L.bs / 32;
+    L.grid = di.sm_count * L.blocks_per_sm;
+    L.smem_bytes = (int)flat4_fixed_smem(a.n, a.dtype, true);
+    L.rows_per_vector = (a.m + (int64_t)L.grid * 8 - 1) / ((int64_t)L.grid * 8);
+    *out = L;
+    return FP_OK;
+  }
   if (L.variant == FP_VAR_CSR_BINNED) {  // one producer CTA of 1024 threads per SM
     L.regs_per_thread = binned_producer_regs(a.y != nullptr);
     L.blocks_per_sm = 1;
@@ -320,6 +338,21 @@ bool plan_colsplit(const PatternArgs& a, int device, int cs_force, CsrSplit* sp,
 // the same (VS, K) runs as plain CSR-vector with the same partial (identical arithmetic).
 fp_launch stream_fallback(const PatternArgs& a, const fp_launch& L) {
   fp_launch o = L;
+  if (L.variant == FP_VAR_CSR_FLAT4_FIXED) {
+    // the chooser picks variant 18 without seeing val: colidx / val aligned differently (or a
+    // row epilogue) run the paper's CSR-vector with the CTA-shared partial instead
+    const size_t es = dtype_size(a.dtype);
+    const bool alike = ((uintptr_t)a.colidx % 4 == 0) && ((uintptr_t)a.val % es == 0) &&
+                       (((uintptr_t)a.colidx / 4) % 4 == ((uintptr_t)a.val / es) % 4);
+    const bool epi = a.y && !(a.epi_kind == 0 && !a.row_out);
+    if (!alike || epi) {
+      o.variant = FP_VAR_CSR_VECTOR;
+      o.vs = 4;
+      o.tl = 4;
+      o.grid = 0;
+    }
+    return o;
+  }
   if (L.variant != FP_VAR_CSR_STREAM && L.variant != FP_VAR_CSR_STREAM_FIXED) return o;
   const bool aligned = ((uintptr_t)a.colidx % 16 == 0) && ((uintptr_t)a.val % 16 == 0);
   const bool epi = a.y && !(a.epi_kind == 0 && !a.row_out);
@@ -330,6 +363,7 @@ fp_launch stream_fallback(const PatternArgs& a, const fp_launch& L) {
 fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s) {
   const fp_launch L = stream_fallback(a, L_in);
   if (L.variant == FP_VAR_CSR_BINNED) return launch_binned(a, L, wide_y_entries(a), s);
+  if (L.variant == FP_VAR_CSR_FLAT4_FIXED) return launch_flat4_fixed(a, L, s);
   if (L.variant == FP_VAR_CSR_COLSPLIT) {
     FP_REQUIRE(a.split && a.split->soff && a.split->cs == L.cluster, FP_ERR_UNSUPPORTED,
                "fp_csr: variant %d (column split) runs from a CSR plan (fp_csr_plan_create)", L.variant);

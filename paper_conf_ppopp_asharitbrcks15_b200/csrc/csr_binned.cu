@@ -32,6 +32,7 @@
 // same for every summation order (deterministic, and bit-exact on integer inputs).  Non-finite
 // terms go to an fp32 spill vector with a global red (IEEE propagation, reading R8).
 #include <algorithm>
+#include <cstdlib>
 
 #include "csr_kernels.cuh"
 
@@ -48,18 +49,29 @@ struct BinPArgs {
   int64_t m, nnz;
   const int64_t* rowptr;
   const int32_t* colidx;
-  const float* val;
-  const float* y;
-  const float* v;
-  float alpha;
+  const void* val;   // T
+  const void* y;     // T
+  const void* v;     // T
+  double alpha;
   int ny_s;          // leading y entries staged in shared memory
   int bw;            // block-0 width (columns >= bw are block 1; bw >= n: one block)
   int mis;           // (address of colidx / 4) mod 4 -- the same for val (checked on launch)
+  int pf;            // nonzeros of colidx / val prefetched into L2 ahead of the next batch
   uint16_t* bcol;    // [nnz] message column within its block
   float* bval;       // [nnz] message value
   int64_t* wsplit;   // [warps][3]: nz0, split (first block-1 slot), nz1
   unsigned* gmax;    // largest finite |term| (float bits)
+  // SINK_FIX (variant 18): the CTA partial w in shared memory + the grid finalize
+  int64_t n;
+  double* acc;
+  unsigned long long* counter;
+  const void* z;
+  double beta;
+  void* w;
+  int add_beta_z, accumulate;
 };
+
+enum { SINK_BINS = 0, SINK_FIX = 1 };
 
 struct BinCArgs {
   const uint16_t* bcol;
@@ -91,13 +103,21 @@ __device__ __forceinline__ int bin_exponent(const unsigned* gmax) {
   return e;
 }
 
-// 16-byte read-once loads of 4 consecutive colidx / val entries (index aligned to 4 in memory)
+// read-once loads of 4 consecutive colidx (16 B) / val (16 or 32 B) entries, index aligned to 4
 __device__ __forceinline__ void ld4(const int32_t* pc, const float* pv, int (&c)[4], float (&x)[4]) {
   asm("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
       : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3])
       : "l"(pc));
   asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
       : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3])
+      : "l"(pv));
+}
+__device__ __forceinline__ void ld4(const int32_t* pc, const double* pv, int (&c)[4], double (&x)[4]) {
+  asm("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+      : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3])
+      : "l"(pc));
+  asm("ld.global.nc.L1::no_allocate.L2::evict_first.v4.f64 {%0,%1,%2,%3}, [%4];"
+      : "=d"(x[0]), "=d"(x[1]), "=d"(x[2]), "=d"(x[3])
       : "l"(pv));
 }
 
@@ -118,24 +138,39 @@ __device__ __forceinline__ void st_msg(uint16_t* pc, float* pv, int c, float t, 
       : "memory");
 }
 
-template <int YM, int NBIN>
-__global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
-  constexpr int NW = kProdBS / 32;
+// SINK_BINS (variant 17, T = float): the scatter writes messages (above).  SINK_FIX (variant
+// 18): the scatter adds into the CTA's partial w held in shared memory as 64-bit fixed point
+// (fixacc.cuh: native 32-bit shared atomics, not the fp CAS loop), y fully staged, and the
+// grid finalize of aggregate.cuh writes w = beta z + sum of the CTA partials (alpha folded into q).
+template <typename T, int YM, int NBIN, int SINK, int BS, int MINB = 1>
+__global__ void __launch_bounds__(BS, MINB) k_flat4(const BinPArgs a) {
+  static_assert(SINK == SINK_FIX || sizeof(T) == 4, "messages are fp32");
+  constexpr int NW = BS / 32;
   constexpr int NT = kNT;
   constexpr int SPAN = 128 * NT;                // nonzero positions of a batch
-  extern __shared__ __align__(16) float y_s[];
-  __shared__ float rs[NW][32];                  // per-warp row sums, compressed (non-empty) row order
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* y_s = reinterpret_cast<T*>(smem_raw);
+  __shared__ T rs[NW][32];                      // per-warp row sums, compressed (non-empty) row order
   __shared__ unsigned hmw[NW][SPAN / 32];       // per-warp head masks
   __shared__ unsigned char cmap[NW][32];        // compressed row -> lane of the batch
+  __shared__ int fix_e;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t* __restrict__ rowptr = a.rowptr;
   const int32_t* __restrict__ colidx = a.colidx;
-  const float* __restrict__ val = a.val;
-  const float* __restrict__ y = a.y;
+  const T* __restrict__ val = (const T*)a.val;
+  const T* __restrict__ y = (const T*)a.y;
   const int ny_s = YM ? a.ny_s : 0;
-  for (int j = threadIdx.x; j < ny_s; j += kProdBS) y_s[j] = y[j];
+  for (int j = threadIdx.x; j < ny_s; j += BS) y_s[j] = y[j];
+  // SINK_FIX: [y (16-byte padded)][sp: n f64][lo: n u32][hi: n u32] behind it
+  const fpd::FixAcc FA = fix_layout(smem_raw + (SINK == SINK_FIX ? fix_y_bytes(YM ? a.n : 0, (int)sizeof(T)) : 0),
+                                    SINK == SINK_FIX ? a.n : 0, &fix_e);
+  fpd::FixScale FS;
+  if constexpr (SINK == SINK_FIX) fpd::fix_init<BS>(FA, a.n);
   __syncthreads();
-  auto Y = [&](int c) -> float { return c < ny_s ? y_s[c] : fpd::ld_keep(y + c); };
+  auto Y = [&](int c) -> T {
+    if constexpr (SINK == SINK_FIX) return y_s[c];
+    else return c < ny_s ? y_s[c] : fpd::ld_keep(y + c);
+  };
   const int mis = a.mis;
 
   const int64_t m = a.m;
@@ -146,22 +181,37 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
   const int64_t base0 = __ldg(rowptr);
   const int64_t nz0 = __ldg(rowptr + r0) - base0, nz1 = __ldg(rowptr + r1) - base0;
   // message slots of this warp: [nz0, nz1); offsets relative to nz0 (< 2^31, checked on launch)
-  uint16_t* const bcol = a.bcol + nz0;
-  float* const bval = a.bval + nz0;
+  uint16_t* const bcol = SINK == SINK_BINS ? a.bcol + nz0 : nullptr;
+  float* const bval = SINK == SINK_BINS ? a.bval + nz0 : nullptr;
   int up = 0, dn = (int)(nz1 - nz0);  // next block-0 slot (upward), one past the last free block-1 slot
   float tmax = 0.f;
   const unsigned lt = lanemask_lt();
   const int bw = a.bw;
-  const float alpha = a.alpha;
+  const T alpha = (T)a.alpha;
 
   // The scatter of one super-tile: lane l's 4 terms (columns c, values t, active bits act),
   // one entry index per step: the step's block-0 lanes take consecutive slots upward from
   // `up`, its block-1 lanes consecutive slots downward from `dn` -- every store instruction
   // covers consecutive slots.  Branch-free: predicated stores, 32-bit slot arithmetic.
-  auto EMIT4 = [&](const int (&c)[4], const float (&t)[4], unsigned act) {
+  auto EMIT4 = [&](const int (&c)[4], const T (&t)[4], unsigned act) {
+    if constexpr (SINK == SINK_FIX) {
+      if (FS.e == fpd::kFixUnset) {  // the CTA's cap exponent from the first terms (fixacc.cuh)
+        double tm = 0.0;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          double at;
+          if (((act >> e) & 1u) && fpd::fix_finite_abs((double)t[e], at)) tm = fmax(tm, at);
+        }
+        fpd::fix_try_set(FA, FS, tm);
+      }
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        if ((act >> e) & 1u) fpd::fix_add(FA, FS, c[e], t[e]);
+      return;
+    }
 #pragma unroll
     for (int e = 0; e < 4; ++e) {
-      tmax = fmaxf(tmax, fabsf(t[e]));  // inactive terms are 0; NaN is ignored, Inf kept
+      tmax = fmaxf(tmax, fabsf((float)t[e]));  // inactive terms are 0; NaN is ignored, Inf kept
       const bool on = (act >> e) & 1u;
       unsigned idx;
       int cl = c[e];
@@ -179,7 +229,7 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
         idx = (unsigned)up + __popc(m0 & lt);
         up += __popc(m0);
       }
-      st_msg(bcol + idx, bval + idx, cl, t[e], on);
+      st_msg(bcol + idx, bval + idx, cl, (float)t[e], on);
     }
   };
 
@@ -187,7 +237,7 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
   auto RP_END = [&](int64_t b) -> int64_t { return __ldg(rowptr + (b + 32 < r1 ? b + 32 : r1)); };
   // 4 entries at aligned index g = A + o (o = 4 * lane + 128 * t): loaded when any is before
   // `hi`; active = inside [lo, hi) (positions relative to A, 32-bit)
-  auto LOAD4 = [&](int64_t A, int o, int lo, int hi, int (&c)[4], float (&x)[4]) -> unsigned {
+  auto LOAD4 = [&](int64_t A, int o, int lo, int hi, int (&c)[4], T (&x)[4]) -> unsigned {
     unsigned act = 0;
     if (o < hi) {
       ld4(colidx + A + o, val + A + o, c, x);
@@ -195,11 +245,11 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       for (int e = 0; e < 4; ++e) {
         const bool in = o + e >= lo && o + e < hi;
         act |= (unsigned)in << e;
-        if (!in) c[e] = 0, x[e] = 0.f;
+        if (!in) c[e] = 0, x[e] = T(0);
       }
     } else {
 #pragma unroll
-      for (int e = 0; e < 4; ++e) c[e] = 0, x[e] = 0.f;
+      for (int e = 0; e < 4; ++e) c[e] = 0, x[e] = T(0);
     }
     return act;
   };
@@ -216,7 +266,7 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
     const bool ok = inr && len <= kLT && nxt - A <= SPAN;
     const int nrows = __ffs(~__ballot_sync(0xffffffffu, ok)) - 1;  // leading ones (-1 if all 32 ok)
     const int nr = nrows < 0 ? 32 : nrows;
-    const float vpre = (a.v && inr) ? fpd::ld_once(a.v + rb + lane) : 1.f;
+    const T vpre = (a.v && inr) ? fpd::ld_once((const T*)a.v + rb + lane) : T(1);
     const int64_t rb_next = rb + (nr == 0 ? 1 : nr);
     rp_cur = RP(rb_next);
     rp_end_cur = RP_END(rb_next);
@@ -227,9 +277,9 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       const int64_t nstart = __shfl_sync(0xffffffffu, nxt, (nr == 0 ? 1 : nr) - 1);
       const int64_t rem = base0 + a.nnz - nstart;  // never past the arrays' end
       if (lane == 0 && rem > 0) {
-        const size_t bytes = (size_t)(rem < SPAN ? rem : SPAN) * 4;
+        const size_t bytes = (size_t)(rem < a.pf ? rem : a.pf) * 4;
         fpd::prefetch_l2(colidx + nstart, bytes);
-        fpd::prefetch_l2(val + nstart, bytes);
+        fpd::prefetch_l2(val + nstart, bytes * (sizeof(T) / 4));
       }
     }
 
@@ -241,11 +291,11 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       const int64_t endA = L + lo;  // end relative to A (may exceed 2^31 only for n > 2^31)
       const int hi0 = (int)(endA < SPAN ? endA : SPAN);
       int cc[NT][4];
-      float xv[NT][4];
+      T xv[NT][4];
       unsigned act[NT];
 #pragma unroll
       for (int t = 0; t < NT; ++t) act[t] = LOAD4(A, 128 * t + 4 * lane, lo, hi0, cc[t], xv[t]);
-      float acc = 0.f;
+      T acc = T(0);
       if constexpr (YM != 0) {
 #pragma unroll
         for (int t = 0; t < NT; ++t)
@@ -257,7 +307,7 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
 #pragma unroll
           for (int t = 0; t < NT; ++t) {
             int c2[4];
-            float x2[4];
+            T x2[4];
             LOAD4(As, 128 * t + 4 * lane, 0, his, c2, x2);
 #pragma unroll
             for (int e = 0; e < 4; ++e) acc = fmaf(x2[e], Y(c2[e]), acc);
@@ -265,11 +315,11 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
         }
         acc = fpd::vector_allreduce<32>(acc);
       }
-      const float vr = __shfl_sync(0xffffffffu, vpre, 0);
-      const float q = (YM != 0 ? acc * vr : vr) * alpha;
+      const T vr = __shfl_sync(0xffffffffu, vpre, 0);
+      const T q = (YM != 0 ? acc * vr : vr) * alpha;
 #pragma unroll
       for (int t = 0; t < NT; ++t) {
-        float tv[4];
+        T tv[4];
 #pragma unroll
         for (int e = 0; e < 4; ++e) tv[e] = xv[t][e] * q;
         EMIT4(cc[t], tv, act[t]);
@@ -277,9 +327,9 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       for (int64_t s0 = SPAN; s0 < endA; s0 += 128) {
         const int his = (int)(endA - s0 < 128 ? endA - s0 : 128);
         int c2[4];
-        float x2[4];
+        T x2[4];
         const unsigned a2 = LOAD4(A + s0, 4 * lane, 0, his, c2, x2);
-        float tv[4];
+        T tv[4];
 #pragma unroll
         for (int e = 0; e < 4; ++e) tv[e] = x2[e] * q;
         EMIT4(c2, tv, a2);
@@ -300,11 +350,11 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       cmap[warp][__popc(nem & lt)] = (unsigned char)lane;
     }
     int cc[NT][4];
-    float xv[NT][4];
+    T xv[NT][4];
     unsigned act[NT];
 #pragma unroll
     for (int t = 0; t < NT; ++t) act[t] = LOAD4(A, 128 * t + 4 * lane, lo, hi, cc[t], xv[t]);
-    rs[warp][lane] = 0.f;
+    rs[warp][lane] = T(0);
     __syncwarp();
     // head bits of this lane's 4 positions per super-tile, and the compressed row index of the
     // lane's first position (heads strictly before it, minus one)
@@ -329,18 +379,18 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
     if constexpr (YM != 0) {
 #pragma unroll
       for (int t = 0; t < NT; ++t) {
-        float sv[4];
+        T sv[4];
 #pragma unroll
         for (int e = 0; e < 4; ++e) sv[e] = xv[t][e] * Y(cc[t][e]);  // Eq. (2) products
         // in-lane: P = sum before the first head, complete segments flushed, the last one kept
-        float sum = 0.f, P = 0.f;
+        T sum = T(0), P = T(0);
         int rid = rbase[t];
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
           if ((hb[t] >> e) & 1u) {
             if (rid == rbase[t]) P = sum;
             else rs[warp][rid] += sum;  // a row entirely inside this lane
-            sum = 0.f;
+            sum = T(0);
             ++rid;
           }
           sum += sv[e];
@@ -350,14 +400,14 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
         const unsigned H = __ballot_sync(0xffffffffu, hb[t] != 0u);
         const unsigned hl = H >> lane;
         const int dist = hl ? __ffs(hl) : 32 - lane;
-        float r = P;
+        T r = P;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
-          const float t2 = __shfl_down_sync(0xffffffffu, r, d);
+          const T t2 = __shfl_down_sync(0xffffffffu, r, d);
           if (d < dist) r += t2;
         }
-        float rn = __shfl_down_sync(0xffffffffu, r, 1);
-        if (lane == 31) rn = 0.f;  // continues in the next super-tile: its lane 0 adds it
+        T rn = __shfl_down_sync(0xffffffffu, r, 1);
+        if (lane == 31) rn = T(0);  // continues in the next super-tile: its lane 0 adds it
         if (hb[t]) rs[warp][rid] += sum + rn;           // the lane's last row: its suffix + what follows
         if (lane == 0 && !(hb[t] & 1u) && rbase[t] >= 0)  // the row running in from the previous tile
           rs[warp][rbase[t]] += r;
@@ -365,18 +415,18 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
       }
     }
     // lane k owns the k-th non-empty row of the batch: q = alpha v p
-    float q = 0.f;
+    T q = T(0);
     {
       const int nne = __popc(nem);
       const int src = lane < nne ? cmap[warp][lane] : 0;
-      const float vr = __shfl_sync(0xffffffffu, vpre, src);
+      const T vr = __shfl_sync(0xffffffffu, vpre, src);
       if (lane < nne) q = (YM != 0 ? rs[warp][lane] * vr : vr) * alpha;
     }
 #pragma unroll
     for (int t = 0; t < NT; ++t) {
       if (128 * t >= hi) break;
       int rid = rbase[t];
-      float tv[4];
+      T tv[4];
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         rid += (hb[t] >> e) & 1u;
@@ -386,14 +436,25 @@ __global__ void __launch_bounds__(kProdBS, 1) k_bin_produce(const BinPArgs a) {
     }
     rb = rb_next;
   }
-  if (lane == 0) {
-    a.wsplit[3 * gw] = nz0;
-    a.wsplit[3 * gw + 1] = nz0 + up;  // == nz0 + dn: every slot of [nz0, nz1) written
-    a.wsplit[3 * gw + 2] = nz1;
-  }
+  if constexpr (SINK == SINK_BINS) {
+    if (lane == 0) {
+      a.wsplit[3 * gw] = nz0;
+      a.wsplit[3 * gw + 1] = nz0 + up;  // == nz0 + dn: every slot of [nz0, nz1) written
+      a.wsplit[3 * gw + 2] = nz1;
+    }
 #pragma unroll
-  for (int d = 16; d > 0; d >>= 1) tmax = fmaxf(tmax, __shfl_xor_sync(0xffffffffu, tmax, d));
-  if (lane == 0 && tmax > 0.f) atomicMax(a.gmax, __float_as_uint(tmax));
+    for (int d = 16; d > 0; d >>= 1) tmax = fmaxf(tmax, __shfl_xor_sync(0xffffffffu, tmax, d));
+    if (lane == 0 && tmax > 0.f) atomicMax(a.gmax, __float_as_uint(tmax));
+  } else {
+    (void)tmax;
+    (void)up;
+    (void)dn;
+    __syncthreads();
+    fpd::fix_to_double<BS>(FA, a.n);
+    __syncthreads();
+    fpd::grid_finalize<T, double>(FA.sp, a.n, a.acc, a.counter, 1.0, a.beta, (const T*)a.z, (T*)a.w, a.add_beta_z,
+                                  a.accumulate);
+  }
 }
 
 __global__ void __launch_bounds__(kConsBS, 1) k_bin_consume(const BinCArgs a) {
@@ -481,6 +542,16 @@ __global__ void k_bin_finalize(int64_t n, int bw, int nbin, int ncons, const int
 
 }  // namespace
 
+// L2 prefetch distance of the flat-4 kernels (nonzeros); FP_BIN_PF overrides (measurement)
+int prefetch_span() {
+  static const int pf = [] {
+    const char* e = std::getenv("FP_BIN_PF");
+    const int v = e ? std::atoi(e) : 0;
+    return v > 0 ? v : 128 * kNT;
+  }();
+  return pf;
+}
+
 // columns one consumer CTA can hold (int32 partial in the opt-in shared memory)
 int binned_max_bw() { return (227 * 1024 - 1024) / 4 / 16 * 16; }
 
@@ -537,14 +608,16 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
   k.nnz = a.nnz;
   k.rowptr = a.rowptr;
   k.colidx = a.colidx;
-  k.val = (const float*)a.val;
-  k.y = (const float*)a.y;
-  k.v = (const float*)a.v;
-  k.alpha = (float)a.alpha;
+  k.val = a.val;
+  k.y = a.y;
+  k.v = a.v;
+  k.alpha = a.alpha;
   // y prefix: what the opt-in shared memory leaves beside the producer's static arrays
   (void)y_prefix;
-  const void* f = a.y ? (nbin == 2 ? (const void*)k_bin_produce<1, 2> : (const void*)k_bin_produce<1, 1>)
-                      : (nbin == 2 ? (const void*)k_bin_produce<0, 2> : (const void*)k_bin_produce<0, 1>);
+  const void* f = a.y ? (nbin == 2 ? (const void*)k_flat4<float, 1, 2, SINK_BINS, kProdBS>
+                                   : (const void*)k_flat4<float, 1, 1, SINK_BINS, kProdBS>)
+                      : (nbin == 2 ? (const void*)k_flat4<float, 0, 2, SINK_BINS, kProdBS>
+                                   : (const void*)k_flat4<float, 0, 1, SINK_BINS, kProdBS>);
   {
     cudaFuncAttributes fa{};
     FP_CUDA(cudaFuncGetAttributes(&fa, f));
@@ -554,6 +627,7 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
   }
   k.bw = nbin == 2 ? bw : INT32_MAX;
   k.mis = mis;
+  k.pf = prefetch_span();
   k.bcol = (uint16_t*)take((size_t)a.nnz * 2);
   k.bval = (float*)take((size_t)a.nnz * 4);
   k.wsplit = (int64_t*)take((size_t)pw * 24);
@@ -579,10 +653,89 @@ fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_pref
   return FP_OK;
 }
 
+// ---- variant 18: the flat-4 kernel with the fixed-point CTA partial (n fits shared memory)
+constexpr int kFixBS = 256;
+
+template <typename T, int YM>
+const void* flat4_fixed_fn() {  // fp64 keeps ~80 registers (3 CTAs of 256 per SM), fp32 64 (4)
+  return (const void*)k_flat4<T, YM, 1, SINK_FIX, kFixBS, sizeof(T) == 8 ? 3 : 4>;
+}
+const void* flat4_fixed_pick(fp_dtype dt, bool has_y) {
+  if (dt == FP_F64) return has_y ? flat4_fixed_fn<double, 1>() : flat4_fixed_fn<double, 0>();
+  return has_y ? flat4_fixed_fn<float, 1>() : flat4_fixed_fn<float, 0>();
+}
+
+size_t flat4_fixed_smem(int64_t n, fp_dtype dt, bool has_y) {
+  return (size_t)(has_y ? fix_y_bytes(n, (int)dtype_size(dt)) : 0) + (size_t)n * 16;
+}
+
+int flat4_fixed_blocks_per_sm(int64_t n, fp_dtype dt, bool has_y) {
+  const void* f = flat4_fixed_pick(dt, has_y);
+  set_max_dynamic_smem(f);
+  int occ = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f, kFixBS, flat4_fixed_smem(n, dt, has_y));
+  return occ;
+}
+
+fp_status launch_flat4_fixed(const PatternArgs& a, const fp_launch& L, cudaStream_t s) {
+  FP_REQUIRE(a.epi_kind == 0 && !a.row_out, FP_ERR_UNSUPPORTED, "fp_csr: variant %d has no row epilogue",
+             L.variant);
+  const bool has_y = a.y != nullptr;
+  const size_t smem = flat4_fixed_smem(a.n, a.dtype, has_y);
+  const void* f = flat4_fixed_pick(a.dtype, has_y);
+  cudaFuncAttributes fa{};
+  FP_CUDA(cudaFuncGetAttributes(&fa, f));
+  FP_REQUIRE(smem + fa.sharedSizeBytes <= (size_t)device_info(current_device()).smem_optin_per_block,
+             FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs n small enough for y + partial w in shared memory",
+             L.variant);
+  const size_t es = dtype_size(a.dtype);
+  const int mis = (int)(((uintptr_t)a.colidx >> 2) & 3);
+  FP_REQUIRE(((uintptr_t)a.colidx & 3) == 0 && ((uintptr_t)a.val % es) == 0 &&
+                 (int)(((uintptr_t)a.val / es) & 3) == mis,
+             FP_ERR_UNSUPPORTED, "fp_csr: variant %d needs colidx and val aligned alike (4-entry groups)",
+             L.variant);
+  const int sms = device_info(current_device()).sm_count;
+  int grid = L.grid;
+  if (grid <= 0) {
+    const int occ = flat4_fixed_blocks_per_sm(a.n, a.dtype, has_y);
+    grid = sms * (occ > 0 ? occ : 1);
+  }
+  FP_REQUIRE(a.nnz / ((int64_t)grid * (kFixBS / 32)) + a.n < INT32_MAX, FP_ERR_UNSUPPORTED,
+             "fp_csr: variant %d: too many nonzeros per warp (grid %d)", L.variant, grid);
+  Workspace* ws = workspace(s, (size_t)a.n, 0);
+  if (!ws) return FP_ERR_NOMEM;
+  BinPArgs k{};
+  k.m = a.m;
+  k.nnz = a.nnz;
+  k.rowptr = a.rowptr;
+  k.colidx = a.colidx;
+  k.val = a.val;
+  k.y = a.y;
+  k.v = a.v;
+  k.alpha = a.alpha;
+  k.ny_s = has_y ? (int)a.n : 0;
+  k.bw = INT32_MAX;
+  k.mis = mis;
+  k.pf = prefetch_span();
+  k.n = a.n;
+  k.acc = ws->acc;
+  k.counter = ws->counters;
+  k.z = a.z;
+  k.beta = a.beta;
+  k.w = a.w;
+  k.add_beta_z = a.add_beta_z ? 1 : 0;
+  k.accumulate = a.accumulate ? 1 : 0;
+  set_max_dynamic_smem(f);
+  void* args[] = {&k};
+  FP_CUDA(cudaLaunchKernel(f, dim3(grid), dim3(kFixBS), args, smem, s));
+  return FP_OK;
+}
+
 // register count of the producer (plan reports)
 int binned_producer_regs(bool has_y) {
   cudaFuncAttributes fa{};
-  if (cudaFuncGetAttributes(&fa, has_y ? (const void*)k_bin_produce<1, 2> : (const void*)k_bin_produce<0, 2>) !=
+  if (cudaFuncGetAttributes(&fa, has_y ? (const void*)k_flat4<float, 1, 2, SINK_BINS, kProdBS>
+                                      : (const void*)k_flat4<float, 0, 2, SINK_BINS, kProdBS>) !=
       cudaSuccess) {
     cudaGetLastError();
     return 0;

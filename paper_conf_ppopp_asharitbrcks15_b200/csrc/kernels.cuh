@@ -68,6 +68,11 @@ PatternArgs csr_args(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, c
 fp_status launch_binned(const PatternArgs& a, const fp_launch& L, int64_t y_prefix, cudaStream_t s);
 int binned_nbin(int64_t n);     // 1 or 2 column blocks; 0 if n is too wide
 int binned_producer_regs(bool has_y);
+// Variant 18 (csr_binned.cu): flat-4 kernel with the fixed-point CTA partial (small n).
+fp_status launch_flat4_fixed(const PatternArgs& a, const fp_launch& L, cudaStream_t s);
+size_t flat4_fixed_smem(int64_t n, fp_dtype dt, bool has_y);
+int flat4_fixed_blocks_per_sm(int64_t n, fp_dtype dt, bool has_y);
+
 size_t binned_ws_bytes(int64_t n, int64_t nnz, int nbin, int producer_grid, int consumers);
 
 // w = beta*z (or 0): the alpha == 0 / m == 0 path, and the pre-initialisation of the L2 path.

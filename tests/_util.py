@@ -30,3 +30,16 @@ def assert_bitexact(w_gpu, w_ref, what=""):
     w = w_gpu.detach().cpu().double().numpy()
     bad = np.nonzero(w != w_ref)[0]
     assert bad.size == 0, f"{what}: {bad.size} entries differ, first at {bad[:5]}: {w[bad[:5]]} vs {w_ref[bad[:5]]}"
+
+
+EXPERIMENTAL_VARIANTS = (10, 12, 14, 15)  # built only with FP_EXPERIMENTAL=1 (Makefile)
+
+
+def skip_unbuilt(variant):
+    """Skip a test of a CSR variant the library was built without (never chosen by the plan)."""
+    import pytest
+
+    import paper_conf_ppopp_asharitbrcks15_b200 as fp
+
+    if variant in EXPERIMENTAL_VARIANTS and b"+experimental" not in fp.lib().fp_version():
+        pytest.skip(f"variant {variant} is built only with FP_EXPERIMENTAL=1")

@@ -133,3 +133,77 @@ def test_binned_chosen_for_c4_shape(cuda_dev):
     st.mean = 40.0
     L = fp.choose(True, st, fp.FP_F32, 0)
     assert (L.variant, L.cluster, L.bs, L.tl) == (17, 2, 1024, 8)
+
+
+# ------------------------------------------------------------------ variant 18 (flat-4, fixed-point CTA partial)
+DT = {"f64": torch.float64, "f32": torch.float32}
+
+
+def launch18(grid=0, variant=18):
+    L = fp.fp_launch()
+    L.variant, L.vs, L.tl, L.bs, L.grid = variant, 32, 8, 256, grid
+    return L
+
+
+def make_dt(m, n, dt, lengths, seed, kind):
+    rp, ci, va = synth.csr(m, n, dt, lengths, kind=kind, seed=seed)
+    integer = kind.startswith("int")
+    y = synth.vector(n, dt, kind="int_small" if integer else "uniform", seed=seed, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="int_pos" if integer else "pos", seed=seed, stream=synth.S_V)
+    z = synth.vector(n, dt, kind="int_small" if integer else "uniform", seed=seed, stream=synth.S_Z)
+    return rp, ci, va, y, v, z
+
+
+@pytest.mark.parametrize("variant", [18])
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("lengths", [("binomial", 0.01), ("powerlaw", 2.0, 3.0), ("uniform", 0, 600), ("uniform", 0, 3)])
+@pytest.mark.parametrize("grid", [0, 1, 37])
+def test_flat4_fixed_bitexact(cuda_dev, variant, dt, lengths, grid):
+    """Variant 18 on integer twins: bit-exact for every instance, short rows (flat batches of 4
+    nonzeros per lane), rows beyond 128 (warp-per-row steps), empty rows, forced grids."""
+    m, n = (20_000, 1000) if lengths[0] != "uniform" or lengths[2] < 100 else (3_000, 1000)
+    rp, ci, va, y, v, z = make_dt(m, n, dt, lengths, seed=grid + 3, kind="int_pm12")
+    for args in ((y, v, z, 1.0, 1.0), (None, v, None, -1.0, 0.0), (y, None, z, 2.0, -0.5)):
+        ref, mag = oracle.csr(m, n, rp, ci, va, *args)
+        assert mag.max() < (2**24 if dt == "f32" else 2**53)
+        w = run(cuda_dev, rp, ci, va, n, *args, launch18(grid, variant))
+        assert_bitexact(w, ref, f"variant {variant} {dt} {lengths} grid={grid} y={args[0] is not None}")
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+def test_flat4_fixed_misaligned_slices(cuda_dev, dt):
+    """colidx / val starting 1..3 entries past a 16-byte boundary (row-shard slices): the 4-entry
+    groups follow the common misalignment."""
+    m, n = 5000, 800
+    rp, ci, va, y, v, z = make_dt(m, n, dt, ("binomial", 0.02), seed=5, kind="int_pm12")
+    ref, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    for off in (1, 2, 3):
+        cib = torch.zeros(ci.numel() + 4, dtype=torch.int32)
+        vab = torch.zeros(va.numel() + 4, dtype=va.dtype)
+        cib[off:off + ci.numel()] = ci
+        vab[off:off + va.numel()] = va
+        cid, vad = cib.to(cuda_dev), vab.to(cuda_dev)
+        w = fp.csr(rp.to(cuda_dev), cid[off:off + ci.numel()], vad[off:off + va.numel()], n, y.to(cuda_dev),
+                   v.to(cuda_dev), z.to(cuda_dev), 1.0, 1.0, launch=launch18())
+        torch.cuda.synchronize()
+        assert_bitexact(w, ref, f"flat4 misaligned by {off}")
+
+
+@pytest.mark.parametrize("variant", [18])
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+def test_flat4_fixed_float_parity(cuda_dev, variant, dt):
+    """U[-1,1) data, C3-shaped rows, plus rows scaled by 2^+-30 (terms far beyond / below the
+    CTA's cap exponent take the fp64 spill / round to the fixed grid): north_star tolerance."""
+    m, n = 30_000, 1000
+    rp, ci, va, y, v, z = make_dt(m, n, dt, ("binomial", 0.01), seed=8, kind="uniform")
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = run(cuda_dev, rp, ci, va, n, y, v, z, 1.0, 1.0, launch18(0, variant))
+    assert_parity(w, ref, mag, DT[dt], "flat4 fixed float")
+    scale = torch.ones(m, dtype=va.dtype)
+    scale[::97] = 2.0**30
+    scale[1::89] = 2.0**-30
+    rows = torch.repeat_interleave(torch.arange(m), rp[1:] - rp[:-1])
+    va2 = va * scale[rows]
+    ref, mag = oracle.csr(m, n, rp, ci, va2, y, v, z, 1.0, 1.0)
+    w = run(cuda_dev, rp, ci, va2, n, y, v, z, 1.0, 1.0, launch18(0, variant))
+    assert_parity(w, ref, mag, DT[dt], "flat4 fixed wide range")

@@ -14,7 +14,7 @@ import torch
 import oracle
 import paper_conf_ppopp_asharitbrcks15_b200 as fp
 import synth
-from _util import TOL, assert_bitexact, assert_parity
+from _util import TOL, assert_bitexact, assert_parity, skip_unbuilt
 
 pytestmark = pytest.mark.gpu
 
@@ -164,8 +164,11 @@ def test_csr_plan_c3_c4(cuda_dev):
     st.m, st.n, st.nnz = 20_000_000, 1000, 200_000_000
     st.mean = 10.0
     L = fp.choose(True, st, fp.FP_F64, 0)
-    # CTA-shared partial; Eq. (4)'s VS = 8 bin runs as 4 lanes x 4 cached entries (B200 sweep,
-    # profiles/r01_sweep2_C3.json: within 3 % of the best of 81 settings)
+    # fp64, y + w on chip: the flat-4 kernel with the fixed-point CTA partial (variant 18, the
+    # best of 936 settings in profiles/r02_sweep_C3.json); fp32: CSR-vector with the CTA-shared
+    # partial, Eq. (4)'s VS = 8 bin run as 4 lanes x 4 cached entries (profiles/r02_sweep_S3.json)
+    assert (L.variant, L.bs) == (18, 256)
+    L = fp.choose(True, st, fp.FP_F32, 0)
     assert (L.vs, L.tl, L.variant) == (4, 4, 3)
     st.m, st.n, st.nnz = 50_000_000, 100_000, 2_000_000_000
     st.mean = 40.0
@@ -182,6 +185,7 @@ def test_csr_plan_c3_c4(cuda_dev):
 def test_csr_flat_bitexact(cuda_dev, dt, variant, nb, lengths):
     """Flat kernels (lanes on consecutive nonzeros, rows longer than 32*NB take the warp-per-
     row path): integer twins bit-exact for every instance."""
+    skip_unbuilt(variant)
     m, n = 4000, 600
     rp, ci, va, y, v, z = make_csr(m, n, dt, lengths, seed=nb + variant, kind="int_pm12")
     L = fp.fp_launch()
@@ -219,6 +223,7 @@ def test_kdd_like_skewed_columns(cuda_dev, dt):
 def test_csr_owner_bitexact(cuda_dev, dt, vs, k, n):
     """Owner-computes aggregation (variant 10): queues, drains, spills -- integer twins exact,
     including heavy rows (power-law) that overflow the queues into the CAS spill partial."""
+    skip_unbuilt(10)
     m = 6000
     for lengths in (("binomial", 0.01), ("powerlaw", 2.0, 4.0)):
         rp, ci, va, y, v, z = make_csr(m, n, dt, lengths, seed=vs + n, kind="int_pm12")
@@ -245,6 +250,7 @@ def test_fixed_point_limb_moves_and_spill_bitexact(cuda_dev, dt, variant, vs, tl
     exponent from terms of 1 (cap 2^7); then 40k terms of 63 push the high limb past 2^29
     (value-preserving moves into the fp64 spill) and terms of 1000 exceed the cap (spill
     path).  Integers: the sum is exact, so w must equal the oracle bit for bit."""
+    skip_unbuilt(variant)
     m = 60000  # one CTA of 8 warps: warp w owns rows [7500 w, 7500 (w + 1)); each starts with 256 rows of 1
     rp, ci, va, y, v = _single_column(m, lambda r: 1.0 if r % 7500 < 256 else (1000.0 if r % 97 == 0 else 63.0), dt)
     ref, _ = oracle.csr(m, 1, rp, ci, va, y, v, None, 1.0, 0.0)
@@ -260,6 +266,7 @@ def test_fixed_point_wide_dynamic_range(cuda_dev, dt, variant):
     """Rows scaled by 2^k, k uniform in [-40, 40] (terms spanning ~2^160): the fixed-point
     partial keeps the stated normwise tolerance (small terms round to the CTA's grid, large
     ones spill to fp64; DESIGN reading R21)."""
+    skip_unbuilt(variant)
     m, n = 30000, 800
     rp, ci, va, y, v, z = make_csr(m, n, dt, ("binomial", 0.01), seed=41)
     k = torch.from_numpy(np.random.default_rng(41).integers(-40, 41, m)).double()
@@ -283,6 +290,7 @@ def test_csr_stream_bitexact(cuda_dev, dt, variant, vsk, lengths):
     the stage (rows read from global), rows longer than VS*K, empty rows, an nnz that is not a
     multiple of the 16-byte chunk (zero-filled tail), warps with no rows -- integer twins must
     equal the oracle bit for bit, with and without y."""
+    skip_unbuilt(variant)
     m, n = 7001, 1000
     rp, ci, va, y, v, z = make_csr(m, n, dt, lengths, seed=vsk[0] * 10 + vsk[1], kind="int_pm12")
     vs, k = vsk
@@ -316,6 +324,7 @@ def test_csr_stream_misaligned_falls_back(cuda_dev, dt):
 @pytest.mark.parametrize("variant", [14, 15])
 def test_csr_stream_float_parity(cuda_dev, dt, variant):
     """Full-precision C3-shaped inputs (scaled down): normwise tolerance of north_star."""
+    skip_unbuilt(variant)
     m, n = 200_000, 1000
     rp, ci, va, y, v, z = make_csr(m, n, dt, ("binomial", 0.01), seed=9)
     ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 0.75, -1.25)
