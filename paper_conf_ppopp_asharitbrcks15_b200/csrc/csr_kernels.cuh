@@ -463,14 +463,14 @@ CsrKFn csr_pick_m(int mode, int vs, int k) {
 #ifdef FP_EXPERIMENTAL_VARIANTS
     // measured and never chosen: built only with FP_EXPERIMENTAL=1
     case DMODE_FLAT_FIXED: return csr_pick_flat<T, YM, MODE_FIXED>(k);
-    case DMODE_FLAT_SHARED: return csr_pick_flat<T, YM, MODE_SHARED>(k);
-    case DMODE_FLAT_L2: return csr_pick_flat<T, YM, MODE_L2>(k);
-    case DMODE_FLAT_PRIVATE: return csr_pick_flat<T, YM, MODE_PRIVATE>(k);
     case DMODE_OWNER4: return csr_pick_owner_n<T, YM, 4>(vs, k);
     case DMODE_OWNER8: return csr_pick_owner_n<T, YM, 8>(vs, k);
     case DMODE_STREAM_SHARED: return csr_pick_stream<T, YM, MODE_SHARED>(vs, k);
     case DMODE_STREAM_FIXED: return csr_pick_stream<T, YM, MODE_FIXED>(vs, k);
 #endif
+    case DMODE_FLAT_SHARED: return csr_pick_flat<T, YM, MODE_SHARED>(k);
+    case DMODE_FLAT_L2: return csr_pick_flat<T, YM, MODE_L2>(k);
+    case DMODE_FLAT_PRIVATE: return csr_pick_flat<T, YM, MODE_PRIVATE>(k);
     case DMODE_FLAT_L2_WIDE: return k == 8 ? k_csr_flat<T, 8, YM, MODE_L2, kWideBS> : nullptr;
     default: return nullptr;
   }
