@@ -252,6 +252,20 @@ def run_gpu(args):
         comm = fp.Comm(device=local)
     name = args.config
     cfg, inp = build_inputs(name, rank, world, dev)
+    exchange = "none"
+    if comm is not None:
+        # the exchange of the partial w: the fused peer-memory path (FP_COMM_PEER, the product),
+        # NVSwitch multicast (FP_COMM_NVLS) or ncclAllReduce (the baseline), --exchange
+        exchange = args.exchange
+        vec_bytes = cfg["n"] * (8 if cfg["dtype"] == "f64" else 4)
+        try:
+            if exchange == "peer":
+                comm.enable_peer(vec_bytes)
+            elif exchange == "nvls":
+                comm.enable_nvls(vec_bytes)
+        except fp.FusedPatError as e:
+            print(f"[bench] {exchange} exchange unavailable ({e}); using NCCL", file=sys.stderr)
+            exchange = "nccl"
     torch.cuda.synchronize()
     alpha, beta = cfg["alpha"], cfg["beta"]
     stream = torch.cuda.current_stream(dev)
@@ -331,7 +345,8 @@ def run_gpu(args):
         step()
     torch.cuda.synchronize()
     graphed = False
-    if args.graph and name != "C5":
+    # (the peer / NVLS exchange advances an epoch per call and is not capturable)
+    if args.graph and name != "C5" and exchange in ("none", "nccl"):
         # Capture one step (the fp_* call; its plan is cached and its workspace exists for the
         # capture stream after the warm-up below) in a CUDA graph, so host-side marshalling is
         # off the timed path -- it matters for the latency config C1.
@@ -438,7 +453,9 @@ def run_gpu(args):
                        "columns": (None if cfg["fmt"] != "csr" else
                                    {0: "stratified-uniform distinct, sorted", -1: "i.i.d. uniform (unsorted)"}.get(
                                        cfg.get("col_skew", 0), f"Zipf-like u^(2^{cfg.get('col_skew')})")), "alpha": alpha, "beta": beta, "v": cfg["use_v"],
-                       "z": cfg["use_z"], "parallelism": f"row-sharded x{world}, one NCCL allreduce of w",
+                       "z": cfg["use_z"],
+                       "parallelism": (f"row-sharded x{world}, one exchange of the partial w ({exchange})"
+                                       if comm is not None else "1 GPU"),
                        "l2": ("flushed (256 MiB memset) between timed steps" if flush is not None else
                               f"inputs larger than L2 (X = {x_bytes / 1e9:.2f} GB >> 126 MB)"),
                        "passes_per_step": passes_per_step, "cuda_graph": graphed,
@@ -673,6 +690,8 @@ def main():
                     help="replay each step from a captured CUDA graph (default)")
     ap.add_argument("--no-graph", dest="graph", action="store_false")
     ap.add_argument("--launch", default=None, help="CSR only: force the plan 'variant,vs,k,grid' (profiling)")
+    ap.add_argument("--exchange", default="peer", choices=["peer", "nvls", "nccl"],
+                    help="N > 1: exchange of the partial w (fused peer memory, NVLS multicast, or NCCL)")
     ap.add_argument("--force-dist", action="store_true",
                     help="use the NCCL row-sharded path (fp_*_dist + allreduce) even with one rank")
     args = ap.parse_args()

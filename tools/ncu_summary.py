@@ -44,10 +44,11 @@ def raw_rows(rep):
     return hdr, units, rows
 
 
-def full(rep, config, alg_bytes):
+def full(rep, config, alg_bytes, variant=None, rnd=None):
     hdr, units, rows = raw_rows(rep)
     print(f"# ncu --set full: {os.path.basename(rep)} ({config})\n")
     traffic_all = []
+    per_kernel = defaultdict(list)
     for row in rows:
         d = dict(zip(hdr, row))
         u = dict(zip(hdr, units))
@@ -61,12 +62,19 @@ def full(rep, config, alg_bytes):
         wb = to_bytes(d["dram__bytes_write.sum"], u["dram__bytes_write.sum"])
         t = rb + wb
         traffic_all.append(t)
+        per_kernel[name].append(t)
         print(f"\nDRAM traffic per launch: {t / 1e9:.4f} GB; algorithmic bytes per launch: {alg_bytes / 1e9:.4f} GB; "
               f"traffic / algorithmic = {t / alg_bytes:.4f}\n")
+    # one step = one launch of every distinct kernel of the fp_* call (variant 17: producer,
+    # consumer, finalize): the step's traffic is the sum of their per-launch means
+    kern = {k: int(sum(v) / len(v)) for k, v in per_kernel.items()}
+    step = sum(kern.values())
+    print(f"\nDRAM traffic per step (sum over the {len(kern)} kernels): {step / 1e9:.4f} GB; "
+          f"traffic / algorithmic = {step / alg_bytes:.4f}\n")
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     db = json.load(open(p)) if os.path.exists(p) else {}
-    db[config] = {"dram_bytes_per_launch": int(sum(traffic_all) / len(traffic_all)),
-                  "algorithmic_bytes_per_launch": int(alg_bytes), "report": os.path.basename(rep)}
+    db[config] = {"dram_bytes_per_step": step, "algorithmic_bytes_per_step": int(alg_bytes),
+                  "kernels": kern, "file": os.path.basename(rep), "variant": variant, "round": rnd}
     json.dump(db, open(p, "w"), indent=1, sort_keys=True)
 
 
@@ -88,6 +96,7 @@ def launches(path):
 
 if __name__ == "__main__":
     if sys.argv[1] == "full":
-        full(sys.argv[2], sys.argv[3], float(sys.argv[4]))
+        full(sys.argv[2], sys.argv[3], float(sys.argv[4]), int(sys.argv[5]) if len(sys.argv) > 5 else None,
+             sys.argv[6] if len(sys.argv) > 6 else None)
     else:
         launches(sys.argv[2])
