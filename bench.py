@@ -258,14 +258,24 @@ def run_gpu(args):
         # NVSwitch multicast (FP_COMM_NVLS) or ncclAllReduce (the baseline), --exchange
         exchange = args.exchange
         vec_bytes = cfg["n"] * (8 if cfg["dtype"] == "f64" else 4)
+        ok = 1
         try:
             if exchange == "peer":
                 comm.enable_peer(vec_bytes)
             elif exchange == "nvls":
                 comm.enable_nvls(vec_bytes)
         except fp.FusedPatError as e:
-            print(f"[bench] {exchange} exchange unavailable ({e}); using NCCL", file=sys.stderr)
-            exchange = "nccl"
+            print(f"[bench] rank {rank}: {exchange} exchange unavailable ({e})", file=sys.stderr)
+            ok = 0
+        # every rank must use the same exchange: fall back to NCCL together if any rank failed
+        import torch.distributed as dist
+
+        flag = torch.tensor([ok], dtype=torch.int32, device=dev)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if exchange != "nccl" and int(flag.item()) == 0:
+            if comm.mode != fp.FP_COMM_NCCL:
+                comm.set_mode(fp.FP_COMM_NCCL)
+            exchange = "nccl (fallback)"
     torch.cuda.synchronize()
     alpha, beta = cfg["alpha"], cfg["beta"]
     stream = torch.cuda.current_stream(dev)
@@ -346,7 +356,7 @@ def run_gpu(args):
     torch.cuda.synchronize()
     graphed = False
     # (the peer / NVLS exchange advances an epoch per call and is not capturable)
-    if args.graph and name != "C5" and exchange in ("none", "nccl"):
+    if args.graph and name != "C5" and exchange in ("none", "nccl", "nccl (fallback)"):
         # Capture one step (the fp_* call; its plan is cached and its workspace exists for the
         # capture stream after the warm-up below) in a CUDA graph, so host-side marshalling is
         # off the timed path -- it matters for the latency config C1.
