@@ -324,15 +324,33 @@ __global__ void __launch_bounds__(BS, MINB) k_flat4(const BinPArgs a) {
         for (int e = 0; e < 4; ++e) tv[e] = xv[t][e] * q;
         EMIT4(cc[t], tv, act[t]);
       }
-      for (int64_t s0 = SPAN; s0 < endA; s0 += 128) {
-        const int his = (int)(endA - s0 < 128 ? endA - s0 : 128);
-        int c2[4];
-        T x2[4];
-        const unsigned a2 = LOAD4(A + s0, 4 * lane, 0, his, c2, x2);
-        T tv[4];
+      // the tail beyond the first SPAN positions is re-read for the scatter: a long row's dot
+      // takes longer than L2 keeps it, so the whole tail is first requested into L2 at once
+      // (its DRAM latency overlapped), then streamed two super-tiles per step
+      if (endA > SPAN) {
+        for (int64_t o = SPAN + (int64_t)lane * 1024; o < endA; o += 32 * 1024) {
+          const int64_t cnt = endA - o < 1024 ? endA - o : 1024;
+          fpd::prefetch_l2(colidx + A + o, (size_t)cnt * 4);
+          fpd::prefetch_l2(val + A + o, (size_t)cnt * sizeof(T));
+        }
+      }
+      for (int64_t s0 = SPAN; s0 < endA; s0 += 256) {
+        int c2[2][4];
+        T x2[2][4];
+        unsigned a2[2];
 #pragma unroll
-        for (int e = 0; e < 4; ++e) tv[e] = x2[e] * q;
-        EMIT4(c2, tv, a2);
+        for (int t = 0; t < 2; ++t) {
+          const int64_t st = s0 + 128 * t;
+          const int his = st < endA ? (int)(endA - st < 128 ? endA - st : 128) : 0;
+          a2[t] = LOAD4(A + st, 4 * lane, 0, his, c2[t], x2[t]);
+        }
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+          T tv[4];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) tv[e] = x2[t][e] * q;
+          EMIT4(c2[t], tv, a2[t]);
+        }
       }
       rb = rb_next;
       continue;
