@@ -2,7 +2,8 @@
 """Small-shape driver for compute-sanitizer (memcheck / racecheck / synccheck): every kernel
 family once -- dense vector / CTA / cluster, CSR vector (shared / L2 / private / owner /
 fixed-point / cp.async stream), flat (shared / L2 / private / fixed / 1024-thread with a y
-prefix), the L2-replica fold, the column-split plan, the row epilogues, CG and TRON drivers --
+prefix), flat-4 with the fixed-point partial (18), the binned scatter (17: producer, consumer,
+finalize), the peer exchange (one-rank local group), the L2-replica fold, the column-split plan, the row epilogues, CG and TRON drivers --
 on tiny inputs.
 
   compute-sanitizer --tool memcheck python tools/sanitize.py
@@ -35,8 +36,11 @@ def main():
         y = synth.vector(700, dt, seed=2, device=dev)
         v = synth.vector(2000, dt, kind="pos", seed=2, stream=synth.S_V, device=dev)
         z = synth.vector(700, dt, seed=2, stream=synth.S_Z, device=dev)
+        experimental = b"+experimental" in fp.lib().fp_version()
         for var, vs, tl in ((3, 8, 2), (3, 4, 4), (4, 32, 4), (5, 8, 2), (6, 32, 4), (7, 32, 8), (8, 32, 2),
-                            (10, 8, 2), (11, 4, 4), (12, 32, 4), (14, 4, 4), (15, 4, 4), (16, 32, 8)):
+                            (10, 8, 2), (11, 4, 4), (12, 32, 4), (14, 4, 4), (15, 4, 4), (16, 32, 8), (18, 32, 8)):
+            if var in (10, 12, 14, 15) and not experimental:
+                continue
             L = fp.fp_launch()
             L.variant, L.vs, L.tl, L.bs, L.grid = var, vs, tl, 1024 if var == 16 else 256, 13
             fp.csr(rp, ci, va, 700, y, v, z, 1.0, 1.0, launch=L)  # 4/7/16: w replicated over L2, folded
@@ -47,6 +51,23 @@ def main():
         L = fp.fp_launch()
         L.variant, L.vs, L.tl, L.bs, L.grid = 16, 32, 8, 1024, 7
         fp.csr(rpw, ciw, vaw, nw, yw, None, yw, 1.0, 1.0, launch=L)
+        # variant 17 (binned scatter, fp32): one and two column blocks, long + empty rows
+        if dt == "f32":
+            for nb, nn in ((1, 700), (2, 90000)):
+                rpb, cib, vab = synth.csr(3000, nn, dt, ("powerlaw", 2.0, 3.0), seed=6, device=dev)
+                yb = synth.vector(nn, dt, seed=6, device=dev)
+                zb = synth.vector(nn, dt, seed=6, stream=synth.S_Z, device=dev)
+                vb = synth.vector(3000, dt, kind="pos", seed=6, stream=synth.S_V, device=dev)
+                L = fp.fp_launch()
+                L.variant, L.vs, L.tl, L.bs, L.grid, L.cluster = 17, 32, 8, 1024, 5, nb
+                fp.csr(rpb, cib, vab, nn, yb, vb, zb, 1.0, 1.0, launch=L)
+                fp.csr(rpb, cib, vab, nn, None, vb, None, 2.0, 0.0, launch=L)
+        # the peer exchange (one-rank local group: the same kernels, a trivially met barrier)
+        g = fp.LocalGroup(1, 0, max_bytes=700 * 8)
+        fp.csr_dist(g.comms[0], rp, ci, va, 700, y, v, z, 1.0, 1.0)
+        g.comms[0].allreduce(y.clone())
+        torch.cuda.synchronize()
+        g.close()
         # CSR plan with the column split of variant 13 (cluster of 2)
         F = fp.fp_launch()
         F.variant, F.cluster = 13, 2
