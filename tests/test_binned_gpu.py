@@ -207,3 +207,21 @@ def test_flat4_fixed_float_parity(cuda_dev, variant, dt):
     ref, mag = oracle.csr(m, n, rp, ci, va2, y, v, z, 1.0, 1.0)
     w = run(cuda_dev, rp, ci, va2, n, y, v, z, 1.0, 1.0, launch18(0, variant))
     assert_parity(w, ref, mag, DT[dt], "flat4 fixed wide range")
+
+
+def test_binned_host_streaming_accumulates_chunks(cuda_dev):
+    """fp_csr_host (P:151 streaming) on a matrix of ~3 chunks of 512 MB: every chunk runs the
+    binned plan (variant 17, > 16M nonzeros) with accumulate = 1 after the first (the finalize
+    adds into w); integer twin bit-exact against the oracle over the whole matrix."""
+    m, n = 4_000_000, 100_000
+    rp, ci, va = synth.csr(m, n, "f32", ("powerlaw", 2.5, 13.64), kind="int_pm12", seed=41)
+    assert int(rp[-1]) > 2 * (512 << 20) // 8  # at least three chunks
+    y = synth.vector(n, "f32", kind="int_small", seed=41, stream=synth.S_Y)
+    v = synth.vector(m, "f32", kind="int_pos", seed=41, stream=synth.S_V)
+    z = synth.vector(n, "f32", kind="int_small", seed=41, stream=synth.S_Z)
+    # v = 1, beta = 0 keep every partial sum below 2^24 (fp32 twin exact in any order, also
+    # across the chunk boundaries where the finalize adds into the fp32 w)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, None, None, 1.0, 0.0)
+    assert mag.max() < 2**24
+    w = fp.csr_host(rp, ci, va, n, y, None, None, 1.0, 0.0)
+    assert_bitexact(w, ref, "binned host streaming")
