@@ -33,6 +33,7 @@
 // terms go to an fp32 spill vector with a global red (IEEE propagation, reading R8).
 #include <algorithm>
 #include <cstdlib>
+#include <type_traits>
 
 #include "csr_kernels.cuh"
 
@@ -491,47 +492,71 @@ __global__ void __launch_bounds__(kConsBS, 1) k_bin_consume(const BinCArgs a) {
   const float sf = fscale ? ldexpf(1.f, ex) : 0.f;
   const double sd = ldexp(1.0, ex);
   const int64_t col0 = (int64_t)b * a.bw;
-  auto ADD = [&](int cl, float t) {
-    if (allspill || !(fabsf(t) <= 3.402823466e38f)) {  // Inf / NaN: IEEE propagation through the spill
+  // one message: fixed point, native returning shared atomic, wrap carried into hi[]; FS =
+  // the float scale is usable (decided once per call, so the two paths are separate loops)
+  auto ADD = [&](int cl, float t, auto fs) {
+    if (!(fabsf(t) <= 3.402823466e38f)) {  // Inf / NaN: IEEE propagation through the spill
       atomicAdd(a.spill + col0 + cl, t);
       return;
     }
-    const int qi = fscale ? __float2int_rn(t * sf) : __double2int_rn((double)t * sd);
+    int qi;
+    if constexpr (decltype(fs)::value) qi = __float2int_rn(t * sf);
+    else qi = __double2int_rn((double)t * sd);
     const int old = atomicAdd(sw + cl, qi);  // native ATOMS.ADD (with return)
     const unsigned nw = (unsigned)old + (unsigned)qi;
     if ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0)  // signed wrap: carry into hi
       atomicAdd(a.hi + col0 + cl, qi > 0 ? 1 : -1);
   };
   // each lane takes 8 consecutive messages per step (a 16-byte column load and a 32-byte value
-  // load at 8-aligned indices), two steps in flight
-  for (int64_t p = pw0 + warp; p < pw1; p += kConsBS / 32) {
-    const int64_t lo = a.wsplit[3 * p + b], hi = a.wsplit[3 * p + b + 1];
-    for (int64_t g0 = (lo & ~int64_t(7)) + 8 * lane; g0 < hi; g0 += 2 * 256) {
-      uint4 cv[2];
-      float tv[2][8];
+  // load at 8-aligned indices), two steps in flight; which of the 8 are inside the warp's
+  // block-b range is one 8-bit mask per step
+  auto RUN = [&](auto fs) {
+    for (int64_t p = pw0 + warp; p < pw1; p += kConsBS / 32) {
+      const int64_t lo = a.wsplit[3 * p + b], hi = a.wsplit[3 * p + b + 1];
+      const int64_t gs = lo & ~int64_t(7);
+      const int nmsg = (int)(hi - gs);  // < 2^31 (a producer warp's range)
+      const int skip = (int)(lo - gs);  // 0..7
+      for (int o0 = 8 * lane; o0 < nmsg; o0 += 2 * 256) {
+        uint4 cv[2];
+        float tv[2][8];
 #pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int64_t g = g0 + u * 256;
-        if (g < hi) {
-          asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-              : "=r"(cv[u].x), "=r"(cv[u].y), "=r"(cv[u].z), "=r"(cv[u].w)
-              : "l"(a.bcol + g));
-          asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-              : "=f"(tv[u][0]), "=f"(tv[u][1]), "=f"(tv[u][2]), "=f"(tv[u][3]), "=f"(tv[u][4]), "=f"(tv[u][5]),
-                "=f"(tv[u][6]), "=f"(tv[u][7])
-              : "l"(a.bval + g));
+        for (int u = 0; u < 2; ++u) {
+          const int o = o0 + u * 256;
+          if (o < nmsg) {
+            asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                : "=r"(cv[u].x), "=r"(cv[u].y), "=r"(cv[u].z), "=r"(cv[u].w)
+                : "l"(a.bcol + gs + o));
+            asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                : "=f"(tv[u][0]), "=f"(tv[u][1]), "=f"(tv[u][2]), "=f"(tv[u][3]), "=f"(tv[u][4]),
+                  "=f"(tv[u][5]), "=f"(tv[u][6]), "=f"(tv[u][7])
+                : "l"(a.bval + gs + o));
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const int o = o0 + u * 256;
+          if (o >= nmsg) continue;
+          // entries e with skip <= o + e < nmsg
+          const int lo_e = skip - o, hi_e = nmsg - o;
+          const unsigned msk = (0xFFu << (lo_e > 0 ? lo_e : 0)) & (hi_e >= 8 ? 0xFFu : ((1u << hi_e) - 1u));
+          const uint32_t cw[4] = {cv[u].x, cv[u].y, cv[u].z, cv[u].w};
+#pragma unroll
+          for (int e = 0; e < 8; ++e)
+            if ((msk >> e) & 1u) ADD((int)((cw[e >> 1] >> (16 * (e & 1))) & 0xffffu), tv[u][e], fs);
         }
       }
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int64_t g = g0 + u * 256;
-        if (g >= hi) continue;
-        const uint32_t cw[4] = {cv[u].x, cv[u].y, cv[u].z, cv[u].w};
-#pragma unroll
-        for (int e = 0; e < 8; ++e)
-          if (g + e >= lo && g + e < hi) ADD((int)((cw[e >> 1] >> (16 * (e & 1))) & 0xffffu), tv[u][e]);
-      }
     }
+  };
+  if (allspill) {
+    // an infinite term: no finite scale, every message through the spill (IEEE semantics)
+    for (int64_t p = pw0 + warp; p < pw1; p += kConsBS / 32) {
+      const int64_t lo = a.wsplit[3 * p + b], hi = a.wsplit[3 * p + b + 1];
+      for (int64_t g = lo + lane; g < hi; g += 32) atomicAdd(a.spill + col0 + a.bcol[g], a.bval[g]);
+    }
+  } else if (fscale) {
+    RUN(std::true_type{});
+  } else {
+    RUN(std::false_type{});
   }
   __syncthreads();
   int32_t* dst = a.part + (int64_t)blockIdx.x * a.bw;
