@@ -401,7 +401,9 @@ fp_status launch_csr(const PatternArgs& a, const fp_launch& L_in, cudaStream_t s
              L.variant, smem);
   // L2 path: number of copies of w the CTAs spread their reds over (copies 1.. live in the
   // all-zero workspace accumulator and are folded into w after the kernel)
-  const int nrep = l2 ? l2_replicas(a) : 1;
+  // copies of w for the L2 reds: the chooser's rule, or an explicit plan's cluster field (1..16;
+  // the sweep varies it -- fp_launch.cluster is otherwise unused by the L2 variants)
+  const int nrep = !l2 ? 1 : (L.cluster > 0 ? std::min(L.cluster, 16) : l2_replicas(a));
   const size_t rep_doubles = nrep > 1 ? ((size_t)(nrep - 1) * a.n * dtype_size(a.dtype) + 7) / 8 : 0;
   Workspace* ws = workspace(s, l2 ? rep_doubles : (size_t)a.n, 0);
   if (!ws) return FP_ERR_NOMEM;

@@ -45,6 +45,7 @@ def main():
     ap.add_argument("--out", default=None)
     ap.add_argument("--variants", default=None, help="comma-separated subset of variants to sweep")
     ap.add_argument("--grids", default="74,148,222,296,370,444,592,740,888,1184,1776,2368")
+    ap.add_argument("--replicas", default="1,2,4,8,16", help="copies of w for the L2-red variants (large n)")
     args = ap.parse_args()
     dev = torch.device("cuda:0")
     cfg, inp = bench.build_inputs(args.config, 0, 1, dev)
@@ -85,18 +86,23 @@ def main():
     if args.variants:
         keep = {int(v) for v in args.variants.split(",")}
         space = [s for s in space if s[0] in keep]
+    # the L2-red variants also sweep the copies of w their reds spread over (fp_launch.cluster)
+    reps_l2 = [int(r) for r in args.replicas.split(",")] if csr and cfg["n"] > 8192 else [0]
+    space = [(var, vs, k, (r if var in (4, 7, 16) else 0)) for (var, vs, k) in space
+             for r in (reps_l2 if var in (4, 7, 16) else [0])]
     rows = []
-    for (var, vs, k), g in itertools.product(space, grids):
+    for (var, vs, k, rep), g in itertools.product(space, grids):
         L = fp.fp_launch()
         L.variant, L.vs, L.tl, L.bs, L.grid = var, vs, k, (1024 if var in (16, 17) else 256), g
+        L.cluster = rep
         try:
             ms = time_call(lambda: run(L), args.reps)
         except fp.FusedPatError as e:
-            rows.append(dict(variant=var, vs=vs, k=k, grid=g, ms=None, err=str(e)[:80]))
+            rows.append(dict(variant=var, vs=vs, k=k, grid=g, replicas=rep, ms=None, err=str(e)[:80]))
             continue
         w = inp["w"].double().cpu().numpy()
         rel = float(np.linalg.norm(w - ref) / max(np.linalg.norm(ref), 1e-300))
-        rows.append(dict(variant=var, vs=vs, k=k, grid=g, ms=ms, gbs=xb / ms / 1e6, rel_vs_chooser=rel,
+        rows.append(dict(variant=var, vs=vs, k=k, grid=g, replicas=rep, ms=ms, gbs=xb / ms / 1e6, rel_vs_chooser=rel,
                          ok=rel <= TOL[dt]))
     timed = sorted([r for r in rows if r["ms"] is not None], key=lambda r: r["ms"])
     rank = sum(1 for r in timed if r["ms"] < t_base) + 1
