@@ -89,6 +89,11 @@ def second_ceiling(cfg, plan, nnz, kern_ms, dev):
         ops = {"smem_gathers": nnz, "smem_fp_atomics": nnz}
         floor = nnz / r["gather_smem_f64"] + nnz / r["atom_smem_f64"]
         what = "y gathers from shared memory + shared-memory fp atomics (a CAS loop) per nonzero"
+    elif v == 19:  # packed: y and the partial w of a column block in shared memory
+        ops = {"smem_gathers": nnz, "smem_int_atomics": nnz}
+        floor = nnz / r["gather_smem_f64"] + nnz / r["atom_smem_u32"]
+        what = ("y gathers from shared memory (rate measured on fp64 words, an upper bound for fp32) + one "
+                "native int32 shared atomic per nonzero")
     elif v in (4, 7, 16, 17):
         prefix = min(n, int(plan.smem_bytes) // s) if v in (16, 17) else 0
         g = int(nnz * (1.0 - prefix / n))
@@ -283,6 +288,7 @@ def run_gpu(args):
 
     plan = None
     plan_ms = None
+    pack_info = None
     if name == "C5":
         iters = args.cg_iters
 
@@ -317,14 +323,27 @@ def run_gpu(args):
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         cplan = None
+        packed = False
         if comm is None:
             cplan = fp.CsrPlan(inp["rowptr"], inp["colidx"], n, inp["val"].dtype, launch=forced)
             torch.cuda.synchronize()
         plan_ms = (time.perf_counter() - t0) * 1e3
+        if comm is None and forced is None and args.pack and cfg["dtype"] == "f32":
+            # the column-blocked copy (fp_csr_plan_pack, variant 19): once per matrix, timed here
+            t0 = time.perf_counter()
+            try:
+                cplan.pack(inp["val"])
+                packed = True
+            except fp.FusedPatError as e:
+                print(f"[bench] no packed plan: {e}", file=sys.stderr)
+            torch.cuda.synchronize()
+            pack_ms = (time.perf_counter() - t0) * 1e3
+            if packed:
+                pack_info = dict(cplan.pack_info, pack_ms=round(pack_ms, 1))
 
         def step():
             if comm is None:
-                cplan(inp["val"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
+                cplan(None if packed else inp["val"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
             else:
                 fp.csr_dist(comm, inp["rowptr"], inp["colidx"], inp["val"], n, inp["y"], inp["v"], inp["z"], alpha,
                             beta, w=inp["w"])
@@ -342,6 +361,8 @@ def run_gpu(args):
         launches_per_step = 1
         if plan.variant == 17:  # producer, consumer, finalize (+ a 16-byte memset)
             launches_per_step = 3
+        elif plan.variant == 19:  # the packed pass + the finalize
+            launches_per_step = 2
         elif plan.variant in (4, 7, 16):
             s_b = 8 if cfg["dtype"] == "f64" else 4
             nrep = int(os.environ.get("FP_L2_REPLICAS", "0")) or (8 if 8 * n * s_b <= (16 << 20) else 1)
@@ -472,7 +493,8 @@ def run_gpu(args):
                        "plan": None if plan is None else {
                            k: int(getattr(plan, k)) for k in ("variant", "vs", "tl", "bs", "grid", "cluster",
                                                               "blocks_per_sm", "smem_bytes", "regs_per_thread")},
-                       "plan_create_ms": None if plan_ms is None else round(plan_ms, 2)},
+                       "plan_create_ms": None if plan_ms is None else round(plan_ms, 2),
+                       "packed_copy": pack_info},
             "evals_per_s": round(evals_per_s * (1 if name != "C5" else 1), 3),
             "pct_hbm_peak": round(100 * value / world / peak, 2),
             "x_bytes_per_eval": x_bytes, "algorithmic_bytes_per_eval": alg_bytes,
@@ -699,6 +721,8 @@ def main():
     ap.add_argument("--graph", dest="graph", action="store_true", default=True,
                     help="replay each step from a captured CUDA graph (default)")
     ap.add_argument("--no-graph", dest="graph", action="store_false")
+    ap.add_argument("--no-pack", dest="pack", action="store_false", default=True,
+                    help="CSR fp32: run the unpacked plan instead of the column-blocked copy (variant 19)")
     ap.add_argument("--launch", default=None, help="CSR only: force the plan 'variant,vs,k,grid' (profiling)")
     ap.add_argument("--exchange", default="peer", choices=["peer", "nvls", "nccl"],
                     help="N > 1: exchange of the partial w (fused peer memory, NVLS multicast, or NCCL)")

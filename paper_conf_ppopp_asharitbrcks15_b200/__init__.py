@@ -87,6 +87,8 @@ _SIGS = {
     "fp_csr_plan_exec": (_int, [_vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _vp]),
     "fp_csr_plan_launch": (_int, [_vp, _P(fp_launch)]),
     "fp_csr_plan_destroy": (_int, [_vp]),
+    "fp_csr_plan_pack": (_int, [_vp, _vp, _vp]),
+    "fp_csr_plan_pack_info": (_int, [_vp, _P(_i64), _P(_i64), _P(_int), _P(_int)]),
     "fp_dense_host": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_csr_host": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_release_workspace": (_int, []),
@@ -267,16 +269,34 @@ class CsrPlan:
         _call("fp_csr_plan_launch", self._h, ctypes.byref(L))
         return L
 
-    def __call__(self, val, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
-        _require_cuda(val, y, v, z, w)
+    def pack(self, val, stream=None):
+        """fp_csr_plan_pack: the column-blocked copy of the matrix with values ``val`` (variant 19);
+        afterwards ``plan(None, y, ...)`` evaluates Eq. (1) on the copy."""
+        _require_cuda(val)
         if val.dtype != self.dtype or val.shape[0] != self.nnz:
             raise ValueError(f"val must be {self.dtype}[{self.nnz}]")
-        y, v, z = _vec(y, self.n, val.dtype, "y"), _vec(v, self.m, val.dtype, "v"), _vec(z, self.n, val.dtype, "z")
+        _call("fp_csr_plan_pack", self._h, _ptr(val), _stream(val.device, stream))
+        self._packed_dev = val.device
+
+    @property
+    def pack_info(self):
+        nt, ne, cs, gr = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int(), ctypes.c_int()
+        _call("fp_csr_plan_pack_info", self._h, ctypes.byref(nt), ctypes.byref(ne), ctypes.byref(cs),
+              ctypes.byref(gr))
+        return {"tiles": nt.value, "entries": ne.value, "blocks": cs.value, "groups": gr.value}
+
+    def __call__(self, val, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
+        """Eq. (1) on the plan's matrix with values ``val``; ``val=None`` uses the packed copy."""
+        _require_cuda(val, y, v, z, w)
+        if val is not None and (val.dtype != self.dtype or val.shape[0] != self.nnz):
+            raise ValueError(f"val must be {self.dtype}[{self.nnz}]")
+        dev = val.device if val is not None else self.rowptr.device
+        y, v, z = _vec(y, self.n, self.dtype, "y"), _vec(v, self.m, self.dtype, "v"), _vec(z, self.n, self.dtype, "z")
         if w is None:
-            w = torch.empty(self.n, dtype=val.dtype, device=val.device)
-        _vec(w, self.n, val.dtype, "w")
+            w = torch.empty(self.n, dtype=self.dtype, device=dev)
+        _vec(w, self.n, self.dtype, "w")
         _call("fp_csr_plan_exec", self._h, _ptr(val), _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w),
-              _stream(val.device, stream))
+              _stream(dev, stream))
         return w
 
     def close(self):

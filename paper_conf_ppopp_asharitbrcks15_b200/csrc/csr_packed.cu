@@ -1,0 +1,809 @@
+// csr_packed.cu -- variant 19 (FP_VAR_CSR_PACKED): Eq. (1) on a column-blocked copy of a CSR
+// matrix whose y and partial w do not fit one SM (C4: n = 1e5 fp32), X read once per call.
+//
+// Why.  For n beyond one SM's shared memory every nonzero costs a random access to the
+// L2-resident y and w (variants 7/16: 2e9 reds + 2e9 gathers, ~11 ms of issuing cost on
+// sm_100a) or a message round trip through HBM (variant 17: 12 GB written + read).  Split the
+// COLUMNS instead: a group of CS CTAs (one per SM) holds y and the partial w of column block k
+// (CTA k) in shared memory, so every gather and every scatter is a shared-memory access (y as
+// fp32, w as 32-bit fixed point with native integer atomics).  Each CTA streams only the
+// nonzeros of its block; the row dots of Eq. (2) are completed by summing the CS block partials
+// of each row (a 32-row exchange per tile through L2), then Eq. (3) scatters the terms from
+// the registers that still hold the row (a7: scale-back from the same registers).
+//
+// The copy (fp_csr_plan_pack, once per matrix, amortised over calls as the paper amortises
+// its baseline's transpose): for each column block k the block-k segments of every row
+// stored contiguously; rows grouped into TILES (<= 32 rows, every block segment <= 256
+// entries, or one long row); each entry one 32-bit word (column inside the block | row inside
+// the tile << 16) + its value; every segment starts 16-byte aligned.  The row structure of a
+// tile is therefore in the entries themselves: no rowptr search and no head masks per call.
+//
+// One call: k_pk (the whole Eq. 1 pass, cooperative launch: the CTAs of a group wait on each
+// other) + k_pk_finalize (sums the groups' partials in a fixed order, adds beta z).
+//
+// Fixed point (reading R25): CTA c adds every term t = x q as round(t / quantum_c)
+// into a 32-bit shared accumulator, quantum_c = 2^(E_c - 26), E_c = (exponent of the largest
+// finite |t| of the CTA's first tile round) + H (H = 3 headroom bits): |t| < 2^E_c gives an
+// int32 of magnitude < 2^26 (error <= quantum_c / 2 per term); larger or non-finite terms and
+// the (rare) int32 wraps go to an fp64 spill vector with global reds.  The partials are
+// converted exactly to fp64 and summed in group order: deterministic except for spills.
+#include <algorithm>
+#include <cstdlib>
+#include <new>
+#include <vector>
+
+#include <cub/device/device_scan.cuh>
+
+#include "kernels.cuh"
+
+namespace fp {
+
+namespace {
+
+constexpr int kPkBS = 1024;
+constexpr int kPkNW = kPkBS / 32;
+constexpr int kPkSpan = 256;          // entries of a block segment held in registers (2 super-tiles)
+constexpr int kPkRowCost = 4;         // work of a row in entries (warp partition)
+constexpr int kPkStatic = 9 * 1024;   // static shared memory reserve of k_pk
+
+struct PkArgs {
+  int64_t n;
+  int bw;                        // columns per block (block k = [k bw, min(n, (k+1) bw)))
+  int groups;
+  int64_t ntiles;
+  const int64_t* tile_row;       // [ntiles + 1]
+  const uint2* tile_seg;         // [cs][ntiles]: (offset / 4, length) of the tile's block-k segment
+  const int32_t* wtile;          // [groups * 32 + 1]: first tile of each warp-quad
+  const uint32_t* cr;            // packed entry words
+  const float* val;
+  const float* y;
+  const float* v;
+  float alpha;
+  int hbits;                     // headroom bits of the fixed-point cap
+  unsigned long long* xch;       // exchange slots [groups][32 warps][2][cs][32 lanes]
+  const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
+  double* part;                  // [groups][n]
+  double* spill;                 // [n], all-zero between calls
+};
+
+__device__ __forceinline__ void pk_ld4(const uint32_t* pc, const float* pv, uint32_t (&c)[4], float (&x)[4]) {
+  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+      : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3])
+      : "l"(pc));
+  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+      : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3])
+      : "l"(pv));
+}
+__device__ __forceinline__ void st_relaxed_gpu(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_gpu(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned pk_lanemask_lt() {
+  unsigned r;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
+  return r;
+}
+
+// Per-warp state of one tile between its dot and its scatter.
+struct PkTile {
+  int64_t row0;
+  int nrows;
+  int64_t A;      // first entry of the segment (multiple of 4)
+  int len;        // entries of the segment (> kPkSpan: long, streamed)
+};
+
+template <int CS, int YM>
+__global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
+  extern __shared__ __align__(16) unsigned char pk_smem[];
+  __shared__ float rs[kPkNW][32];   // the tile's block partials of the row dots (by row in tile)
+  __shared__ float qsm[kPkNW][32];  // q of the tile's rows (rare spill path)
+  __shared__ unsigned s_tmax;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int k = CS == 1 ? 0 : (int)(blockIdx.x % CS);
+  const int g = CS == 1 ? (int)blockIdx.x : (int)(blockIdx.x / CS);
+  const int bw = a.bw;
+  const int64_t c0 = (int64_t)k * bw;
+  const int bwk = (int)max((int64_t)0, min((int64_t)bw, a.n - c0));  // columns of this block
+  float* y_s = reinterpret_cast<float*>(pk_smem);
+  int* acc = reinterpret_cast<int*>(pk_smem + (YM ? (size_t)bw * 4 : 0));
+  for (int j = threadIdx.x; j < bw; j += kPkBS) {
+    if (YM) y_s[j] = j < bwk ? a.y[c0 + j] : 0.f;
+    acc[j] = 0;
+  }
+  if (threadIdx.x == 0) s_tmax = 0u;
+  __syncthreads();
+
+  const int gq = g * kPkNW + warp;
+  const int64_t t0 = a.wtile[gq], t1 = a.wtile[gq + 1];
+  const uint2* __restrict__ seg = a.tile_seg + (int64_t)k * a.ntiles;
+  const unsigned tag0 = *a.epoch << 20;
+  unsigned long long* const xslot = a.xch + (int64_t)gq * 2 * CS * 32;
+  const float alpha = a.alpha;
+
+  auto info = [&](int64_t t) -> PkTile {
+    PkTile T;
+    const int64_t r0 = __ldg(a.tile_row + t), r1 = __ldg(a.tile_row + t + 1);
+    const uint2 s = __ldg(seg + t);
+    T.row0 = r0;
+    T.nrows = (int)(r1 - r0);
+    T.A = (int64_t)s.x * 4;
+    T.len = (int)s.y;
+    return T;
+  };
+
+  // ---- the two halves of a tile.  Window registers: two super-tiles of 128 entries, lane l
+  // holding entries 4l..4l+3 of each (16-byte loads).
+  uint32_t cw[2][4];
+  float xv[2][4];
+  float q = 0.f;  // q of row `lane` of the tile
+  float qs = 0.f; // q / quantum
+
+  // dot + exchange + q.  Returns the largest finite |x q| of the tile's active entries.
+  auto dot_q = [&](const PkTile& T, int64_t seq, bool need_tm) -> float {
+    const float vr = (lane < T.nrows) ? (a.v ? __ldg(a.v + T.row0 + lane) : 1.f) : 0.f;
+    const bool lng = T.len > kPkSpan;
+    if (!lng) {
+#pragma unroll
+      for (int st = 0; st < 2; ++st) {
+        const int o = 128 * st + 4 * lane;
+        if (o < T.len) {
+          pk_ld4(a.cr + T.A + o, a.val + T.A + o, cw[st], xv[st]);
+        } else {
+#pragma unroll
+          for (int e = 0; e < 4; ++e) cw[st][e] = 31u << 16, xv[st][e] = 0.f;
+        }
+      }
+    }
+    float p = 0.f;
+    if constexpr (YM != 0) {
+      if (!lng) {
+        rs[warp][lane] = 0.f;
+        __syncwarp();
+        int carry = -1;  // row of the previous super-tile's last entry
+#pragma unroll
+        for (int st = 0; st < 2; ++st) {
+          if (128 * st >= T.len) break;
+          int rid[4];
+          float s[4];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const bool act = 128 * st + 4 * lane + e < T.len;
+            rid[e] = act ? (int)(cw[st][e] >> 16) : 31;
+            const float yy = y_s[cw[st][e] & 0xffffu];
+            s[e] = act ? xv[st][e] * yy : 0.f;  // Eq. (2) products (inactive: exactly 0)
+          }
+          int prev = __shfl_up_sync(0xffffffffu, rid[3], 1);
+          if (lane == 0) prev = carry;
+          unsigned hb = 0;
+#pragma unroll
+          for (int e = 0; e < 4; ++e) hb |= (unsigned)(rid[e] != (e ? rid[e - 1] : prev)) << e;
+          // in-lane: P = entries before the first head; complete runs stored; `sum` = last run
+          float sum = 0.f, P = 0.f;
+          bool first = true;
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            if ((hb >> e) & 1u) {
+              if (first) P = sum;
+              else rs[warp][rid[e - 1]] = sum;  // a row entirely inside this lane
+              first = false;
+              sum = 0.f;
+            }
+            sum += s[e];
+          }
+          if (!hb) P = sum;
+          // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a head
+          const unsigned H = __ballot_sync(0xffffffffu, hb != 0u);
+          const unsigned hl = H >> lane;
+          const int dist = hl ? __ffs(hl) : 32 - lane;
+          float r = P;
+#pragma unroll
+          for (int d = 1; d < 32; d <<= 1) {
+            const float t2 = __shfl_down_sync(0xffffffffu, r, d);
+            if (d < dist) r += t2;
+          }
+          float rn = __shfl_down_sync(0xffffffffu, r, 1);
+          if (lane == 31) rn = 0.f;
+          if (hb) rs[warp][rid[3]] = sum + rn;            // the lane's last row: its run + what follows
+          if (lane == 0 && !(hb & 1u) && prev >= 0) rs[warp][prev] += r;  // row running in
+          carry = __shfl_sync(0xffffffffu, rid[3], 31);
+          __syncwarp();
+        }
+        p = rs[warp][lane];
+      } else {
+        // a long row (the tile's only row): stream the segment, every load of a step in flight
+        float s = 0.f;
+        for (int s0 = 0; s0 < T.len; s0 += kPkSpan) {
+          uint32_t c2[2][4];
+          float x2[2][4];
+#pragma unroll
+          for (int st = 0; st < 2; ++st) {
+            const int o = s0 + 128 * st + 4 * lane;
+            if (o < T.len) pk_ld4(a.cr + T.A + o, a.val + T.A + o, c2[st], x2[st]);
+            else {
+#pragma unroll
+              for (int e = 0; e < 4; ++e) c2[st][e] = 0u, x2[st][e] = 0.f;
+            }
+          }
+#pragma unroll
+          for (int st = 0; st < 2; ++st)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const bool act = s0 + 128 * st + 4 * lane + e < T.len;
+              const float pr = x2[st][e] * y_s[c2[st][e] & 0xffffu];
+              s += act ? pr : 0.f;
+            }
+        }
+        s = fpd::vector_allreduce<32>(s);
+        p = lane == 0 ? s : 0.f;
+      }
+      // exchange of the block partials inside the group (the CS CTAs' warps `warp` walk the
+      // same tile list): value + tag in one 64-bit word, so no flag and no fence is needed
+      if constexpr (CS > 1) {
+        const unsigned tag = tag0 + (unsigned)seq;
+        unsigned long long* slot = xslot + (int64_t)(seq & 1) * CS * 32;
+        st_relaxed_gpu(slot + k * 32 + lane, ((unsigned long long)tag << 32) | __float_as_uint(p));
+        unsigned long long wv[CS];
+        bool done;
+        do {
+          done = true;
+#pragma unroll
+          for (int j = 0; j < CS; ++j) {
+            if (j != k) {
+              wv[j] = ld_relaxed_gpu(slot + j * 32 + lane);
+              done &= (unsigned)(wv[j] >> 32) == tag;
+            }
+          }
+        } while (!done);
+        float tot = 0.f;
+#pragma unroll
+        for (int j = 0; j < CS; ++j) tot += j == k ? p : __uint_as_float((unsigned)wv[j]);  // fixed order
+        p = tot;
+      }
+      q = alpha * (vr * p);
+    } else {
+      (void)seq;
+      q = alpha * vr;
+    }
+    if (lane >= T.nrows) q = 0.f;
+    qsm[warp][lane] = q;
+    // largest finite |term| of the tile (the fixed-point cap of the first round)
+    float tm = 0.f;
+    if (!need_tm) return tm;
+    if (!lng) {
+#pragma unroll
+      for (int st = 0; st < 2; ++st)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const bool act = 128 * st + 4 * lane + e < T.len;
+          const float qe = __shfl_sync(0xffffffffu, q, (int)(cw[st][e] >> 16) & 31);
+          const float t = fabsf(xv[st][e] * qe);
+          if (act && t <= 3.402823466e38f) tm = fmaxf(tm, t);
+        }
+    } else {
+      const float q0 = fabsf(__shfl_sync(0xffffffffu, q, 0));
+      for (int o = 4 * lane; o < T.len; o += 128) {
+        uint32_t c2[4];
+        float x2[4];
+        pk_ld4(a.cr + T.A + o, a.val + T.A + o, c2, x2);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float t = fabsf(x2[e]) * q0;
+          if (o + e < T.len && t <= 3.402823466e38f) tm = fmaxf(tm, t);
+        }
+      }
+    }
+    return tm;
+  };
+
+  int E = 0;          // cap exponent: |t| < 2^E goes fixed point
+  float sc = 1.f;     // 2^(26 - E)
+  double quantum = 0; // 2^(E - 26)
+  auto set_scale = [&](int e) {
+    E = min(max(e, -95), 100);
+    sc = ldexpf(1.f, 26 - E);
+    quantum = ldexp(1.0, E - 26);
+  };
+  set_scale(0);
+
+  // one term into the CTA's fixed-point partial (or the spill)
+  auto add_term = [&](int col, float x, float qe, int rid) {
+    const float ts = x * qe;
+    if (fabsf(ts) < 67108864.f) {  // 2^26
+      const int qi = __float2int_rn(ts);
+      const int old = atomicAdd(acc + col, qi);  // native ATOMS.ADD
+      const unsigned nw = (unsigned)old + (unsigned)qi;
+      if ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0)  // int32 wrap: carry 2^32 quanta
+        atomicAdd(a.spill + c0 + col, qi > 0 ? 4294967296.0 * quantum : -4294967296.0 * quantum);
+    } else {  // beyond the cap, or Inf / NaN (IEEE propagation, reading R8)
+      atomicAdd(a.spill + c0 + col, (double)(x * qsm[warp][rid]));
+    }
+  };
+
+  auto scatter = [&](const PkTile& T) {
+    qs = q * sc;
+    if (T.len <= kPkSpan) {
+#pragma unroll
+      for (int st = 0; st < 2; ++st) {
+        if (128 * st >= T.len) break;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int rid = (int)(cw[st][e] >> 16) & 31;
+          const float qe = __shfl_sync(0xffffffffu, qs, rid);
+          if (128 * st + 4 * lane + e < T.len) add_term((int)(cw[st][e] & 0xffffu), xv[st][e], qe, rid);
+        }
+      }
+    } else {
+      // the long row's segment is re-read (just streamed: mostly an L2 hit)
+      const float q0 = __shfl_sync(0xffffffffu, qs, 0);
+      for (int s0 = 0; s0 < T.len; s0 += kPkSpan) {
+        uint32_t c2[2][4];
+        float x2[2][4];
+#pragma unroll
+        for (int st = 0; st < 2; ++st) {
+          const int o = s0 + 128 * st + 4 * lane;
+          if (o < T.len) pk_ld4(a.cr + T.A + o, a.val + T.A + o, c2[st], x2[st]);
+        }
+#pragma unroll
+        for (int st = 0; st < 2; ++st)
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            if (s0 + 128 * st + 4 * lane + e < T.len) add_term((int)(c2[st][e] & 0xffffu), x2[st][e], q0, 0);
+      }
+    }
+  };
+
+  // ---- first rounds: one tile per warp until some finite term is nonzero, then the CTA's cap
+  int64_t t = t0;
+  for (;;) {
+    const bool have = t < t1;
+    PkTile T{};
+    float tm = 0.f;
+    if (have) {
+      T = info(t);
+      tm = dot_q(T, t - t0, true);
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) tm = fmaxf(tm, __shfl_xor_sync(0xffffffffu, tm, d));
+    if (lane == 0 && tm > 0.f) atomicMax(&s_tmax, __float_as_uint(tm));
+    const int any = __syncthreads_or(have);
+    const float mx = __uint_as_float(*(volatile unsigned*)&s_tmax);
+    const bool done = mx > 0.f || !any;
+    if (mx > 0.f) {
+      int e0;
+      frexpf(mx, &e0);  // mx < 2^e0
+      set_scale(e0 + a.hbits);
+    }
+    // (while every finite term so far is 0, scale 2^26 adds zeros; non-finite terms spill)
+    if (have) scatter(T);
+    if (have) ++t;
+    if (done) break;
+  }
+
+  // ---- steady state
+  for (; t < t1; ++t) {
+    const PkTile T = info(t);
+    if (lane == 0 && t + 1 < t1) {  // the next tile's segment on its way into L2
+      const uint2 s1 = __ldg(seg + t + 1);
+      const int n1 = (int)min((unsigned)s1.y, 4096u);
+      if (n1 > 0) {
+        fpd::prefetch_l2(a.cr + (int64_t)s1.x * 4, (size_t)n1 * 4);
+        fpd::prefetch_l2(a.val + (int64_t)s1.x * 4, (size_t)n1 * 4);
+      }
+    }
+    (void)dot_q(T, t - t0, false);
+    scatter(T);
+  }
+
+  __syncthreads();
+  double* dst = a.part + (int64_t)g * a.n + c0;
+  for (int j = threadIdx.x; j < bwk; j += kPkBS) dst[j] = (double)acc[j] * quantum;
+}
+
+__global__ void k_pk_finalize(int64_t n, int groups, const double* __restrict__ part, double* __restrict__ spill,
+                              const float* __restrict__ z, double beta, int add_beta_z, int accumulate, float* w,
+                              unsigned* epoch) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+    for (int gi = 0; gi < groups; ++gi) s += part[(int64_t)gi * n + j];  // fixed order
+    s += spill[j];
+    if (add_beta_z && beta != 0.0) s += beta * (double)z[j];
+    if (accumulate) s += (double)w[j];
+    w[j] = (float)s;
+    spill[j] = 0.0;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) *epoch += 1u;
+}
+
+// ------------------------------------------------------------------------------ plan side
+// (1) entries of each row in each column block
+__global__ void k_pk_count(int64_t m, const int64_t* __restrict__ rowptr, const int32_t* __restrict__ colidx,
+                           int cs, int bw, uint32_t* __restrict__ cnt) {
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t c[kPkMaxCS] = {};
+    const int64_t e = rowptr[r + 1];
+    for (int64_t i = rowptr[r]; i < e; ++i) {
+      const int b = colidx[i] / bw;
+#pragma unroll
+      for (int kk = 0; kk < kPkMaxCS; ++kk) c[kk] += (uint32_t)(b == kk);
+    }
+    for (int kk = 0; kk < cs; ++kk) cnt[(int64_t)kk * m + r] = c[kk];
+  }
+}
+
+// (2) tiles of each 32-row group (greedy): bit i of gmask set where a tile starts at row 32 g + i
+__device__ __forceinline__ bool pk_is_long(const uint32_t* cnt, int64_t m, int cs, int64_t r) {
+  for (int kk = 0; kk < cs; ++kk)
+    if (cnt[(int64_t)kk * m + r] > (uint32_t)kPkSpan) return true;
+  return false;
+}
+__global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, uint32_t* __restrict__ gmask,
+                           int64_t* __restrict__ gcount) {
+  const int64_t ng = (m + 31) / 32;
+  for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t accs[kPkMaxCS] = {};
+    uint32_t mask = 0;
+    int ntl = 0;
+    bool fresh = true;  // the next row starts a tile
+    for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
+      const int64_t r = gi * 32 + i;
+      if (pk_is_long(cnt, m, cs, r)) {
+        mask |= 1u << i;
+        ++ntl;
+        fresh = true;
+        continue;
+      }
+      bool fit = !fresh;
+      for (int kk = 0; kk < cs && fit; ++kk) fit = accs[kk] + cnt[(int64_t)kk * m + r] <= (uint32_t)kPkSpan;
+      if (!fit) {
+        mask |= 1u << i;
+        ++ntl;
+        for (int kk = 0; kk < cs; ++kk) accs[kk] = 0;
+      }
+      for (int kk = 0; kk < cs; ++kk) accs[kk] += cnt[(int64_t)kk * m + r];
+      fresh = false;
+    }
+    gmask[gi] = mask;
+    gcount[gi] = ntl;
+  }
+}
+
+// (3) tile rows and segment lengths; al = the lengths rounded up to 4 (scanned into offsets)
+__global__ void k_pk_tile_rows(int64_t m, int cs, int64_t ntiles, const uint32_t* __restrict__ cnt,
+                               const uint32_t* __restrict__ gmask, const int64_t* __restrict__ gbase,
+                               int64_t* __restrict__ tile_row, uint32_t* __restrict__ tlen, int64_t* __restrict__ al) {
+  const int64_t ng = (m + 31) / 32;
+  for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t mask = gmask[gi];
+    int64_t t = gbase[gi] - 1;
+    uint32_t len[kPkMaxCS] = {};
+    auto flush = [&]() {
+      if (t < 0) return;
+      for (int kk = 0; kk < cs; ++kk) {
+        tlen[(int64_t)kk * ntiles + t] = len[kk];
+        al[(int64_t)kk * ntiles + t] = (int64_t)((len[kk] + 3u) & ~3u);
+        len[kk] = 0;
+      }
+    };
+    for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
+      const int64_t r = gi * 32 + i;
+      if ((mask >> i) & 1u) {
+        flush();
+        ++t;
+        tile_row[t] = r;
+      }
+      for (int kk = 0; kk < cs; ++kk) len[kk] += cnt[(int64_t)kk * m + r];
+    }
+    flush();
+    if (gi == ng - 1) tile_row[ntiles] = m;
+  }
+}
+
+__global__ void k_pk_seg(int64_t total, const int64_t* __restrict__ off, const uint32_t* __restrict__ tlen,
+                         uint2* __restrict__ seg) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
+    seg[i] = make_uint2((unsigned)(off[i] >> 2), tlen[i]);
+}
+
+// (4) the entries: a warp per 32-row group, lanes over a row's entries; block-k entries keep
+// their order (stable), so non-canonical rows are packed as given (reading R7)
+__global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const int64_t* __restrict__ rowptr,
+                             const int32_t* __restrict__ colidx, const float* __restrict__ val,
+                             const uint32_t* __restrict__ gmask, const int64_t* __restrict__ gbase,
+                             const uint2* __restrict__ seg, uint32_t* __restrict__ cr, float* __restrict__ pval) {
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = pk_lanemask_lt();
+  const int64_t ng = (m + 31) / 32;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
+  for (int64_t gi = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5); gi < ng; gi += nw) {
+    const uint32_t mask = gmask[gi];
+    int64_t t = gbase[gi] - 1;
+    int64_t run[kPkMaxCS] = {};
+    int rid = 0;
+    for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
+      const int64_t r = gi * 32 + i;
+      if ((mask >> i) & 1u) {
+        ++t;
+        rid = 0;
+        for (int kk = 0; kk < cs; ++kk) run[kk] = (int64_t)seg[(int64_t)kk * ntiles + t].x * 4;
+      }
+      const int64_t e = rowptr[r + 1];
+      for (int64_t i0 = rowptr[r]; i0 < e; i0 += 32) {
+        const int64_t ii = i0 + lane;
+        const bool ok = ii < e;
+        const int col = ok ? colidx[ii] : 0;
+        const int b = col / bw;
+        int64_t pos = -1;
+        for (int kk = 0; kk < cs; ++kk) {
+          const unsigned bm = __ballot_sync(0xffffffffu, ok && b == kk);
+          if (ok && b == kk) pos = run[kk] + __popc(bm & lt);
+          run[kk] += __popc(bm);
+        }
+        if (ok) {
+          cr[pos] = (uint32_t)(col - b * bw) | ((uint32_t)rid << 16);
+          pval[pos] = val ? val[ii] : 0.f;
+        }
+      }
+      ++rid;
+    }
+  }
+}
+
+// (5) warp-quad partition: tile ranges of equal nonzero + row cost
+__global__ void k_pk_partition(int64_t ntiles, int nq, const int64_t* __restrict__ tile_row,
+                               const int64_t* __restrict__ rowptr, int32_t* __restrict__ wtile) {
+  const int qi = blockIdx.x * blockDim.x + threadIdx.x;
+  if (qi > nq) return;
+  auto cost = [&](int64_t t) { const int64_t r = tile_row[t]; return rowptr[r] - rowptr[0] + kPkRowCost * r; };
+  const int64_t total = cost(ntiles);
+  const int64_t target = (int64_t)((__int128)total * qi / nq);
+  int64_t lo = 0, hi = ntiles;  // smallest t with cost(t) >= target
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) / 2;
+    if (cost(mid) >= target) hi = mid;
+    else lo = mid + 1;
+  }
+  wtile[qi] = (int32_t)(qi == nq ? ntiles : lo);
+}
+
+template <int CS, int YM>
+const void* pk_kernel() {
+  return (const void*)k_pk<CS, YM>;
+}
+const void* pk_pick(int cs, bool has_y) {
+  switch (cs) {
+    case 1: return has_y ? pk_kernel<1, 1>() : pk_kernel<1, 0>();
+    case 2: return has_y ? pk_kernel<2, 1>() : pk_kernel<2, 0>();
+    case 4: return has_y ? pk_kernel<4, 1>() : pk_kernel<4, 0>();
+    case 8: return has_y ? pk_kernel<8, 1>() : pk_kernel<8, 0>();
+  }
+  return nullptr;
+}
+
+int pk_headroom() {
+  static const int h = [] {
+    const char* e = std::getenv("FP_PK_HEADROOM");
+    return e ? std::atoi(e) : 3;
+  }();
+  return h;
+}
+
+}  // namespace
+
+// columns one CTA holds (y fp32 + int32 partial in the opt-in shared memory)
+int packed_max_bw() {
+  const size_t room = device_info(current_device()).smem_optin_per_block - kPkStatic;
+  return (int)std::min<size_t>(room / 8, 65535);
+}
+
+int packed_cs(int64_t n) {
+  const int64_t mb = packed_max_bw();
+  for (int cs : {1, 2, 4, 8})
+    if ((n + cs - 1) / cs <= mb) return cs;
+  return 0;
+}
+
+void packed_free(Packed* p) {
+  if (!p) return;
+  for (void* b : {(void*)p->tile_row, (void*)p->tile_seg, (void*)p->wtile, (void*)p->cr, (void*)p->val,
+                  (void*)p->xch, (void*)p->epoch, (void*)p->part, (void*)p->spill})
+    if (b) cudaFree(b);
+  delete p;
+}
+
+fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                       const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s) {
+  *out = nullptr;
+  FP_REQUIRE(dtype == FP_F32, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: the packed variant is fp32 only");
+  FP_REQUIRE(val || nnz == 0, FP_ERR_INVALID_ARG, "fp_csr_plan_pack: val is NULL");
+  FP_REQUIRE(m >= 1 && n >= 1, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: empty matrix");
+  const int cs = cs_force > 0 ? cs_force : packed_cs(n);
+  FP_REQUIRE(cs == 1 || cs == 2 || cs == 4 || cs == 8, FP_ERR_UNSUPPORTED,
+             "fp_csr_plan_pack: n = %lld needs more than 8 column blocks", (long long)n);
+  const int bw = (int)((n + cs - 1) / cs);
+  FP_REQUIRE(bw <= packed_max_bw(), FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: n = %lld too wide for %d blocks",
+             (long long)n, cs);
+  const DeviceInfo& di = device_info(current_device());
+  const int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
+  Packed* p = new (std::nothrow) Packed;
+  FP_REQUIRE(p, FP_ERR_NOMEM, "fp_csr_plan_pack: out of host memory");
+  p->m = m;
+  p->n = n;
+  p->nnz = nnz;
+  p->cs = cs;
+  p->bw = bw;
+  p->groups = groups;
+  p->rowptr = rowptr;
+  const int64_t ng = (m + 31) / 32;
+  uint32_t* cnt = nullptr;
+  uint32_t* gmask = nullptr;
+  int64_t* gcount = nullptr;
+  int64_t* gbase = nullptr;
+  int64_t* al = nullptr;
+  int64_t* off = nullptr;
+  uint32_t* tlen = nullptr;
+  void* tmp = nullptr;
+  auto cleanup = [&]() {
+    for (void* b : {(void*)cnt, (void*)gmask, (void*)gcount, (void*)gbase, (void*)al, (void*)off, (void*)tlen, tmp})
+      if (b) cudaFree(b);
+  };
+  auto fail = [&](cudaError_t e, const char* what) {
+    cudaGetLastError();
+    set_error("fp_csr_plan_pack: %s: %s", what, cudaGetErrorString(e));
+    cleanup();
+    packed_free(p);
+    return e == cudaErrorMemoryAllocation ? FP_ERR_NOMEM : FP_ERR_CUDA;
+  };
+#define PK_TRY(call, what)                 \
+  do {                                     \
+    cudaError_t e_ = (call);               \
+    if (e_ != cudaSuccess) return fail(e_, what); \
+  } while (0)
+  PK_TRY(cudaMalloc((void**)&cnt, (size_t)cs * m * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&gmask, (size_t)ng * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&gcount, (size_t)ng * 8), "alloc");
+  PK_TRY(cudaMalloc((void**)&gbase, (size_t)ng * 8), "alloc");
+  const int tb = 256;
+  const int grid_r = (int)std::min<int64_t>((m + tb - 1) / tb, (int64_t)di.sm_count * 32);
+  const int grid_g = (int)std::min<int64_t>((ng + tb - 1) / tb, (int64_t)di.sm_count * 32);
+  k_pk_count<<<grid_r, tb, 0, s>>>(m, rowptr, colidx, cs, bw, cnt);
+  k_pk_tiles<<<grid_g, tb, 0, s>>>(m, cs, cnt, gmask, gcount);
+  size_t tb_bytes = 0;
+  PK_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, gcount, gbase, ng, s), "scan");
+  size_t tmp_bytes = tb_bytes;
+  PK_TRY(cudaMalloc(&tmp, tmp_bytes), "alloc");
+  PK_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb_bytes, gcount, gbase, ng, s), "scan");
+  int64_t hb[2] = {0, 0};
+  PK_TRY(cudaMemcpyAsync(&hb[0], gbase + ng - 1, 8, cudaMemcpyDeviceToHost, s), "copy");
+  PK_TRY(cudaMemcpyAsync(&hb[1], gcount + ng - 1, 8, cudaMemcpyDeviceToHost, s), "copy");
+  PK_TRY(cudaStreamSynchronize(s), "sync");
+  const int64_t ntiles = hb[0] + hb[1];
+  p->ntiles = ntiles;
+  const int64_t segs = (int64_t)cs * ntiles;
+  PK_TRY(cudaMalloc((void**)&p->tile_row, (size_t)(ntiles + 1) * 8), "alloc");
+  PK_TRY(cudaMalloc((void**)&tlen, (size_t)segs * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&al, (size_t)segs * 8), "alloc");
+  PK_TRY(cudaMalloc((void**)&off, (size_t)segs * 8), "alloc");
+  k_pk_tile_rows<<<grid_g, tb, 0, s>>>(m, cs, ntiles, cnt, gmask, gbase, p->tile_row, tlen, al);
+  PK_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, al, off, segs, s), "scan");
+  if (tb_bytes > tmp_bytes) {
+    cudaFree(tmp);
+    tmp = nullptr;
+    tmp_bytes = tb_bytes;
+    PK_TRY(cudaMalloc(&tmp, tmp_bytes), "alloc");
+  }
+  PK_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb_bytes, al, off, segs, s), "scan");
+  int64_t ht[2] = {0, 0};
+  PK_TRY(cudaMemcpyAsync(&ht[0], off + segs - 1, 8, cudaMemcpyDeviceToHost, s), "copy");
+  PK_TRY(cudaMemcpyAsync(&ht[1], al + segs - 1, 8, cudaMemcpyDeviceToHost, s), "copy");
+  PK_TRY(cudaStreamSynchronize(s), "sync");
+  const int64_t total = ht[0] + ht[1];
+  if (total / 4 >= (int64_t)UINT32_MAX) return fail(cudaErrorInvalidValue, "too many nonzeros for 32-bit offsets");
+  p->entries = total;
+  PK_TRY(cudaMalloc((void**)&p->tile_seg, (size_t)segs * sizeof(uint2)), "alloc");
+  k_pk_seg<<<(int)std::min<int64_t>((segs + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(segs, off, tlen,
+                                                                                                   p->tile_seg);
+  PK_TRY(cudaMalloc((void**)&p->cr, (size_t)std::max<int64_t>(total, 4) * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&p->val, (size_t)std::max<int64_t>(total, 4) * 4), "alloc");
+  PK_TRY(cudaMemsetAsync(p->cr, 0, (size_t)std::max<int64_t>(total, 4) * 4, s), "memset");
+  PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)std::max<int64_t>(total, 4) * 4, s), "memset");
+  k_pk_scatter<<<(int)std::min<int64_t>((ng + 7) / 8, (int64_t)di.sm_count * 16), 256, 0, s>>>(
+      m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase, p->tile_seg, p->cr, p->val);
+  const int nq = groups * kPkNW;
+  if (ntiles >= INT32_MAX) return fail(cudaErrorInvalidValue, "too many tiles");
+  PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
+  k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, p->tile_row, rowptr, p->wtile);
+  // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
+  const size_t xbytes = (size_t)groups * kPkNW * 2 * cs * 32 * 8;
+  PK_TRY(cudaMalloc((void**)&p->xch, xbytes), "alloc");
+  PK_TRY(cudaMemsetAsync(p->xch, 0, xbytes, s), "memset");
+  PK_TRY(cudaMalloc((void**)&p->epoch, 16), "alloc");
+  const unsigned one = 1;
+  PK_TRY(cudaMemcpyAsync(p->epoch, &one, 4, cudaMemcpyHostToDevice, s), "copy");
+  PK_TRY(cudaMalloc((void**)&p->part, (size_t)groups * n * 8), "alloc");
+  PK_TRY(cudaMalloc((void**)&p->spill, (size_t)n * 8), "alloc");
+  PK_TRY(cudaMemsetAsync(p->spill, 0, (size_t)n * 8, s), "memset");
+  // tiles per warp-quad must stay below 2^20 (the exchange tag)
+  {
+    std::vector<int32_t> hw(nq + 1);
+    PK_TRY(cudaMemcpyAsync(hw.data(), p->wtile, (size_t)(nq + 1) * 4, cudaMemcpyDeviceToHost, s), "copy");
+    PK_TRY(cudaStreamSynchronize(s), "sync");
+    int64_t mx = 0;
+    for (int i = 0; i < nq; ++i) mx = std::max<int64_t>(mx, (int64_t)hw[i + 1] - hw[i]);
+    p->max_tiles_per_warp = mx;
+    if (mx >= (1 << 20)) {
+      cleanup();
+      packed_free(p);
+      set_error("fp_csr_plan_pack: %lld tiles for one warp (limit 2^20)", (long long)mx);
+      return FP_ERR_UNSUPPORTED;
+    }
+  }
+#undef PK_TRY
+  cleanup();
+  *out = p;
+  return FP_OK;
+}
+
+fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
+  const bool has_y = a.y != nullptr;
+  const void* f = pk_pick(p->cs, has_y);
+  FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr_plan_exec: no packed kernel for %d blocks", p->cs);
+  set_max_dynamic_smem(f);
+  PkArgs k{};
+  k.n = p->n;
+  k.bw = p->bw;
+  k.groups = p->groups;
+  k.ntiles = p->ntiles;
+  k.tile_row = p->tile_row;
+  k.tile_seg = p->tile_seg;
+  k.wtile = p->wtile;
+  k.cr = p->cr;
+  k.val = p->val;
+  k.y = (const float*)a.y;
+  k.v = (const float*)a.v;
+  k.alpha = (float)a.alpha;
+  k.hbits = pk_headroom();
+  k.xch = p->xch;
+  k.epoch = p->epoch;
+  k.part = p->part;
+  k.spill = p->spill;
+  const size_t smem = (size_t)p->bw * (has_y ? 8 : 4);
+  void* args[] = {&k};
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(p->groups * p->cs);
+  cfg.blockDim = dim3(kPkBS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;  // the CTAs of a group wait on each other
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = p->cs > 1 ? 1 : 0;
+  FP_CUDA(cudaLaunchKernelExC(&cfg, f, args));
+  const int fb = 256;
+  const int fg = (int)std::min<int64_t>((p->n + fb - 1) / fb, 8 * (int64_t)device_info(current_device()).sm_count);
+  k_pk_finalize<<<fg, fb, 0, s>>>(p->n, p->groups, p->part, p->spill, (const float*)a.z, a.beta,
+                                  a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (float*)a.w, p->epoch);
+  FP_CUDA(cudaGetLastError());
+  return FP_OK;
+}
+
+void packed_launch(const Packed* p, fp_launch* L) {
+  *L = fp_launch{};
+  L->variant = FP_VAR_CSR_PACKED;
+  L->vs = 32;
+  L->tl = kPkSpan;
+  L->bs = kPkBS;
+  L->grid = p->groups * p->cs;
+  L->cluster = p->cs;
+  L->smem_bytes = p->bw * 8;
+  L->blocks_per_sm = 1;
+  cudaFuncAttributes fa{};
+  if (cudaFuncGetAttributes(&fa, pk_pick(p->cs, true)) == cudaSuccess) L->regs_per_thread = fa.numRegs;
+  else cudaGetLastError();
+}
+
+}  // namespace fp

@@ -2,6 +2,7 @@
 // -> launch parameters) and, for n too wide for one SM's shared memory, the
 // column split of the cluster kernel (csr_colsplit.cuh): CS-1 int32 segment offsets per row.
 // The paper amortises its baseline's transpose the same way.
+#include <cstdlib>
 #include <new>
 
 #include "csr_kernels.cuh"
@@ -15,6 +16,7 @@ struct fp_csr_plan {
   fp::CsrSplit split;
   int32_t* soff = nullptr;  // device, owned
   int device = 0;
+  fp::Packed* packed = nullptr;  // fp_csr_plan_pack: the column-blocked copy (owned)
 };
 
 namespace {
@@ -146,6 +148,21 @@ fp_status fp_csr_plan_create(int64_t m, int64_t n, int64_t nnz, const int64_t* r
 fp_status fp_csr_plan_exec(const fp_csr_plan* p, const void* val, const void* y, const void* v, const void* z,
                            double alpha, double beta, void* w, fp_stream stream) {
   FP_REQUIRE(p, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: plan is NULL");
+  if (!val && p->nnz > 0) {  // the packed copy (fp_csr_plan_pack)
+    FP_REQUIRE(p->packed, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: val is NULL and the plan is not packed");
+    FP_REQUIRE(p->n == 0 || w, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: w is NULL");
+    FP_REQUIRE(beta == 0.0 || z, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: beta != 0 needs z");
+    FP_REQUIRE(fp::current_device() == p->device, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: plan is on device %d",
+               p->device);
+    const size_t wb = (size_t)p->n * 4;
+    FP_REQUIRE(!fp::overlaps(w, wb, y, wb) && !fp::overlaps(w, wb, v, (size_t)p->m * 4), FP_ERR_ALIAS,
+               "fp_csr_plan_exec: w overlaps y or v");
+    fp::PatternArgs a =
+        fp::csr_args(p->m, p->n, p->nnz, p->rowptr, p->colidx, nullptr, y, v, z, alpha, beta, w, p->dtype);
+    if (p->n == 0) return FP_OK;
+    if (alpha == 0.0 || p->m == 0) return fp::launch_scale_z(p->n, z, beta, w, p->dtype, (cudaStream_t)stream);
+    return fp::packed_exec(p->packed, a, (cudaStream_t)stream);
+  }
   fp::PatternArgs a = fp::csr_args(p->m, p->n, p->nnz, p->rowptr, p->colidx, val, y, v, z, alpha, beta, w, p->dtype);
   a.split = p->soff ? &p->split : nullptr;
   return fp::run_csr(a, &p->L, (cudaStream_t)stream);
@@ -153,13 +170,42 @@ fp_status fp_csr_plan_exec(const fp_csr_plan* p, const void* val, const void* y,
 
 fp_status fp_csr_plan_launch(const fp_csr_plan* p, fp_launch* out) {
   FP_REQUIRE(p && out, FP_ERR_INVALID_ARG, "fp_csr_plan_launch: NULL argument");
-  *out = p->L;
+  if (p->packed) fp::packed_launch(p->packed, out);
+  else *out = p->L;
+  return FP_OK;
+}
+
+fp_status fp_csr_plan_pack(fp_csr_plan* p, const void* val, fp_stream stream) {
+  FP_REQUIRE(p, FP_ERR_INVALID_ARG, "fp_csr_plan_pack: plan is NULL");
+  FP_REQUIRE(fp::current_device() == p->device, FP_ERR_INVALID_ARG, "fp_csr_plan_pack: plan is on device %d",
+             p->device);
+  fp::Packed* q = nullptr;
+  const int cs_env = [] {
+    const char* e = std::getenv("FP_PK_CS");  // force the column blocks (measurement)
+    return e ? std::atoi(e) : 0;
+  }();
+  fp_status st = fp::packed_build(p->m, p->n, p->nnz, p->rowptr, p->colidx, val, p->dtype, cs_env, &q,
+                                  (cudaStream_t)stream);
+  if (st != FP_OK) return st;
+  fp::packed_free(p->packed);
+  p->packed = q;
+  return FP_OK;
+}
+
+fp_status fp_csr_plan_pack_info(const fp_csr_plan* p, int64_t* ntiles, int64_t* entries, int* blocks, int* groups) {
+  FP_REQUIRE(p, FP_ERR_INVALID_ARG, "fp_csr_plan_pack_info: plan is NULL");
+  FP_REQUIRE(p->packed, FP_ERR_INVALID_ARG, "fp_csr_plan_pack_info: the plan is not packed");
+  if (ntiles) *ntiles = p->packed->ntiles;
+  if (entries) *entries = p->packed->entries;
+  if (blocks) *blocks = p->packed->cs;
+  if (groups) *groups = p->packed->groups;
   return FP_OK;
 }
 
 fp_status fp_csr_plan_destroy(fp_csr_plan* p) {
   if (!p) return FP_OK;
   if (p->soff) cudaFree(p->soff);
+  fp::packed_free(p->packed);
   delete p;
   return FP_OK;
 }

@@ -73,6 +73,31 @@ fp_status launch_flat4_fixed(const PatternArgs& a, const fp_launch& L, cudaStrea
 size_t flat4_fixed_smem(int64_t n, fp_dtype dt, bool has_y);
 int flat4_fixed_blocks_per_sm(int64_t n, fp_dtype dt, bool has_y);
 
+// Variant 19 (csr_packed.cu): a column-blocked copy of a CSR matrix (fp_csr_plan_pack) and
+// Eq. (1) on it with one CTA group per column split (y + fixed-point w in shared memory).
+constexpr int kPkMaxCS = 8;
+struct Packed {
+  int64_t m = 0, n = 0, nnz = 0;
+  int cs = 0, bw = 0, groups = 0;
+  int64_t ntiles = 0, entries = 0, max_tiles_per_warp = 0;
+  const int64_t* rowptr = nullptr;
+  int64_t* tile_row = nullptr;          // [ntiles + 1]
+  uint2* tile_seg = nullptr;            // [cs][ntiles] (offset / 4, length)
+  int32_t* wtile = nullptr;             // [groups * 32 + 1]
+  uint32_t* cr = nullptr;               // [entries] column in block | row in tile << 16
+  float* val = nullptr;                 // [entries]
+  unsigned long long* xch = nullptr;    // exchange slots
+  unsigned* epoch = nullptr;            // call counter
+  double* part = nullptr;               // [groups][n]
+  double* spill = nullptr;              // [n]
+};
+int packed_cs(int64_t n);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
+fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                       const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s);
+fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s);
+void packed_free(Packed* p);
+void packed_launch(const Packed* p, fp_launch* L);
+
 size_t binned_ws_bytes(int64_t n, int64_t nnz, int nbin, int producer_grid, int consumers);
 
 // w = beta*z (or 0): the alpha == 0 / m == 0 path, and the pre-initialisation of the L2 path.

@@ -1,0 +1,227 @@
+"""GPU parity of variant 19 (FP_VAR_CSR_PACKED, csr_packed.cu) against the fp64 oracle.
+
+The packed plan (fp_csr_plan_pack) splits the columns into CS = 1/2/4/8 blocks, one CTA per
+block and SM holding y and the partial w of its block in shared memory (SURVEY 8 rows a3/a7/
+a9/a10 at large n); the row dots of Eq. (2) are completed across the CTAs of a group
+(one tagged word per row through L2), the scatter of Eq. (3) (Alg. 2 l.13-14) runs
+from the registers that hold the row, into a 32-bit fixed-point partial (reading R25).
+Checked here, at sizes the oracle finishes in seconds:
+* integer twins bit-exact for every block count, every instance (with/without y, v, beta*z),
+  power-law / binomial / long rows (segments beyond the 256-entry register window), empty rows,
+  non-canonical rows (i.i.d. columns: unsorted, repeats), ragged m;
+* the int32 wrap and the terms beyond the CTA's cap carried by the fp64 spill;
+* U[-1,1) fp32 data within the north_star 2e-5 normwise tolerance, rows scaled by 2^+-30;
+* IEEE propagation of Inf/NaN terms (reading R8);
+* determinism (bit-identical reruns), re-packing with new values, CUDA-graph replays (the
+  per-call exchange tag lives in device memory);
+* what it refuses (fp64, exec without values on an unpacked plan).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_ppopp_asharitbrcks15_b200 as fp
+import synth
+from _util import assert_bitexact, assert_parity
+
+pytestmark = pytest.mark.gpu
+
+
+def make(m, n, lengths, seed, kind, col_skew=0):
+    rp, ci, va = synth.csr(m, n, "f32", lengths, kind=kind, seed=seed, col_skew=col_skew)
+    integer = kind.startswith("int")
+    y = synth.vector(n, "f32", kind="int_small" if integer else "uniform", seed=seed, stream=synth.S_Y)
+    v = synth.vector(m, "f32", kind="int_pos" if integer else "pos", seed=seed, stream=synth.S_V)
+    z = synth.vector(n, "f32", kind="int_small" if integer else "uniform", seed=seed, stream=synth.S_Z)
+    return rp, ci, va, y, v, z
+
+
+def packed_plan(dev, rp, ci, va, n, blocks=0, monkeypatch=None):
+    if monkeypatch is not None:
+        monkeypatch.setenv("FP_PK_CS", str(blocks))
+    plan = fp.CsrPlan(rp.to(dev), ci.to(dev), n, torch.float32)
+    plan.pack(va.to(dev))
+    torch.cuda.synchronize()
+    if monkeypatch is not None:
+        monkeypatch.delenv("FP_PK_CS")
+    return plan
+
+
+def run(plan, dev, y, v, z, alpha, beta):
+    cu = lambda t: None if t is None else t.to(dev)
+    w = plan(None, cu(y), cu(v), cu(z), alpha, beta)
+    torch.cuda.synchronize()
+    return w
+
+
+INSTANCES = lambda y, v, z: ((y, v, z, 1.0, 1.0), (y, None, None, 2.0, 0.0), (None, v, z, -1.0, 0.5),
+                             (y, v, z, 0.5, -2.0))
+
+
+@pytest.mark.parametrize("n,blocks", [(1000, 1), (1000, 2), (40_000, 2), (100_000, 4), (100_000, 8),
+                                      (150_000, 8), (57_001, 4)])
+@pytest.mark.parametrize("lengths", [("powerlaw", 2.5, 13.64), ("binomial", 0.01), ("uniform", 0, 1500)])
+def test_packed_integer_twin_bitexact(cuda_dev, monkeypatch, n, blocks, lengths):
+    m = 20_011 if lengths[0] != "uniform" else 2_003
+    if lengths[0] == "binomial":
+        lengths = ("binomial", min(0.01, 200.0 / n))
+    if lengths[0] == "uniform":
+        lengths = ("uniform", 0, min(1500, n))
+    rp, ci, va, y, v, z = make(m, n, lengths, seed=n % 97 + blocks, kind="int_pm12")
+    plan = packed_plan(cuda_dev, rp, ci, va, n, blocks, monkeypatch)
+    info = plan.pack_info
+    assert info["blocks"] == blocks and info["entries"] >= ci.numel()
+    assert plan.launch.variant == 19 and plan.launch.cluster == blocks
+    for args in INSTANCES(y, v, z):
+        ref, mag = oracle.csr(m, n, rp, ci, va, *args)
+        assert mag.max() < 2**24
+        w = run(plan, cuda_dev, *args)
+        assert_bitexact(w, ref, f"packed n={n} cs={blocks} {lengths} y={args[0] is not None}")
+
+
+@pytest.mark.parametrize("blocks", [1, 4])
+def test_packed_edge_shapes(cuda_dev, monkeypatch, blocks):
+    """m = 1, m < 32, ragged m, empty rows (lengths from 0), one row longer than n/2, nnz = 0."""
+    n = 60_000
+    for m, lengths in ((1, ("uniform", 1, 40)), (5, ("uniform", 0, 3)), (33, ("uniform", 0, 9)),
+                       (1000, ("uniform", 0, 2)), (7, ("uniform", 30_000, 40_000))):
+        rp, ci, va, y, v, z = make(m, n, lengths, seed=m, kind="int_pm12")
+        plan = packed_plan(cuda_dev, rp, ci, va, n, blocks, monkeypatch)
+        for args in INSTANCES(y, v, z):
+            ref, _ = oracle.csr(m, n, rp, ci, va, *args)
+            w = run(plan, cuda_dev, *args)
+            assert_bitexact(w, ref, f"packed edge m={m} {lengths} cs={blocks}")
+    # nnz = 0: w = beta z
+    m = 50
+    rp = torch.zeros(m + 1, dtype=torch.int64)
+    ci = torch.zeros(0, dtype=torch.int32)
+    va = torch.zeros(0, dtype=torch.float32)
+    y = torch.ones(n)
+    z = torch.arange(n, dtype=torch.float32)
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, torch.float32)
+    w = plan(va.to(cuda_dev), y.to(cuda_dev), None, z.to(cuda_dev), 1.0, 2.0)
+    assert torch.equal(w.cpu(), 2 * z)
+
+
+@pytest.mark.parametrize("blocks", [2, 4])
+def test_packed_noncanonical_rows(cuda_dev, monkeypatch, blocks):
+    """i.i.d. columns: unsorted rows with repeated columns (reading R7: duplicates summed)."""
+    m, n = 10_000, 80_000
+    rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.0, 20.0), seed=11, kind="int_pm12", col_skew=-1)
+    plan = packed_plan(cuda_dev, rp, ci, va, n, blocks, monkeypatch)
+    for args in INSTANCES(y, v, z):
+        ref, _ = oracle.csr(m, n, rp, ci, va, *args)
+        w = run(plan, cuda_dev, *args)
+        assert_bitexact(w, ref, f"packed iid cs={blocks}")
+
+
+def test_packed_int32_wrap_and_cap_spill(cuda_dev):
+    """Every row holds column 0 and n-1 with the largest same-sign term: each CTA's int32 sum of
+    those columns wraps many times (carried through the fp64 spill); a late row 64x larger than
+    everything before it goes beyond the CTA's cap (spilled)."""
+    m, n = 60_000, 90_000
+    rp, ci, va = synth.csr(m, n, "f32", ("uniform", 2, 12), kind="int_pm12", seed=5)
+    rp, ci, va = rp.clone(), ci.clone(), va.clone()
+    ci[rp[:-1]] = 0
+    ci[rp[1:] - 1] = n - 1
+    va[rp[:-1]] = 2.0
+    va[rp[1:] - 1] = 2.0
+    va[rp[m - 7]:rp[m - 6]] *= 64.0
+    y = torch.zeros(n, dtype=torch.float32)
+    y[0] = 3.0
+    y[n - 1] = 3.0
+    v = torch.full((m,), 3.0)
+    ref, _ = oracle.csr(m, n, rp, ci, va, y, v, None, 1.0, 0.0)
+    assert abs(ref[0]) > 2**21
+    plan = packed_plan(cuda_dev, rp, ci, va, n)
+    w = run(plan, cuda_dev, y, v, None, 1.0, 0.0)
+    assert_bitexact(w, ref, "packed wraps")
+
+
+@pytest.mark.parametrize("n", [100_000, 30_000])
+def test_packed_float_parity_deterministic(cuda_dev, n):
+    m = 40_000
+    rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=7, kind="uniform")
+    plan = packed_plan(cuda_dev, rp, ci, va, n)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = run(plan, cuda_dev, y, v, z, 1.0, 1.0)
+    err = assert_parity(w, ref, mag, torch.float32, f"packed float n={n}")
+    assert err < 2e-6, f"fixed-point error {err:.2e} well inside the tolerance expected"
+    w2 = run(plan, cuda_dev, y, v, z, 1.0, 1.0)
+    assert torch.equal(w, w2), "the packed sum must be order-independent (bit-identical reruns)"
+
+
+def test_packed_dynamic_range(cuda_dev):
+    """Rows scaled by 2^+-30 at random: terms far beyond the first round's cap (spill) and far
+    below the quantum (rounded): the normwise bound still holds."""
+    m, n = 30_000, 70_000
+    rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=8, kind="uniform")
+    g = torch.Generator().manual_seed(3)
+    sc = torch.pow(2.0, torch.randint(-30, 31, (m,), generator=g).float())
+    va = va * torch.repeat_interleave(sc, (rp[1:] - rp[:-1]))
+    plan = packed_plan(cuda_dev, rp, ci, va, n)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = run(plan, cuda_dev, y, v, z, 1.0, 1.0)
+    assert_parity(w, ref, mag, torch.float32, "packed dynamic range")
+
+
+def test_packed_nonfinite_propagates(cuda_dev):
+    m, n = 5000, 80_000
+    rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=9, kind="uniform")
+    va = va.clone()
+    va[100] = float("inf")
+    va[2000] = float("nan")
+    plan = packed_plan(cuda_dev, rp, ci, va, n)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = run(plan, cuda_dev, y, v, z, 1.0, 1.0)
+    assert_parity(w, ref, mag, torch.float32, "packed non-finite")
+
+
+def test_packed_repack_unpacked_exec_alpha0(cuda_dev):
+    """pack again with new values; exec with val on a packed plan runs the unpacked path; alpha
+    = 0 writes beta z; exec without val on an unpacked plan and fp64 packing are refused."""
+    m, n = 8000, 100_000
+    rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=4, kind="int_pm12")
+    plan = packed_plan(cuda_dev, rp, ci, va, n)
+    va2 = -2 * va
+    plan.pack(va2.to(cuda_dev))
+    ref, _ = oracle.csr(m, n, rp, ci, va2, y, v, z, 1.0, 1.0)
+    assert_bitexact(run(plan, cuda_dev, y, v, z, 1.0, 1.0), ref, "repacked")
+    ref1, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = plan(va.to(cuda_dev), y.to(cuda_dev), v.to(cuda_dev), z.to(cuda_dev), 1.0, 1.0)
+    torch.cuda.synchronize()
+    assert_bitexact(w, ref1, "packed plan, exec with val")
+    w0 = run(plan, cuda_dev, y, v, z, 0.0, 3.0)
+    assert torch.equal(w0.cpu(), 3 * z)
+    plain = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, torch.float32)
+    with pytest.raises(fp.FusedPatError):
+        plain(None, y.to(cuda_dev), v.to(cuda_dev), z.to(cuda_dev), 1.0, 1.0)
+    rp64, ci64, va64 = synth.csr(500, 3000, "f64", ("uniform", 0, 20), seed=3)
+    p64 = fp.CsrPlan(rp64.to(cuda_dev), ci64.to(cuda_dev), 3000, torch.float64)
+    with pytest.raises(fp.FusedPatError):
+        p64.pack(va64.to(cuda_dev))
+
+
+def test_packed_graph_replay(cuda_dev):
+    """A captured exec replayed many times (the exchange tag is a device counter advanced by the
+    finalize, so replays never read a previous call's row partials)."""
+    m, n = 20_000, 100_000
+    rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=12, kind="int_pm12")
+    plan = packed_plan(cuda_dev, rp, ci, va, n)
+    ref, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    yd, vd, zd = y.to(cuda_dev), v.to(cuda_dev), z.to(cuda_dev)
+    w = torch.empty(n, device=cuda_dev)
+    s = torch.cuda.Stream(device=cuda_dev)
+    s.wait_stream(torch.cuda.current_stream(cuda_dev))
+    with torch.cuda.stream(s):
+        plan(None, yd, vd, zd, 1.0, 1.0, w=w)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        plan(None, yd, vd, zd, 1.0, 1.0, w=w)
+    for i in range(5):
+        w.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert_bitexact(w, ref, f"graph replay {i}")
