@@ -60,7 +60,7 @@ struct PkArgs {
   const float* v;
   float alpha;
   int hbits;                     // headroom bits of the fixed-point cap
-  unsigned long long* xch;       // exchange slots [groups][32 warps][2][cs][32 lanes]
+  unsigned long long* xch;       // exchange slots [groups][32 warps][kPkNS][cs][32 lanes]
   const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
   double* part;                  // [groups][n]
   double* spill;                 // [n], all-zero between calls
@@ -88,19 +88,36 @@ __device__ __forceinline__ unsigned pk_lanemask_lt() {
   return r;
 }
 
-// Per-warp state of one tile between its dot and its scatter.
+// One tile as a warp sees it: its block-k segment (16-byte aligned) and its rows.
 struct PkTile {
+  const uint32_t* pc;
+  const float* pv;
   int64_t row0;
   int nrows;
-  int64_t A;      // first entry of the segment (multiple of 4)
-  int len;        // entries of the segment (> kPkSpan: long, streamed)
+  int len;
 };
 
+constexpr int kPkNS = 8;  // exchange slots per warp: >= 2 D + 1 (a slot is rewritten only after its
+                          // tile was consumed by every CTA of the group)
+
+// The pass.  Warp `warp` of CTA k (block k) in group g walks the tile list of warp-quad
+// (g, warp) -- the same list in every CTA of the group -- as a pipeline:
+//   DOT(i):  stream tile i's segment (two 128-entry super-tiles per step, lane l holding
+//            entries 4l..4l+3 of each), Eq. (2) products y[col] x, segmented sums by row ->
+//            the block partial of the row dots, published as one tagged word per row;
+//   Q(j):    j = i - D: wait for the CS words of row `lane` of tile j, sum them in block order
+//            (identical in every CTA), q = alpha v p;
+//   SCAT(j): stream tile j's segment again (read D tiles ago: an L2 hit) and add every
+//            term x q into the block's fixed-point partial.
+// The dot runs D tiles ahead of the scatter, so the exchange latency hides behind the warp's
+// own work.
 template <int CS, int YM>
 __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
+  constexpr int D = (CS > 1 && YM != 0) ? 2 : 0;
+  static_assert(kPkNS >= 2 * D + 1, "exchange slots");
   extern __shared__ __align__(16) unsigned char pk_smem[];
   __shared__ float rs[kPkNW][32];   // the tile's block partials of the row dots (by row in tile)
-  __shared__ float qsm[kPkNW][32];  // q of the tile's rows (rare spill path)
+  __shared__ float qsm[kPkNW][32];  // q of the tile's rows (spill path)
   __shared__ unsigned s_tmax;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int k = CS == 1 ? 0 : (int)(blockIdx.x % CS);
@@ -118,190 +135,151 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   __syncthreads();
 
   const int gq = g * kPkNW + warp;
-  const int64_t t0 = a.wtile[gq], t1 = a.wtile[gq + 1];
-  const uint2* __restrict__ seg = a.tile_seg + (int64_t)k * a.ntiles;
+  const int64_t t0 = a.wtile[gq];
+  const int nt = a.wtile[gq + 1] - a.wtile[gq];
+  const uint2* __restrict__ seg = a.tile_seg + (int64_t)k * a.ntiles + t0;
+  const int64_t* __restrict__ trow = a.tile_row + t0;
   const unsigned tag0 = *a.epoch << 20;
-  unsigned long long* const xslot = a.xch + (int64_t)gq * 2 * CS * 32;
+  unsigned long long* const xslot = a.xch + (int64_t)gq * kPkNS * CS * 32;
   const float alpha = a.alpha;
 
-  auto info = [&](int64_t t) -> PkTile {
+  auto info = [&](int i) -> PkTile {
     PkTile T;
-    const int64_t r0 = __ldg(a.tile_row + t), r1 = __ldg(a.tile_row + t + 1);
-    const uint2 s = __ldg(seg + t);
+    const int64_t r0 = __ldg(trow + i), r1 = __ldg(trow + i + 1);
+    const uint2 s = __ldg(seg + i);
+    T.pc = a.cr + (int64_t)s.x * 4;
+    T.pv = a.val + (int64_t)s.x * 4;
     T.row0 = r0;
     T.nrows = (int)(r1 - r0);
-    T.A = (int64_t)s.x * 4;
     T.len = (int)s.y;
     return T;
   };
-
-  // ---- the two halves of a tile.  Window registers: two super-tiles of 128 entries, lane l
-  // holding entries 4l..4l+3 of each (16-byte loads).
-  uint32_t cw[2][4];
-  float xv[2][4];
-  float q = 0.f;  // q of row `lane` of the tile
-  float qs = 0.f; // q / quantum
-
-  // dot + exchange + q.  Returns the largest finite |x q| of the tile's active entries.
-  auto dot_q = [&](const PkTile& T, int64_t seq, bool need_tm) -> float {
-    const float vr = (lane < T.nrows) ? (a.v ? __ldg(a.v + T.row0 + lane) : 1.f) : 0.f;
-    const bool lng = T.len > kPkSpan;
-    if (!lng) {
+  // one step of a segment: entries s0 .. s0 + 255 (those at or beyond len are not loaded)
+  auto load_win = [&](const PkTile& T, int s0, uint32_t (&cw)[2][4], float (&xv)[2][4]) {
 #pragma unroll
-      for (int st = 0; st < 2; ++st) {
-        const int o = 128 * st + 4 * lane;
-        if (o < T.len) {
-          pk_ld4(a.cr + T.A + o, a.val + T.A + o, cw[st], xv[st]);
-        } else {
+    for (int st = 0; st < 2; ++st) {
+      const int o = s0 + 128 * st + 4 * lane;
+      if (o < T.len) {
+        pk_ld4(T.pc + o, T.pv + o, cw[st], xv[st]);
+      } else {
 #pragma unroll
-          for (int e = 0; e < 4; ++e) cw[st][e] = 31u << 16, xv[st][e] = 0.f;
-        }
+        for (int e = 0; e < 4; ++e) cw[st][e] = 31u << 16, xv[st][e] = 0.f;
       }
     }
-    float p = 0.f;
-    if constexpr (YM != 0) {
-      if (!lng) {
-        rs[warp][lane] = 0.f;
-        __syncwarp();
-        int carry = -1;  // row of the previous super-tile's last entry
-#pragma unroll
-        for (int st = 0; st < 2; ++st) {
-          if (128 * st >= T.len) break;
-          int rid[4];
-          float s[4];
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const bool act = 128 * st + 4 * lane + e < T.len;
-            rid[e] = act ? (int)(cw[st][e] >> 16) : 31;
-            const float yy = y_s[cw[st][e] & 0xffffu];
-            s[e] = act ? xv[st][e] * yy : 0.f;  // Eq. (2) products (inactive: exactly 0)
-          }
-          int prev = __shfl_up_sync(0xffffffffu, rid[3], 1);
-          if (lane == 0) prev = carry;
-          unsigned hb = 0;
-#pragma unroll
-          for (int e = 0; e < 4; ++e) hb |= (unsigned)(rid[e] != (e ? rid[e - 1] : prev)) << e;
-          // in-lane: P = entries before the first head; complete runs stored; `sum` = last run
-          float sum = 0.f, P = 0.f;
-          bool first = true;
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            if ((hb >> e) & 1u) {
-              if (first) P = sum;
-              else rs[warp][rid[e - 1]] = sum;  // a row entirely inside this lane
-              first = false;
-              sum = 0.f;
-            }
-            sum += s[e];
-          }
-          if (!hb) P = sum;
-          // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a head
-          const unsigned H = __ballot_sync(0xffffffffu, hb != 0u);
-          const unsigned hl = H >> lane;
-          const int dist = hl ? __ffs(hl) : 32 - lane;
-          float r = P;
-#pragma unroll
-          for (int d = 1; d < 32; d <<= 1) {
-            const float t2 = __shfl_down_sync(0xffffffffu, r, d);
-            if (d < dist) r += t2;
-          }
-          float rn = __shfl_down_sync(0xffffffffu, r, 1);
-          if (lane == 31) rn = 0.f;
-          if (hb) rs[warp][rid[3]] = sum + rn;            // the lane's last row: its run + what follows
-          if (lane == 0 && !(hb & 1u) && prev >= 0) rs[warp][prev] += r;  // row running in
-          carry = __shfl_sync(0xffffffffu, rid[3], 31);
-          __syncwarp();
-        }
-        p = rs[warp][lane];
-      } else {
-        // a long row (the tile's only row): stream the segment, every load of a step in flight
-        float s = 0.f;
-        for (int s0 = 0; s0 < T.len; s0 += kPkSpan) {
-          uint32_t c2[2][4];
-          float x2[2][4];
-#pragma unroll
-          for (int st = 0; st < 2; ++st) {
-            const int o = s0 + 128 * st + 4 * lane;
-            if (o < T.len) pk_ld4(a.cr + T.A + o, a.val + T.A + o, c2[st], x2[st]);
-            else {
-#pragma unroll
-              for (int e = 0; e < 4; ++e) c2[st][e] = 0u, x2[st][e] = 0.f;
-            }
-          }
-#pragma unroll
-          for (int st = 0; st < 2; ++st)
-#pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const bool act = s0 + 128 * st + 4 * lane + e < T.len;
-              const float pr = x2[st][e] * y_s[c2[st][e] & 0xffffu];
-              s += act ? pr : 0.f;
-            }
-        }
-        s = fpd::vector_allreduce<32>(s);
-        p = lane == 0 ? s : 0.f;
+  };
+
+  // DOT(i): returns the block partial of row `lane` of tile i (0 beyond its rows)
+  auto dot = [&](int i) -> float {
+    const PkTile T = info(i);
+    if (lane == 0 && i + 1 < nt) {  // the next tile's segment on its way into L2
+      const uint2 s1 = __ldg(seg + i + 1);
+      const int n1 = (int)min(s1.y, 4096u);
+      if (n1 > 0) {
+        fpd::prefetch_l2(a.cr + (int64_t)s1.x * 4, (size_t)n1 * 4);
+        fpd::prefetch_l2(a.val + (int64_t)s1.x * 4, (size_t)n1 * 4);
       }
-      // exchange of the block partials inside the group (the CS CTAs' warps `warp` walk the
-      // same tile list): value + tag in one 64-bit word, so no flag and no fence is needed
+    }
+    rs[warp][lane] = 0.f;
+    __syncwarp();
+    int carry = -1;  // row of the previous super-tile's last entry
+    for (int s0 = 0; s0 < T.len; s0 += 2 * 128) {
+      uint32_t cw[2][4];
+      float xv[2][4];
+      load_win(T, s0, cw, xv);
+#pragma unroll
+      for (int st = 0; st < 2; ++st) {
+        if (s0 + 128 * st >= T.len) break;
+        int rid[4];
+        float sv[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const bool act = s0 + 128 * st + 4 * lane + e < T.len;
+          rid[e] = act ? (int)(cw[st][e] >> 16) : 31;
+          const float yy = y_s[cw[st][e] & 0xffffu];
+          sv[e] = act ? xv[st][e] * yy : 0.f;  // Eq. (2) products (inactive: exactly 0)
+        }
+        int prev = __shfl_up_sync(0xffffffffu, rid[3], 1);
+        if (lane == 0) prev = carry;
+        unsigned hb = 0;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) hb |= (unsigned)(rid[e] != (e ? rid[e - 1] : prev)) << e;
+        // in-lane: P = entries before the first head; complete runs stored; `sum` = last run
+        float sum = 0.f, P = 0.f;
+        bool first = true;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          if ((hb >> e) & 1u) {
+            if (first) P = sum;
+            else rs[warp][rid[e - 1]] = sum;  // a row entirely inside this lane
+            first = false;
+            sum = 0.f;
+          }
+          sum += sv[e];
+        }
+        if (!hb) P = sum;
+        // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a head
+        const unsigned H = __ballot_sync(0xffffffffu, hb != 0u);
+        const unsigned hl = H >> lane;
+        const int dist = hl ? __ffs(hl) : 32 - lane;
+        float r = P;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const float t2 = __shfl_down_sync(0xffffffffu, r, d);
+          if (d < dist) r += t2;
+        }
+        float rn = __shfl_down_sync(0xffffffffu, r, 1);
+        if (lane == 31) rn = 0.f;
+        if (hb) rs[warp][rid[3]] = sum + rn;                            // the lane's last row
+        if (lane == 0 && !(hb & 1u) && prev >= 0) rs[warp][prev] += r;  // the row running in
+        carry = __shfl_sync(0xffffffffu, rid[3], 31);
+        __syncwarp();
+      }
+    }
+    const float p = rs[warp][lane];
+    if constexpr (CS > 1)
+      st_relaxed_gpu(xslot + (int64_t)(i % kPkNS) * CS * 32 + k * 32 + lane,
+                     ((unsigned long long)(tag0 + (unsigned)i) << 32) | __float_as_uint(p));
+    return p;
+  };
+
+  // Q(j): q of row `lane` of tile j; p_own = this CTA's partial when D == 0
+  auto qcalc = [&](const PkTile& T, int j, float p_own) -> float {
+    const float vr = lane < T.nrows ? (a.v ? __ldg(a.v + T.row0 + lane) : 1.f) : 0.f;
+    float q;
+    if constexpr (YM == 0) {
+      (void)j;
+      (void)p_own;
+      q = alpha * vr;
+    } else {
+      float p = p_own;
       if constexpr (CS > 1) {
-        const unsigned tag = tag0 + (unsigned)seq;
-        unsigned long long* slot = xslot + (int64_t)(seq & 1) * CS * 32;
-        st_relaxed_gpu(slot + k * 32 + lane, ((unsigned long long)tag << 32) | __float_as_uint(p));
+        // the exchange: value + tag in one 64-bit word, so no flag and no fence is needed
+        const unsigned tag = tag0 + (unsigned)j;
+        const unsigned long long* slot = xslot + (int64_t)(j % kPkNS) * CS * 32 + lane;
         unsigned long long wv[CS];
         bool done;
         do {
           done = true;
 #pragma unroll
-          for (int j = 0; j < CS; ++j) {
-            if (j != k) {
-              wv[j] = ld_relaxed_gpu(slot + j * 32 + lane);
-              done &= (unsigned)(wv[j] >> 32) == tag;
-            }
+          for (int b = 0; b < CS; ++b) {
+            wv[b] = ld_relaxed_gpu(slot + b * 32);
+            done &= (unsigned)(wv[b] >> 32) == tag;
           }
         } while (!done);
-        float tot = 0.f;
+        p = 0.f;
 #pragma unroll
-        for (int j = 0; j < CS; ++j) tot += j == k ? p : __uint_as_float((unsigned)wv[j]);  // fixed order
-        p = tot;
+        for (int b = 0; b < CS; ++b) p += __uint_as_float((unsigned)wv[b]);  // block order: identical in every CTA
       }
       q = alpha * (vr * p);
-    } else {
-      (void)seq;
-      q = alpha * vr;
     }
     if (lane >= T.nrows) q = 0.f;
     qsm[warp][lane] = q;
-    // largest finite |term| of the tile (the fixed-point cap of the first round)
-    float tm = 0.f;
-    if (!need_tm) return tm;
-    if (!lng) {
-#pragma unroll
-      for (int st = 0; st < 2; ++st)
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const bool act = 128 * st + 4 * lane + e < T.len;
-          const float qe = __shfl_sync(0xffffffffu, q, (int)(cw[st][e] >> 16) & 31);
-          const float t = fabsf(xv[st][e] * qe);
-          if (act && t <= 3.402823466e38f) tm = fmaxf(tm, t);
-        }
-    } else {
-      const float q0 = fabsf(__shfl_sync(0xffffffffu, q, 0));
-      for (int o = 4 * lane; o < T.len; o += 128) {
-        uint32_t c2[4];
-        float x2[4];
-        pk_ld4(a.cr + T.A + o, a.val + T.A + o, c2, x2);
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const float t = fabsf(x2[e]) * q0;
-          if (o + e < T.len && t <= 3.402823466e38f) tm = fmaxf(tm, t);
-        }
-      }
-    }
-    return tm;
+    return q;
   };
 
-  int E = 0;          // cap exponent: |t| < 2^E goes fixed point
-  float sc = 1.f;     // 2^(26 - E)
-  double quantum = 0; // 2^(E - 26)
+  int E = 0;           // cap exponent: |t| < 2^E goes fixed point
+  float sc = 1.f;      // 2^(26 - E)
+  double quantum = 0;  // 2^(E - 26)
   auto set_scale = [&](int e) {
     E = min(max(e, -95), 100);
     sc = ldexpf(1.f, 26 - E);
@@ -323,84 +301,93 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     }
   };
 
-  auto scatter = [&](const PkTile& T) {
-    qs = q * sc;
-    if (T.len <= kPkSpan) {
+  // SCAT(j): Eq. (3) from the segment, re-read
+  auto scatter = [&](const PkTile& T, float q) {
+    const float qs = q * sc;
+    for (int s0 = 0; s0 < T.len; s0 += 2 * 128) {
+      uint32_t cw[2][4];
+      float xv[2][4];
+      load_win(T, s0, cw, xv);
 #pragma unroll
       for (int st = 0; st < 2; ++st) {
-        if (128 * st >= T.len) break;
+        if (s0 + 128 * st >= T.len) break;
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
           const int rid = (int)(cw[st][e] >> 16) & 31;
           const float qe = __shfl_sync(0xffffffffu, qs, rid);
-          if (128 * st + 4 * lane + e < T.len) add_term((int)(cw[st][e] & 0xffffu), xv[st][e], qe, rid);
+          if (s0 + 128 * st + 4 * lane + e < T.len) add_term((int)(cw[st][e] & 0xffffu), xv[st][e], qe, rid);
         }
-      }
-    } else {
-      // the long row's segment is re-read (just streamed: mostly an L2 hit)
-      const float q0 = __shfl_sync(0xffffffffu, qs, 0);
-      for (int s0 = 0; s0 < T.len; s0 += kPkSpan) {
-        uint32_t c2[2][4];
-        float x2[2][4];
-#pragma unroll
-        for (int st = 0; st < 2; ++st) {
-          const int o = s0 + 128 * st + 4 * lane;
-          if (o < T.len) pk_ld4(a.cr + T.A + o, a.val + T.A + o, c2[st], x2[st]);
-        }
-#pragma unroll
-        for (int st = 0; st < 2; ++st)
-#pragma unroll
-          for (int e = 0; e < 4; ++e)
-            if (s0 + 128 * st + 4 * lane + e < T.len) add_term((int)(c2[st][e] & 0xffffu), x2[st][e], q0, 0);
       }
     }
   };
 
-  // ---- first rounds: one tile per warp until some finite term is nonzero, then the CTA's cap
-  int64_t t = t0;
-  for (;;) {
-    const bool have = t < t1;
-    PkTile T{};
+  // largest finite |x q| of a tile (the first rounds only)
+  auto tmax_of = [&](const PkTile& T, float q) -> float {
     float tm = 0.f;
+    for (int s0 = 0; s0 < T.len; s0 += 2 * 128) {
+      uint32_t cw[2][4];
+      float xv[2][4];
+      load_win(T, s0, cw, xv);
+#pragma unroll
+      for (int st = 0; st < 2; ++st)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float qe = __shfl_sync(0xffffffffu, q, (int)(cw[st][e] >> 16) & 31);
+          const float t = fabsf(xv[st][e] * qe);
+          if (s0 + 128 * st + 4 * lane + e < T.len && t <= 3.402823466e38f) tm = fmaxf(tm, t);
+        }
+    }
+    return tm;
+  };
+
+  // ---- the dots of the first D tiles, then rounds of one scatter per warp until the CTA's
+  // cap is set (all warps take part in every round: the loop condition is CTA-uniform)
+  float pown = 0.f;
+  if constexpr (YM != 0)
+    for (int i = 0; i < D; ++i)
+      if (i < nt) (void)dot(i);
+  int j = 0;
+  for (;;) {
+    const bool have = j < nt;
+    PkTile T{};
+    float q = 0.f, tm = 0.f;
     if (have) {
-      T = info(t);
-      tm = dot_q(T, t - t0, true);
+      if constexpr (YM != 0)
+        if (j + D < nt) pown = dot(j + D);
+      T = info(j);
+      q = qcalc(T, j, pown);
+      tm = tmax_of(T, q);
     }
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) tm = fmaxf(tm, __shfl_xor_sync(0xffffffffu, tm, d));
     if (lane == 0 && tm > 0.f) atomicMax(&s_tmax, __float_as_uint(tm));
     const int any = __syncthreads_or(have);
     const float mx = __uint_as_float(*(volatile unsigned*)&s_tmax);
-    const bool done = mx > 0.f || !any;
     if (mx > 0.f) {
       int e0;
       frexpf(mx, &e0);  // mx < 2^e0
       set_scale(e0 + a.hbits);
     }
-    // (while every finite term so far is 0, scale 2^26 adds zeros; non-finite terms spill)
-    if (have) scatter(T);
-    if (have) ++t;
-    if (done) break;
+    // (while every finite term so far is 0, the provisional scale adds zeros; non-finite terms spill)
+    if (have) {
+      scatter(T, q);
+      ++j;
+    }
+    if (mx > 0.f || !any) break;
   }
 
   // ---- steady state
-  for (; t < t1; ++t) {
-    const PkTile T = info(t);
-    if (lane == 0 && t + 1 < t1) {  // the next tile's segment on its way into L2
-      const uint2 s1 = __ldg(seg + t + 1);
-      const int n1 = (int)min((unsigned)s1.y, 4096u);
-      if (n1 > 0) {
-        fpd::prefetch_l2(a.cr + (int64_t)s1.x * 4, (size_t)n1 * 4);
-        fpd::prefetch_l2(a.val + (int64_t)s1.x * 4, (size_t)n1 * 4);
-      }
-    }
-    (void)dot_q(T, t - t0, false);
-    scatter(T);
+  for (; j < nt; ++j) {
+    if constexpr (YM != 0)
+      if (j + D < nt) pown = dot(j + D);
+    const PkTile T = info(j);
+    const float q = qcalc(T, j, pown);
+    scatter(T, q);
   }
 
   __syncthreads();
   double* dst = a.part + (int64_t)g * a.n + c0;
-  for (int j = threadIdx.x; j < bwk; j += kPkBS) dst[j] = (double)acc[j] * quantum;
+  for (int i = threadIdx.x; i < bwk; i += kPkBS) dst[i] = (double)acc[i] * quantum;
 }
 
 __global__ void k_pk_finalize(int64_t n, int groups, const double* __restrict__ part, double* __restrict__ spill,
@@ -717,7 +704,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
   k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, p->tile_row, rowptr, p->wtile);
   // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
-  const size_t xbytes = (size_t)groups * kPkNW * 2 * cs * 32 * 8;
+  const size_t xbytes = (size_t)groups * kPkNW * kPkNS * cs * 32 * 8;
   PK_TRY(cudaMalloc((void**)&p->xch, xbytes), "alloc");
   PK_TRY(cudaMemsetAsync(p->xch, 0, xbytes, s), "memset");
   PK_TRY(cudaMalloc((void**)&p->epoch, 16), "alloc");

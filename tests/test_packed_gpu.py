@@ -80,12 +80,12 @@ def test_packed_integer_twin_bitexact(cuda_dev, monkeypatch, n, blocks, lengths)
         assert_bitexact(w, ref, f"packed n={n} cs={blocks} {lengths} y={args[0] is not None}")
 
 
-@pytest.mark.parametrize("blocks", [1, 4])
+@pytest.mark.parametrize("blocks", [2, 4])
 def test_packed_edge_shapes(cuda_dev, monkeypatch, blocks):
     """m = 1, m < 32, ragged m, empty rows (lengths from 0), one row longer than n/2, nnz = 0."""
-    n = 60_000
+    n = 50_000
     for m, lengths in ((1, ("uniform", 1, 40)), (5, ("uniform", 0, 3)), (33, ("uniform", 0, 9)),
-                       (1000, ("uniform", 0, 2)), (7, ("uniform", 30_000, 40_000))):
+                       (1000, ("uniform", 0, 2)), (7, ("uniform", 26_000, 40_000))):
         rp, ci, va, y, v, z = make(m, n, lengths, seed=m, kind="int_pm12")
         plan = packed_plan(cuda_dev, rp, ci, va, n, blocks, monkeypatch)
         for args in INSTANCES(y, v, z):

@@ -5,7 +5,8 @@ mkdir -p gpurun_out
 timeout 900 python -m pytest tests/test_packed_gpu.py -q -x -p no:cacheprovider --timeout 300 -rf > gpurun_out/pk_pytest.log 2>&1
 tail -15 gpurun_out/pk_pytest.log
 timeout 600 python bench.py --config C4 --steps 10 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/pk_c4.json 2> gpurun_out/pk_c4.err
-tail -c 1500 gpurun_out/pk_c4.json; tail -3 gpurun_out/pk_c4.err
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/pk_c4_launches.csv python bench.py --config C4 --steps 2 --warmup 1 --no-e2e --no-cpu-baseline --no-graph > /dev/null 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_pk -s 1 -c 1 -o gpurun_out/pk_c4_full -f python bench.py --config C4 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-graph > gpurun_out/pk_ncu.log 2>&1
+python -c "
+import json; d=json.loads(open('gpurun_out/pk_c4.json').read().strip().splitlines()[-1]); print(d['ms_per_step'], d['roofline']['frac'], d['config']['packed_copy'])"
+tail -3 gpurun_out/pk_c4.err
+timeout 900 ncu --set full --clock-control none --import-source on -k k_pk -c 1 -o gpurun_out/pk_c4_full -f python bench.py --config C4 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-graph > gpurun_out/pk_ncu.log 2>&1
 tail -3 gpurun_out/pk_ncu.log
