@@ -42,17 +42,20 @@ namespace {
 
 constexpr int kPkBS = 1024;
 constexpr int kPkNW = kPkBS / 32;
-constexpr int kPkSpan = 256;          // entries of a block segment held in registers (2 super-tiles)
+constexpr int kPkLong = 1024;         // a block segment longer than this makes its row a tile of its own
 constexpr int kPkRowCost = 4;         // work of a row in entries (warp partition)
-constexpr int kPkStatic = 9 * 1024;   // static shared memory reserve of k_pk
+constexpr int kPkStatic = 11 * 1024;  // static shared memory reserve of k_pk
+constexpr int kPkNS = 8;              // exchange slots per warp (>= 2 D + 1)
+constexpr int kPkRing = 4;            // tile descriptors a warp keeps between DOT and SCATTER (>= D + 1)
+constexpr unsigned kPkOffMask = 0x3FFFFu;  // entry word: byte offset of the column in the block (18 bits)
+constexpr int kPkRidShift = 18;            //             | row in tile << 18
 
 struct PkArgs {
   int64_t n;
   int bw;                        // columns per block (block k = [k bw, min(n, (k+1) bw)))
   int groups;
   int64_t ntiles;
-  const int64_t* tile_row;       // [ntiles + 1]
-  const uint2* tile_seg;         // [cs][ntiles]: (offset / 4, length) of the tile's block-k segment
+  const uint4* tile_desc;        // [cs][ntiles]: (offset / 4, length, first row, rows)
   const int32_t* wtile;          // [groups * 32 + 1]: first tile of each warp-quad
   const uint32_t* cr;            // packed entry words
   const float* val;
@@ -60,10 +63,10 @@ struct PkArgs {
   const float* v;
   float alpha;
   int hbits;                     // headroom bits of the fixed-point cap
-  unsigned long long* xch;       // exchange slots [groups][32 warps][kPkNS][cs][32 lanes]
+  unsigned long long* xch;       // exchange slots [groups][32 warps][kPkNS][cs + 1][32 lanes]
   const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
   double* part;                  // [groups][n]
-  double* spill;                 // [n], all-zero between calls
+  double* spill;                 // [cs][bw + 1], all-zero between calls
 };
 
 __device__ __forceinline__ void pk_ld4(const uint32_t* pc, const float* pv, uint32_t (&c)[4], float (&x)[4]) {
@@ -87,37 +90,42 @@ __device__ __forceinline__ unsigned pk_lanemask_lt() {
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
   return r;
 }
-
-// One tile as a warp sees it: its block-k segment (16-byte aligned) and its rows.
-struct PkTile {
-  const uint32_t* pc;
-  const float* pv;
-  int64_t row0;
-  int nrows;
-  int len;
-};
-
-constexpr int kPkNS = 8;  // exchange slots per warp: >= 2 D + 1 (a slot is rewritten only after its
-                          // tile was consumed by every CTA of the group)
+// y (read-only after staging) and the fixed-point partial through 32-bit shared addresses
+__device__ __forceinline__ float pk_lds(unsigned addr) {
+  float v;
+  asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ int pk_atom_add(unsigned addr, int v) {
+  int old;
+  asm volatile("atom.shared.add.s32 %0, [%1], %2;" : "=r"(old) : "r"(addr), "r"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ void pk_prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
 
 // The pass.  Warp `warp` of CTA k (block k) in group g walks the tile list of warp-quad
 // (g, warp) -- the same list in every CTA of the group -- as a pipeline:
 //   DOT(i):  stream tile i's segment (two 128-entry super-tiles per step, lane l holding
 //            entries 4l..4l+3 of each), Eq. (2) products y[col] x, segmented sums by row ->
-//            the block partial of the row dots, published as one tagged word per row;
-//   Q(j):    j = i - D: wait for the CS words of row `lane` of tile j, sum them in block order
-//            (identical in every CTA), q = alpha v p;
+//            the block partial of the row dots, published as one tagged word per row (CTA 0
+//            also publishes v of the rows);
+//   Q(j):    j = i - D: wait for the CS (+ v) words of row `lane` of tile j, sum them in block
+//            order (identical in every CTA), q = alpha v p;
 //   SCAT(j): stream tile j's segment again (read D tiles ago: an L2 hit) and add every
 //            term x q into the block's fixed-point partial.
 // The dot runs D tiles ahead of the scatter, so the exchange latency hides behind the warp's
-// own work.
+// own work.  Padding entries (column = the block's zero / dummy slot, row 31, value 0) make
+// every lane of a loaded 4-entry group valid: no per-entry predicates.
 template <int CS, int YM>
 __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
-  constexpr int D = (CS > 1 && YM != 0) ? 2 : 0;
-  static_assert(kPkNS >= 2 * D + 1, "exchange slots");
+  constexpr int D = (CS > 1 && YM != 0) ? 3 : 0;
+  static_assert(kPkNS >= 2 * D + 1 && kPkRing >= D + 1, "exchange slots / descriptor ring");
   extern __shared__ __align__(16) unsigned char pk_smem[];
-  __shared__ float rs[kPkNW][32];   // the tile's block partials of the row dots (by row in tile)
-  __shared__ float qsm[kPkNW][32];  // q of the tile's rows (spill path)
+  __shared__ float rs[kPkNW][32];        // the tile's block partials of the row dots (by row in tile)
+  __shared__ float qsm[kPkNW][32];       // q of the tile's rows (spill path)
+  __shared__ uint4 ring[kPkNW][kPkRing]; // descriptors of the tiles between DOT and SCATTER
   __shared__ unsigned s_tmax;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int k = CS == 1 ? 0 : (int)(blockIdx.x % CS);
@@ -125,100 +133,99 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   const int bw = a.bw;
   const int64_t c0 = (int64_t)k * bw;
   const int bwk = (int)max((int64_t)0, min((int64_t)bw, a.n - c0));  // columns of this block
+  // [y: bw + 1 floats, y[bw] = 0 (padding entries)][acc: bw + 1 ints, acc[bw] = dummy]
+  const int ystride = YM ? (bw + 4) & ~3 : 0;
   float* y_s = reinterpret_cast<float*>(pk_smem);
-  int* acc = reinterpret_cast<int*>(pk_smem + (YM ? (size_t)bw * 4 : 0));
-  for (int j = threadIdx.x; j < bw; j += kPkBS) {
+  int* acc = reinterpret_cast<int*>(pk_smem) + ystride;
+  for (int j = threadIdx.x; j <= bw; j += kPkBS) {
     if (YM) y_s[j] = j < bwk ? a.y[c0 + j] : 0.f;
     acc[j] = 0;
   }
   if (threadIdx.x == 0) s_tmax = 0u;
   __syncthreads();
+  const unsigned ys_base = fpd::smem_u32(y_s), acc_base = fpd::smem_u32(acc);
 
   const int gq = g * kPkNW + warp;
   const int64_t t0 = a.wtile[gq];
   const int nt = a.wtile[gq + 1] - a.wtile[gq];
-  const uint2* __restrict__ seg = a.tile_seg + (int64_t)k * a.ntiles + t0;
-  const int64_t* __restrict__ trow = a.tile_row + t0;
+  const uint4* __restrict__ desc = a.tile_desc + (int64_t)k * a.ntiles + t0;
   const unsigned tag0 = *a.epoch << 20;
-  unsigned long long* const xslot = a.xch + (int64_t)gq * kPkNS * CS * 32;
+  unsigned long long* const xslot = a.xch + (int64_t)gq * kPkNS * (CS + 1) * 32;
   const float alpha = a.alpha;
+  double* const spill = a.spill + (int64_t)k * (bw + 1);
 
-  auto info = [&](int i) -> PkTile {
-    PkTile T;
-    const int64_t r0 = __ldg(trow + i), r1 = __ldg(trow + i + 1);
-    const uint2 s = __ldg(seg + i);
-    T.pc = a.cr + (int64_t)s.x * 4;
-    T.pv = a.val + (int64_t)s.x * 4;
-    T.row0 = r0;
-    T.nrows = (int)(r1 - r0);
-    T.len = (int)s.y;
-    return T;
-  };
-  // one step of a segment: entries s0 .. s0 + 255 (those at or beyond len are not loaded)
-  auto load_win = [&](const PkTile& T, int s0, uint32_t (&cw)[2][4], float (&xv)[2][4]) {
+  // one step of a segment: entries s0 .. s0 + 255 of the 16-byte aligned segment at off4 * 4
+  auto load_win = [&](const uint4& T, int s0, uint32_t (&cw)[2][4], float (&xv)[2][4]) {
+    const int64_t base = (int64_t)T.x * 4;
 #pragma unroll
     for (int st = 0; st < 2; ++st) {
       const int o = s0 + 128 * st + 4 * lane;
-      if (o < T.len) {
-        pk_ld4(T.pc + o, T.pv + o, cw[st], xv[st]);
+      if (o < (int)T.y) {
+        pk_ld4(a.cr + base + o, a.val + base + o, cw[st], xv[st]);
       } else {
 #pragma unroll
-        for (int e = 0; e < 4; ++e) cw[st][e] = 31u << 16, xv[st][e] = 0.f;
+        for (int e = 0; e < 4; ++e) cw[st][e] = ((unsigned)bw * 4u) | (31u << kPkRidShift), xv[st][e] = 0.f;
       }
     }
   };
 
-  // DOT(i): returns the block partial of row `lane` of tile i (0 beyond its rows)
-  auto dot = [&](int i) -> float {
-    const PkTile T = info(i);
-    if (lane == 0 && i + 1 < nt) {  // the next tile's segment on its way into L2
-      const uint2 s1 = __ldg(seg + i + 1);
-      const int n1 = (int)min(s1.y, 4096u);
-      if (n1 > 0) {
-        fpd::prefetch_l2(a.cr + (int64_t)s1.x * 4, (size_t)n1 * 4);
-        fpd::prefetch_l2(a.val + (int64_t)s1.x * 4, (size_t)n1 * 4);
+  // ---- DOT(i): tile i's block partials of the row dots, published (YM), descriptor -> ring
+  uint4 cd = make_uint4(0, 0, 0, 0);  // lane l: descriptor of tile (i & ~31) + l
+  float pown = 0.f, vown = 1.f;       // D == 0: this CTA's partial / v of row `lane`
+  auto dot = [&](int i) {
+    if ((i & 31) == 0 && i + lane < nt) cd = __ldg(desc + i + lane);
+    uint4 T;
+    T.x = __shfl_sync(0xffffffffu, cd.x, i & 31);
+    T.y = __shfl_sync(0xffffffffu, cd.y, i & 31);
+    T.z = __shfl_sync(0xffffffffu, cd.z, i & 31);
+    T.w = __shfl_sync(0xffffffffu, cd.w, i & 31);
+    if (lane == 0) ring[warp][i % kPkRing] = T;
+    __syncwarp();
+    // the next tile's segment on its way into L2 (lanes 0-15: 128-byte lines of cr, 16-31: val)
+    {
+      const int i1 = i + 1;
+      const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
+      if ((i1 & 31) != 0 && i1 < nt) {
+        const int l = lane & 15;
+        if (32 * l < (int)min(len1, 512u)) {
+          const int64_t e = (int64_t)off1 * 4 + 32 * l;
+          pk_prefetch_l2(lane < 16 ? (const void*)(a.cr + e) : (const void*)(a.val + e));
+        }
       }
     }
+    const float vr = (YM != 0 && (CS == 1 || k == 0) && lane < (int)T.w)
+                         ? (a.v ? __ldg(a.v + (int)T.z + lane) : 1.f) : 1.f;
+    if constexpr (YM == 0) return;
     rs[warp][lane] = 0.f;
     __syncwarp();
     int carry = -1;  // row of the previous super-tile's last entry
-    for (int s0 = 0; s0 < T.len; s0 += 2 * 128) {
+    for (int s0 = 0; s0 < (int)T.y; s0 += 2 * 128) {
       uint32_t cw[2][4];
       float xv[2][4];
       load_win(T, s0, cw, xv);
 #pragma unroll
       for (int st = 0; st < 2; ++st) {
-        if (s0 + 128 * st >= T.len) break;
+        if (s0 + 128 * st >= (int)T.y) break;
         int rid[4];
-        float sv[4];
+        float c[4];  // in-lane inclusive segmented sums of the Eq. (2) products
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
-          const bool act = s0 + 128 * st + 4 * lane + e < T.len;
-          rid[e] = act ? (int)(cw[st][e] >> 16) : 31;
-          const float yy = y_s[cw[st][e] & 0xffffu];
-          sv[e] = act ? xv[st][e] * yy : 0.f;  // Eq. (2) products (inactive: exactly 0)
+          rid[e] = (int)(cw[st][e] >> kPkRidShift);
+          const float pr = xv[st][e] * pk_lds(ys_base + (cw[st][e] & kPkOffMask));
+          c[e] = (e == 0 || rid[e] != rid[e - 1]) ? pr : c[e - 1] + pr;
         }
         int prev = __shfl_up_sync(0xffffffffu, rid[3], 1);
         if (lane == 0) prev = carry;
-        unsigned hb = 0;
-#pragma unroll
-        for (int e = 0; e < 4; ++e) hb |= (unsigned)(rid[e] != (e ? rid[e - 1] : prev)) << e;
-        // in-lane: P = entries before the first head; complete runs stored; `sum` = last run
-        float sum = 0.f, P = 0.f;
-        bool first = true;
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          if ((hb >> e) & 1u) {
-            if (first) P = sum;
-            else rs[warp][rid[e - 1]] = sum;  // a row entirely inside this lane
-            first = false;
-            sum = 0.f;
-          }
-          sum += sv[e];
-        }
-        if (!hb) P = sum;
-        // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a head
-        const unsigned H = __ballot_sync(0xffffffffu, hb != 0u);
+        const bool h0 = rid[0] != prev, h1 = rid[1] != rid[0], h2 = rid[2] != rid[1], h3 = rid[3] != rid[2];
+        const bool any = h0 | h1 | h2 | h3;
+        // P = the entries before the lane's first row start (continuing a row from before)
+        const float P = h0 ? 0.f : (h1 ? c[0] : (h2 ? c[1] : (h3 ? c[2] : c[3])));
+        // rows that start and end inside the lane
+        if (h1 && h0) rs[warp][rid[0]] = c[0];
+        if (h2 && (h0 | h1)) rs[warp][rid[1]] = c[1];
+        if (h3 && (h0 | h1 | h2)) rs[warp][rid[2]] = c[2];
+        // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a row start
+        const unsigned H = __ballot_sync(0xffffffffu, any);
         const unsigned hl = H >> lane;
         const int dist = hl ? __ffs(hl) : 32 - lane;
         float r = P;
@@ -229,50 +236,54 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
         }
         float rn = __shfl_down_sync(0xffffffffu, r, 1);
         if (lane == 31) rn = 0.f;
-        if (hb) rs[warp][rid[3]] = sum + rn;                            // the lane's last row
-        if (lane == 0 && !(hb & 1u) && prev >= 0) rs[warp][prev] += r;  // the row running in
+        if (any) rs[warp][rid[3]] = c[3] + rn;                     // the lane's last row
+        if (lane == 0 && !h0 && prev >= 0) rs[warp][prev] += r;    // the row running in
         carry = __shfl_sync(0xffffffffu, rid[3], 31);
         __syncwarp();
       }
     }
     const float p = rs[warp][lane];
-    if constexpr (CS > 1)
-      st_relaxed_gpu(xslot + (int64_t)(i % kPkNS) * CS * 32 + k * 32 + lane,
-                     ((unsigned long long)(tag0 + (unsigned)i) << 32) | __float_as_uint(p));
-    return p;
+    if constexpr (CS > 1) {
+      const unsigned long long tg = (unsigned long long)(tag0 + (unsigned)i) << 32;
+      unsigned long long* slot = xslot + (int64_t)(i % kPkNS) * (CS + 1) * 32 + lane;
+      st_relaxed_gpu(slot + k * 32, tg | __float_as_uint(p));
+      if (k == 0) st_relaxed_gpu(slot + CS * 32, tg | __float_as_uint(vr));
+    } else {
+      pown = p;
+      vown = vr;
+    }
   };
 
-  // Q(j): q of row `lane` of tile j; p_own = this CTA's partial when D == 0
-  auto qcalc = [&](const PkTile& T, int j, float p_own) -> float {
-    const float vr = lane < T.nrows ? (a.v ? __ldg(a.v + T.row0 + lane) : 1.f) : 0.f;
+  // ---- Q(j): q of row `lane` of tile j (descriptor T)
+  auto qcalc = [&](const uint4& T, int j) -> float {
     float q;
     if constexpr (YM == 0) {
       (void)j;
-      (void)p_own;
+      const float vr = lane < (int)T.w ? (a.v ? __ldg(a.v + (int)T.z + lane) : 1.f) : 0.f;
       q = alpha * vr;
+    } else if constexpr (CS == 1) {
+      (void)j;
+      q = alpha * (vown * pown);
     } else {
-      float p = p_own;
-      if constexpr (CS > 1) {
-        // the exchange: value + tag in one 64-bit word, so no flag and no fence is needed
-        const unsigned tag = tag0 + (unsigned)j;
-        const unsigned long long* slot = xslot + (int64_t)(j % kPkNS) * CS * 32 + lane;
-        unsigned long long wv[CS];
-        bool done;
-        do {
-          done = true;
+      // the exchange: value + tag in one 64-bit word, so no flag and no fence is needed
+      const unsigned tag = tag0 + (unsigned)j;
+      const unsigned long long* slot = xslot + (int64_t)(j % kPkNS) * (CS + 1) * 32 + lane;
+      unsigned long long wv[CS + 1];
+      bool done;
+      do {
+        done = true;
 #pragma unroll
-          for (int b = 0; b < CS; ++b) {
-            wv[b] = ld_relaxed_gpu(slot + b * 32);
-            done &= (unsigned)(wv[b] >> 32) == tag;
-          }
-        } while (!done);
-        p = 0.f;
+        for (int b = 0; b <= CS; ++b) {
+          wv[b] = ld_relaxed_gpu(slot + b * 32);
+          done &= (unsigned)(wv[b] >> 32) == tag;
+        }
+      } while (!done);
+      float p = 0.f;
 #pragma unroll
-        for (int b = 0; b < CS; ++b) p += __uint_as_float((unsigned)wv[b]);  // block order: identical in every CTA
-      }
-      q = alpha * (vr * p);
+      for (int b = 0; b < CS; ++b) p += __uint_as_float((unsigned)wv[b]);  // block order: identical in every CTA
+      q = alpha * (__uint_as_float((unsigned)wv[CS]) * p);
     }
-    if (lane >= T.nrows) q = 0.f;
+    if (lane >= (int)T.w) q = 0.f;
     qsm[warp][lane] = q;
     return q;
   };
@@ -287,44 +298,50 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   };
   set_scale(0);
 
-  // one term into the CTA's fixed-point partial (or the spill)
-  auto add_term = [&](int col, float x, float qe, int rid) {
-    const float ts = x * qe;
-    if (fabsf(ts) < 67108864.f) {  // 2^26
-      const int qi = __float2int_rn(ts);
-      const int old = atomicAdd(acc + col, qi);  // native ATOMS.ADD
-      const unsigned nw = (unsigned)old + (unsigned)qi;
-      if ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0)  // int32 wrap: carry 2^32 quanta
-        atomicAdd(a.spill + c0 + col, qi > 0 ? 4294967296.0 * quantum : -4294967296.0 * quantum);
-    } else {  // beyond the cap, or Inf / NaN (IEEE propagation, reading R8)
-      atomicAdd(a.spill + c0 + col, (double)(x * qsm[warp][rid]));
-    }
-  };
-
-  // SCAT(j): Eq. (3) from the segment, re-read
-  auto scatter = [&](const PkTile& T, float q) {
+  // ---- SCAT(j): Eq. (3) from the segment, re-read.  Common path branch-free; terms beyond the
+  // cap, non-finite terms and int32 wraps (rare) are collected in a mask and spilled after.
+  auto scatter = [&](const uint4& T, float q) {
     const float qs = q * sc;
-    for (int s0 = 0; s0 < T.len; s0 += 2 * 128) {
+    for (int s0 = 0; s0 < (int)T.y; s0 += 2 * 128) {
       uint32_t cw[2][4];
       float xv[2][4];
       load_win(T, s0, cw, xv);
+      unsigned rare = 0;
 #pragma unroll
       for (int st = 0; st < 2; ++st) {
-        if (s0 + 128 * st >= T.len) break;
+        if (s0 + 128 * st >= (int)T.y) break;
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
-          const int rid = (int)(cw[st][e] >> 16) & 31;
-          const float qe = __shfl_sync(0xffffffffu, qs, rid);
-          if (s0 + 128 * st + 4 * lane + e < T.len) add_term((int)(cw[st][e] & 0xffffu), xv[st][e], qe, rid);
+          const float qe = __shfl_sync(0xffffffffu, qs, (int)(cw[st][e] >> kPkRidShift));
+          const float ts = xv[st][e] * qe;
+          const bool big = !(fabsf(ts) < 67108864.f);  // >= 2^26 or NaN
+          const int qi = big ? 0 : __float2int_rn(ts);
+          const int old = pk_atom_add(acc_base + (cw[st][e] & kPkOffMask), qi);  // native ATOMS.ADD
+          const unsigned nw = (unsigned)old + (unsigned)qi;
+          const bool ovf = (int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0;
+          rare |= (unsigned)(big | ovf) << (4 * st + e);
+        }
+      }
+      if (rare) {
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+          if ((rare >> b) & 1u) {
+            const uint32_t w = cw[b >> 2][b & 3];
+            const float x = xv[b >> 2][b & 3];
+            const float t = x * qsm[warp][w >> kPkRidShift];
+            const int col = (int)((w & kPkOffMask) >> 2);
+            if (!(fabsf(t * sc) < 67108864.f)) atomicAdd(spill + col, (double)t);  // beyond the cap / Inf / NaN
+            else atomicAdd(spill + col, t > 0.f ? 4294967296.0 * quantum : -4294967296.0 * quantum);  // wrap
+          }
         }
       }
     }
   };
 
   // largest finite |x q| of a tile (the first rounds only)
-  auto tmax_of = [&](const PkTile& T, float q) -> float {
+  auto tmax_of = [&](const uint4& T, float q) -> float {
     float tm = 0.f;
-    for (int s0 = 0; s0 < T.len; s0 += 2 * 128) {
+    for (int s0 = 0; s0 < (int)T.y; s0 += 2 * 128) {
       uint32_t cw[2][4];
       float xv[2][4];
       load_win(T, s0, cw, xv);
@@ -332,9 +349,9 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
       for (int st = 0; st < 2; ++st)
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
-          const float qe = __shfl_sync(0xffffffffu, q, (int)(cw[st][e] >> 16) & 31);
+          const float qe = __shfl_sync(0xffffffffu, q, (int)(cw[st][e] >> kPkRidShift));
           const float t = fabsf(xv[st][e] * qe);
-          if (s0 + 128 * st + 4 * lane + e < T.len && t <= 3.402823466e38f) tm = fmaxf(tm, t);
+          if (t <= 3.402823466e38f) tm = fmaxf(tm, t);
         }
     }
     return tm;
@@ -342,20 +359,17 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
 
   // ---- the dots of the first D tiles, then rounds of one scatter per warp until the CTA's
   // cap is set (all warps take part in every round: the loop condition is CTA-uniform)
-  float pown = 0.f;
-  if constexpr (YM != 0)
-    for (int i = 0; i < D; ++i)
-      if (i < nt) (void)dot(i);
+  for (int i = 0; i < D; ++i)
+    if (i < nt) dot(i);
   int j = 0;
   for (;;) {
     const bool have = j < nt;
-    PkTile T{};
+    uint4 T = make_uint4(0, 0, 0, 0);
     float q = 0.f, tm = 0.f;
     if (have) {
-      if constexpr (YM != 0)
-        if (j + D < nt) pown = dot(j + D);
-      T = info(j);
-      q = qcalc(T, j, pown);
+      if (j + D < nt) dot(j + D);
+      T = ring[warp][j % kPkRing];
+      q = qcalc(T, j);
       tm = tmax_of(T, q);
     }
 #pragma unroll
@@ -378,10 +392,9 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
 
   // ---- steady state
   for (; j < nt; ++j) {
-    if constexpr (YM != 0)
-      if (j + D < nt) pown = dot(j + D);
-    const PkTile T = info(j);
-    const float q = qcalc(T, j, pown);
+    if (j + D < nt) dot(j + D);
+    const uint4 T = ring[warp][j % kPkRing];
+    const float q = qcalc(T, j);
     scatter(T, q);
   }
 
@@ -390,17 +403,19 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   for (int i = threadIdx.x; i < bwk; i += kPkBS) dst[i] = (double)acc[i] * quantum;
 }
 
-__global__ void k_pk_finalize(int64_t n, int groups, const double* __restrict__ part, double* __restrict__ spill,
-                              const float* __restrict__ z, double beta, int add_beta_z, int accumulate, float* w,
-                              unsigned* epoch) {
+__global__ void k_pk_finalize(int64_t n, int bw, int groups, const double* __restrict__ part,
+                              double* __restrict__ spill, const float* __restrict__ z, double beta, int add_beta_z,
+                              int accumulate, float* w, unsigned* epoch) {
   for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
     double s = 0.0;
     for (int gi = 0; gi < groups; ++gi) s += part[(int64_t)gi * n + j];  // fixed order
-    s += spill[j];
+    const int64_t b = j / bw;
+    double* sp = spill + j + b;  // [block][bw + 1]
+    s += *sp;
     if (add_beta_z && beta != 0.0) s += beta * (double)z[j];
     if (accumulate) s += (double)w[j];
     w[j] = (float)s;
-    spill[j] = 0.0;
+    *sp = 0.0;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) *epoch += 1u;
 }
@@ -424,7 +439,7 @@ __global__ void k_pk_count(int64_t m, const int64_t* __restrict__ rowptr, const 
 // (2) tiles of each 32-row group (greedy): bit i of gmask set where a tile starts at row 32 g + i
 __device__ __forceinline__ bool pk_is_long(const uint32_t* cnt, int64_t m, int cs, int64_t r) {
   for (int kk = 0; kk < cs; ++kk)
-    if (cnt[(int64_t)kk * m + r] > (uint32_t)kPkSpan) return true;
+    if (cnt[(int64_t)kk * m + r] > (uint32_t)kPkLong) return true;
   return false;
 }
 __global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, uint32_t* __restrict__ gmask,
@@ -444,7 +459,7 @@ __global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, 
         continue;
       }
       bool fit = !fresh;
-      for (int kk = 0; kk < cs && fit; ++kk) fit = accs[kk] + cnt[(int64_t)kk * m + r] <= (uint32_t)kPkSpan;
+      for (int kk = 0; kk < cs && fit; ++kk) fit = accs[kk] + cnt[(int64_t)kk * m + r] <= (uint32_t)kPkLong;
       if (!fit) {
         mask |= 1u << i;
         ++ntl;
@@ -489,18 +504,27 @@ __global__ void k_pk_tile_rows(int64_t m, int cs, int64_t ntiles, const uint32_t
   }
 }
 
-__global__ void k_pk_seg(int64_t total, const int64_t* __restrict__ off, const uint32_t* __restrict__ tlen,
-                         uint2* __restrict__ seg) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
-    seg[i] = make_uint2((unsigned)(off[i] >> 2), tlen[i]);
+__global__ void k_pk_desc(int64_t total, int64_t ntiles, const int64_t* __restrict__ off,
+                          const uint32_t* __restrict__ tlen, const int64_t* __restrict__ tile_row,
+                          uint4* __restrict__ desc) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t t = i % ntiles;
+    desc[i] = make_uint4((unsigned)(off[i] >> 2), tlen[i], (unsigned)tile_row[t],
+                         (unsigned)(tile_row[t + 1] - tile_row[t]));
+  }
+}
+
+__global__ void k_pk_fill(int64_t n, uint32_t* __restrict__ p, uint32_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
 }
 
 // (4) the entries: a warp per 32-row group, lanes over a row's entries; block-k entries keep
-// their order (stable), so non-canonical rows are packed as given (reading R7)
+// their order (stable), so non-canonical rows are packed as given (reading R7).  Entry word:
+// byte offset of the column inside its block | row inside the tile << 18.
 __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const int64_t* __restrict__ rowptr,
                              const int32_t* __restrict__ colidx, const float* __restrict__ val,
                              const uint32_t* __restrict__ gmask, const int64_t* __restrict__ gbase,
-                             const uint2* __restrict__ seg, uint32_t* __restrict__ cr, float* __restrict__ pval) {
+                             const uint4* __restrict__ desc, uint32_t* __restrict__ cr, float* __restrict__ pval) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = pk_lanemask_lt();
   const int64_t ng = (m + 31) / 32;
@@ -509,13 +533,13 @@ __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const in
     const uint32_t mask = gmask[gi];
     int64_t t = gbase[gi] - 1;
     int64_t run[kPkMaxCS] = {};
-    int rid = 0;
+    unsigned rid = 0;
     for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
       const int64_t r = gi * 32 + i;
       if ((mask >> i) & 1u) {
         ++t;
         rid = 0;
-        for (int kk = 0; kk < cs; ++kk) run[kk] = (int64_t)seg[(int64_t)kk * ntiles + t].x * 4;
+        for (int kk = 0; kk < cs; ++kk) run[kk] = (int64_t)desc[(int64_t)kk * ntiles + t].x * 4;
       }
       const int64_t e = rowptr[r + 1];
       for (int64_t i0 = rowptr[r]; i0 < e; i0 += 32) {
@@ -530,7 +554,7 @@ __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const in
           run[kk] += __popc(bm);
         }
         if (ok) {
-          cr[pos] = (uint32_t)(col - b * bw) | ((uint32_t)rid << 16);
+          cr[pos] = ((uint32_t)(col - b * bw) * 4u) | (rid << kPkRidShift);
           pval[pos] = val ? val[ii] : 0.f;
         }
       }
@@ -583,7 +607,7 @@ int pk_headroom() {
 // columns one CTA holds (y fp32 + int32 partial in the opt-in shared memory)
 int packed_max_bw() {
   const size_t room = device_info(current_device()).smem_optin_per_block - kPkStatic;
-  return (int)std::min<size_t>(room / 8, 65535);
+  return (int)std::min<size_t>(room / 8 - 4, (kPkOffMask >> 2) - 1);  // + the zero / dummy slot
 }
 
 int packed_cs(int64_t n) {
@@ -595,7 +619,7 @@ int packed_cs(int64_t n) {
 
 void packed_free(Packed* p) {
   if (!p) return;
-  for (void* b : {(void*)p->tile_row, (void*)p->tile_seg, (void*)p->wtile, (void*)p->cr, (void*)p->val,
+  for (void* b : {(void*)p->tile_desc, (void*)p->wtile, (void*)p->cr, (void*)p->val,
                   (void*)p->xch, (void*)p->epoch, (void*)p->part, (void*)p->spill})
     if (b) cudaFree(b);
   delete p;
@@ -607,6 +631,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   FP_REQUIRE(dtype == FP_F32, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: the packed variant is fp32 only");
   FP_REQUIRE(val || nnz == 0, FP_ERR_INVALID_ARG, "fp_csr_plan_pack: val is NULL");
   FP_REQUIRE(m >= 1 && n >= 1, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: empty matrix");
+  FP_REQUIRE(m < INT32_MAX, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: m >= 2^31");
   const int cs = cs_force > 0 ? cs_force : packed_cs(n);
   FP_REQUIRE(cs == 1 || cs == 2 || cs == 4 || cs == 8, FP_ERR_UNSUPPORTED,
              "fp_csr_plan_pack: n = %lld needs more than 8 column blocks", (long long)n);
@@ -632,9 +657,11 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   int64_t* al = nullptr;
   int64_t* off = nullptr;
   uint32_t* tlen = nullptr;
+  int64_t* tile_row = nullptr;
   void* tmp = nullptr;
   auto cleanup = [&]() {
-    for (void* b : {(void*)cnt, (void*)gmask, (void*)gcount, (void*)gbase, (void*)al, (void*)off, (void*)tlen, tmp})
+    for (void* b : {(void*)cnt, (void*)gmask, (void*)gcount, (void*)gbase, (void*)al, (void*)off, (void*)tlen,
+                    (void*)tile_row, tmp})
       if (b) cudaFree(b);
   };
   auto fail = [&](cudaError_t e, const char* what) {
@@ -670,11 +697,11 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const int64_t ntiles = hb[0] + hb[1];
   p->ntiles = ntiles;
   const int64_t segs = (int64_t)cs * ntiles;
-  PK_TRY(cudaMalloc((void**)&p->tile_row, (size_t)(ntiles + 1) * 8), "alloc");
+  PK_TRY(cudaMalloc((void**)&tile_row, (size_t)(ntiles + 1) * 8), "alloc");
   PK_TRY(cudaMalloc((void**)&tlen, (size_t)segs * 4), "alloc");
   PK_TRY(cudaMalloc((void**)&al, (size_t)segs * 8), "alloc");
   PK_TRY(cudaMalloc((void**)&off, (size_t)segs * 8), "alloc");
-  k_pk_tile_rows<<<grid_g, tb, 0, s>>>(m, cs, ntiles, cnt, gmask, gbase, p->tile_row, tlen, al);
+  k_pk_tile_rows<<<grid_g, tb, 0, s>>>(m, cs, ntiles, cnt, gmask, gbase, tile_row, tlen, al);
   PK_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, al, off, segs, s), "scan");
   if (tb_bytes > tmp_bytes) {
     cudaFree(tmp);
@@ -690,29 +717,34 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const int64_t total = ht[0] + ht[1];
   if (total / 4 >= (int64_t)UINT32_MAX) return fail(cudaErrorInvalidValue, "too many nonzeros for 32-bit offsets");
   p->entries = total;
-  PK_TRY(cudaMalloc((void**)&p->tile_seg, (size_t)segs * sizeof(uint2)), "alloc");
-  k_pk_seg<<<(int)std::min<int64_t>((segs + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(segs, off, tlen,
-                                                                                                   p->tile_seg);
-  PK_TRY(cudaMalloc((void**)&p->cr, (size_t)std::max<int64_t>(total, 4) * 4), "alloc");
-  PK_TRY(cudaMalloc((void**)&p->val, (size_t)std::max<int64_t>(total, 4) * 4), "alloc");
-  PK_TRY(cudaMemsetAsync(p->cr, 0, (size_t)std::max<int64_t>(total, 4) * 4, s), "memset");
-  PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)std::max<int64_t>(total, 4) * 4, s), "memset");
+  PK_TRY(cudaMalloc((void**)&p->tile_desc, (size_t)segs * sizeof(uint4)), "alloc");
+  k_pk_desc<<<(int)std::min<int64_t>((segs + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(
+      segs, ntiles, off, tlen, tile_row, p->tile_desc);
+  const int64_t cap = std::max<int64_t>(total, 4);
+  PK_TRY(cudaMalloc((void**)&p->cr, (size_t)cap * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&p->val, (size_t)cap * 4), "alloc");
+  // padding entries (segment tails up to the next 16-byte boundary): the block's zero / dummy
+  // column, the tile's last row slot, value 0
+  k_pk_fill<<<(int)std::min<int64_t>((cap + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(
+      cap, p->cr, ((uint32_t)bw * 4u) | (31u << kPkRidShift));
+  PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)cap * 4, s), "memset");
   k_pk_scatter<<<(int)std::min<int64_t>((ng + 7) / 8, (int64_t)di.sm_count * 16), 256, 0, s>>>(
-      m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase, p->tile_seg, p->cr, p->val);
+      m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase, p->tile_desc, p->cr, p->val);
   const int nq = groups * kPkNW;
   if (ntiles >= INT32_MAX) return fail(cudaErrorInvalidValue, "too many tiles");
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
-  k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, p->tile_row, rowptr, p->wtile);
+  k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile);
   // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
-  const size_t xbytes = (size_t)groups * kPkNW * kPkNS * cs * 32 * 8;
+  const size_t xbytes = (size_t)groups * kPkNW * kPkNS * (cs + 1) * 32 * 8;
   PK_TRY(cudaMalloc((void**)&p->xch, xbytes), "alloc");
   PK_TRY(cudaMemsetAsync(p->xch, 0, xbytes, s), "memset");
   PK_TRY(cudaMalloc((void**)&p->epoch, 16), "alloc");
   const unsigned one = 1;
   PK_TRY(cudaMemcpyAsync(p->epoch, &one, 4, cudaMemcpyHostToDevice, s), "copy");
   PK_TRY(cudaMalloc((void**)&p->part, (size_t)groups * n * 8), "alloc");
-  PK_TRY(cudaMalloc((void**)&p->spill, (size_t)n * 8), "alloc");
-  PK_TRY(cudaMemsetAsync(p->spill, 0, (size_t)n * 8, s), "memset");
+  const size_t spb = (size_t)cs * (bw + 1) * 8;  // [block][bw + 1] (+ the dummy column)
+  PK_TRY(cudaMalloc((void**)&p->spill, spb), "alloc");
+  PK_TRY(cudaMemsetAsync(p->spill, 0, spb, s), "memset");
   // tiles per warp-quad must stay below 2^20 (the exchange tag)
   {
     std::vector<int32_t> hw(nq + 1);
@@ -744,8 +776,7 @@ fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.bw = p->bw;
   k.groups = p->groups;
   k.ntiles = p->ntiles;
-  k.tile_row = p->tile_row;
-  k.tile_seg = p->tile_seg;
+  k.tile_desc = p->tile_desc;
   k.wtile = p->wtile;
   k.cr = p->cr;
   k.val = p->val;
@@ -757,7 +788,7 @@ fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.epoch = p->epoch;
   k.part = p->part;
   k.spill = p->spill;
-  const size_t smem = (size_t)p->bw * (has_y ? 8 : 4);
+  const size_t smem = ((has_y ? (size_t)((p->bw + 4) & ~3) : 0) + (size_t)p->bw + 1) * 4;
   void* args[] = {&k};
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(p->groups * p->cs);
@@ -772,7 +803,7 @@ fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
   FP_CUDA(cudaLaunchKernelExC(&cfg, f, args));
   const int fb = 256;
   const int fg = (int)std::min<int64_t>((p->n + fb - 1) / fb, 8 * (int64_t)device_info(current_device()).sm_count);
-  k_pk_finalize<<<fg, fb, 0, s>>>(p->n, p->groups, p->part, p->spill, (const float*)a.z, a.beta,
+  k_pk_finalize<<<fg, fb, 0, s>>>(p->n, p->bw, p->groups, p->part, p->spill, (const float*)a.z, a.beta,
                                   a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (float*)a.w, p->epoch);
   FP_CUDA(cudaGetLastError());
   return FP_OK;
@@ -782,11 +813,11 @@ void packed_launch(const Packed* p, fp_launch* L) {
   *L = fp_launch{};
   L->variant = FP_VAR_CSR_PACKED;
   L->vs = 32;
-  L->tl = kPkSpan;
+  L->tl = kPkLong;
   L->bs = kPkBS;
   L->grid = p->groups * p->cs;
   L->cluster = p->cs;
-  L->smem_bytes = p->bw * 8;
+  L->smem_bytes = ((p->bw + 4) & ~3) * 4 + (p->bw + 1) * 4;
   L->blocks_per_sm = 1;
   cudaFuncAttributes fa{};
   if (cudaFuncGetAttributes(&fa, pk_pick(p->cs, true)) == cudaSuccess) L->regs_per_thread = fa.numRegs;

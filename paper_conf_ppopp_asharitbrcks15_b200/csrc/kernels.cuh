@@ -81,15 +81,14 @@ struct Packed {
   int cs = 0, bw = 0, groups = 0;
   int64_t ntiles = 0, entries = 0, max_tiles_per_warp = 0;
   const int64_t* rowptr = nullptr;
-  int64_t* tile_row = nullptr;          // [ntiles + 1]
-  uint2* tile_seg = nullptr;            // [cs][ntiles] (offset / 4, length)
+  uint4* tile_desc = nullptr;           // [cs][ntiles] (offset / 4, length, first row, rows)
   int32_t* wtile = nullptr;             // [groups * 32 + 1]
   uint32_t* cr = nullptr;               // [entries] column in block | row in tile << 16
   float* val = nullptr;                 // [entries]
   unsigned long long* xch = nullptr;    // exchange slots
   unsigned* epoch = nullptr;            // call counter
   double* part = nullptr;               // [groups][n]
-  double* spill = nullptr;              // [n]
+  double* spill = nullptr;              // [cs][bw + 1]
 };
 int packed_cs(int64_t n);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
