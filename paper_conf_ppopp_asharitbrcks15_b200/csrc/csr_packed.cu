@@ -13,9 +13,9 @@
 //
 // The copy (fp_csr_plan_pack, once per matrix, amortised over calls as the paper amortises
 // its baseline's transpose): for each column block k the block-k segments of every row
-// stored contiguously; rows grouped into TILES (<= 32 rows, every block segment <= 256
-// entries, or one long row); each entry one 32-bit word (column inside the block | row inside
-// the tile << 16) + its value; every segment starts 16-byte aligned.  The row structure of a
+// stored contiguously; rows grouped into TILES (<= 64 rows, every block segment <= 1024
+// entries, or one long row); each entry one 32-bit word (byte offset of the column inside the
+// block | row inside the tile << 26) + its value; every segment padded to 8 entries (32 bytes).  The row structure of a
 // tile is therefore in the entries themselves: no rowptr search and no head masks per call.
 //
 // One call: k_pk (the whole Eq. 1 pass, cooperative launch: the CTAs of a group wait on each
@@ -42,20 +42,27 @@ namespace {
 
 constexpr int kPkBS = 1024;
 constexpr int kPkNW = kPkBS / 32;
+constexpr int kPkRows = 64;           // rows per tile (at most)
 constexpr int kPkLong = 1024;         // a block segment longer than this makes its row a tile of its own
 constexpr int kPkRowCost = 4;         // work of a row in entries (warp partition)
-constexpr int kPkStatic = 11 * 1024;  // static shared memory reserve of k_pk
-constexpr int kPkNS = 8;              // exchange slots per warp (>= 2 D + 1)
+constexpr int kPkStatic = 27 * 1024;  // static shared memory reserve of k_pk
 constexpr int kPkRing = 4;            // tile descriptors a warp keeps between DOT and SCATTER (>= D + 1)
 constexpr unsigned kPkOffMask = 0x3FFFFu;  // entry word: byte offset of the column in the block (18 bits)
-constexpr int kPkRidShift = 18;            //             | row in tile << 18
+constexpr int kPkRidShift = 26;            //             | row in tile << 26 (rid * 4 = word >> 24)
+constexpr float kPkCap = 67108864.f;       // 2^26: |term / quantum| below this goes fixed point
+
+template <int D>
+struct PkSlots {
+  static constexpr int NS = 2 * D + 2;  // exchange slots per warp: a slot is rewritten only after
+};                                      // every CTA of the group consumed its tile
 
 struct PkArgs {
   int64_t n;
   int bw;                        // columns per block (block k = [k bw, min(n, (k+1) bw)))
   int groups;
   int64_t ntiles;
-  const uint4* tile_desc;        // [cs][ntiles]: (offset / 4, length, first row, rows)
+  int64_t padidx;                // 8 padding entries (the inactive lanes' loads)
+  const uint4* tile_desc;        // [cs][ntiles]: (offset / 8, length | rows << 25, first row, max |x| bits)
   const int32_t* wtile;          // [groups * 32 + 1]: first tile of each warp-quad
   const uint32_t* cr;            // packed entry words
   const float* val;
@@ -63,19 +70,31 @@ struct PkArgs {
   const float* v;
   float alpha;
   int hbits;                     // headroom bits of the fixed-point cap
-  unsigned long long* xch;       // exchange slots [groups][32 warps][kPkNS][cs + 1][32 lanes]
+  unsigned long long* xch;       // exchange slots [groups][32 warps][NS][cs + 1][64 rows]
   const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
   double* part;                  // [groups][n]
   double* spill;                 // [cs][bw + 1], all-zero between calls
 };
 
-__device__ __forceinline__ void pk_ld4(const uint32_t* pc, const float* pv, uint32_t (&c)[4], float (&x)[4]) {
-  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-      : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3])
-      : "l"(pc));
-  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
-      : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3])
-      : "l"(pv));
+// 8 consecutive entries (32 bytes) with an L2 eviction priority: the dot's read keeps the
+// segment (evict_last) for the scatter's re-read, which releases it (evict_first)
+template <bool KEEP>
+__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t (&c)[8], float (&x)[8]) {
+  if constexpr (KEEP) {
+    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
+        : "l"(pc));
+    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])
+        : "l"(pv));
+  } else {
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
+        : "l"(pc));
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])
+        : "l"(pv));
+  }
 }
 __device__ __forceinline__ void st_relaxed_gpu(unsigned long long* p, unsigned long long v) {
   asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -90,11 +109,19 @@ __device__ __forceinline__ unsigned pk_lanemask_lt() {
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
   return r;
 }
-// y (read-only after staging) and the fixed-point partial through 32-bit shared addresses
+// shared memory through 32-bit addresses (y and q are read-only while read)
 __device__ __forceinline__ float pk_lds(unsigned addr) {
   float v;
   asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr));
   return v;
+}
+__device__ __forceinline__ float pk_lds_v(unsigned addr) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ void pk_sts(unsigned addr, float v) {
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
 }
 __device__ __forceinline__ int pk_atom_add(unsigned addr, int v) {
   int old;
@@ -102,29 +129,34 @@ __device__ __forceinline__ int pk_atom_add(unsigned addr, int v) {
   return old;
 }
 __device__ __forceinline__ void pk_prefetch_l2(const void* p) {
-  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+  asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(p));
 }
+// (acc << 1) | (x >> 31): collect one sign bit per entry
+__device__ __forceinline__ unsigned pk_push_sign(unsigned acc, unsigned x) { return __funnelshift_l(x, acc, 1); }
 
 // The pass.  Warp `warp` of CTA k (block k) in group g walks the tile list of warp-quad
 // (g, warp) -- the same list in every CTA of the group -- as a pipeline:
-//   DOT(i):  stream tile i's segment (two 128-entry super-tiles per step, lane l holding
-//            entries 4l..4l+3 of each), Eq. (2) products y[col] x, segmented sums by row ->
-//            the block partial of the row dots, published as one tagged word per row (CTA 0
+//   DOT(i):  stream tile i's segment (256 entries per step, lane l holding entries 8l..8l+7
+//            from two 32-byte loads), Eq. (2) products y[col] x, segmented sums by row ->
+//            the block partials of the row dots, published as one tagged word per row (CTA 0
 //            also publishes v of the rows);
-//   Q(j):    j = i - D: wait for the CS (+ v) words of row `lane` of tile j, sum them in block
-//            order (identical in every CTA), q = alpha v p;
+//   Q(j):    j = i - D: wait for the CS (+ v) words of rows `lane` and `lane + 32` of tile j,
+//            sum them in block order (identical in every CTA), q = alpha v p;
 //   SCAT(j): stream tile j's segment again (read D tiles ago: an L2 hit) and add every
 //            term x q into the block's fixed-point partial.
 // The dot runs D tiles ahead of the scatter, so the exchange latency hides behind the warp's
-// own work.  Padding entries (column = the block's zero / dummy slot, row 31, value 0) make
-// every lane of a loaded 4-entry group valid: no per-entry predicates.
+// own work.  Padding entries (column = the block's zero / dummy slot, row 63, value 0) fill the
+// segments to 8 entries and the lanes beyond a segment load a padding block: no per-entry
+// predicates.
 template <int CS, int YM>
 __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
-  constexpr int D = (CS > 1 && YM != 0) ? 3 : 0;
-  static_assert(kPkNS >= 2 * D + 1 && kPkRing >= D + 1, "exchange slots / descriptor ring");
+  constexpr int D = (CS > 1 && YM != 0) ? 2 : 0;
+  constexpr int NS = PkSlots<D>::NS;
+  static_assert(kPkRing >= D + 1, "descriptor ring");
   extern __shared__ __align__(16) unsigned char pk_smem[];
-  __shared__ float rs[kPkNW][32];        // the tile's block partials of the row dots (by row in tile)
-  __shared__ float qsm[kPkNW][32];       // q of the tile's rows (spill path)
+  __shared__ float rs[kPkNW][kPkRows];   // the tile's block partials of the row dots (by row in tile)
+  __shared__ float qsm[kPkNW][kPkRows];  // q / quantum of the tile's rows
+  __shared__ float qus[kPkNW][kPkRows];  // q of the tile's rows (spill path, first rounds)
   __shared__ uint4 ring[kPkNW][kPkRing]; // descriptors of the tiles between DOT and SCATTER
   __shared__ unsigned s_tmax;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -144,34 +176,32 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   if (threadIdx.x == 0) s_tmax = 0u;
   __syncthreads();
   const unsigned ys_base = fpd::smem_u32(y_s), acc_base = fpd::smem_u32(acc);
+  const unsigned rs_base = fpd::smem_u32(&rs[warp][0]), qs_base = fpd::smem_u32(&qsm[warp][0]),
+                 qu_base = fpd::smem_u32(&qus[warp][0]);
 
   const int gq = g * kPkNW + warp;
   const int64_t t0 = a.wtile[gq];
   const int nt = a.wtile[gq + 1] - a.wtile[gq];
   const uint4* __restrict__ desc = a.tile_desc + (int64_t)k * a.ntiles + t0;
   const unsigned tag0 = *a.epoch << 20;
-  unsigned long long* const xslot = a.xch + (int64_t)gq * kPkNS * (CS + 1) * 32;
+  constexpr int SW = (CS + 1) * kPkRows;  // words of one slot
+  unsigned long long* const xslot = a.xch + (int64_t)gq * NS * SW;
   const float alpha = a.alpha;
   double* const spill = a.spill + (int64_t)k * (bw + 1);
+  const int64_t padidx = a.padidx;
 
-  // one step of a segment: entries s0 .. s0 + 255 of the 16-byte aligned segment at off4 * 4
-  auto load_win = [&](const uint4& T, int s0, uint32_t (&cw)[2][4], float (&xv)[2][4]) {
-    const int64_t base = (int64_t)T.x * 4;
-#pragma unroll
-    for (int st = 0; st < 2; ++st) {
-      const int o = s0 + 128 * st + 4 * lane;
-      if (o < (int)T.y) {
-        pk_ld4(a.cr + base + o, a.val + base + o, cw[st], xv[st]);
-      } else {
-#pragma unroll
-        for (int e = 0; e < 4; ++e) cw[st][e] = ((unsigned)bw * 4u) | (31u << kPkRidShift), xv[st][e] = 0.f;
-      }
-    }
+  auto seg_len = [](const uint4& T) { return (int)(T.y & 0x1FFFFFFu); };
+  auto seg_rows = [](const uint4& T) { return (int)(T.y >> 25); };
+  // the lane's 8 entries of step s0 (the padding block beyond the segment)
+  auto ld_step = [&](const uint4& T, int s0, auto keep, uint32_t (&cw)[8], float (&xv)[8]) {
+    const int o = s0 + 8 * lane;
+    const int64_t idx = o < seg_len(T) ? (int64_t)T.x * 8 + o : padidx;
+    pk_ld8<decltype(keep)::value>(a.cr + idx, a.val + idx, cw, xv);
   };
 
   // ---- DOT(i): tile i's block partials of the row dots, published (YM), descriptor -> ring
   uint4 cd = make_uint4(0, 0, 0, 0);  // lane l: descriptor of tile (i & ~31) + l
-  float pown = 0.f, vown = 1.f;       // D == 0: this CTA's partial / v of row `lane`
+  float pown0 = 0.f, pown1 = 0.f, vown0 = 0.f, vown1 = 0.f;  // D == 0: partials / v of rows lane, lane + 32
   auto dot = [&](int i) {
     if ((i & 31) == 0 && i + lane < nt) cd = __ldg(desc + i + lane);
     uint4 T;
@@ -180,179 +210,213 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     T.z = __shfl_sync(0xffffffffu, cd.z, i & 31);
     T.w = __shfl_sync(0xffffffffu, cd.w, i & 31);
     if (lane == 0) ring[warp][i % kPkRing] = T;
-    __syncwarp();
     // the next tile's segment on its way into L2 (lanes 0-15: 128-byte lines of cr, 16-31: val)
     {
       const int i1 = i + 1;
       const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
       if ((i1 & 31) != 0 && i1 < nt) {
         const int l = lane & 15;
-        if (32 * l < (int)min(len1, 512u)) {
-          const int64_t e = (int64_t)off1 * 4 + 32 * l;
+        if (32 * l < (int)min(len1 & 0x1FFFFFFu, 512u)) {
+          const int64_t e = (int64_t)off1 * 8 + 32 * l;
           pk_prefetch_l2(lane < 16 ? (const void*)(a.cr + e) : (const void*)(a.val + e));
         }
       }
     }
-    const float vr = (YM != 0 && (CS == 1 || k == 0) && lane < (int)T.w)
-                         ? (a.v ? __ldg(a.v + (int)T.z + lane) : 1.f) : 1.f;
-    if constexpr (YM == 0) return;
-    rs[warp][lane] = 0.f;
     __syncwarp();
-    int carry = -1;  // row of the previous super-tile's last entry
-    for (int s0 = 0; s0 < (int)T.y; s0 += 2 * 128) {
-      uint32_t cw[2][4];
-      float xv[2][4];
-      load_win(T, s0, cw, xv);
-#pragma unroll
-      for (int st = 0; st < 2; ++st) {
-        if (s0 + 128 * st >= (int)T.y) break;
-        int rid[4];
-        float c[4];  // in-lane inclusive segmented sums of the Eq. (2) products
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          rid[e] = (int)(cw[st][e] >> kPkRidShift);
-          const float pr = xv[st][e] * pk_lds(ys_base + (cw[st][e] & kPkOffMask));
-          c[e] = (e == 0 || rid[e] != rid[e - 1]) ? pr : c[e - 1] + pr;
-        }
-        int prev = __shfl_up_sync(0xffffffffu, rid[3], 1);
-        if (lane == 0) prev = carry;
-        const bool h0 = rid[0] != prev, h1 = rid[1] != rid[0], h2 = rid[2] != rid[1], h3 = rid[3] != rid[2];
-        const bool any = h0 | h1 | h2 | h3;
-        // P = the entries before the lane's first row start (continuing a row from before)
-        const float P = h0 ? 0.f : (h1 ? c[0] : (h2 ? c[1] : (h3 ? c[2] : c[3])));
-        // rows that start and end inside the lane
-        if (h1 && h0) rs[warp][rid[0]] = c[0];
-        if (h2 && (h0 | h1)) rs[warp][rid[1]] = c[1];
-        if (h3 && (h0 | h1 | h2)) rs[warp][rid[2]] = c[2];
-        // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a row start
-        const unsigned H = __ballot_sync(0xffffffffu, any);
-        const unsigned hl = H >> lane;
-        const int dist = hl ? __ffs(hl) : 32 - lane;
-        float r = P;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const float t2 = __shfl_down_sync(0xffffffffu, r, d);
-          if (d < dist) r += t2;
-        }
-        float rn = __shfl_down_sync(0xffffffffu, r, 1);
-        if (lane == 31) rn = 0.f;
-        if (any) rs[warp][rid[3]] = c[3] + rn;                     // the lane's last row
-        if (lane == 0 && !h0 && prev >= 0) rs[warp][prev] += r;    // the row running in
-        carry = __shfl_sync(0xffffffffu, rid[3], 31);
-        __syncwarp();
-      }
+    if constexpr (YM == 0) return;
+    const int nr = seg_rows(T), len = seg_len(T);
+    float v0 = 0.f, v1 = 0.f;
+    if (CS == 1 || k == 0) {
+      const float* vp = a.v + (int)T.z;
+      if (lane < nr) v0 = a.v ? __ldg(vp + lane) : 1.f;
+      if (lane + 32 < nr) v1 = a.v ? __ldg(vp + lane + 32) : 1.f;
     }
-    const float p = rs[warp][lane];
+    pk_sts(rs_base + 4 * lane, 0.f);
+    pk_sts(rs_base + 128 + 4 * lane, 0.f);
+    __syncwarp();
+    int carry = -4;  // rid * 4 of the previous step's last entry
+    for (int s0 = 0; s0 < len; s0 += 256) {
+      uint32_t cw[8];
+      float xv[8];
+      ld_step(T, s0, std::true_type{}, cw, xv);
+      int r4[8];
+      float c[8];  // in-lane inclusive segmented sums of the Eq. (2) products
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        r4[e] = (int)(cw[e] >> 24);
+        const float pr = xv[e] * pk_lds(ys_base + (cw[e] & kPkOffMask));
+        c[e] = (e == 0 || r4[e] != r4[e - 1]) ? pr : c[e - 1] + pr;
+      }
+      int prev = __shfl_up_sync(0xffffffffu, r4[7], 1);
+      if (lane == 0) prev = carry;
+      const bool h0 = r4[0] != prev;
+      bool seen = h0;
+      // rows that start and end inside the lane
+#pragma unroll
+      for (int e = 0; e < 7; ++e) {
+        const bool h = r4[e + 1] != r4[e];
+        if (h && seen) pk_sts(rs_base + r4[e], c[e]);
+        seen |= h;
+      }
+      // P = the entries before the lane's first row start (continuing a row from before)
+      float P = c[7];
+#pragma unroll
+      for (int e = 7; e >= 1; --e)
+        if (r4[e] != r4[e - 1]) P = c[e - 1];
+      if (h0) P = 0.f;
+      // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a row start
+      const unsigned H = __ballot_sync(0xffffffffu, seen);
+      const unsigned hl = H >> lane;
+      const int dist = hl ? __ffs(hl) : 32 - lane;
+      float r = P;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const float t2 = __shfl_down_sync(0xffffffffu, r, d);
+        if (d < dist) r += t2;
+      }
+      float rn = __shfl_down_sync(0xffffffffu, r, 1);
+      if (lane == 31) rn = 0.f;
+      if (seen) pk_sts(rs_base + r4[7], c[7] + rn);                                  // the lane's last row
+      if (lane == 0 && !h0 && prev >= 0) pk_sts(rs_base + prev, pk_lds_v(rs_base + prev) + r);  // running in
+      carry = __shfl_sync(0xffffffffu, r4[7], 31);
+      __syncwarp();
+    }
+    const float p0 = pk_lds_v(rs_base + 4 * lane), p1 = pk_lds_v(rs_base + 128 + 4 * lane);
     if constexpr (CS > 1) {
       const unsigned long long tg = (unsigned long long)(tag0 + (unsigned)i) << 32;
-      unsigned long long* slot = xslot + (int64_t)(i % kPkNS) * (CS + 1) * 32 + lane;
-      st_relaxed_gpu(slot + k * 32, tg | __float_as_uint(p));
-      if (k == 0) st_relaxed_gpu(slot + CS * 32, tg | __float_as_uint(vr));
+      unsigned long long* slot = xslot + (int64_t)(i % NS) * SW + lane;
+      st_relaxed_gpu(slot + k * kPkRows, tg | __float_as_uint(p0));
+      st_relaxed_gpu(slot + k * kPkRows + 32, tg | __float_as_uint(p1));
+      if (k == 0) {
+        st_relaxed_gpu(slot + CS * kPkRows, tg | __float_as_uint(v0));
+        st_relaxed_gpu(slot + CS * kPkRows + 32, tg | __float_as_uint(v1));
+      }
     } else {
-      pown = p;
-      vown = vr;
+      pown0 = p0;
+      pown1 = p1;
+      vown0 = v0;
+      vown1 = v1;
     }
   };
 
-  // ---- Q(j): q of row `lane` of tile j (descriptor T)
-  auto qcalc = [&](const uint4& T, int j) -> float {
-    float q;
+  // ---- Q(j): q of rows lane and lane + 32 of tile j (descriptor T) -> qus
+  auto qcalc = [&](const uint4& T, int j) {
+    const int nr = seg_rows(T);
+    float q0, q1;
     if constexpr (YM == 0) {
       (void)j;
-      const float vr = lane < (int)T.w ? (a.v ? __ldg(a.v + (int)T.z + lane) : 1.f) : 0.f;
-      q = alpha * vr;
+      const float* vp = a.v + (int)T.z;
+      q0 = lane < nr ? alpha * (a.v ? __ldg(vp + lane) : 1.f) : 0.f;
+      q1 = lane + 32 < nr ? alpha * (a.v ? __ldg(vp + lane + 32) : 1.f) : 0.f;
     } else if constexpr (CS == 1) {
       (void)j;
-      q = alpha * (vown * pown);
+      q0 = alpha * (vown0 * pown0);
+      q1 = alpha * (vown1 * pown1);
     } else {
       // the exchange: value + tag in one 64-bit word, so no flag and no fence is needed
       const unsigned tag = tag0 + (unsigned)j;
-      const unsigned long long* slot = xslot + (int64_t)(j % kPkNS) * (CS + 1) * 32 + lane;
-      unsigned long long wv[CS + 1];
-      bool done;
-      do {
-        done = true;
+      const unsigned long long* slot = xslot + (int64_t)(j % NS) * SW + lane;
+      unsigned long long wv[2 * (CS + 1)];
+      for (;;) {
+        bool done = true;
 #pragma unroll
-        for (int b = 0; b <= CS; ++b) {
-          wv[b] = ld_relaxed_gpu(slot + b * 32);
+        for (int b = 0; b < 2 * (CS + 1); ++b) {
+          wv[b] = ld_relaxed_gpu(slot + (b >> 1) * kPkRows + (b & 1) * 32);
           done &= (unsigned)(wv[b] >> 32) == tag;
         }
-      } while (!done);
-      float p = 0.f;
+        if (done) break;
+        __nanosleep(64);
+      }
+      float p0 = 0.f, p1 = 0.f;
 #pragma unroll
-      for (int b = 0; b < CS; ++b) p += __uint_as_float((unsigned)wv[b]);  // block order: identical in every CTA
-      q = alpha * (__uint_as_float((unsigned)wv[CS]) * p);
+      for (int b = 0; b < CS; ++b) {  // block order: identical in every CTA
+        p0 += __uint_as_float((unsigned)wv[2 * b]);
+        p1 += __uint_as_float((unsigned)wv[2 * b + 1]);
+      }
+      q0 = alpha * (__uint_as_float((unsigned)wv[2 * CS]) * p0);
+      q1 = alpha * (__uint_as_float((unsigned)wv[2 * CS + 1]) * p1);
     }
-    if (lane >= (int)T.w) q = 0.f;
-    qsm[warp][lane] = q;
-    return q;
+    if (lane >= nr) q0 = 0.f;
+    if (lane + 32 >= nr) q1 = 0.f;
+    pk_sts(qu_base + 4 * lane, q0);
+    pk_sts(qu_base + 128 + 4 * lane, q1);
   };
 
-  int E = 0;           // cap exponent: |t| < 2^E goes fixed point
-  float sc = 1.f;      // 2^(26 - E)
+  float sc = 1.f;      // 2^(26 - E): the cap is 2^E
   double quantum = 0;  // 2^(E - 26)
   auto set_scale = [&](int e) {
-    E = min(max(e, -95), 100);
-    sc = ldexpf(1.f, 26 - E);
-    quantum = ldexp(1.0, E - 26);
+    e = min(max(e, -95), 100);
+    sc = ldexpf(1.f, 26 - e);
+    quantum = ldexp(1.0, e - 26);
   };
   set_scale(0);
 
-  // ---- SCAT(j): Eq. (3) from the segment, re-read.  Common path branch-free; terms beyond the
-  // cap, non-finite terms and int32 wraps (rare) are collected in a mask and spilled after.
-  auto scatter = [&](const uint4& T, float q) {
-    const float qs = q * sc;
-    for (int s0 = 0; s0 < (int)T.y; s0 += 2 * 128) {
-      uint32_t cw[2][4];
-      float xv[2][4];
-      load_win(T, s0, cw, xv);
-      unsigned rare = 0;
+  // ---- SCAT(j): Eq. (3) from the segment, re-read.  SAFE (every |x q| of the tile below the
+  // cap, from the plan's max |x| of the tile): no per-entry checks; else terms beyond the cap
+  // and non-finite terms are flagged too.  Flagged entries (and int32 wraps) spill after.
+  auto scatter = [&](const uint4& T) {
+    __syncwarp();
+    const float q0 = pk_lds_v(qu_base + 4 * lane), q1 = pk_lds_v(qu_base + 128 + 4 * lane);
+    const float qs0 = q0 * sc, qs1 = q1 * sc;
+    pk_sts(qs_base + 4 * lane, qs0);
+    pk_sts(qs_base + 128 + 4 * lane, qs1);
+    const float xm = __uint_as_float(T.w);
+    const bool safe = __all_sync(0xffffffffu, fabsf(qs0) * xm < 67108000.f && fabsf(qs1) * xm < 67108000.f);
+    __syncwarp();
+    const int len = seg_len(T);
+    auto run = [&](auto SAFE) {
+      for (int s0 = 0; s0 < len; s0 += 256) {
+        uint32_t cw[8];
+        float xv[8];
+        ld_step(T, s0, std::false_type{}, cw, xv);
+        unsigned rare = 0;
 #pragma unroll
-      for (int st = 0; st < 2; ++st) {
-        if (s0 + 128 * st >= (int)T.y) break;
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const float qe = __shfl_sync(0xffffffffu, qs, (int)(cw[st][e] >> kPkRidShift));
-          const float ts = xv[st][e] * qe;
-          const bool big = !(fabsf(ts) < 67108864.f);  // >= 2^26 or NaN
-          const int qi = big ? 0 : __float2int_rn(ts);
-          const int old = pk_atom_add(acc_base + (cw[st][e] & kPkOffMask), qi);  // native ATOMS.ADD
+        for (int e = 0; e < 8; ++e) {
+          const float ts = xv[e] * pk_lds(qs_base + (cw[e] >> 24));
+          int qi = __float2int_rn(ts);
+          if constexpr (!decltype(SAFE)::value) {
+            const bool big = !(fabsf(ts) < kPkCap);  // >= 2^26 or NaN
+            if (big) qi = 0;
+            rare = (rare << 1) | (unsigned)big;
+          }
+          const int old = pk_atom_add(acc_base + (cw[e] & kPkOffMask), qi);  // native ATOMS.ADD
           const unsigned nw = (unsigned)old + (unsigned)qi;
-          const bool ovf = (int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0;
-          rare |= (unsigned)(big | ovf) << (4 * st + e);
+          const unsigned ovf = ((unsigned)old ^ nw) & ((unsigned)qi ^ nw);  // sign bit: int32 wrap
+          if constexpr (decltype(SAFE)::value) rare = pk_push_sign(rare, ovf);
+          else rare |= ovf >> 31;
         }
-      }
-      if (rare) {
+        if (rare) {  // rare: bit 7 - e flags entry e
 #pragma unroll
-        for (int b = 0; b < 8; ++b) {
-          if ((rare >> b) & 1u) {
-            const uint32_t w = cw[b >> 2][b & 3];
-            const float x = xv[b >> 2][b & 3];
-            const float t = x * qsm[warp][w >> kPkRidShift];
-            const int col = (int)((w & kPkOffMask) >> 2);
-            if (!(fabsf(t * sc) < 67108864.f)) atomicAdd(spill + col, (double)t);  // beyond the cap / Inf / NaN
-            else atomicAdd(spill + col, t > 0.f ? 4294967296.0 * quantum : -4294967296.0 * quantum);  // wrap
+          for (int e = 0; e < 8; ++e) {
+            if ((rare >> (7 - e)) & 1u) {
+              const float ts = xv[e] * pk_lds_v(qs_base + (cw[e] >> 24));
+              const int col = (int)((cw[e] & kPkOffMask) >> 2);
+              if (!(fabsf(ts) < kPkCap))  // beyond the cap / Inf / NaN (IEEE propagation, reading R8)
+                atomicAdd(spill + col, (double)(xv[e] * pk_lds_v(qu_base + (cw[e] >> 24))));
+              else  // the int32 sum wrapped: carry 2^32 quanta
+                atomicAdd(spill + col, ts > 0.f ? 4294967296.0 * quantum : -4294967296.0 * quantum);
+            }
           }
         }
       }
-    }
+    };
+    if (safe) run(std::true_type{});
+    else run(std::false_type{});
   };
 
   // largest finite |x q| of a tile (the first rounds only)
-  auto tmax_of = [&](const uint4& T, float q) -> float {
+  auto tmax_of = [&](const uint4& T) -> float {
+    __syncwarp();
     float tm = 0.f;
-    for (int s0 = 0; s0 < (int)T.y; s0 += 2 * 128) {
-      uint32_t cw[2][4];
-      float xv[2][4];
-      load_win(T, s0, cw, xv);
+    for (int s0 = 0; s0 < seg_len(T); s0 += 256) {
+      uint32_t cw[8];
+      float xv[8];
+      ld_step(T, s0, std::true_type{}, cw, xv);
 #pragma unroll
-      for (int st = 0; st < 2; ++st)
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const float qe = __shfl_sync(0xffffffffu, q, (int)(cw[st][e] >> kPkRidShift));
-          const float t = fabsf(xv[st][e] * qe);
-          if (t <= 3.402823466e38f) tm = fmaxf(tm, t);
-        }
+      for (int e = 0; e < 8; ++e) {
+        const float t = fabsf(xv[e] * pk_lds_v(qu_base + (cw[e] >> 24)));
+        if (t <= 3.402823466e38f) tm = fmaxf(tm, t);
+      }
     }
     return tm;
   };
@@ -365,12 +429,12 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   for (;;) {
     const bool have = j < nt;
     uint4 T = make_uint4(0, 0, 0, 0);
-    float q = 0.f, tm = 0.f;
+    float tm = 0.f;
     if (have) {
       if (j + D < nt) dot(j + D);
       T = ring[warp][j % kPkRing];
-      q = qcalc(T, j);
-      tm = tmax_of(T, q);
+      qcalc(T, j);
+      tm = tmax_of(T);
     }
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) tm = fmaxf(tm, __shfl_xor_sync(0xffffffffu, tm, d));
@@ -384,7 +448,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     }
     // (while every finite term so far is 0, the provisional scale adds zeros; non-finite terms spill)
     if (have) {
-      scatter(T, q);
+      scatter(T);
       ++j;
     }
     if (mx > 0.f || !any) break;
@@ -394,8 +458,8 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   for (; j < nt; ++j) {
     if (j + D < nt) dot(j + D);
     const uint4 T = ring[warp][j % kPkRing];
-    const float q = qcalc(T, j);
-    scatter(T, q);
+    qcalc(T, j);
+    scatter(T);
   }
 
   __syncthreads();
@@ -436,24 +500,24 @@ __global__ void k_pk_count(int64_t m, const int64_t* __restrict__ rowptr, const 
   }
 }
 
-// (2) tiles of each 32-row group (greedy): bit i of gmask set where a tile starts at row 32 g + i
+// (2) tiles of each 64-row group (greedy): bit i of gmask set where a tile starts at row 64 g + i
 __device__ __forceinline__ bool pk_is_long(const uint32_t* cnt, int64_t m, int cs, int64_t r) {
   for (int kk = 0; kk < cs; ++kk)
     if (cnt[(int64_t)kk * m + r] > (uint32_t)kPkLong) return true;
   return false;
 }
-__global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, uint32_t* __restrict__ gmask,
+__global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, unsigned long long* __restrict__ gmask,
                            int64_t* __restrict__ gcount) {
-  const int64_t ng = (m + 31) / 32;
+  const int64_t ng = (m + kPkRows - 1) / kPkRows;
   for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
     uint32_t accs[kPkMaxCS] = {};
-    uint32_t mask = 0;
+    unsigned long long mask = 0;
     int ntl = 0;
     bool fresh = true;  // the next row starts a tile
-    for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
-      const int64_t r = gi * 32 + i;
+    for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
+      const int64_t r = gi * kPkRows + i;
       if (pk_is_long(cnt, m, cs, r)) {
-        mask |= 1u << i;
+        mask |= 1ull << i;
         ++ntl;
         fresh = true;
         continue;
@@ -461,7 +525,7 @@ __global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, 
       bool fit = !fresh;
       for (int kk = 0; kk < cs && fit; ++kk) fit = accs[kk] + cnt[(int64_t)kk * m + r] <= (uint32_t)kPkLong;
       if (!fit) {
-        mask |= 1u << i;
+        mask |= 1ull << i;
         ++ntl;
         for (int kk = 0; kk < cs; ++kk) accs[kk] = 0;
       }
@@ -473,26 +537,26 @@ __global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, 
   }
 }
 
-// (3) tile rows and segment lengths; al = the lengths rounded up to 4 (scanned into offsets)
+// (3) tile rows and segment lengths; al = the lengths rounded up to 8 (scanned into offsets)
 __global__ void k_pk_tile_rows(int64_t m, int cs, int64_t ntiles, const uint32_t* __restrict__ cnt,
-                               const uint32_t* __restrict__ gmask, const int64_t* __restrict__ gbase,
+                               const unsigned long long* __restrict__ gmask, const int64_t* __restrict__ gbase,
                                int64_t* __restrict__ tile_row, uint32_t* __restrict__ tlen, int64_t* __restrict__ al) {
-  const int64_t ng = (m + 31) / 32;
+  const int64_t ng = (m + kPkRows - 1) / kPkRows;
   for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t mask = gmask[gi];
+    const unsigned long long mask = gmask[gi];
     int64_t t = gbase[gi] - 1;
     uint32_t len[kPkMaxCS] = {};
     auto flush = [&]() {
       if (t < 0) return;
       for (int kk = 0; kk < cs; ++kk) {
         tlen[(int64_t)kk * ntiles + t] = len[kk];
-        al[(int64_t)kk * ntiles + t] = (int64_t)((len[kk] + 3u) & ~3u);
+        al[(int64_t)kk * ntiles + t] = (int64_t)((len[kk] + 7u) & ~7u);
         len[kk] = 0;
       }
     };
-    for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
-      const int64_t r = gi * 32 + i;
-      if ((mask >> i) & 1u) {
+    for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
+      const int64_t r = gi * kPkRows + i;
+      if ((mask >> i) & 1ull) {
         flush();
         ++t;
         tile_row[t] = r;
@@ -509,8 +573,8 @@ __global__ void k_pk_desc(int64_t total, int64_t ntiles, const int64_t* __restri
                           uint4* __restrict__ desc) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t t = i % ntiles;
-    desc[i] = make_uint4((unsigned)(off[i] >> 2), tlen[i], (unsigned)tile_row[t],
-                         (unsigned)(tile_row[t + 1] - tile_row[t]));
+    const unsigned nr = (unsigned)(tile_row[t + 1] - tile_row[t]);
+    desc[i] = make_uint4((unsigned)(off[i] >> 3), tlen[i] | (nr << 25), (unsigned)tile_row[t], 0u);
   }
 }
 
@@ -518,28 +582,41 @@ __global__ void k_pk_fill(int64_t n, uint32_t* __restrict__ p, uint32_t v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
 }
 
-// (4) the entries: a warp per 32-row group, lanes over a row's entries; block-k entries keep
+// (4) the entries: a warp per 64-row group, lanes over a row's entries; block-k entries keep
 // their order (stable), so non-canonical rows are packed as given (reading R7).  Entry word:
-// byte offset of the column inside its block | row inside the tile << 18.
+// byte offset of the column inside its block | row inside the tile << 26.  Also the largest
+// |x| of every (tile, block) segment (+Inf if a value is not finite): the scatter's no-check test.
 __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const int64_t* __restrict__ rowptr,
                              const int32_t* __restrict__ colidx, const float* __restrict__ val,
-                             const uint32_t* __restrict__ gmask, const int64_t* __restrict__ gbase,
-                             const uint4* __restrict__ desc, uint32_t* __restrict__ cr, float* __restrict__ pval) {
+                             const unsigned long long* __restrict__ gmask, const int64_t* __restrict__ gbase,
+                             uint4* __restrict__ desc, uint32_t* __restrict__ cr, float* __restrict__ pval) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = pk_lanemask_lt();
-  const int64_t ng = (m + 31) / 32;
+  const int64_t ng = (m + kPkRows - 1) / kPkRows;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
   for (int64_t gi = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5); gi < ng; gi += nw) {
-    const uint32_t mask = gmask[gi];
+    const unsigned long long mask = gmask[gi];
     int64_t t = gbase[gi] - 1;
     int64_t run[kPkMaxCS] = {};
+    float xm[kPkMaxCS] = {};
     unsigned rid = 0;
-    for (int i = 0; i < 32 && gi * 32 + i < m; ++i) {
-      const int64_t r = gi * 32 + i;
-      if ((mask >> i) & 1u) {
+    auto flush = [&]() {
+      if (t < 0) return;
+      for (int kk = 0; kk < cs; ++kk) {
+        float v = xm[kk];
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, d));
+        if (lane == 0) desc[(int64_t)kk * ntiles + t].w = __float_as_uint(v);
+        xm[kk] = 0.f;
+      }
+    };
+    for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
+      const int64_t r = gi * kPkRows + i;
+      if ((mask >> i) & 1ull) {
+        flush();
         ++t;
         rid = 0;
-        for (int kk = 0; kk < cs; ++kk) run[kk] = (int64_t)desc[(int64_t)kk * ntiles + t].x * 4;
+        for (int kk = 0; kk < cs; ++kk) run[kk] = (int64_t)desc[(int64_t)kk * ntiles + t].x * 8;
       }
       const int64_t e = rowptr[r + 1];
       for (int64_t i0 = rowptr[r]; i0 < e; i0 += 32) {
@@ -548,18 +625,24 @@ __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const in
         const int col = ok ? colidx[ii] : 0;
         const int b = col / bw;
         int64_t pos = -1;
+        const float x = ok && val ? val[ii] : 0.f;
+        const float ax = fabsf(x) <= 3.402823466e38f ? fabsf(x) : __int_as_float(0x7f800000);
         for (int kk = 0; kk < cs; ++kk) {
           const unsigned bm = __ballot_sync(0xffffffffu, ok && b == kk);
-          if (ok && b == kk) pos = run[kk] + __popc(bm & lt);
+          if (ok && b == kk) {
+            pos = run[kk] + __popc(bm & lt);
+            xm[kk] = fmaxf(xm[kk], ax);
+          }
           run[kk] += __popc(bm);
         }
         if (ok) {
           cr[pos] = ((uint32_t)(col - b * bw) * 4u) | (rid << kPkRidShift);
-          pval[pos] = val ? val[ii] : 0.f;
+          pval[pos] = x;
         }
       }
       ++rid;
     }
+    flush();
   }
 }
 
@@ -649,9 +732,9 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   p->bw = bw;
   p->groups = groups;
   p->rowptr = rowptr;
-  const int64_t ng = (m + 31) / 32;
+  const int64_t ng = (m + kPkRows - 1) / kPkRows;
   uint32_t* cnt = nullptr;
-  uint32_t* gmask = nullptr;
+  unsigned long long* gmask = nullptr;
   int64_t* gcount = nullptr;
   int64_t* gbase = nullptr;
   int64_t* al = nullptr;
@@ -677,7 +760,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
     if (e_ != cudaSuccess) return fail(e_, what); \
   } while (0)
   PK_TRY(cudaMalloc((void**)&cnt, (size_t)cs * m * 4), "alloc");
-  PK_TRY(cudaMalloc((void**)&gmask, (size_t)ng * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&gmask, (size_t)ng * 8), "alloc");
   PK_TRY(cudaMalloc((void**)&gcount, (size_t)ng * 8), "alloc");
   PK_TRY(cudaMalloc((void**)&gbase, (size_t)ng * 8), "alloc");
   const int tb = 256;
@@ -715,18 +798,18 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   PK_TRY(cudaMemcpyAsync(&ht[1], al + segs - 1, 8, cudaMemcpyDeviceToHost, s), "copy");
   PK_TRY(cudaStreamSynchronize(s), "sync");
   const int64_t total = ht[0] + ht[1];
-  if (total / 4 >= (int64_t)UINT32_MAX) return fail(cudaErrorInvalidValue, "too many nonzeros for 32-bit offsets");
+  if (total / 8 >= (int64_t)UINT32_MAX) return fail(cudaErrorInvalidValue, "too many nonzeros for 32-bit offsets");
   p->entries = total;
   PK_TRY(cudaMalloc((void**)&p->tile_desc, (size_t)segs * sizeof(uint4)), "alloc");
   k_pk_desc<<<(int)std::min<int64_t>((segs + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(
       segs, ntiles, off, tlen, tile_row, p->tile_desc);
-  const int64_t cap = std::max<int64_t>(total, 4);
+  const int64_t cap = total + 8;  // + the padding block the inactive lanes load
   PK_TRY(cudaMalloc((void**)&p->cr, (size_t)cap * 4), "alloc");
   PK_TRY(cudaMalloc((void**)&p->val, (size_t)cap * 4), "alloc");
   // padding entries (segment tails up to the next 16-byte boundary): the block's zero / dummy
   // column, the tile's last row slot, value 0
   k_pk_fill<<<(int)std::min<int64_t>((cap + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(
-      cap, p->cr, ((uint32_t)bw * 4u) | (31u << kPkRidShift));
+      cap, p->cr, ((uint32_t)bw * 4u) | ((uint32_t)(kPkRows - 1) << kPkRidShift));
   PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)cap * 4, s), "memset");
   k_pk_scatter<<<(int)std::min<int64_t>((ng + 7) / 8, (int64_t)di.sm_count * 16), 256, 0, s>>>(
       m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase, p->tile_desc, p->cr, p->val);
@@ -735,7 +818,8 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
   k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile);
   // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
-  const size_t xbytes = (size_t)groups * kPkNW * kPkNS * (cs + 1) * 32 * 8;
+  const int ns = cs > 1 ? PkSlots<2>::NS : 1;
+  const size_t xbytes = (size_t)groups * kPkNW * ns * (cs + 1) * kPkRows * 8;
   PK_TRY(cudaMalloc((void**)&p->xch, xbytes), "alloc");
   PK_TRY(cudaMemsetAsync(p->xch, 0, xbytes, s), "memset");
   PK_TRY(cudaMalloc((void**)&p->epoch, 16), "alloc");
@@ -777,6 +861,7 @@ fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.groups = p->groups;
   k.ntiles = p->ntiles;
   k.tile_desc = p->tile_desc;
+  k.padidx = p->entries;
   k.wtile = p->wtile;
   k.cr = p->cr;
   k.val = p->val;
