@@ -109,7 +109,9 @@ __device__ __forceinline__ unsigned pk_lanemask_lt() {
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
   return r;
 }
-// shared memory through 32-bit addresses (y and q are read-only while read)
+// shared memory through 32-bit addresses (y and q are read-only while read).  No "memory"
+// clobbers: they would pin the next step's global loads behind this step's atomics; the
+// volatile ones keep their order among themselves, __syncwarp orders them across lanes.
 __device__ __forceinline__ float pk_lds(unsigned addr) {
   float v;
   asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr));
@@ -117,15 +119,15 @@ __device__ __forceinline__ float pk_lds(unsigned addr) {
 }
 __device__ __forceinline__ float pk_lds_v(unsigned addr) {
   float v;
-  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr));
   return v;
 }
 __device__ __forceinline__ void pk_sts(unsigned addr, float v) {
-  asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v));
 }
 __device__ __forceinline__ int pk_atom_add(unsigned addr, int v) {
   int old;
-  asm volatile("atom.shared.add.s32 %0, [%1], %2;" : "=r"(old) : "r"(addr), "r"(v) : "memory");
+  asm volatile("atom.shared.add.s32 %0, [%1], %2;" : "=r"(old) : "r"(addr), "r"(v));
   return old;
 }
 __device__ __forceinline__ void pk_prefetch_l2(const void* p) {
