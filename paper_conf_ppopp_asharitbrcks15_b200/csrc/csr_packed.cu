@@ -74,6 +74,7 @@ struct PkArgs {
   const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
   double* part;                  // [groups][n]
   double* spill;                 // [cs][bw + 1], all-zero between calls
+  unsigned long long* trace;     // FP_PK_TRACE: per warp (start, end of the pass, tiles, prologue end)
 };
 
 // 8 consecutive entries (32 bytes) with an L2 eviction priority: the dot's read keeps the
@@ -181,6 +182,8 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   const unsigned rs_base = fpd::smem_u32(&rs[warp][0]), qs_base = fpd::smem_u32(&qsm[warp][0]),
                  qu_base = fpd::smem_u32(&qus[warp][0]);
 
+  unsigned long long tr0 = 0, tr1 = 0;
+  if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr0));
   const int gq = g * kPkNW + warp;
   const int64_t t0 = a.wtile[gq];
   const int nt = a.wtile[gq + 1] - a.wtile[gq];
@@ -456,12 +459,22 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     if (mx > 0.f || !any) break;
   }
 
+  if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr1));
   // ---- steady state
   for (; j < nt; ++j) {
     if (j + D < nt) dot(j + D);
     const uint4 T = ring[warp][j % kPkRing];
     qcalc(T, j);
     scatter(T);
+  }
+  if (a.trace && lane == 0) {
+    unsigned long long tr2;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr2));
+    unsigned long long* tp = a.trace + ((int64_t)blockIdx.x * kPkNW + warp) * 4;
+    tp[0] = tr0;
+    tp[1] = tr2;
+    tp[2] = (unsigned long long)nt;
+    tp[3] = tr1;
   }
 
   __syncthreads();
@@ -705,7 +718,7 @@ int packed_cs(int64_t n) {
 void packed_free(Packed* p) {
   if (!p) return;
   for (void* b : {(void*)p->tile_desc, (void*)p->wtile, (void*)p->cr, (void*)p->val,
-                  (void*)p->xch, (void*)p->epoch, (void*)p->part, (void*)p->spill})
+                  (void*)p->xch, (void*)p->epoch, (void*)p->part, (void*)p->spill, (void*)p->trace})
     if (b) cudaFree(b);
   delete p;
 }
@@ -852,7 +865,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   return FP_OK;
 }
 
-fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
+fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   const bool has_y = a.y != nullptr;
   const void* f = pk_pick(p->cs, has_y);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr_plan_exec: no packed kernel for %d blocks", p->cs);
@@ -875,6 +888,11 @@ fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.epoch = p->epoch;
   k.part = p->part;
   k.spill = p->spill;
+  k.trace = nullptr;
+  if (std::getenv("FP_PK_TRACE")) {  // measurement: per-warp timing of the pass (kept in the plan)
+    if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 32);
+    k.trace = p->trace;
+  }
   const size_t smem = ((has_y ? (size_t)((p->bw + 4) & ~3) : 0) + (size_t)p->bw + 1) * 4;
   void* args[] = {&k};
   cudaLaunchConfig_t cfg{};

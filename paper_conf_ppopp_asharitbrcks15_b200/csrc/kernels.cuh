@@ -89,11 +89,12 @@ struct Packed {
   unsigned* epoch = nullptr;            // call counter
   double* part = nullptr;               // [groups][n]
   double* spill = nullptr;              // [cs][bw + 1]
+  unsigned long long* trace = nullptr;  // FP_PK_TRACE measurement buffer
 };
 int packed_cs(int64_t n);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                        const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s);
-fp_status packed_exec(const Packed* p, const PatternArgs& a, cudaStream_t s);
+fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s);
 void packed_free(Packed* p);
 void packed_launch(const Packed* p, fp_launch* L);
 
