@@ -23,9 +23,11 @@
 //
 // Fixed point (reading R25): CTA c adds every term t = x q as round(t / quantum_c)
 // into a 32-bit shared accumulator, quantum_c = 2^(E_c - 26), E_c = (exponent of the largest
-// finite |t| of the CTA's first tile round) + H (H = 3 headroom bits): |t| < 2^E_c gives an
-// int32 of magnitude < 2^26 (error <= quantum_c / 2 per term); larger or non-finite terms and
-// the (rare) int32 wraps go to an fp64 spill vector with global reds.  The partials are
+// finite |t| of the CTA's first tile round) + H (H = 3 headroom bits), so the first round's
+// terms are int32s of magnitude < 2^26 (error <= quantum_c / 2 per term) and terms up to
+// 2^(E_c + 5) (power-law rows: |q| grows like sqrt(row length)) still fit an int32 exactly;
+// an add that wraps the int32 sum is detected from the returned old value and carries 2^32
+// quanta into an fp64 spill vector; larger or non-finite terms go to the spill themselves.  The partials are
 // converted exactly to fp64 and summed in group order: deterministic except for spills.
 #include <algorithm>
 #include <cstdlib>
@@ -49,7 +51,8 @@ constexpr int kPkStatic = 27 * 1024;  // static shared memory reserve of k_pk
 constexpr int kPkRing = 4;            // tile descriptors a warp keeps between DOT and SCATTER (>= D + 1)
 constexpr unsigned kPkOffMask = 0x3FFFFu;  // entry word: byte offset of the column in the block (18 bits)
 constexpr int kPkRidShift = 26;            //             | row in tile << 26 (rid * 4 = word >> 24)
-constexpr float kPkCap = 67108864.f;       // 2^26: |term / quantum| below this goes fixed point
+constexpr float kPkCap = 2147483520.f;     // 2^31 - 128: |term / quantum| below this is an exact-range int32
+                                           // (one int32 wrap at most per add: detected, carried)
 
 template <int D>
 struct PkSlots {
@@ -366,7 +369,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     pk_sts(qs_base + 4 * lane, qs0);
     pk_sts(qs_base + 128 + 4 * lane, qs1);
     const float xm = __uint_as_float(T.w);
-    const bool safe = __all_sync(0xffffffffu, fabsf(qs0) * xm < 67108000.f && fabsf(qs1) * xm < 67108000.f);
+    const bool safe = __all_sync(0xffffffffu, fabsf(qs0) * xm < 2.0e9f && fabsf(qs1) * xm < 2.0e9f);
     __syncwarp();
     const int len = seg_len(T);
     auto run = [&](auto SAFE) {
@@ -380,7 +383,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
           const float ts = xv[e] * pk_lds(qs_base + (cw[e] >> 24));
           int qi = __float2int_rn(ts);
           if constexpr (!decltype(SAFE)::value) {
-            const bool big = !(fabsf(ts) < kPkCap);  // >= 2^26 or NaN
+            const bool big = !(fabsf(ts) < kPkCap);  // beyond the int32 range, or NaN
             if (big) qi = 0;
             rare = (rare << 1) | (unsigned)big;
           }

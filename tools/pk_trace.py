@@ -38,3 +38,9 @@ print("per group: max end, min/median/max us:", grp.max(1).min().round(1), np.me
       grp.max(1).max().round(1))
 slow = np.argsort(end)[-5:]
 print("slowest warps (cta, warp, end us, tiles):", [(int(i // 32), int(i % 32), round(end[i], 1), int(tiles[i])) for i in slow])
+w = end.reshape(-1, 32)
+print("mean end by warp index:", w.mean(0).round(0).astype(int).tolist())
+print("corr(end, tiles):", np.corrcoef(end, tiles)[0, 1].round(3))
+c = end.reshape(-1, 32).mean(1)
+print("mean end by CTA (first 16):", c[:16].round(0).astype(int).tolist())
+print("by block k (cta % blocks):", [round(float(c[k::info['blocks']].mean()), 1) for k in range(info['blocks'])])
