@@ -185,7 +185,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   const unsigned rs_base = fpd::smem_u32(&rs[warp][0]), qs_base = fpd::smem_u32(&qsm[warp][0]),
                  qu_base = fpd::smem_u32(&qus[warp][0]);
 
-  unsigned long long tr0 = 0, tr1 = 0;
+  unsigned long long tr0 = 0, tr1 = 0, twait = 0, nrare = 0, nsafe = 0, tdot = 0;
   if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr0));
   const int gq = g * kPkNW + warp;
   const int64_t t0 = a.wtile[gq];
@@ -325,6 +325,8 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
       const unsigned tag = tag0 + (unsigned)j;
       const unsigned long long* slot = xslot + (int64_t)(j % NS) * SW + lane;
       unsigned long long wv[2 * (CS + 1)];
+      unsigned long long c0w = 0;
+      if (a.trace) c0w = clock64();
       for (;;) {
         bool done = true;
 #pragma unroll
@@ -335,6 +337,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
         if (done) break;
         __nanosleep(64);
       }
+      if (a.trace) twait += clock64() - c0w;
       float p0 = 0.f, p1 = 0.f;
 #pragma unroll
       for (int b = 0; b < CS; ++b) {  // block order: identical in every CTA
@@ -393,6 +396,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
           if constexpr (decltype(SAFE)::value) rare = pk_push_sign(rare, ovf);
           else rare |= ovf >> 31;
         }
+        if (a.trace && rare) nrare += __popc(rare);
         if (rare) {  // rare: bit 7 - e flags entry e
 #pragma unroll
           for (int e = 0; e < 8; ++e) {
@@ -408,6 +412,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
         }
       }
     };
+    if (a.trace) nsafe += safe ? 1 : 0;
     if (safe) run(std::true_type{});
     else run(std::false_type{});
   };
@@ -465,7 +470,10 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr1));
   // ---- steady state
   for (; j < nt; ++j) {
+    unsigned long long cd0 = 0;
+    if (a.trace) cd0 = clock64();
     if (j + D < nt) dot(j + D);
+    if (a.trace) tdot += clock64() - cd0;
     const uint4 T = ring[warp][j % kPkRing];
     qcalc(T, j);
     scatter(T);
@@ -473,11 +481,15 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   if (a.trace && lane == 0) {
     unsigned long long tr2;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr2));
-    unsigned long long* tp = a.trace + ((int64_t)blockIdx.x * kPkNW + warp) * 4;
+    unsigned long long* tp = a.trace + ((int64_t)blockIdx.x * kPkNW + warp) * 8;
     tp[0] = tr0;
     tp[1] = tr2;
     tp[2] = (unsigned long long)nt;
     tp[3] = tr1;
+    tp[4] = twait;
+    tp[5] = nrare;
+    tp[6] = nsafe;
+    tp[7] = tdot;
   }
 
   __syncthreads();
@@ -893,7 +905,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.spill = p->spill;
   k.trace = nullptr;
   if (std::getenv("FP_PK_TRACE")) {  // measurement: per-warp timing of the pass (kept in the plan)
-    if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 32);
+    if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 64);
     k.trace = p->trace;
   }
   const size_t smem = ((has_y ? (size_t)((p->bw + 4) & ~3) : 0) + (size_t)p->bw + 1) * 4;

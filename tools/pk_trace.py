@@ -22,9 +22,9 @@ for _ in range(3):
 torch.cuda.synchronize()
 info = plan.pack_info
 nw = info["groups"] * info["blocks"] * 32
-buf = (ctypes.c_ulonglong * (4 * nw))()
-k = fp.lib().fpx_pack_trace(plan._h, buf, ctypes.c_int64(4 * nw))
-t = np.frombuffer(buf, dtype=np.uint64).reshape(-1, 4).astype(np.float64)
+buf = (ctypes.c_ulonglong * (8 * nw))()
+k = fp.lib().fpx_pack_trace(plan._h, buf, ctypes.c_int64(8 * nw))
+t = np.frombuffer(buf, dtype=np.uint64).reshape(-1, 8).astype(np.float64)
 t0 = t[:, 0].min()
 start, end, tiles, pro = (t[:, 0] - t0) / 1e3, (t[:, 1] - t0) / 1e3, t[:, 2], (t[:, 3] - t0) / 1e3
 print(f"warps {len(t)}  start us: max {start.max():.1f}  prologue end us: median {np.median(pro):.1f} max {pro.max():.1f}")
@@ -44,3 +44,8 @@ print("corr(end, tiles):", np.corrcoef(end, tiles)[0, 1].round(3))
 c = end.reshape(-1, 32).mean(1)
 print("mean end by CTA (first 16):", c[:16].round(0).astype(int).tolist())
 print("by block k (cta % blocks):", [round(float(c[k::info['blocks']].mean()), 1) for k in range(info['blocks'])])
+wait_ms, rare, safe, dotms = t[:, 4] / 1.965e6, t[:, 5], t[:, 6], t[:, 7] / 1.965e6
+print("poll wait ms: median/max", np.median(wait_ms).round(2), wait_ms.max().round(2), " corr(end, wait):", np.corrcoef(end, wait_ms)[0, 1].round(3))
+print("dot ms: median/max", np.median(dotms).round(2), dotms.max().round(2), " corr(end, dot):", np.corrcoef(end, dotms)[0, 1].round(3))
+print("flagged entries: total", int(rare.sum()), " max per warp", int(rare.max()), " corr(end, flagged):", np.corrcoef(end, rare)[0, 1].round(3))
+print("check-free tiles fraction:", (safe.sum() / tiles.sum()).round(4))
