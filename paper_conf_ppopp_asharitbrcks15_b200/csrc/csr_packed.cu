@@ -31,6 +31,7 @@
 // converted exactly to fp64 and summed in group order: deterministic except for spills.
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
 #include <new>
 #include <vector>
 
@@ -77,29 +78,30 @@ struct PkArgs {
   const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
   double* part;                  // [groups][n]
   double* spill;                 // [cs][bw + 1], all-zero between calls
+  int pol_keep, pol_release;     // L2 hints of the dot's read / the scatter's re-read (pk_ld8)
+  int nap;                       // ns a warp sleeps between polls of the exchange (0: spin)
   unsigned long long* trace;     // FP_PK_TRACE: per warp (start, end of the pass, tiles, prologue end)
 };
 
-// 8 consecutive entries (32 bytes) with an L2 eviction priority: the dot's read keeps the
-// segment (evict_last) for the scatter's re-read, which releases it (evict_first)
-template <bool KEEP>
-__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t (&c)[8], float (&x)[8]) {
-  if constexpr (KEEP) {
-    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-        : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
-        : "l"(pc));
-    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])
-        : "l"(pv));
+// 8 consecutive entries (32 bytes).  POL: 0 = no L2 hint, 1 = evict_last (the dot's read keeps
+// the segment for the scatter's re-read), 2 = evict_first (the re-read releases it)
+#define PK_LD8(Q)                                                                                      \
+  asm("ld.global.nc.L1::no_allocate" Q ".v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                      \
+      : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])  \
+      : "l"(pc));                                                                                      \
+  asm("ld.global.nc.L1::no_allocate" Q ".v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                      \
+      : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])  \
+      : "l"(pv))
+__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t (&c)[8], float (&x)[8], int pol) {
+  if (pol == 1) {
+    PK_LD8(".L2::evict_last");
+  } else if (pol == 2) {
+    PK_LD8(".L2::evict_first");
   } else {
-    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-        : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
-        : "l"(pc));
-    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])
-        : "l"(pv));
+    PK_LD8("");
   }
 }
+#undef PK_LD8
 __device__ __forceinline__ void st_relaxed_gpu(unsigned long long* p, unsigned long long v) {
   asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -204,7 +206,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   auto ld_step = [&](const uint4& T, int s0, auto keep, uint32_t (&cw)[8], float (&xv)[8]) {
     const int o = s0 + 8 * lane;
     const int64_t idx = o < seg_len(T) ? (int64_t)T.x * 8 + o : padidx;
-    pk_ld8<decltype(keep)::value>(a.cr + idx, a.val + idx, cw, xv);
+    pk_ld8(a.cr + idx, a.val + idx, cw, xv, decltype(keep)::value ? a.pol_keep : a.pol_release);
   };
 
   // ---- DOT(i): tile i's block partials of the row dots, published (YM), descriptor -> ring
@@ -335,7 +337,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
           done &= (unsigned)(wv[b] >> 32) == tag;
         }
         if (done) break;
-        __nanosleep(64);
+        if (a.nap) __nanosleep(a.nap);
       }
       if (a.trace) twait += clock64() - c0w;
       float p0 = 0.f, p1 = 0.f;
@@ -904,6 +906,17 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.part = p->part;
   k.spill = p->spill;
   k.trace = nullptr;
+  {  // measurement knobs: FP_PK_POL="keep,release" (0 none, 1 evict_last, 2 evict_first), FP_PK_NAP=ns
+    const char* e = std::getenv("FP_PK_POL");
+    k.pol_keep = 1;
+    k.pol_release = 2;
+    if (e && std::strlen(e) >= 3) {
+      k.pol_keep = e[0] - '0';
+      k.pol_release = e[2] - '0';
+    }
+    const char* n = std::getenv("FP_PK_NAP");
+    k.nap = n ? std::atoi(n) : 64;
+  }
   if (std::getenv("FP_PK_TRACE")) {  // measurement: per-warp timing of the pass (kept in the plan)
     if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 64);
     k.trace = p->trace;
