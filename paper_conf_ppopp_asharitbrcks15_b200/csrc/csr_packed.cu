@@ -915,7 +915,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
       k.pol_release = e[2] - '0';
     }
     const char* n = std::getenv("FP_PK_NAP");
-    k.nap = n ? std::atoi(n) : 64;
+    k.nap = n ? std::atoi(n) : 0;
   }
   if (std::getenv("FP_PK_TRACE")) {  // measurement: per-warp timing of the pass (kept in the plan)
     if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 64);
