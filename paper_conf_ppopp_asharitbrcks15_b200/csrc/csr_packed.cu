@@ -78,13 +78,12 @@ struct PkArgs {
   const unsigned* epoch;         // call counter (advanced by k_pk_finalize)
   double* part;                  // [groups][n]
   double* spill;                 // [cs][bw + 1], all-zero between calls
-  int pol_keep, pol_release;     // L2 hints of the dot's read / the scatter's re-read (pk_ld8)
   int nap;                       // ns a warp sleeps between polls of the exchange (0: spin)
   unsigned long long* trace;     // FP_PK_TRACE: per warp (start, end of the pass, tiles, prologue end)
 };
 
-// 8 consecutive entries (32 bytes).  POL: 0 = no L2 hint, 1 = evict_last (the dot's read keeps
-// the segment for the scatter's re-read), 2 = evict_first (the re-read releases it)
+// 8 consecutive entries (32 bytes).  KEEP: the dot's read asks L2 to keep the segment
+// (evict_last) for the scatter's re-read, which releases it (evict_first)
 #define PK_LD8(Q)                                                                                      \
   asm("ld.global.nc.L1::no_allocate" Q ".v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                      \
       : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])  \
@@ -92,13 +91,12 @@ struct PkArgs {
   asm("ld.global.nc.L1::no_allocate" Q ".v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                      \
       : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])  \
       : "l"(pv))
-__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t (&c)[8], float (&x)[8], int pol) {
-  if (pol == 1) {
+template <bool KEEP>
+__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t (&c)[8], float (&x)[8]) {
+  if constexpr (KEEP) {
     PK_LD8(".L2::evict_last");
-  } else if (pol == 2) {
-    PK_LD8(".L2::evict_first");
   } else {
-    PK_LD8("");
+    PK_LD8(".L2::evict_first");
   }
 }
 #undef PK_LD8
@@ -156,9 +154,9 @@ __device__ __forceinline__ unsigned pk_push_sign(unsigned acc, unsigned x) { ret
 // own work.  Padding entries (column = the block's zero / dummy slot, row 63, value 0) fill the
 // segments to 8 entries and the lanes beyond a segment load a padding block: no per-entry
 // predicates.
-template <int CS, int YM>
+template <int CS, int YM, int DD>
 __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
-  constexpr int D = (CS > 1 && YM != 0) ? 2 : 0;
+  constexpr int D = (CS > 1 && YM != 0) ? DD : 0;
   constexpr int NS = PkSlots<D>::NS;
   static_assert(kPkRing >= D + 1, "descriptor ring");
   extern __shared__ __align__(16) unsigned char pk_smem[];
@@ -173,12 +171,14 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   const int bw = a.bw;
   const int64_t c0 = (int64_t)k * bw;
   const int bwk = (int)max((int64_t)0, min((int64_t)bw, a.n - c0));  // columns of this block
-  // [y: bw + 1 floats, y[bw] = 0 (padding entries)][acc: bw + 1 ints, acc[bw] = dummy]
+  // [y: bw + 1 floats, y[bw] = 0 (padding entries)][acc: bw + 1 + 32 ints: acc[bw] = the padding
+  // entries' dummy, acc[bw + 1 + l] = lane l's dummy when it is beyond the segment (the
+  // padding block: 32 lanes on one word would serialise the atomic 32 ways)]
   const int ystride = YM ? (bw + 4) & ~3 : 0;
   float* y_s = reinterpret_cast<float*>(pk_smem);
   int* acc = reinterpret_cast<int*>(pk_smem) + ystride;
-  for (int j = threadIdx.x; j <= bw; j += kPkBS) {
-    if (YM) y_s[j] = j < bwk ? a.y[c0 + j] : 0.f;
+  for (int j = threadIdx.x; j <= bw + 32; j += kPkBS) {
+    if (YM && j <= bw) y_s[j] = j < bwk ? a.y[c0 + j] : 0.f;
     acc[j] = 0;
   }
   if (threadIdx.x == 0) s_tmax = 0u;
@@ -206,7 +206,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   auto ld_step = [&](const uint4& T, int s0, auto keep, uint32_t (&cw)[8], float (&xv)[8]) {
     const int o = s0 + 8 * lane;
     const int64_t idx = o < seg_len(T) ? (int64_t)T.x * 8 + o : padidx;
-    pk_ld8(a.cr + idx, a.val + idx, cw, xv, decltype(keep)::value ? a.pol_keep : a.pol_release);
+    pk_ld8<decltype(keep)::value>(a.cr + idx, a.val + idx, cw, xv);
   };
 
   // ---- DOT(i): tile i's block partials of the row dots, published (YM), descriptor -> ring
@@ -382,6 +382,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
         uint32_t cw[8];
         float xv[8];
         ld_step(T, s0, std::false_type{}, cw, xv);
+        const unsigned abase = acc_base + (s0 + 8 * lane < len ? 0u : 4u * (lane + 1));  // lane's dummy
         unsigned rare = 0;
 #pragma unroll
         for (int e = 0; e < 8; ++e) {
@@ -392,7 +393,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
             if (big) qi = 0;
             rare = (rare << 1) | (unsigned)big;
           }
-          const int old = pk_atom_add(acc_base + (cw[e] & kPkOffMask), qi);  // native ATOMS.ADD
+          const int old = pk_atom_add(abase + (cw[e] & kPkOffMask), qi);  // native ATOMS.ADD
           const unsigned nw = (unsigned)old + (unsigned)qi;
           const unsigned ovf = ((unsigned)old ^ nw) & ((unsigned)qi ^ nw);  // sign bit: int32 wrap
           if constexpr (decltype(SAFE)::value) rare = pk_push_sign(rare, ovf);
@@ -695,16 +696,25 @@ __global__ void k_pk_partition(int64_t ntiles, int nq, const int64_t* __restrict
   wtile[qi] = (int32_t)(qi == nq ? ntiles : lo);
 }
 
-template <int CS, int YM>
+template <int CS, int YM, int DD>
 const void* pk_kernel() {
-  return (const void*)k_pk<CS, YM>;
+  return (const void*)k_pk<CS, YM, DD>;
+}
+// pipeline depth D of the exchange (FP_PK_D = 1 or 2; measurement)
+int pk_depth() {
+  static const int d = [] {
+    const char* e = std::getenv("FP_PK_D");
+    return e && std::atoi(e) == 2 ? 2 : 1;
+  }();
+  return d;
 }
 const void* pk_pick(int cs, bool has_y) {
+  const bool d2 = pk_depth() == 2;
   switch (cs) {
-    case 1: return has_y ? pk_kernel<1, 1>() : pk_kernel<1, 0>();
-    case 2: return has_y ? pk_kernel<2, 1>() : pk_kernel<2, 0>();
-    case 4: return has_y ? pk_kernel<4, 1>() : pk_kernel<4, 0>();
-    case 8: return has_y ? pk_kernel<8, 1>() : pk_kernel<8, 0>();
+    case 1: return has_y ? pk_kernel<1, 1, 1>() : pk_kernel<1, 0, 1>();
+    case 2: return has_y ? (d2 ? pk_kernel<2, 1, 2>() : pk_kernel<2, 1, 1>()) : pk_kernel<2, 0, 1>();
+    case 4: return has_y ? (d2 ? pk_kernel<4, 1, 2>() : pk_kernel<4, 1, 1>()) : pk_kernel<4, 0, 1>();
+    case 8: return has_y ? (d2 ? pk_kernel<8, 1, 2>() : pk_kernel<8, 1, 1>()) : pk_kernel<8, 0, 1>();
   }
   return nullptr;
 }
@@ -722,7 +732,7 @@ int pk_headroom() {
 // columns one CTA holds (y fp32 + int32 partial in the opt-in shared memory)
 int packed_max_bw() {
   const size_t room = device_info(current_device()).smem_optin_per_block - kPkStatic;
-  return (int)std::min<size_t>(room / 8 - 4, (kPkOffMask >> 2) - 1);  // + the zero / dummy slot
+  return (int)std::min<size_t>(room / 8 - 40, (kPkOffMask >> 2) - 1);  // + the zero / dummy slots
 }
 
 int packed_cs(int64_t n) {
@@ -906,14 +916,8 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.part = p->part;
   k.spill = p->spill;
   k.trace = nullptr;
-  {  // measurement knobs: FP_PK_POL="keep,release" (0 none, 1 evict_last, 2 evict_first), FP_PK_NAP=ns
-    const char* e = std::getenv("FP_PK_POL");
-    k.pol_keep = 1;
-    k.pol_release = 2;
-    if (e && std::strlen(e) >= 3) {
-      k.pol_keep = e[0] - '0';
-      k.pol_release = e[2] - '0';
-    }
+  {  // measurement knob: FP_PK_NAP = ns a warp sleeps between polls (0: spin, the default;
+     // 64 ns left some warp-quads 2x behind on C4: 13.4 vs 7.9 ms)
     const char* n = std::getenv("FP_PK_NAP");
     k.nap = n ? std::atoi(n) : 0;
   }
@@ -921,7 +925,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 64);
     k.trace = p->trace;
   }
-  const size_t smem = ((has_y ? (size_t)((p->bw + 4) & ~3) : 0) + (size_t)p->bw + 1) * 4;
+  const size_t smem = ((has_y ? (size_t)((p->bw + 4) & ~3) : 0) + (size_t)p->bw + 33) * 4;
   void* args[] = {&k};
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(p->groups * p->cs);
@@ -950,7 +954,7 @@ void packed_launch(const Packed* p, fp_launch* L) {
   L->bs = kPkBS;
   L->grid = p->groups * p->cs;
   L->cluster = p->cs;
-  L->smem_bytes = ((p->bw + 4) & ~3) * 4 + (p->bw + 1) * 4;
+  L->smem_bytes = ((p->bw + 4) & ~3) * 4 + (p->bw + 33) * 4;
   L->blocks_per_sm = 1;
   cudaFuncAttributes fa{};
   if (cudaFuncGetAttributes(&fa, pk_pick(p->cs, true)) == cudaSuccess) L->regs_per_thread = fa.numRegs;
