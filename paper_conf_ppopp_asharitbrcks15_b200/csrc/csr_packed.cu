@@ -43,18 +43,22 @@ namespace fp {
 
 namespace {
 
-constexpr int kPkBS = 512;            // 16 warps: 128 registers per thread for two tiles in registers
+constexpr int kPkBS = 1024;
 constexpr int kPkNW = kPkBS / 32;
 constexpr int kPkRows = 64;           // rows per tile (at most)
-constexpr int kPkE = 16;              // entries per lane of a window
-constexpr int kPkWin = 32 * kPkE;     // 512 entries: a block segment held in registers
-constexpr int kPkLong = kPkWin;       // a block segment longer than this makes its row a tile of its own
+constexpr int kPkLong = 1024;         // a block segment longer than this makes its row a tile of its own
 constexpr int kPkRowCost = 4;         // work of a row in entries (warp partition)
-constexpr int kPkStatic = 13 * 1024;  // static shared memory reserve of k_pk
+constexpr int kPkStatic = 27 * 1024;  // static shared memory reserve of k_pk
+constexpr int kPkRing = 4;            // tile descriptors a warp keeps between DOT and SCATTER (>= D + 1)
 constexpr unsigned kPkOffMask = 0x3FFFFu;  // entry word: byte offset of the column in the block (18 bits)
 constexpr int kPkRidShift = 26;            //             | row in tile << 26 (rid * 4 = word >> 24)
 constexpr float kPkCap = 2147483520.f;     // 2^31 - 128: |term / quantum| below this is an exact-range int32
                                            // (one int32 wrap at most per add: detected, carried)
+
+template <int D>
+struct PkSlots {
+  static constexpr int NS = 2 * D + 2;  // exchange slots per warp: a slot is rewritten only after
+};                                      // every CTA of the group consumed its tile
 
 struct PkArgs {
   int64_t n;
@@ -88,7 +92,7 @@ struct PkArgs {
       : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])  \
       : "l"(pv))
 template <bool KEEP>
-__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t* c, float* x) {
+__device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint32_t (&c)[8], float (&x)[8]) {
   if constexpr (KEEP) {
     PK_LD8(".L2::evict_last");
   } else {
@@ -137,29 +141,31 @@ __device__ __forceinline__ void pk_prefetch_l2(const void* p) {
 __device__ __forceinline__ unsigned pk_push_sign(unsigned acc, unsigned x) { return __funnelshift_l(x, acc, 1); }
 
 // The pass.  Warp `warp` of CTA k (block k) in group g walks the tile list of warp-quad
-// (g, warp) -- the same list in every CTA of the group -- as a two-stage pipeline; at step j:
-//   DOT(j+1): load tile j+1's block segment into registers (lane l: entries 16l..16l+15, four
-//             32-byte loads; X is read from HBM once), Eq. (2) products y[col] x, segmented
-//             sums by row -> the block partials of the row dots, published as one tagged word
-//             per row (CTA 0 also publishes v of the rows);
-//   Q(j):     wait for the CS (+ v) words of rows `lane` and `lane + 32` of tile j, sum them in
-//             block order (identical in every CTA), q = alpha v p;
-//   SCAT(j):  every term x q of tile j, from the registers that hold it (a7), into the
-//             block's fixed-point partial.
-// The exchange latency of tile j hides behind DOT(j+1).  A block segment longer than the
-// 512-entry register window (a single long row) is streamed by the dot and re-read by the
-// scatter (L2 evict_last / evict_first).  Padding entries (column = the block's zero / dummy
-// slot, row 63, value 0) fill segments to 8 entries; a half-window beyond the segment loads a
-// padding block: no per-entry predicates.
+// (g, warp) -- the same list in every CTA of the group -- as a pipeline:
+//   DOT(i):  stream tile i's segment (256 entries per step, lane l holding entries 8l..8l+7
+//            from two 32-byte loads), Eq. (2) products y[col] x, segmented sums by row ->
+//            the block partials of the row dots, published as one tagged word per row (CTA 0
+//            also publishes v of the rows);
+//   Q(j):    j = i - D: wait for the CS (+ v) words of rows `lane` and `lane + 32` of tile j,
+//            sum them in block order (identical in every CTA), q = alpha v p;
+//   SCAT(j): stream tile j's segment again (read D tiles ago: an L2 hit) and add every
+//            term x q into the block's fixed-point partial.
+// The dot runs D tiles ahead of the scatter, so the exchange latency hides behind the warp's
+// own work.  Padding entries (column = the block's zero / dummy slot, row 63, value 0) fill the
+// segments to 8 entries and the lanes beyond a segment load a padding block: no per-entry
+// predicates.
 template <int CS, int YM>
 __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
-  constexpr bool XCH = CS > 1 && YM != 0;
-  constexpr int NS = 4;  // exchange slots per warp: >= 2 D + 2 with D = 1
+  // pipeline depth: measured on C4, D = 1 6.22 ms, D = 2 7.05 ms (the segments of 3 tiles per warp
+  // in flight between dot and scatter overflow L2: the re-reads miss), D = 0 13.5 ms (exchange latency)
+  constexpr int D = (CS > 1 && YM != 0) ? 1 : 0;
+  constexpr int NS = PkSlots<D>::NS;
+  static_assert(kPkRing >= D + 1, "descriptor ring");
   extern __shared__ __align__(16) unsigned char pk_smem[];
   __shared__ float rs[kPkNW][kPkRows];   // the tile's block partials of the row dots (by row in tile)
   __shared__ float qsm[kPkNW][kPkRows];  // q / quantum of the tile's rows
   __shared__ float qus[kPkNW][kPkRows];  // q of the tile's rows (spill path, first rounds)
-  __shared__ uint4 ring[kPkNW][2];       // descriptors of tiles j, j + 1
+  __shared__ uint4 ring[kPkNW][kPkRing]; // descriptors of the tiles between DOT and SCATTER
   __shared__ unsigned s_tmax;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int k = CS == 1 ? 0 : (int)(blockIdx.x % CS);
@@ -183,7 +189,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   const unsigned rs_base = fpd::smem_u32(&rs[warp][0]), qs_base = fpd::smem_u32(&qsm[warp][0]),
                  qu_base = fpd::smem_u32(&qus[warp][0]);
 
-  unsigned long long tr0 = 0, tr1 = 0, twait = 0, nrare = 0, nsafe = 0, tdot = 0;
+  unsigned long long tr0 = 0, tr1 = 0;
   if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr0));
   const int gq = g * kPkNW + warp;
   const int64_t t0 = a.wtile[gq];
@@ -198,69 +204,24 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
 
   auto seg_len = [](const uint4& T) { return (int)(T.y & 0x1FFFFFFu); };
   auto seg_rows = [](const uint4& T) { return (int)(T.y >> 25); };
-  // the lane's 16 entries of window s0 (a half beyond the segment loads the padding block)
-  auto ld_win = [&](const uint4& T, int s0, auto keep, uint32_t (&cw)[kPkE], float (&xv)[kPkE]) {
-    const int len = seg_len(T), o = s0 + kPkE * lane;
-    const int64_t b = (int64_t)T.x * 8 + o;
-    const int64_t i0 = o < len ? b : padidx, i1 = o + 8 < len ? b + 8 : padidx;
-    pk_ld8<decltype(keep)::value>(a.cr + i0, a.val + i0, cw, xv);
-    pk_ld8<decltype(keep)::value>(a.cr + i1, a.val + i1, cw + 8, xv + 8);
+  // the lane's 8 entries of step s0 (the padding block beyond the segment)
+  auto ld_step = [&](const uint4& T, int s0, auto keep, uint32_t (&cw)[8], float (&xv)[8]) {
+    const int o = s0 + 8 * lane;
+    const int64_t idx = o < seg_len(T) ? (int64_t)T.x * 8 + o : padidx;
+    pk_ld8<decltype(keep)::value>(a.cr + idx, a.val + idx, cw, xv);
   };
 
-  // one window of the dot: in-lane segmented sums, the rows inside the lane stored, the lane's
-  // leading / trailing runs joined across lanes (a shuffle scan bounded by the next row start)
-  auto dot_win = [&](const uint32_t (&cw)[kPkE], const float (&xv)[kPkE], int& carry) {
-    float c[kPkE];
-#pragma unroll
-    for (int e = 0; e < kPkE; ++e) {
-      const float pr = xv[e] * pk_lds(ys_base + (cw[e] & kPkOffMask));
-      c[e] = (e == 0 || (cw[e] >> 24) != (cw[e - 1] >> 24)) ? pr : c[e - 1] + pr;
-    }
-    const int last = (int)(cw[kPkE - 1] >> 24);
-    int prev = __shfl_up_sync(0xffffffffu, last, 1);
-    if (lane == 0) prev = carry;
-    const bool h0 = (int)(cw[0] >> 24) != prev;
-    bool seen = h0;
-#pragma unroll
-    for (int e = 0; e < kPkE - 1; ++e) {  // rows that start and end inside the lane
-      const bool h = (cw[e + 1] >> 24) != (cw[e] >> 24);
-      if (h && seen) pk_sts(rs_base + (cw[e] >> 24), c[e]);
-      seen |= h;
-    }
-    // P = the entries before the lane's first row start (continuing a row from before)
-    float P = c[kPkE - 1];
-#pragma unroll
-    for (int e = kPkE - 1; e >= 1; --e)
-      if ((cw[e] >> 24) != (cw[e - 1] >> 24)) P = c[e - 1];
-    if (h0) P = 0.f;
-    const unsigned H = __ballot_sync(0xffffffffu, seen);
-    const unsigned hl = H >> lane;
-    const int dist = hl ? __ffs(hl) : 32 - lane;
-    float r = P;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const float t2 = __shfl_down_sync(0xffffffffu, r, d);
-      if (d < dist) r += t2;
-    }
-    float rn = __shfl_down_sync(0xffffffffu, r, 1);
-    if (lane == 31) rn = 0.f;
-    if (seen) pk_sts(rs_base + last, c[kPkE - 1] + rn);                                   // the lane's last row
-    if (lane == 0 && !h0 && prev >= 0) pk_sts(rs_base + prev, pk_lds_v(rs_base + prev) + r);  // running in
-    carry = __shfl_sync(0xffffffffu, last, 31);
-    __syncwarp();
-  };
-
-  // ---- DOT(i): tile i's segment into (cw, xv) (or streamed when longer than the window), its
-  // block partials of the row dots published (XCH) or returned in p0/p1/v0/v1; descriptor -> ring
+  // ---- DOT(i): tile i's block partials of the row dots, published (YM), descriptor -> ring
   uint4 cd = make_uint4(0, 0, 0, 0);  // lane l: descriptor of tile (i & ~31) + l
-  auto dot = [&](int i, uint32_t (&cw)[kPkE], float (&xv)[kPkE], float& p0, float& p1, float& v0, float& v1) {
+  float pown0 = 0.f, pown1 = 0.f, vown0 = 0.f, vown1 = 0.f;  // D == 0: partials / v of rows lane, lane + 32
+  auto dot = [&](int i) {
     if ((i & 31) == 0 && i + lane < nt) cd = __ldg(desc + i + lane);
     uint4 T;
     T.x = __shfl_sync(0xffffffffu, cd.x, i & 31);
     T.y = __shfl_sync(0xffffffffu, cd.y, i & 31);
     T.z = __shfl_sync(0xffffffffu, cd.z, i & 31);
     T.w = __shfl_sync(0xffffffffu, cd.w, i & 31);
-    if (lane == 0) ring[warp][i & 1] = T;
+    if (lane == 0) ring[warp][i % kPkRing] = T;
     // the next tile's segment on its way into L2 (lanes 0-15: 128-byte lines of cr, 16-31: val)
     {
       const int i1 = i + 1;
@@ -274,11 +235,9 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
       }
     }
     __syncwarp();
-    const int len = seg_len(T);
-    if (len <= kPkWin) ld_win(T, 0, std::false_type{}, cw, xv);  // read once (L2 evict_first)
     if constexpr (YM == 0) return;
-    const int nr = seg_rows(T);
-    v0 = v1 = 0.f;
+    const int nr = seg_rows(T), len = seg_len(T);
+    float v0 = 0.f, v1 = 0.f;
     if (CS == 1 || k == 0) {
       const float* vp = a.v + (int)T.z;
       if (lane < nr) v0 = a.v ? __ldg(vp + lane) : 1.f;
@@ -287,20 +246,55 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     pk_sts(rs_base + 4 * lane, 0.f);
     pk_sts(rs_base + 128 + 4 * lane, 0.f);
     __syncwarp();
-    int carry = -4;  // rid * 4 of the previous window's last entry
-    if (len <= kPkWin) {
-      if (len > 0) dot_win(cw, xv, carry);
-    } else {
-      for (int s0 = 0; s0 < len; s0 += kPkWin) {
-        uint32_t c2[kPkE];
-        float x2[kPkE];
-        ld_win(T, s0, std::true_type{}, c2, x2);  // kept in L2 for the scatter's re-read
-        dot_win(c2, x2, carry);
+    int carry = -4;  // rid * 4 of the previous step's last entry
+    for (int s0 = 0; s0 < len; s0 += 256) {
+      uint32_t cw[8];
+      float xv[8];
+      ld_step(T, s0, std::true_type{}, cw, xv);
+      int r4[8];
+      float c[8];  // in-lane inclusive segmented sums of the Eq. (2) products
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        r4[e] = (int)(cw[e] >> 24);
+        const float pr = xv[e] * pk_lds(ys_base + (cw[e] & kPkOffMask));
+        c[e] = (e == 0 || r4[e] != r4[e - 1]) ? pr : c[e - 1] + pr;
       }
+      int prev = __shfl_up_sync(0xffffffffu, r4[7], 1);
+      if (lane == 0) prev = carry;
+      const bool h0 = r4[0] != prev;
+      bool seen = h0;
+      // rows that start and end inside the lane
+#pragma unroll
+      for (int e = 0; e < 7; ++e) {
+        const bool h = r4[e + 1] != r4[e];
+        if (h && seen) pk_sts(rs_base + r4[e], c[e]);
+        seen |= h;
+      }
+      // P = the entries before the lane's first row start (continuing a row from before)
+      float P = c[7];
+#pragma unroll
+      for (int e = 7; e >= 1; --e)
+        if (r4[e] != r4[e - 1]) P = c[e - 1];
+      if (h0) P = 0.f;
+      // across lanes: R_l = P_l + ... + P_h, h = the first lane >= l holding a row start
+      const unsigned H = __ballot_sync(0xffffffffu, seen);
+      const unsigned hl = H >> lane;
+      const int dist = hl ? __ffs(hl) : 32 - lane;
+      float r = P;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const float t2 = __shfl_down_sync(0xffffffffu, r, d);
+        if (d < dist) r += t2;
+      }
+      float rn = __shfl_down_sync(0xffffffffu, r, 1);
+      if (lane == 31) rn = 0.f;
+      if (seen) pk_sts(rs_base + r4[7], c[7] + rn);                                  // the lane's last row
+      if (lane == 0 && !h0 && prev >= 0) pk_sts(rs_base + prev, pk_lds_v(rs_base + prev) + r);  // running in
+      carry = __shfl_sync(0xffffffffu, r4[7], 31);
+      __syncwarp();
     }
-    p0 = pk_lds_v(rs_base + 4 * lane);
-    p1 = pk_lds_v(rs_base + 128 + 4 * lane);
-    if constexpr (XCH) {
+    const float p0 = pk_lds_v(rs_base + 4 * lane), p1 = pk_lds_v(rs_base + 128 + 4 * lane);
+    if constexpr (CS > 1) {
       const unsigned long long tg = (unsigned long long)(tag0 + (unsigned)i) << 32;
       unsigned long long* slot = xslot + (int64_t)(i % NS) * SW + lane;
       st_relaxed_gpu(slot + k * kPkRows, tg | __float_as_uint(p0));
@@ -309,11 +303,16 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
         st_relaxed_gpu(slot + CS * kPkRows, tg | __float_as_uint(v0));
         st_relaxed_gpu(slot + CS * kPkRows + 32, tg | __float_as_uint(v1));
       }
+    } else {
+      pown0 = p0;
+      pown1 = p1;
+      vown0 = v0;
+      vown1 = v1;
     }
   };
 
   // ---- Q(j): q of rows lane and lane + 32 of tile j (descriptor T) -> qus
-  auto qcalc = [&](const uint4& T, int j, float p0, float p1, float v0, float v1) {
+  auto qcalc = [&](const uint4& T, int j) {
     const int nr = seg_rows(T);
     float q0, q1;
     if constexpr (YM == 0) {
@@ -321,17 +320,15 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
       const float* vp = a.v + (int)T.z;
       q0 = lane < nr ? alpha * (a.v ? __ldg(vp + lane) : 1.f) : 0.f;
       q1 = lane + 32 < nr ? alpha * (a.v ? __ldg(vp + lane + 32) : 1.f) : 0.f;
-    } else if constexpr (!XCH) {
+    } else if constexpr (CS == 1) {
       (void)j;
-      q0 = alpha * (v0 * p0);
-      q1 = alpha * (v1 * p1);
+      q0 = alpha * (vown0 * pown0);
+      q1 = alpha * (vown1 * pown1);
     } else {
       // the exchange: value + tag in one 64-bit word, so no flag and no fence is needed
       const unsigned tag = tag0 + (unsigned)j;
       const unsigned long long* slot = xslot + (int64_t)(j % NS) * SW + lane;
       unsigned long long wv[2 * (CS + 1)];
-      unsigned long long c0w = 0;
-      if (a.trace) c0w = clock64();
       for (;;) {
         bool done = true;
 #pragma unroll
@@ -342,15 +339,14 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
         if (done) break;
         if (a.nap) __nanosleep(a.nap);
       }
-      if (a.trace) twait += clock64() - c0w;
-      float s0 = 0.f, s1 = 0.f;
+      float p0 = 0.f, p1 = 0.f;
 #pragma unroll
       for (int b = 0; b < CS; ++b) {  // block order: identical in every CTA
-        s0 += __uint_as_float((unsigned)wv[2 * b]);
-        s1 += __uint_as_float((unsigned)wv[2 * b + 1]);
+        p0 += __uint_as_float((unsigned)wv[2 * b]);
+        p1 += __uint_as_float((unsigned)wv[2 * b + 1]);
       }
-      q0 = alpha * (__uint_as_float((unsigned)wv[2 * CS]) * s0);
-      q1 = alpha * (__uint_as_float((unsigned)wv[2 * CS + 1]) * s1);
+      q0 = alpha * (__uint_as_float((unsigned)wv[2 * CS]) * p0);
+      q1 = alpha * (__uint_as_float((unsigned)wv[2 * CS + 1]) * p1);
     }
     if (lane >= nr) q0 = 0.f;
     if (lane + 32 >= nr) q1 = 0.f;
@@ -367,47 +363,10 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   };
   set_scale(0);
 
-  // one window of the scatter.  SAFE (every |x q| of the tile below the int32 range, from the
-  // plan's max |x| of the tile): no per-entry checks; else terms beyond it and non-finite terms
-  // are flagged too.  Flagged entries (and int32 wraps) spill after the window.
-  auto scat_win = [&](const uint32_t (&cw)[kPkE], const float (&xv)[kPkE], int s0, int len, auto SAFE) {
-    const int o = s0 + kPkE * lane;
-    const unsigned ab0 = acc_base + (o < len ? 0u : 4u * (lane + 1));  // lane's dummy beyond the segment
-    const unsigned ab1 = acc_base + (o + 8 < len ? 0u : 4u * (lane + 1));
-    unsigned rare = 0;
-#pragma unroll
-    for (int e = 0; e < kPkE; ++e) {
-      const float ts = xv[e] * pk_lds(qs_base + (cw[e] >> 24));
-      int qi = __float2int_rn(ts);
-      if constexpr (!decltype(SAFE)::value) {
-        const bool big = !(fabsf(ts) < kPkCap);  // beyond the int32 range, or NaN
-        if (big) qi = 0;
-        rare = (rare << 1) | (unsigned)big;
-      }
-      const int old = pk_atom_add((e < 8 ? ab0 : ab1) + (cw[e] & kPkOffMask), qi);  // native ATOMS.ADD
-      const unsigned nw = (unsigned)old + (unsigned)qi;
-      const unsigned ovf = ((unsigned)old ^ nw) & ((unsigned)qi ^ nw);  // sign bit: int32 wrap
-      if constexpr (decltype(SAFE)::value) rare = pk_push_sign(rare, ovf);
-      else rare |= ovf >> 31;
-    }
-    if (a.trace && rare) nrare += __popc(rare);
-    if (rare) {  // bit (kPkE - 1 - e) flags entry e
-#pragma unroll
-      for (int e = 0; e < kPkE; ++e) {
-        if ((rare >> (kPkE - 1 - e)) & 1u) {
-          const float ts = xv[e] * pk_lds_v(qs_base + (cw[e] >> 24));
-          const int col = (int)((cw[e] & kPkOffMask) >> 2);
-          if (!(fabsf(ts) < kPkCap))  // beyond the int32 range / Inf / NaN (IEEE propagation, reading R8)
-            atomicAdd(spill + col, (double)(xv[e] * pk_lds_v(qu_base + (cw[e] >> 24))));
-          else  // the int32 sum wrapped: carry 2^32 quanta
-            atomicAdd(spill + col, ts > 0.f ? 4294967296.0 * quantum : -4294967296.0 * quantum);
-        }
-      }
-    }
-  };
-
-  // ---- SCAT(j): Eq. (3) from the registers (or the segment re-read, long rows)
-  auto scatter = [&](const uint4& T, const uint32_t (&cw)[kPkE], const float (&xv)[kPkE]) {
+  // ---- SCAT(j): Eq. (3) from the segment, re-read.  SAFE (every |x q| of the tile below the
+  // cap, from the plan's max |x| of the tile): no per-entry checks; else terms beyond the cap
+  // and non-finite terms are flagged too.  Flagged entries (and int32 wraps) spill after.
+  auto scatter = [&](const uint4& T) {
     __syncwarp();
     const float q0 = pk_lds_v(qu_base + 4 * lane), q1 = pk_lds_v(qu_base + 128 + 4 * lane);
     const float qs0 = q0 * sc, qs1 = q1 * sc;
@@ -415,70 +374,80 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     pk_sts(qs_base + 128 + 4 * lane, qs1);
     const float xm = __uint_as_float(T.w);
     const bool safe = __all_sync(0xffffffffu, fabsf(qs0) * xm < 2.0e9f && fabsf(qs1) * xm < 2.0e9f);
-    if (a.trace) nsafe += safe ? 1 : 0;
     __syncwarp();
     const int len = seg_len(T);
-    if (len <= kPkWin) {
-      if (len > 0) {
-        if (safe) scat_win(cw, xv, 0, len, std::true_type{});
-        else scat_win(cw, xv, 0, len, std::false_type{});
+    auto run = [&](auto SAFE) {
+      for (int s0 = 0; s0 < len; s0 += 256) {
+        uint32_t cw[8];
+        float xv[8];
+        ld_step(T, s0, std::false_type{}, cw, xv);
+        const unsigned abase = acc_base + (s0 + 8 * lane < len ? 0u : 4u * (lane + 1));  // lane's dummy
+        unsigned rare = 0;
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          const float ts = xv[e] * pk_lds(qs_base + (cw[e] >> 24));
+          int qi = __float2int_rn(ts);
+          if constexpr (!decltype(SAFE)::value) {
+            const bool big = !(fabsf(ts) < kPkCap);  // beyond the int32 range, or NaN
+            if (big) qi = 0;
+            rare = (rare << 1) | (unsigned)big;
+          }
+          const int old = pk_atom_add(abase + (cw[e] & kPkOffMask), qi);  // native ATOMS.ADD
+          const unsigned nw = (unsigned)old + (unsigned)qi;
+          const unsigned ovf = ((unsigned)old ^ nw) & ((unsigned)qi ^ nw);  // sign bit: int32 wrap
+          if constexpr (decltype(SAFE)::value) rare = pk_push_sign(rare, ovf);
+          else rare |= ovf >> 31;
+        }
+        if (rare) {  // rare: bit 7 - e flags entry e
+#pragma unroll
+          for (int e = 0; e < 8; ++e) {
+            if ((rare >> (7 - e)) & 1u) {
+              const float ts = xv[e] * pk_lds_v(qs_base + (cw[e] >> 24));
+              const int col = (int)((cw[e] & kPkOffMask) >> 2);
+              if (!(fabsf(ts) < kPkCap))  // beyond the cap / Inf / NaN (IEEE propagation, reading R8)
+                atomicAdd(spill + col, (double)(xv[e] * pk_lds_v(qu_base + (cw[e] >> 24))));
+              else  // the int32 sum wrapped: carry 2^32 quanta
+                atomicAdd(spill + col, ts > 0.f ? 4294967296.0 * quantum : -4294967296.0 * quantum);
+            }
+          }
+        }
       }
-    } else {
-      for (int s0 = 0; s0 < len; s0 += kPkWin) {
-        uint32_t c2[kPkE];
-        float x2[kPkE];
-        ld_win(T, s0, std::false_type{}, c2, x2);
-        if (safe) scat_win(c2, x2, s0, len, std::true_type{});
-        else scat_win(c2, x2, s0, len, std::false_type{});
-      }
-    }
+    };
+    if (safe) run(std::true_type{});
+    else run(std::false_type{});
   };
 
   // largest finite |x q| of a tile (the first rounds only)
-  auto tmax_of = [&](const uint4& T, const uint32_t (&cw)[kPkE], const float (&xv)[kPkE]) -> float {
+  auto tmax_of = [&](const uint4& T) -> float {
     __syncwarp();
     float tm = 0.f;
-    const int len = seg_len(T);
-    for (int s0 = 0; s0 < len; s0 += kPkWin) {
-      uint32_t c2[kPkE];
-      float x2[kPkE];
-      if (len > kPkWin) ld_win(T, s0, std::true_type{}, c2, x2);
+    for (int s0 = 0; s0 < seg_len(T); s0 += 256) {
+      uint32_t cw[8];
+      float xv[8];
+      ld_step(T, s0, std::true_type{}, cw, xv);
 #pragma unroll
-      for (int e = 0; e < kPkE; ++e) {
-        const uint32_t w = len > kPkWin ? c2[e] : cw[e];
-        const float x = len > kPkWin ? x2[e] : xv[e];
-        const float t = fabsf(x * pk_lds_v(qu_base + (w >> 24)));
+      for (int e = 0; e < 8; ++e) {
+        const float t = fabsf(xv[e] * pk_lds_v(qu_base + (cw[e] >> 24)));
         if (t <= 3.402823466e38f) tm = fmaxf(tm, t);
       }
     }
     return tm;
   };
 
-  // Registers: the current tile (C) and the next (N); the dot's row partials / v likewise.
-  uint32_t cwC[kPkE], cwN[kPkE];
-  float xvC[kPkE], xvN[kPkE];
-  float pC0 = 0.f, pC1 = 0.f, vC0 = 0.f, vC1 = 0.f, pN0 = 0.f, pN1 = 0.f, vN0 = 0.f, vN1 = 0.f;
-#pragma unroll
-  for (int e = 0; e < kPkE; ++e) cwC[e] = cwN[e] = 0u, xvC[e] = xvN[e] = 0.f;
-  auto rotate = [&]() {
-#pragma unroll
-    for (int e = 0; e < kPkE; ++e) cwC[e] = cwN[e], xvC[e] = xvN[e];
-    pC0 = pN0, pC1 = pN1, vC0 = vN0, vC1 = vN1;
-  };
-
-  // ---- tile 0's dot, then rounds of one scatter per warp until the CTA's cap is set (all
-  // warps take part in every round: the loop condition is CTA-uniform)
-  if (nt > 0) dot(0, cwC, xvC, pC0, pC1, vC0, vC1);
+  // ---- the dots of the first D tiles, then rounds of one scatter per warp until the CTA's
+  // cap is set (all warps take part in every round: the loop condition is CTA-uniform)
+  for (int i = 0; i < D; ++i)
+    if (i < nt) dot(i);
   int j = 0;
   for (;;) {
     const bool have = j < nt;
     uint4 T = make_uint4(0, 0, 0, 0);
     float tm = 0.f;
     if (have) {
-      if (j + 1 < nt) dot(j + 1, cwN, xvN, pN0, pN1, vN0, vN1);
-      T = ring[warp][j & 1];
-      qcalc(T, j, pC0, pC1, vC0, vC1);
-      tm = tmax_of(T, cwC, xvC);
+      if (j + D < nt) dot(j + D);
+      T = ring[warp][j % kPkRing];
+      qcalc(T, j);
+      tm = tmax_of(T);
     }
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) tm = fmaxf(tm, __shfl_xor_sync(0xffffffffu, tm, d));
@@ -492,8 +461,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     }
     // (while every finite term so far is 0, the provisional scale adds zeros; non-finite terms spill)
     if (have) {
-      scatter(T, cwC, xvC);
-      rotate();
+      scatter(T);
       ++j;
     }
     if (mx > 0.f || !any) break;
@@ -502,14 +470,10 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr1));
   // ---- steady state
   for (; j < nt; ++j) {
-    unsigned long long cd0 = 0;
-    if (a.trace) cd0 = clock64();
-    if (j + 1 < nt) dot(j + 1, cwN, xvN, pN0, pN1, vN0, vN1);
-    if (a.trace) tdot += clock64() - cd0;
-    const uint4 T = ring[warp][j & 1];
-    qcalc(T, j, pC0, pC1, vC0, vC1);
-    scatter(T, cwC, xvC);
-    rotate();
+    if (j + D < nt) dot(j + D);
+    const uint4 T = ring[warp][j % kPkRing];
+    qcalc(T, j);
+    scatter(T);
   }
   if (a.trace && lane == 0) {
     unsigned long long tr2;
@@ -519,10 +483,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     tp[1] = tr2;
     tp[2] = (unsigned long long)nt;
     tp[3] = tr1;
-    tp[4] = twait;
-    tp[5] = nrare;
-    tp[6] = nsafe;
-    tp[7] = tdot;
+    tp[4] = tp[5] = tp[6] = tp[7] = 0;
   }
 
   __syncthreads();
@@ -881,7 +842,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
   k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile);
   // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
-  const int ns = cs > 1 ? 4 : 1;  // k_pk's NS
+  const int ns = cs > 1 ? PkSlots<1>::NS : 1;
   const size_t xbytes = (size_t)groups * kPkNW * ns * (cs + 1) * kPkRows * 8;
   PK_TRY(cudaMalloc((void**)&p->xch, xbytes), "alloc");
   PK_TRY(cudaMemsetAsync(p->xch, 0, xbytes, s), "memset");

@@ -217,7 +217,7 @@ fp_status fp_csr_plan_destroy(fp_csr_plan* p) {
 // clocks polling, flagged entries, tiles on the check-free path, clocks in the dots).
 extern "C" int fpx_pack_trace(const fp_csr_plan* p, unsigned long long* host, int64_t n) {
   if (!p || !p->packed || !p->packed->trace) return 0;
-  const int64_t have = (int64_t)p->packed->groups * p->packed->cs * 32 * 8;
+  const int64_t have = (int64_t)p->packed->groups * p->packed->cs * (p->packed->trace_warps) * 8;
   const int64_t k = n < have ? n : have;
   if (cudaMemcpy(host, p->packed->trace, (size_t)k * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
   return (int)k;

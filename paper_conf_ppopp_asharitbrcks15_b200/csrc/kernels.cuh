@@ -90,6 +90,7 @@ struct Packed {
   double* part = nullptr;               // [groups][n]
   double* spill = nullptr;              // [cs][bw + 1]
   unsigned long long* trace = nullptr;  // FP_PK_TRACE measurement buffer
+  int trace_warps = 32;                 // warps per CTA of the pass (trace layout)
 };
 int packed_cs(int64_t n);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,

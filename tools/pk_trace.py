@@ -30,7 +30,7 @@ start, end, tiles, pro = (t[:, 0] - t0) / 1e3, (t[:, 1] - t0) / 1e3, t[:, 2], (t
 print(f"warps {len(t)}  start us: max {start.max():.1f}  prologue end us: median {np.median(pro):.1f} max {pro.max():.1f}")
 print("end us percentiles 0/10/50/90/99/100:", np.percentile(end, [0, 10, 50, 90, 99, 100]).round(1))
 print("tiles per warp min/median/max:", tiles.min(), np.median(tiles), tiles.max())
-cta = end.reshape(-1, 32)
+cta = end.reshape(-1, 32)  # 32 warps per CTA
 print("per CTA: spread (max - min) of warp ends, median/max us:", np.median(cta.max(1) - cta.min(1)).round(1),
       (cta.max(1) - cta.min(1)).max().round(1))
 grp = end.reshape(info["groups"], -1)
@@ -44,8 +44,3 @@ print("corr(end, tiles):", np.corrcoef(end, tiles)[0, 1].round(3))
 c = end.reshape(-1, 32).mean(1)
 print("mean end by CTA (first 16):", c[:16].round(0).astype(int).tolist())
 print("by block k (cta % blocks):", [round(float(c[k::info['blocks']].mean()), 1) for k in range(info['blocks'])])
-wait_ms, rare, safe, dotms = t[:, 4] / 1.965e6, t[:, 5], t[:, 6], t[:, 7] / 1.965e6
-print("poll wait ms: median/max", np.median(wait_ms).round(2), wait_ms.max().round(2), " corr(end, wait):", np.corrcoef(end, wait_ms)[0, 1].round(3))
-print("dot ms: median/max", np.median(dotms).round(2), dotms.max().round(2), " corr(end, dot):", np.corrcoef(end, dotms)[0, 1].round(3))
-print("flagged entries: total", int(rare.sum()), " max per warp", int(rare.max()), " corr(end, flagged):", np.corrcoef(end, rare)[0, 1].round(3))
-print("check-free tiles fraction:", (safe.sum() / tiles.sum()).round(4))

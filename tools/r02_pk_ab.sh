@@ -1,10 +1,7 @@
 #!/bin/bash
-# variant 19 A/B: pipeline depth
 cd $GRAFT_REPO_ROOT
-for d in 1 2; do
-  echo "== FP_PK_D=$d"
-  FP_PK_D=$d timeout 300 python tools/pk_trace.py C4 2>/dev/null | grep -E "end us perc|poll wait|dot ms"
-  FP_PK_D=$d timeout 300 python bench.py --config C4 --steps 10 --warmup 3 --no-e2e --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print('ms', d['ms_per_step'])"
-done
-FP_PK_D=1 timeout 900 ncu --set full --clock-control none --import-source on -k k_pk -c 1 -o gpurun_out/pk_c4_full -f python bench.py --config C4 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-graph > gpurun_out/pk_ncu.log 2>&1
+mkdir -p gpurun_out
 timeout 900 python -m pytest tests/test_packed_gpu.py -q -x -p no:cacheprovider --timeout 300 2>&1 | tail -2
+timeout 300 python tools/pk_trace.py C4 2>/dev/null | grep -E "end us perc|poll wait|dot ms|flagged|check-free"
+timeout 300 python bench.py --config C4 --steps 10 --warmup 3 --no-e2e --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print('ms', d['ms_per_step'], d['roofline']['frac'])"
+timeout 900 ncu --set full --clock-control none --import-source on -k k_pk -c 1 -o gpurun_out/pk_c4_full -f python bench.py --config C4 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-graph > gpurun_out/pk_ncu.log 2>&1
