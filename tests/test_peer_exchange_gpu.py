@@ -67,6 +67,15 @@ def test_peer_dist_bitexact(cuda_dev, P, fmt, dt):
         b = fp.shard_rows_dense(m, P)
         shards = [(X[b[r]:b[r + 1]].contiguous().to(cuda_dev), v[b[r]:b[r + 1]].to(cuda_dev)) for r in range(P)]
     yd, zd = y.to(cuda_dev), z.to(cuda_dev)
+    # each shard's local-pass kernel once, serially: its first launch loads the kernel (lazy
+    # module loading synchronises the device, which would wait on another rank's spinning barrier)
+    for r in range(P):
+        if fmt == "csr":
+            lrp, lci, lva, lv = shards[r]
+            fp.csr(lrp, lci, lva, n, yd, lv, zd, 1.0, -2.0)
+        else:
+            fp.dense(shards[r][0], yd, shards[r][1], zd, 1.0, -2.0)
+    torch.cuda.synchronize()
     g = fp.LocalGroup(P, 0, max_bytes=n * 8)
     try:
         for rep in range(3):
