@@ -324,11 +324,11 @@ def run_gpu(args):
         t0 = time.perf_counter()
         cplan = None
         packed = False
-        if comm is None:
-            cplan = fp.CsrPlan(inp["rowptr"], inp["colidx"], n, inp["val"].dtype, launch=forced)
-            torch.cuda.synchronize()
+        # the rank's plan (its row shard when N > 1: fp_csr_plan_dist)
+        cplan = fp.CsrPlan(inp["rowptr"], inp["colidx"], n, inp["val"].dtype, launch=forced)
+        torch.cuda.synchronize()
         plan_ms = (time.perf_counter() - t0) * 1e3
-        if comm is None and forced is None and args.pack and cfg["dtype"] == "f32":
+        if forced is None and args.pack and cfg["dtype"] == "f32":
             # the column-blocked copy (fp_csr_plan_pack, variant 19): once per matrix, timed here
             t0 = time.perf_counter()
             try:
@@ -345,15 +345,9 @@ def run_gpu(args):
             if comm is None:
                 cplan(None if packed else inp["val"], inp["y"], inp["v"], inp["z"], alpha, beta, w=inp["w"])
             else:
-                fp.csr_dist(comm, inp["rowptr"], inp["colidx"], inp["val"], n, inp["y"], inp["v"], inp["z"], alpha,
-                            beta, w=inp["w"])
-        if cplan is not None:
-            plan = cplan.launch
-        else:
-            st = fp.fp_row_stats()
-            st.m, st.n, st.nnz = inp["m_local"], n, inp["nnz_local"]
-            st.mean = st.nnz / max(1, st.m)
-            plan = fp.choose(True, st, fp.FP_F64 if cfg["dtype"] == "f64" else fp.FP_F32, local)
+                cplan.dist(comm, None if packed else inp["val"], inp["y"], inp["v"], inp["z"], alpha, beta,
+                           w=inp["w"])
+        plan = cplan.launch
         passes_per_step = 1
         # the L2 variants write beta*z (k_scale_z) before the main kernel and, when w is
         # replicated over L2 (csr.cu l2_replicas: 8 copies while they take <= 16 MB), fold the

@@ -88,6 +88,7 @@ _SIGS = {
     "fp_csr_plan_launch": (_int, [_vp, _P(fp_launch)]),
     "fp_csr_plan_destroy": (_int, [_vp]),
     "fp_csr_plan_pack": (_int, [_vp, _vp, _vp]),
+    "fp_csr_plan_dist": (_int, [_vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _vp]),
     "fp_csr_plan_pack_info": (_int, [_vp, _P(_i64), _P(_i64), _P(_int), _P(_int)]),
     "fp_dense_host": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_csr_host": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
@@ -297,6 +298,19 @@ class CsrPlan:
         _vec(w, self.n, self.dtype, "w")
         _call("fp_csr_plan_exec", self._h, _ptr(val), _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta), _ptr(w),
               _stream(dev, stream))
+        return w
+
+    def dist(self, comm, val, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
+        """fp_csr_plan_dist: this plan is the rank's row shard; every rank gets the full w
+        (``val=None``: the packed copy)."""
+        _require_cuda(val, y, v, z, w)
+        dev = val.device if val is not None else self.rowptr.device
+        y, v, z = _vec(y, self.n, self.dtype, "y"), _vec(v, self.m, self.dtype, "v"), _vec(z, self.n, self.dtype, "z")
+        if w is None:
+            w = torch.empty(self.n, dtype=self.dtype, device=dev)
+        _vec(w, self.n, self.dtype, "w")
+        _call("fp_csr_plan_dist", self._h, comm.handle, _ptr(val), _ptr(y), _ptr(v), _ptr(z), float(alpha), float(beta),
+              _ptr(w), _stream(dev, stream))
         return w
 
     def close(self):

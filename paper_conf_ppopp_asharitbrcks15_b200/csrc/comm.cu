@@ -90,6 +90,22 @@ namespace {
 fp_status peer_begin(fp_comm* c, size_t bytes, cudaStream_t s, void** D);
 fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double beta, void* w, cudaStream_t s);
 
+// Peer-mode pattern with a CSR plan (fp_csr_plan_dist): as dist_peer, the local pass on the plan
+fp_status dist_peer_plan(fp::PatternArgs a, const fp_csr_plan* plan, fp_comm* comm, cudaStream_t s) {
+  if (a.n == 0) return FP_OK;
+  void* D = nullptr;
+  fp_status st = peer_begin(comm, (size_t)a.n * fp::dtype_size(a.dtype), s, &D);
+  if (st != FP_OK) return st;
+  void* w = a.w;
+  const void* z = a.z;
+  const double beta = a.beta;
+  a.w = D;
+  a.add_beta_z = false;
+  st = fp::plan_run(plan, a, s);
+  if (st != FP_OK) return st;
+  return peer_finish(comm, a.n, a.dtype, beta != 0.0 ? z : nullptr, beta, w, s);
+}
+
 // Peer-mode pattern: the local pass writes this rank's partial alpha X_r^T(v_r (.) X_r y)
 // straight into its symmetric D buffer (no beta z), then the exchange sums the ranks' D in
 // rank order and adds beta z once: every rank ends with the same bits.
@@ -707,6 +723,22 @@ fp_status fp_csr_dist(int64_t m_local, int64_t n, int64_t nnz_local, const int64
   fp_status st = fp::run_csr(a, nullptr, (cudaStream_t)stream);
   if (st != FP_OK) return st;
   return fp_allreduce(comm, w, n, dtype, stream);
+}
+
+fp_status fp_csr_plan_dist(const fp_csr_plan* plan, fp_comm* comm, const void* val, const void* y, const void* v,
+                           const void* z, double alpha, double beta, void* w, fp_stream stream) {
+  FP_REQUIRE(plan && comm, FP_ERR_INVALID_ARG, "fp_csr_plan_dist: plan or comm is NULL");
+  int64_t m = 0, n = 0, nnz = 0;
+  const int64_t* rowptr = nullptr;
+  const int32_t* colidx = nullptr;
+  fp_dtype dt = FP_F32;
+  fp::plan_shape(plan, &m, &n, &nnz, &rowptr, &colidx, &dt);
+  fp::PatternArgs a = fp::csr_args(m, n, nnz, rowptr, colidx, val, y, v, z, alpha, beta, w, dt);
+  if (comm->mode != FP_COMM_NCCL) return dist_peer_plan(a, plan, comm, (cudaStream_t)stream);
+  a.add_beta_z = comm->rank == 0;
+  fp_status st = fp::plan_run(plan, a, (cudaStream_t)stream);
+  if (st != FP_OK) return st;
+  return fp_allreduce(comm, w, n, dt, stream);
 }
 
 }  // extern "C"

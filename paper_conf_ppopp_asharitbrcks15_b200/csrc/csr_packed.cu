@@ -811,7 +811,11 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   FP_REQUIRE(bw <= packed_max_bw(), FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: n = %lld too wide for %d blocks",
              (long long)n, cs);
   const DeviceInfo& di = device_info(current_device());
-  const int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
+  int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
+  if (const char* e = std::getenv("FP_PK_GROUPS")) {  // fewer CTA groups (tests: several local ranks
+    const int gg = std::atoi(e);                       // must fit the GPU at once)
+    if (gg > 0 && gg < groups) groups = gg;
+  }
   Packed* p = new (std::nothrow) Packed;
   FP_REQUIRE(p, FP_ERR_NOMEM, "fp_csr_plan_pack: out of host memory");
   p->m = m;

@@ -48,6 +48,39 @@ __global__ void k_split_offsets(int64_t m, const int64_t* __restrict__ rowptr, c
 
 }  // namespace
 
+namespace fp {
+// One evaluation on a plan's matrix: the packed copy when a.val is NULL (fp_csr_plan_pack),
+// else the unpacked plan.  a carries the call's vectors and the dist layer's flags (add_beta_z,
+// w = a rank's partial buffer).
+fp_status plan_run(const fp_csr_plan* p, PatternArgs& a, cudaStream_t s) {
+  if (!a.val && p->nnz > 0) {
+    FP_REQUIRE(p->packed, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: val is NULL and the plan is not packed");
+    FP_REQUIRE(p->n == 0 || a.w, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: w is NULL");
+    FP_REQUIRE(a.beta == 0.0 || a.z || !a.add_beta_z, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: beta != 0 needs z");
+    FP_REQUIRE(current_device() == p->device, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: plan is on device %d",
+               p->device);
+    const size_t wb = (size_t)p->n * 4;
+    FP_REQUIRE(!overlaps(a.w, wb, a.y, wb) && !overlaps(a.w, wb, a.v, (size_t)p->m * 4), FP_ERR_ALIAS,
+               "fp_csr_plan_exec: w overlaps y or v");
+    if (p->n == 0) return FP_OK;
+    if (a.alpha == 0.0 || p->m == 0)
+      return launch_scale_z(p->n, a.add_beta_z ? a.z : nullptr, a.add_beta_z ? a.beta : 0.0, a.w, p->dtype, s);
+    return packed_exec(p->packed, a, s);
+  }
+  a.split = p->soff ? &p->split : nullptr;
+  return run_csr(a, &p->L, s);
+}
+void plan_shape(const fp_csr_plan* p, int64_t* m, int64_t* n, int64_t* nnz, const int64_t** rowptr,
+                const int32_t** colidx, fp_dtype* dt) {
+  *m = p->m;
+  *n = p->n;
+  *nnz = p->nnz;
+  *rowptr = p->rowptr;
+  *colidx = p->colidx;
+  *dt = p->dtype;
+}
+}  // namespace fp
+
 extern "C" {
 
 fp_status fp_csr_plan_create(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
@@ -148,24 +181,8 @@ fp_status fp_csr_plan_create(int64_t m, int64_t n, int64_t nnz, const int64_t* r
 fp_status fp_csr_plan_exec(const fp_csr_plan* p, const void* val, const void* y, const void* v, const void* z,
                            double alpha, double beta, void* w, fp_stream stream) {
   FP_REQUIRE(p, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: plan is NULL");
-  if (!val && p->nnz > 0) {  // the packed copy (fp_csr_plan_pack)
-    FP_REQUIRE(p->packed, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: val is NULL and the plan is not packed");
-    FP_REQUIRE(p->n == 0 || w, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: w is NULL");
-    FP_REQUIRE(beta == 0.0 || z, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: beta != 0 needs z");
-    FP_REQUIRE(fp::current_device() == p->device, FP_ERR_INVALID_ARG, "fp_csr_plan_exec: plan is on device %d",
-               p->device);
-    const size_t wb = (size_t)p->n * 4;
-    FP_REQUIRE(!fp::overlaps(w, wb, y, wb) && !fp::overlaps(w, wb, v, (size_t)p->m * 4), FP_ERR_ALIAS,
-               "fp_csr_plan_exec: w overlaps y or v");
-    fp::PatternArgs a =
-        fp::csr_args(p->m, p->n, p->nnz, p->rowptr, p->colidx, nullptr, y, v, z, alpha, beta, w, p->dtype);
-    if (p->n == 0) return FP_OK;
-    if (alpha == 0.0 || p->m == 0) return fp::launch_scale_z(p->n, z, beta, w, p->dtype, (cudaStream_t)stream);
-    return fp::packed_exec(p->packed, a, (cudaStream_t)stream);
-  }
   fp::PatternArgs a = fp::csr_args(p->m, p->n, p->nnz, p->rowptr, p->colidx, val, y, v, z, alpha, beta, w, p->dtype);
-  a.split = p->soff ? &p->split : nullptr;
-  return fp::run_csr(a, &p->L, (cudaStream_t)stream);
+  return fp::plan_run(p, a, (cudaStream_t)stream);
 }
 
 fp_status fp_csr_plan_launch(const fp_csr_plan* p, fp_launch* out) {

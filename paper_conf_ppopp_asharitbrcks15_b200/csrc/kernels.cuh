@@ -96,6 +96,13 @@ int packed_cs(int64_t n);  // column blocks (1, 2, 4, 8) for n columns, 0 if too
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                        const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s);
 fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s);
+}  // namespace fp
+struct fp_csr_plan;
+namespace fp {
+// csr_plan.cu: one evaluation on a plan's matrix (packed copy when a.val == NULL)
+fp_status plan_run(const fp_csr_plan* p, PatternArgs& a, cudaStream_t s);
+void plan_shape(const fp_csr_plan* p, int64_t* m, int64_t* n, int64_t* nnz, const int64_t** rowptr,
+                const int32_t** colidx, fp_dtype* dt);
 void packed_free(Packed* p);
 void packed_launch(const Packed* p, fp_launch* L);
 

@@ -166,6 +166,13 @@ def _worker(rank, world, port, q):
                             yy.to(dev), lv.contiguous().to(dev), zz.to(dev), 1.0, 1.0)
             torch.cuda.synchronize()
             assert_bitexact(w, full, f"csr_dist {dt} rank {rank}")
+            if dt == "f32":  # the packed plan of the shard through NCCL
+                plan = fp.CsrPlan(lrp.contiguous().to(dev), lci.contiguous().to(dev), nn, torch.float32)
+                plan.pack(lva.contiguous().to(dev))
+                w = plan.dist(comm, None, yy.to(dev), lv.contiguous().to(dev), zz.to(dev), 1.0, 1.0)
+                torch.cuda.synchronize()
+                assert_bitexact(w, full, f"packed plan dist (NCCL) rank {rank}")
+                plan.close()
             msgs.append(f"csr-int-{dt}")
 
         # ---- the same exchange over peer memory (CUDA IPC) and over NVLS multicast
@@ -191,6 +198,14 @@ def _worker(rank, world, port, q):
                     w = fp.csr_dist(cm, lrp, lci, lva, nn, yy.to(dev), lv, zz.to(dev), 1.0, 1.0)
                     torch.cuda.synchronize()
                     assert_bitexact(w, full, f"csr_dist mode {mode} rank {rank}")
+                # the packed plan of the shard (variant 19) through the same exchange
+                plan = fp.CsrPlan(lrp, lci, nn, torch.float32)
+                plan.pack(lva)
+                for _ in range(3):
+                    w = plan.dist(cm, None, yy.to(dev), lv, zz.to(dev), 1.0, 1.0)
+                    torch.cuda.synchronize()
+                    assert_bitexact(w, full, f"packed plan dist mode {mode} rank {rank}")
+                plan.close()
                 msgs.append(f"mode-{mode}")
             finally:
                 cm.close()

@@ -134,3 +134,46 @@ def test_peer_cg_matches_single_gpu(cuda_dev):
             assert float((w - w1).norm() / w1.norm()) < 1e-8
     finally:
         g.close()
+
+
+@pytest.mark.parametrize("P", [2, 4])
+@pytest.mark.parametrize("packed", [True, False])
+def test_peer_plan_dist_bitexact(cuda_dev, monkeypatch, P, packed):
+    """fp_csr_plan_dist: every rank runs its shard's plan (packed copy: variant 19, or the
+    unpacked plan) and the peer exchange; every rank bit-identical and bit-exact against the
+    full-matrix oracle on an integer twin, over three calls.  The ranks share one GPU here, so
+    the packed passes (cooperative launches) use 4 CTA groups each (FP_PK_GROUPS)."""
+    m, n = 30_011, 60_000
+    y = synth.vector(n, "f32", kind="int_small", seed=P, stream=synth.S_Y)
+    z = synth.vector(n, "f32", kind="int_small", seed=P, stream=synth.S_Z)
+    v = synth.vector(m, "f32", kind="int_pos", seed=P, stream=synth.S_V)
+    rp, ci, va = synth.csr(m, n, "f32", ("powerlaw", 2.5, 13.64), kind="int_pm12", seed=P)
+    full, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, -2.0)
+    b = fp.shard_rows_csr(rp, P)
+    shards = [tuple(t.contiguous().to(cuda_dev) for t in fp.shard_slice_csr(rp, ci, va, v, b, r)) for r in range(P)]
+    monkeypatch.setenv("FP_PK_GROUPS", "4")
+    plans = []
+    for lrp, lci, lva, lv in shards:
+        pl = fp.CsrPlan(lrp, lci, n, torch.float32)
+        if packed:
+            pl.pack(lva)
+        plans.append(pl)
+    torch.cuda.synchronize()
+    yd, zd = y.to(cuda_dev), z.to(cuda_dev)
+    for r in range(P):  # load the kernels before the ranks run concurrently
+        plans[r](None if packed else shards[r][2], yd, shards[r][3], zd, 1.0, -2.0)
+    torch.cuda.synchronize()
+    g = fp.LocalGroup(P, 0, max_bytes=n * 8)
+    try:
+        for rep in range(3):
+            def fn(r, s):
+                return plans[r].dist(g.comms[r], None if packed else shards[r][2], yd, shards[r][3], zd, 1.0, -2.0,
+                                     stream=s)
+            ws = run_ranks(P, fn)
+            torch.cuda.synchronize()
+            assert not g.timed_out()
+            for r in range(P):
+                assert torch.equal(ws[r], ws[0]), f"rank {r} differs from rank 0 (call {rep})"
+            assert_bitexact(ws[0], full, f"plan dist packed={packed} P={P} call {rep}")
+    finally:
+        g.close()
