@@ -79,6 +79,7 @@ struct PkArgs {
   double* part;                  // [groups][n]
   double* spill;                 // [cs][bw + 1], all-zero between calls
   int nap;                       // ns a warp sleeps between polls of the exchange (0: spin)
+  int pf;                        // L2 prefetch of the next tile: 0 none, 1 per-lane lines, 2 bulk (FP_PK_PF)
   unsigned long long* trace;     // FP_PK_TRACE: per warp (start, end of the pass, tiles, prologue end)
 };
 
@@ -227,10 +228,17 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
       const int i1 = i + 1;
       const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
       if ((i1 & 31) != 0 && i1 < nt) {
-        const int l = lane & 15;
-        if (32 * l < (int)min(len1 & 0x1FFFFFFu, 512u)) {
-          const int64_t e = (int64_t)off1 * 8 + 32 * l;
-          pk_prefetch_l2(lane < 16 ? (const void*)(a.cr + e) : (const void*)(a.val + e));
+        if (a.pf == 1) {
+          const int l = lane & 15;
+          if (32 * l < (int)min(len1 & 0x1FFFFFFu, 512u)) {
+            const int64_t e = (int64_t)off1 * 8 + 32 * l;
+            pk_prefetch_l2(lane < 16 ? (const void*)(a.cr + e) : (const void*)(a.val + e));
+          }
+        } else if (a.pf == 2 && lane == 0) {  // bulk prefetch (TMA unit, not the LSU pipe)
+          const int64_t e = (int64_t)off1 * 8;
+          const unsigned nb = min(len1 & 0x1FFFFFFu, 2048u) * 4u;
+          fpd::prefetch_l2(a.cr + e, nb);
+          fpd::prefetch_l2(a.val + e, nb);
         }
       }
     }
@@ -972,6 +980,8 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.trace = nullptr;
   {  // measurement knob: FP_PK_NAP = ns a warp sleeps between polls (0: spin, the default;
      // 64 ns left some warp-quads 2x behind on C4: 13.4 vs 7.9 ms)
+    const char* f = std::getenv("FP_PK_PF");
+    k.pf = f ? std::atoi(f) : 1;
     const char* n = std::getenv("FP_PK_NAP");
     k.nap = n ? std::atoi(n) : 0;
   }
