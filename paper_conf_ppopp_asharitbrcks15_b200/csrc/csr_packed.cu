@@ -981,7 +981,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   {  // measurement knob: FP_PK_NAP = ns a warp sleeps between polls (0: spin, the default;
      // 64 ns left some warp-quads 2x behind on C4: 13.4 vs 7.9 ms)
     const char* f = std::getenv("FP_PK_PF");
-    k.pf = f ? std::atoi(f) : 1;
+    k.pf = f ? std::atoi(f) : 2;  // measured on C4: none 5.71, per-lane 5.69, bulk 5.63 ms
     const char* n = std::getenv("FP_PK_NAP");
     k.nap = n ? std::atoi(n) : 0;
   }
