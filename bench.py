@@ -328,7 +328,7 @@ def run_gpu(args):
         cplan = fp.CsrPlan(inp["rowptr"], inp["colidx"], n, inp["val"].dtype, launch=forced)
         torch.cuda.synchronize()
         plan_ms = (time.perf_counter() - t0) * 1e3
-        if forced is None and args.pack and cfg["dtype"] == "f32":
+        if forced is None and args.pack:
             # the column-blocked copy (fp_csr_plan_pack, variant 19): once per matrix, timed here
             t0 = time.perf_counter()
             try:

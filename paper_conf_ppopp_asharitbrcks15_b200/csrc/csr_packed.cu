@@ -141,6 +141,453 @@ __device__ __forceinline__ void pk_prefetch_l2(const void* p) {
 // (acc << 1) | (x >> 31): collect one sign bit per entry
 __device__ __forceinline__ unsigned pk_push_sign(unsigned acc, unsigned x) { return __funnelshift_l(x, acc, 1); }
 
+// typed shared-memory accesses (the single-block pass, fp32 / fp64)
+__device__ __forceinline__ double pk_lds(unsigned addr, double) {
+  double v;
+  asm("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ float pk_lds(unsigned addr, float) { return pk_lds(addr); }
+__device__ __forceinline__ double pk_lds_v(unsigned addr, double) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ float pk_lds_v(unsigned addr, float) { return pk_lds_v(addr); }
+__device__ __forceinline__ void pk_sts(unsigned addr, double v) {
+  asm volatile("st.shared.f64 [%0], %1;" ::"r"(addr), "d"(v));
+}
+__device__ __forceinline__ unsigned pk_atom_addu(unsigned addr, unsigned v) {
+  unsigned old;
+  asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(addr), "r"(v));
+  return old;
+}
+// 8 values of a window: fp32 one 32-byte load, fp64 two
+template <bool KEEP>
+__device__ __forceinline__ void pk_ldv(const float* pv, float* x) {
+  if constexpr (KEEP)
+    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])
+        : "l"(pv));
+  else
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]), "=f"(x[7])
+        : "l"(pv));
+}
+template <bool KEEP>
+__device__ __forceinline__ void pk_ldv(const double* pv, double* x) {
+  if constexpr (KEEP) {
+    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(x[0]), "=d"(x[1]), "=d"(x[2]), "=d"(x[3]) : "l"(pv));
+    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(x[4]), "=d"(x[5]), "=d"(x[6]), "=d"(x[7]) : "l"(pv + 4));
+  } else {
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(x[0]), "=d"(x[1]), "=d"(x[2]), "=d"(x[3]) : "l"(pv));
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(x[4]), "=d"(x[5]), "=d"(x[6]), "=d"(x[7]) : "l"(pv + 4));
+  }
+}
+template <bool KEEP>
+__device__ __forceinline__ void pk_ldc(const uint32_t* pc, uint32_t* c) {
+  if constexpr (KEEP)
+    asm("ld.global.nc.L1::no_allocate.L2::evict_last.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
+        : "l"(pc));
+  else
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
+        : "l"(pc));
+}
+
+struct PkTileRes {
+  uint4 D;
+  bool one;
+};
+
+struct Pk1Args {
+  int64_t n;
+  int64_t ntiles;
+  int64_t padidx;
+  const uint4* tile_desc;        // [ntiles]
+  const int32_t* wtile;          // [ctas * 32 + 1]
+  const uint32_t* cr;
+  const void* val;               // T
+  const void* y;                 // T
+  const void* v;                 // T
+  double alpha;
+  int hbits;
+  int pf;
+  double* part;                  // [ctas][n]
+  double* spill;                 // [n + 1]
+};
+
+// The single-block pass (one column block, CS = 1: y and the whole partial w in each CTA's
+// shared memory, no exchange).  Every tile (<= 256 entries) is loaded ONCE: the dot, q and the
+// scatter all run from the registers that hold it (a7) -- X is read from HBM once.  A
+// longer segment (one long row) is streamed by the dot and re-read by the scatter.  fp32: the
+// partial w is one int32 per column (reading R25); fp64: a 64-bit fixed point in two native
+// int32 limbs, quantum 2^(E - 50) (the low limb's returned value gives the carry; a wrap of
+// the high limb carries 2^64 quanta into the spill).
+template <typename T, int YM, int BS1>
+__global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
+  constexpr int NW1 = BS1 / 32;
+  constexpr bool F64 = sizeof(T) == 8;
+  constexpr int QB = F64 ? 50 : 26;  // bits of the first round's largest term
+  extern __shared__ __align__(16) unsigned char pk_smem[];
+  __shared__ unsigned s_tmax;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int n = (int)a.n;
+  // dynamic: [rs | q / quantum | q: 3 x 32 warps x 64 rows][y: n + 1 (y[n] = 0: padding
+  // entries)][lo: n + 33][hi (fp64): n + 33] (+ a dummy word per lane)
+  T (*rs)[kPkRows] = reinterpret_cast<T (*)[kPkRows]>(pk_smem);
+  T (*qsm)[kPkRows] = rs + NW1;
+  T (*qus)[kPkRows] = rs + 2 * NW1;
+  T* y_s = reinterpret_cast<T*>(pk_smem + (size_t)3 * NW1 * kPkRows * sizeof(T));
+  const int ystride = YM ? (n + 4) & ~3 : 0;
+  unsigned* lo = reinterpret_cast<unsigned*>(reinterpret_cast<unsigned char*>(y_s) + (size_t)ystride * sizeof(T));
+  int* hi = reinterpret_cast<int*>(lo + ((n + 36) & ~3));
+  for (int j = threadIdx.x; j <= n + 32; j += BS1) {
+    if (YM && j <= n) y_s[j] = j < n ? reinterpret_cast<const T*>(a.y)[j] : T(0);
+    lo[j] = 0u;
+    if (F64) hi[j] = 0;
+  }
+  if (threadIdx.x == 0) s_tmax = 0u;
+  __syncthreads();
+  const unsigned ys_base = fpd::smem_u32(y_s), lo_base = fpd::smem_u32(lo), hi_base = fpd::smem_u32(hi);
+  const unsigned rs_base = fpd::smem_u32(&rs[warp][0]), qs_base = fpd::smem_u32(&qsm[warp][0]),
+                 qu_base = fpd::smem_u32(&qus[warp][0]);
+  constexpr int TS = (int)sizeof(T);
+  const int gq = (int)blockIdx.x * NW1 + warp;
+  const int64_t t0 = a.wtile[gq];
+  const int nt = a.wtile[gq + 1] - a.wtile[gq];
+  const uint4* __restrict__ desc = a.tile_desc + t0;
+  const T* __restrict__ val = reinterpret_cast<const T*>(a.val);
+  const T* __restrict__ vv = reinterpret_cast<const T*>(a.v);
+  const T alpha = (T)a.alpha;
+  double* const spill = a.spill;
+  const int64_t padidx = a.padidx;
+  auto seg_len = [](const uint4& D) { return (int)(D.y & 0x1FFFFFFu); };
+  auto seg_rows = [](const uint4& D) { return (int)(D.y >> 25); };
+  auto ld_step = [&](const uint4& D, int s0, auto keep, uint32_t (&cw)[8], T (&xv)[8]) {
+    const int o = s0 + 8 * lane;
+    const int64_t idx = o < seg_len(D) ? (int64_t)D.x * 8 + o : padidx;
+    pk_ldc<decltype(keep)::value>(a.cr + idx, cw);
+    pk_ldv<decltype(keep)::value>(val + idx, xv);
+  };
+  // y[col]: the entry word holds col * 4
+  auto yaddr = [&](uint32_t w) { return ys_base + (F64 ? 2u : 1u) * (w & kPkOffMask); };
+  auto qaddr = [&](unsigned base, uint32_t w) { return base + (F64 ? 2u : 1u) * (w >> 24); };
+
+  // one window of the dot into rs (as k_pk's, typed)
+  auto dot_win = [&](const uint32_t (&cw)[8], const T (&xv)[8], int& carry) {
+    T c[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) {
+      const T pr = xv[e] * pk_lds(yaddr(cw[e]), T(0));
+      c[e] = (e == 0 || (cw[e] >> 24) != (cw[e - 1] >> 24)) ? pr : c[e - 1] + pr;
+    }
+    const int last = (int)(cw[7] >> 24);
+    int prev = __shfl_up_sync(0xffffffffu, last, 1);
+    if (lane == 0) prev = carry;
+    const bool h0 = (int)(cw[0] >> 24) != prev;
+    bool seen = h0;
+#pragma unroll
+    for (int e = 0; e < 7; ++e) {
+      const bool h = (cw[e + 1] >> 24) != (cw[e] >> 24);
+      if (h && seen) pk_sts(qaddr(rs_base, cw[e]), c[e]);
+      seen |= h;
+    }
+    T P = c[7];
+#pragma unroll
+    for (int e = 7; e >= 1; --e)
+      if ((cw[e] >> 24) != (cw[e - 1] >> 24)) P = c[e - 1];
+    if (h0) P = T(0);
+    const unsigned H = __ballot_sync(0xffffffffu, seen);
+    const unsigned hl = H >> lane;
+    const int dist = hl ? __ffs(hl) : 32 - lane;
+    T r = P;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const T t2 = __shfl_down_sync(0xffffffffu, r, d);
+      if (d < dist) r += t2;
+    }
+    T rn = __shfl_down_sync(0xffffffffu, r, 1);
+    if (lane == 31) rn = T(0);
+    if (seen) pk_sts(qaddr(rs_base, cw[7]), c[7] + rn);
+    if (lane == 0 && !h0 && prev >= 0) {
+      const unsigned ad = rs_base + (F64 ? 2 : 1) * (unsigned)prev;
+      pk_sts(ad, pk_lds_v(ad, T(0)) + r);
+    }
+    carry = __shfl_sync(0xffffffffu, last, 31);
+    __syncwarp();
+  };
+
+  double sc = 1.0;     // 2^(QB - E)
+  double quantum = 0;  // 2^(E - QB)
+  auto set_scale = [&](int e) {
+    e = min(max(e, F64 ? -900 : -95), F64 ? 900 : 100);
+    sc = ldexp(1.0, QB - e);
+    quantum = ldexp(1.0, e - QB);
+  };
+  set_scale(0);
+
+  // one window of the scatter: every x q into the fixed-point partial; terms beyond the
+  // int32 / int64 range, non-finite terms and wraps spill (rare)
+  auto scat_win = [&](const uint32_t (&cw)[8], const T (&xv)[8], int s0, int len) {
+    const unsigned dm = (s0 + 8 * lane < len) ? 0u : 4u * (lane + 1);  // lane's dummy beyond the segment
+    unsigned rare = 0;
+#pragma unroll
+    for (int e = 0; e < 8; ++e) {
+      const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
+      const unsigned off = dm + (cw[e] & kPkOffMask);
+      if constexpr (!F64) {
+        const bool big = !(fabsf(ts) < kPkCap);
+        const int qi = big ? 0 : __float2int_rn(ts);
+        const int old = pk_atom_add(lo_base + off, qi);
+        const unsigned nw = (unsigned)old + (unsigned)qi;
+        rare = (rare << 1) | (unsigned)(big | ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0));
+      } else {
+        const bool big = !(fabs(ts) < 4.6e18);  // |term| < 2^62 quanta
+        const long long I = big ? 0ll : __double2ll_rn(ts);
+        const unsigned l = (unsigned)I;
+        const unsigned ol = pk_atom_addu(lo_base + off, l);
+        const int h = (int)(I >> 32) + ((ol + l < ol) ? 1 : 0);
+        bool ovf = false;
+        if (h != 0) {
+          const int oh = pk_atom_add(hi_base + off, h);
+          const unsigned nw = (unsigned)oh + (unsigned)h;
+          ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
+        }
+        rare = (rare << 1) | (unsigned)(big | ovf);
+      }
+    }
+    if (rare) {  // bit 7 - e flags entry e
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        if ((rare >> (7 - e)) & 1u) {
+          const T ts = xv[e] * pk_lds_v(qaddr(qs_base, cw[e]), T(0));
+          const int col = (int)((cw[e] & kPkOffMask) >> 2);
+          const bool big = F64 ? !(fabs((double)ts) < 4.6e18) : !(fabsf((float)ts) < kPkCap);
+          if (big)
+            atomicAdd(spill + col, (double)(xv[e] * pk_lds_v(qaddr(qu_base, cw[e]), T(0))));
+          else  // the int32 (fp32: the sum; fp64: the high limb) wrapped
+            atomicAdd(spill + col, (ts > T(0) ? 1.0 : -1.0) * (F64 ? 18446744073709551616.0 : 4294967296.0) * quantum);
+        }
+      }
+    }
+  };
+
+  // ---- per tile: dot (registers), q, scatter (registers); long segments streamed twice
+  uint4 cd = make_uint4(0, 0, 0, 0);
+  auto tile = [&](int i, bool first) {
+    if ((i & 31) == 0 && i + lane < nt) cd = __ldg(desc + i + lane);
+    uint4 D;
+    D.x = __shfl_sync(0xffffffffu, cd.x, i & 31);
+    D.y = __shfl_sync(0xffffffffu, cd.y, i & 31);
+    D.z = __shfl_sync(0xffffffffu, cd.z, i & 31);
+    D.w = __shfl_sync(0xffffffffu, cd.w, i & 31);
+    {
+      const int i1 = i + 1;
+      const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
+      if ((i1 & 31) != 0 && i1 < nt && a.pf && lane == 0) {
+        const int64_t e = (int64_t)off1 * 8;
+        const unsigned ne = min(len1 & 0x1FFFFFFu, 2048u);
+        fpd::prefetch_l2(a.cr + e, ne * 4u);
+        fpd::prefetch_l2(val + e, ne * (unsigned)TS);
+      }
+    }
+    const int len = seg_len(D), nr = seg_rows(D);
+    const T* vp = vv + (int)D.z;
+    const T v0 = lane < nr ? (vv ? __ldg(vp + lane) : T(1)) : T(0);
+    const T v1 = lane + 32 < nr ? (vv ? __ldg(vp + lane + 32) : T(1)) : T(0);
+    uint32_t cw[8];
+    T xv[8];
+    const bool one = len <= 256;
+    if (one) ld_step(D, 0, std::false_type{}, cw, xv);
+    T q0, q1;
+    if constexpr (YM != 0) {
+      pk_sts(rs_base + TS * lane, T(0));
+      pk_sts(rs_base + TS * (lane + 32), T(0));
+      __syncwarp();
+      int carry = -4;
+      if (one) {
+        if (len > 0) dot_win(cw, xv, carry);
+      } else {
+        for (int s0 = 0; s0 < len; s0 += 256) {
+          uint32_t c2[8];
+          T x2[8];
+          ld_step(D, s0, std::true_type{}, c2, x2);
+          dot_win(c2, x2, carry);
+        }
+      }
+      q0 = alpha * (v0 * pk_lds_v(rs_base + TS * lane, T(0)));
+      q1 = alpha * (v1 * pk_lds_v(rs_base + TS * (lane + 32), T(0)));
+    } else {
+      q0 = alpha * v0;
+      q1 = alpha * v1;
+    }
+    pk_sts(qu_base + TS * lane, q0);
+    pk_sts(qu_base + TS * (lane + 32), q1);
+    // the first rounds: the CTA's cap from every warp's first tile (one barrier per round)
+    if (first) {
+      __syncwarp();
+      float tm = 0.f;
+      for (int s0 = 0; s0 < len; s0 += 256) {
+        uint32_t c2[8];
+        T x2[8];
+        if (!one) ld_step(D, s0, std::true_type{}, c2, x2);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          const double t = fabs((double)((one ? xv[e] : x2[e]) * pk_lds_v(qaddr(qu_base, one ? cw[e] : c2[e]), T(0))));
+          if (t <= 1.7976931348623157e308) tm = fmaxf(tm, (float)fmin(t, 3.0e38));
+        }
+      }
+#pragma unroll
+      for (int d = 16; d > 0; d >>= 1) tm = fmaxf(tm, __shfl_xor_sync(0xffffffffu, tm, d));
+      if (lane == 0 && tm > 0.f) atomicMax(&s_tmax, __float_as_uint(tm));
+    }
+    return PkTileRes{D, one};
+  };
+
+  // The scatter half of a tile (registers when `one`)
+  auto finish = [&](const uint4& D, bool one, const uint32_t (&cw)[8], const T (&xv)[8]) {
+    __syncwarp();
+    const T s = (T)sc;
+    pk_sts(qs_base + TS * lane, pk_lds_v(qu_base + TS * lane, T(0)) * s);
+    pk_sts(qs_base + TS * (lane + 32), pk_lds_v(qu_base + TS * (lane + 32), T(0)) * s);
+    __syncwarp();
+    const int len = seg_len(D);
+    if (one) {
+      if (len > 0) scat_win(cw, xv, 0, len);
+    } else {
+      for (int s0 = 0; s0 < len; s0 += 256) {
+        uint32_t c2[8];
+        T x2[8];
+        ld_step(D, s0, std::false_type{}, c2, x2);
+        scat_win(c2, x2, s0, len);
+      }
+    }
+  };
+  (void)finish;
+
+  // Both halves share the window registers: written out per tile below.
+  int j = 0;
+  for (;;) {  // first rounds (CTA-uniform loop)
+    const bool have = j < nt;
+    uint32_t cw[8];
+    T xv[8];
+    uint4 D = make_uint4(0, 0, 0, 0);
+    bool one = true;
+    if (have) {
+      // the tile's dot (and its cap contribution); the window is reloaded for the scatter
+      const PkTileRes r = tile(j, true);
+      D = r.D;
+      one = r.one;
+    }
+    const int any = __syncthreads_or(have);
+    const float mx = __uint_as_float(*(volatile unsigned*)&s_tmax);
+    if (mx > 0.f) {
+      int e0;
+      frexpf(mx, &e0);
+      set_scale(e0 + a.hbits);
+    }
+    if (have) {
+      if (one) ld_step(D, 0, std::false_type{}, cw, xv);
+      finish(D, one, cw, xv);
+      ++j;
+    }
+    if (mx > 0.f || !any) break;
+  }
+  for (; j < nt; ++j) {
+    // steady state: one load of the tile for dot and scatter
+    if ((j & 31) == 0 && j + lane < nt) cd = __ldg(desc + j + lane);
+    uint4 D;
+    D.x = __shfl_sync(0xffffffffu, cd.x, j & 31);
+    D.y = __shfl_sync(0xffffffffu, cd.y, j & 31);
+    D.z = __shfl_sync(0xffffffffu, cd.z, j & 31);
+    D.w = __shfl_sync(0xffffffffu, cd.w, j & 31);
+    {
+      const int i1 = j + 1;
+      const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
+      if ((i1 & 31) != 0 && i1 < nt && a.pf && lane == 0) {
+        const int64_t e = (int64_t)off1 * 8;
+        const unsigned ne = min(len1 & 0x1FFFFFFu, 2048u);
+        fpd::prefetch_l2(a.cr + e, ne * 4u);
+        fpd::prefetch_l2(val + e, ne * (unsigned)TS);
+      }
+    }
+    const int len = seg_len(D), nr = seg_rows(D);
+    const T* vp = vv + (int)D.z;
+    const T v0 = lane < nr ? (vv ? __ldg(vp + lane) : T(1)) : T(0);
+    const T v1 = lane + 32 < nr ? (vv ? __ldg(vp + lane + 32) : T(1)) : T(0);
+    const bool one = len <= 256;
+    uint32_t cw[8];
+    T xv[8];
+    if (one) ld_step(D, 0, std::false_type{}, cw, xv);
+    T q0, q1;
+    if constexpr (YM != 0) {
+      pk_sts(rs_base + TS * lane, T(0));
+      pk_sts(rs_base + TS * (lane + 32), T(0));
+      __syncwarp();
+      int carry = -4;
+      if (one) {
+        if (len > 0) dot_win(cw, xv, carry);
+      } else {
+        for (int s0 = 0; s0 < len; s0 += 256) {
+          uint32_t c2[8];
+          T x2[8];
+          ld_step(D, s0, std::true_type{}, c2, x2);
+          dot_win(c2, x2, carry);
+        }
+      }
+      q0 = alpha * (v0 * pk_lds_v(rs_base + TS * lane, T(0)));
+      q1 = alpha * (v1 * pk_lds_v(rs_base + TS * (lane + 32), T(0)));
+    } else {
+      q0 = alpha * v0;
+      q1 = alpha * v1;
+    }
+    const T s = (T)sc;
+    pk_sts(qu_base + TS * lane, q0);
+    pk_sts(qu_base + TS * (lane + 32), q1);
+    pk_sts(qs_base + TS * lane, q0 * s);
+    pk_sts(qs_base + TS * (lane + 32), q1 * s);
+    __syncwarp();
+    if (one) {
+      if (len > 0) scat_win(cw, xv, 0, len);
+    } else {
+      for (int s0 = 0; s0 < len; s0 += 256) {
+        uint32_t c2[8];
+        T x2[8];
+        ld_step(D, s0, std::false_type{}, c2, x2);
+        scat_win(c2, x2, s0, len);
+      }
+    }
+  }
+
+  __syncthreads();
+  double* dst = a.part + (int64_t)blockIdx.x * a.n;
+  for (int i = threadIdx.x; i < n; i += BS1) {
+    const long long I = F64 ? (long long)(((unsigned long long)(long long)hi[i] << 32) | (unsigned long long)lo[i])
+                            : (long long)(int)lo[i];
+    dst[i] = (double)I * quantum;
+  }
+}
+
+template <typename T>
+__global__ void k_pk1_finalize(int64_t n, int ctas, const double* __restrict__ part, double* __restrict__ spill,
+                               const T* __restrict__ z, double beta, int add_beta_z, int accumulate, T* w) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+    for (int gi = 0; gi < ctas; ++gi) s += part[(int64_t)gi * n + j];  // fixed order
+    s += spill[j];
+    if (add_beta_z && beta != 0.0) s += beta * (double)z[j];
+    if (accumulate) s += (double)w[j];
+    w[j] = (T)s;
+    spill[j] = 0.0;
+  }
+}
+
 // The pass.  Warp `warp` of CTA k (block k) in group g walks the tile list of warp-quad
 // (g, warp) -- the same list in every CTA of the group -- as a pipeline:
 //   DOT(i):  stream tile i's segment (256 entries per step, lane l holding entries 8l..8l+7
@@ -533,13 +980,13 @@ __global__ void k_pk_count(int64_t m, const int64_t* __restrict__ rowptr, const 
 }
 
 // (2) tiles of each 64-row group (greedy): bit i of gmask set where a tile starts at row 64 g + i
-__device__ __forceinline__ bool pk_is_long(const uint32_t* cnt, int64_t m, int cs, int64_t r) {
+__device__ __forceinline__ bool pk_is_long(const uint32_t* cnt, int64_t m, int cs, int64_t r, int span) {
   for (int kk = 0; kk < cs; ++kk)
-    if (cnt[(int64_t)kk * m + r] > (uint32_t)kPkLong) return true;
+    if (cnt[(int64_t)kk * m + r] > (uint32_t)span) return true;
   return false;
 }
-__global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, unsigned long long* __restrict__ gmask,
-                           int64_t* __restrict__ gcount) {
+__global__ void k_pk_tiles(int64_t m, int cs, int span, const uint32_t* __restrict__ cnt,
+                           unsigned long long* __restrict__ gmask, int64_t* __restrict__ gcount) {
   const int64_t ng = (m + kPkRows - 1) / kPkRows;
   for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
     uint32_t accs[kPkMaxCS] = {};
@@ -548,14 +995,14 @@ __global__ void k_pk_tiles(int64_t m, int cs, const uint32_t* __restrict__ cnt, 
     bool fresh = true;  // the next row starts a tile
     for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
       const int64_t r = gi * kPkRows + i;
-      if (pk_is_long(cnt, m, cs, r)) {
+      if (pk_is_long(cnt, m, cs, r, span)) {
         mask |= 1ull << i;
         ++ntl;
         fresh = true;
         continue;
       }
       bool fit = !fresh;
-      for (int kk = 0; kk < cs && fit; ++kk) fit = accs[kk] + cnt[(int64_t)kk * m + r] <= (uint32_t)kPkLong;
+      for (int kk = 0; kk < cs && fit; ++kk) fit = accs[kk] + cnt[(int64_t)kk * m + r] <= (uint32_t)span;
       if (!fit) {
         mask |= 1ull << i;
         ++ntl;
@@ -618,10 +1065,11 @@ __global__ void k_pk_fill(int64_t n, uint32_t* __restrict__ p, uint32_t v) {
 // their order (stable), so non-canonical rows are packed as given (reading R7).  Entry word:
 // byte offset of the column inside its block | row inside the tile << 26.  Also the largest
 // |x| of every (tile, block) segment (+Inf if a value is not finite): the scatter's no-check test.
+template <typename V>
 __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const int64_t* __restrict__ rowptr,
-                             const int32_t* __restrict__ colidx, const float* __restrict__ val,
+                             const int32_t* __restrict__ colidx, const V* __restrict__ val,
                              const unsigned long long* __restrict__ gmask, const int64_t* __restrict__ gbase,
-                             uint4* __restrict__ desc, uint32_t* __restrict__ cr, float* __restrict__ pval) {
+                             uint4* __restrict__ desc, uint32_t* __restrict__ cr, V* __restrict__ pval) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = pk_lanemask_lt();
   const int64_t ng = (m + kPkRows - 1) / kPkRows;
@@ -657,8 +1105,8 @@ __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const in
         const int col = ok ? colidx[ii] : 0;
         const int b = col / bw;
         int64_t pos = -1;
-        const float x = ok && val ? val[ii] : 0.f;
-        const float ax = fabsf(x) <= 3.402823466e38f ? fabsf(x) : __int_as_float(0x7f800000);
+        const V x = ok && val ? val[ii] : V(0);
+        const float ax = fabs((double)x) <= 3.0e38 ? (float)fabs((double)x) : __int_as_float(0x7f800000);
         for (int kk = 0; kk < cs; ++kk) {
           const unsigned bm = __ballot_sync(0xffffffffu, ok && b == kk);
           if (ok && b == kk) {
@@ -686,10 +1134,11 @@ __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const in
 // e the entry of its current row whose bank is least used by the lanes placed so far.  On
 // C4-shaped rows this lowers the mean max bank load from 3.5 to 2.4 (tools/banksim.py).
 // A warp per (tile, block) segment; the window staged in shared memory.
+template <typename V>
 __global__ void __launch_bounds__(256) k_pk_bankopt(int64_t nseg, const uint4* __restrict__ desc,
-                                                    uint32_t* __restrict__ cr, float* __restrict__ pval) {
+                                                    uint32_t* __restrict__ cr, V* __restrict__ pval, int bmask) {
   __shared__ uint32_t sc[8][32][9];
-  __shared__ float sv[8][32][9];
+  __shared__ V sv[8][32][9];
   __shared__ int cnt[8][32];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   const int64_t nw = (int64_t)gridDim.x * 8;
@@ -721,16 +1170,16 @@ __global__ void __launch_bounds__(256) k_pk_bankopt(int64_t nseg, const uint4* _
             if (lane == l) {
               int best = e, bc = 1 << 30;
               for (int jj = e; jj < e + k; ++jj) {
-                const int c = cnt[wi][(sc[wi][lane][jj] >> 2) & 31];
+                const int c = cnt[wi][(sc[wi][lane][jj] >> 2) & bmask];
                 if (c < bc) bc = c, best = jj;
               }
               const uint32_t tw = sc[wi][lane][e];
-              const float tv = sv[wi][lane][e];
+              const V tv = sv[wi][lane][e];
               sc[wi][lane][e] = sc[wi][lane][best];
               sv[wi][lane][e] = sv[wi][lane][best];
               sc[wi][lane][best] = tw;
               sv[wi][lane][best] = tv;
-              ++cnt[wi][(sc[wi][lane][e] >> 2) & 31];
+              ++cnt[wi][(sc[wi][lane][e] >> 2) & bmask];
             }
             __syncwarp();
           }
@@ -784,15 +1233,37 @@ int pk_headroom() {
 
 }  // namespace
 
-// columns one CTA holds (y fp32 + int32 partial in the opt-in shared memory)
+// the single-block pass (cs == 1, fp32 / fp64)
+template <int BS1>
+const void* pk1_pick_bs(fp_dtype dt, bool has_y) {
+  if (dt == FP_F64) return has_y ? (const void*)k_pk1<double, 1, BS1> : (const void*)k_pk1<double, 0, BS1>;
+  return has_y ? (const void*)k_pk1<float, 1, BS1> : (const void*)k_pk1<float, 0, BS1>;
+}
+const void* pk1_pick(fp_dtype dt, bool has_y, int bs) {
+  return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y) : pk1_pick_bs<512>(dt, has_y);
+}
+size_t pk1_smem_n(int64_t n, fp_dtype dt, bool has_y, int bs) {
+  const size_t ts = dtype_size(dt);
+  const size_t ys = has_y ? (size_t)((n + 4) & ~3) * ts : 0;
+  return (size_t)3 * (bs / 32) * kPkRows * ts + ys + (size_t)((n + 36) & ~3) * 4 * (dt == FP_F64 ? 2 : 1);
+}
+// columns one CTA holds (y + the fixed-point partial in the opt-in shared memory)
 int packed_max_bw() {
   const size_t room = device_info(current_device()).smem_optin_per_block - kPkStatic;
   return (int)std::min<size_t>(room / 8 - 40, (kPkOffMask >> 2) - 1);  // + the zero / dummy slots
 }
+// the single-block pass k_pk1 (static shared memory: 3 x 32 x 64 values)
+int packed1_max_n(fp_dtype dt) {
+  const size_t stat = (size_t)3 * 16 * kPkRows * dtype_size(dt) + 1024;  // 512-thread CTAs
+  const size_t room = device_info(current_device()).smem_optin_per_block - stat;
+  return (int)std::min<size_t>(room / (dt == FP_F64 ? 16 : 8) - 48, (kPkOffMask >> 2) - 1);
+}
 
-int packed_cs(int64_t n) {
+int packed_cs(int64_t n, fp_dtype dt) {
+  if (n <= packed1_max_n(dt)) return 1;
+  if (dt == FP_F64) return 0;
   const int64_t mb = packed_max_bw();
-  for (int cs : {1, 2, 4, 8})
+  for (int cs : {2, 4, 8})
     if ((n + cs - 1) / cs <= mb) return cs;
   return 0;
 }
@@ -808,18 +1279,32 @@ void packed_free(Packed* p) {
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                        const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s) {
   *out = nullptr;
-  FP_REQUIRE(dtype == FP_F32, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: the packed variant is fp32 only");
+  FP_REQUIRE(valid_dtype(dtype), FP_ERR_INVALID_ARG, "fp_csr_plan_pack: bad dtype");
   FP_REQUIRE(val || nnz == 0, FP_ERR_INVALID_ARG, "fp_csr_plan_pack: val is NULL");
   FP_REQUIRE(m >= 1 && n >= 1, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: empty matrix");
   FP_REQUIRE(m < INT32_MAX, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: m >= 2^31");
-  const int cs = cs_force > 0 ? cs_force : packed_cs(n);
+  const int cs = cs_force > 0 ? cs_force : packed_cs(n, dtype);
   FP_REQUIRE(cs == 1 || cs == 2 || cs == 4 || cs == 8, FP_ERR_UNSUPPORTED,
-             "fp_csr_plan_pack: n = %lld needs more than 8 column blocks", (long long)n);
+             "fp_csr_plan_pack: n = %lld needs more than %s column blocks", (long long)n,
+             dtype == FP_F64 ? "one (fp64)" : "8");
+  FP_REQUIRE(dtype == FP_F32 || cs == 1, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: fp64 packs one column block only");
   const int bw = (int)((n + cs - 1) / cs);
-  FP_REQUIRE(bw <= packed_max_bw(), FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: n = %lld too wide for %d blocks",
-             (long long)n, cs);
+  FP_REQUIRE(cs == 1 ? n <= packed1_max_n(dtype) : bw <= packed_max_bw(), FP_ERR_UNSUPPORTED,
+             "fp_csr_plan_pack: n = %lld too wide for %d blocks", (long long)n, cs);
+  const size_t vs = dtype_size(dtype);
+  const int span = cs == 1 ? 256 : kPkLong;  // one block: a tile is one window (loaded once)
   const DeviceInfo& di = device_info(current_device());
   int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
+  int bs = kPkBS;
+  if (cs == 1) {  // the single-block pass: CTAs of FP_PK_BS1 (512 default) threads, as many as fit
+    const char* e = std::getenv("FP_PK_BS1");
+    bs = e && std::atoi(e) == 1024 ? 1024 : 512;
+    const void* f1 = pk1_pick(dtype, true, bs);
+    set_max_dynamic_smem(f1);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f1, bs, pk1_smem_n(n, dtype, true, bs));
+    groups = di.sm_count * std::max(1, occ);
+  }
   if (const char* e = std::getenv("FP_PK_GROUPS")) {  // fewer CTA groups (tests: several local ranks
     const int gg = std::atoi(e);                       // must fit the GPU at once)
     if (gg > 0 && gg < groups) groups = gg;
@@ -833,6 +1318,8 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   p->bw = bw;
   p->groups = groups;
   p->rowptr = rowptr;
+  p->dtype = dtype;
+  p->bs = bs;
   const int64_t ng = (m + kPkRows - 1) / kPkRows;
   uint32_t* cnt = nullptr;
   unsigned long long* gmask = nullptr;
@@ -868,7 +1355,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const int grid_r = (int)std::min<int64_t>((m + tb - 1) / tb, (int64_t)di.sm_count * 32);
   const int grid_g = (int)std::min<int64_t>((ng + tb - 1) / tb, (int64_t)di.sm_count * 32);
   k_pk_count<<<grid_r, tb, 0, s>>>(m, rowptr, colidx, cs, bw, cnt);
-  k_pk_tiles<<<grid_g, tb, 0, s>>>(m, cs, cnt, gmask, gcount);
+  k_pk_tiles<<<grid_g, tb, 0, s>>>(m, cs, span, cnt, gmask, gcount);
   size_t tb_bytes = 0;
   PK_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, gcount, gbase, ng, s), "scan");
   size_t tmp_bytes = tb_bytes;
@@ -906,18 +1393,28 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
       segs, ntiles, off, tlen, tile_row, p->tile_desc);
   const int64_t cap = total + 8;  // + the padding block the inactive lanes load
   PK_TRY(cudaMalloc((void**)&p->cr, (size_t)cap * 4), "alloc");
-  PK_TRY(cudaMalloc((void**)&p->val, (size_t)cap * 4), "alloc");
+  PK_TRY(cudaMalloc((void**)&p->val, (size_t)cap * vs), "alloc");
   // padding entries (segment tails up to the next 16-byte boundary): the block's zero / dummy
   // column, the tile's last row slot, value 0
   k_pk_fill<<<(int)std::min<int64_t>((cap + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(
       cap, p->cr, ((uint32_t)bw * 4u) | ((uint32_t)(kPkRows - 1) << kPkRidShift));
-  PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)cap * 4, s), "memset");
-  k_pk_scatter<<<(int)std::min<int64_t>((ng + 7) / 8, (int64_t)di.sm_count * 16), 256, 0, s>>>(
-      m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase, p->tile_desc, p->cr, p->val);
+  PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)cap * vs, s), "memset");
+  const int sgrid = (int)std::min<int64_t>((ng + 7) / 8, (int64_t)di.sm_count * 16);
+  if (dtype == FP_F64)
+    k_pk_scatter<double><<<sgrid, 256, 0, s>>>(m, cs, bw, ntiles, rowptr, colidx, (const double*)val, gmask, gbase,
+                                              p->tile_desc, p->cr, (double*)p->val);
+  else
+    k_pk_scatter<float><<<sgrid, 256, 0, s>>>(m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase,
+                                             p->tile_desc, p->cr, (float*)p->val);
   if (std::getenv("FP_PK_NOBANK") == nullptr)  // measurement: FP_PK_NOBANK=1 keeps the row order
-    k_pk_bankopt<<<(int)std::min<int64_t>((segs + 7) / 8, (int64_t)di.sm_count * 8), 256, 0, s>>>(segs, p->tile_desc,
-                                                                                                   p->cr, p->val);
-  const int nq = groups * kPkNW;
+  {
+    const int bgrid = (int)std::min<int64_t>((segs + 7) / 8, (int64_t)di.sm_count * 8);
+    if (dtype == FP_F64)  // 8-byte y gathers: bank pairs (col mod 16)
+      k_pk_bankopt<double><<<bgrid, 256, 0, s>>>(segs, p->tile_desc, p->cr, (double*)p->val, 15);
+    else
+      k_pk_bankopt<float><<<bgrid, 256, 0, s>>>(segs, p->tile_desc, p->cr, (float*)p->val, 31);
+  }
+  const int nq = groups * (bs / 32);
   if (ntiles >= INT32_MAX) return fail(cudaErrorInvalidValue, "too many tiles");
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
   k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile);
@@ -954,8 +1451,42 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   return FP_OK;
 }
 
+size_t pk1_smem(const Packed* p, bool has_y) { return pk1_smem_n(p->n, p->dtype, has_y, p->bs); }
+
 fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   const bool has_y = a.y != nullptr;
+  if (p->cs == 1) {
+    const void* f1 = pk1_pick(p->dtype, has_y, p->bs);
+    set_max_dynamic_smem(f1);
+    Pk1Args k{};
+    k.n = p->n;
+    k.ntiles = p->ntiles;
+    k.padidx = p->entries;
+    k.tile_desc = p->tile_desc;
+    k.wtile = p->wtile;
+    k.cr = p->cr;
+    k.val = p->val;
+    k.y = a.y;
+    k.v = a.v;
+    k.alpha = a.alpha;
+    k.hbits = pk_headroom();
+    const char* f = std::getenv("FP_PK_PF");
+    k.pf = f ? std::atoi(f) : 2;
+    k.part = p->part;
+    k.spill = p->spill;
+    void* args[] = {&k};
+    FP_CUDA(cudaLaunchKernel(f1, dim3(p->groups), dim3(p->bs), args, pk1_smem(p, has_y), s));
+    const int fb = 256;
+    const int fg = (int)std::min<int64_t>((p->n + fb - 1) / fb, 8 * (int64_t)device_info(current_device()).sm_count);
+    if (p->dtype == FP_F64)
+      k_pk1_finalize<double><<<fg, fb, 0, s>>>(p->n, p->groups, p->part, p->spill, (const double*)a.z, a.beta,
+                                               a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (double*)a.w);
+    else
+      k_pk1_finalize<float><<<fg, fb, 0, s>>>(p->n, p->groups, p->part, p->spill, (const float*)a.z, a.beta,
+                                              a.add_beta_z ? 1 : 0, a.accumulate ? 1 : 0, (float*)a.w);
+    FP_CUDA(cudaGetLastError());
+    return FP_OK;
+  }
   const void* f = pk_pick(p->cs, has_y);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr_plan_exec: no packed kernel for %d blocks", p->cs);
   set_max_dynamic_smem(f);
@@ -968,7 +1499,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   k.padidx = p->entries;
   k.wtile = p->wtile;
   k.cr = p->cr;
-  k.val = p->val;
+  k.val = (const float*)p->val;
   k.y = (const float*)a.y;
   k.v = (const float*)a.v;
   k.alpha = (float)a.alpha;
@@ -1015,13 +1546,15 @@ void packed_launch(const Packed* p, fp_launch* L) {
   L->variant = FP_VAR_CSR_PACKED;
   L->vs = 32;
   L->tl = kPkLong;
-  L->bs = kPkBS;
+  L->bs = p->bs;
   L->grid = p->groups * p->cs;
   L->cluster = p->cs;
-  L->smem_bytes = ((p->bw + 4) & ~3) * 4 + (p->bw + 33) * 4;
+  L->smem_bytes = p->cs == 1 ? (int)pk1_smem(p, true) : ((p->bw + 4) & ~3) * 4 + (p->bw + 33) * 4;
+  L->tl = p->cs == 1 ? 256 : kPkLong;
   L->blocks_per_sm = 1;
   cudaFuncAttributes fa{};
-  if (cudaFuncGetAttributes(&fa, pk_pick(p->cs, true)) == cudaSuccess) L->regs_per_thread = fa.numRegs;
+  if (cudaFuncGetAttributes(&fa, p->cs == 1 ? pk1_pick(p->dtype, true, p->bs) : pk_pick(p->cs, true)) == cudaSuccess)
+    L->regs_per_thread = fa.numRegs;
   else cudaGetLastError();
 }
 

@@ -84,7 +84,9 @@ struct Packed {
   uint4* tile_desc = nullptr;           // [cs][ntiles] (offset / 4, length, first row, rows)
   int32_t* wtile = nullptr;             // [groups * 32 + 1]
   uint32_t* cr = nullptr;               // [entries] column in block | row in tile << 16
-  float* val = nullptr;                 // [entries]
+  void* val = nullptr;                  // [entries] fp32 / fp64
+  fp_dtype dtype = FP_F32;
+  int bs = 1024;                        // threads per CTA of the pass
   unsigned long long* xch = nullptr;    // exchange slots
   unsigned* epoch = nullptr;            // call counter
   double* part = nullptr;               // [groups][n]
@@ -92,7 +94,7 @@ struct Packed {
   unsigned long long* trace = nullptr;  // FP_PK_TRACE measurement buffer
   int trace_warps = 32;                 // warps per CTA of the pass (trace layout)
 };
-int packed_cs(int64_t n);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
+int packed_cs(int64_t n, fp_dtype dt);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                        const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s);
 fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s);

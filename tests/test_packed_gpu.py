@@ -14,7 +14,8 @@ Checked here, at sizes the oracle finishes in seconds:
 * IEEE propagation of Inf/NaN terms (reading R8);
 * determinism (bit-identical reruns), re-packing with new values, CUDA-graph replays (the
   per-call exchange tag lives in device memory);
-* what it refuses (fp64, exec without values on an unpacked plan).
+* what it refuses (fp64 wider than one block, exec without values on an unpacked plan);
+* the single-block pass (k_pk1, fp32 and fp64) on C3/S3-shaped matrices.
 """
 import numpy as np
 import pytest
@@ -197,9 +198,9 @@ def test_packed_repack_unpacked_exec_alpha0(cuda_dev):
     plain = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, torch.float32)
     with pytest.raises(fp.FusedPatError):
         plain(None, y.to(cuda_dev), v.to(cuda_dev), z.to(cuda_dev), 1.0, 1.0)
-    rp64, ci64, va64 = synth.csr(500, 3000, "f64", ("uniform", 0, 20), seed=3)
-    p64 = fp.CsrPlan(rp64.to(cuda_dev), ci64.to(cuda_dev), 3000, torch.float64)
-    with pytest.raises(fp.FusedPatError):
+    rp64, ci64, va64 = synth.csr(500, 60_000, "f64", ("uniform", 0, 20), seed=3)
+    p64 = fp.CsrPlan(rp64.to(cuda_dev), ci64.to(cuda_dev), 60_000, torch.float64)
+    with pytest.raises(fp.FusedPatError):  # fp64 packs one column block only
         p64.pack(va64.to(cuda_dev))
 
 
@@ -225,3 +226,68 @@ def test_packed_graph_replay(cuda_dev):
         g.replay()
         torch.cuda.synchronize()
         assert_bitexact(w, ref, f"graph replay {i}")
+
+
+# ------------------------------------------------------------------ the single-block pass (k_pk1), fp32 and fp64
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+@pytest.mark.parametrize("lengths", [("binomial", 0.01), ("powerlaw", 2.5, 13.64), ("uniform", 0, 700)])
+def test_packed1_integer_twin_bitexact(cuda_dev, dt, lengths):
+    """One column block (small n, C3/S3 shapes): every tile loaded once, dot / q / scatter from the
+    same registers; long rows (beyond the 256-entry window) streamed twice.  fp64: the 64-bit
+    fixed point in two int32 limbs.  Integer twins bit-exact, every instance."""
+    m, n = (20_011, 1000) if lengths[0] != "uniform" else (4_001, 1000)
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rp, ci, va = synth.csr(m, n, dt, lengths, kind="int_pm12", seed=21)
+    y = synth.vector(n, dt, kind="int_small", seed=21, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="int_pos", seed=21, stream=synth.S_V)
+    z = synth.vector(n, dt, kind="int_small", seed=21, stream=synth.S_Z)
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, tdt)
+    plan.pack(va.to(cuda_dev))
+    assert plan.launch.variant == 19 and plan.launch.cluster == 1
+    for args in INSTANCES(y, v, z):
+        ref, mag = oracle.csr(m, n, rp, ci, va, *args)
+        assert mag.max() < 2**24
+        w = run(plan, cuda_dev, *args)
+        assert_bitexact(w, ref, f"packed1 {dt} {lengths} y={args[0] is not None}")
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+def test_packed1_float_parity(cuda_dev, dt):
+    """U[-1,1) data (C3 rows) plus rows scaled by 2^+-30: the north_star tolerance (1e-11 fp64,
+    2e-5 fp32); reruns bit-identical."""
+    m, n = 30_000, 1000
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rp, ci, va = synth.csr(m, n, dt, ("binomial", 0.01), seed=8)
+    y = synth.vector(n, dt, seed=8, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="pos", seed=8, stream=synth.S_V)
+    z = synth.vector(n, dt, seed=8, stream=synth.S_Z)
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, tdt)
+    plan.pack(va.to(cuda_dev))
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    w = run(plan, cuda_dev, y, v, z, 1.0, 1.0)
+    assert_parity(w, ref, mag, tdt, f"packed1 {dt}")
+    assert torch.equal(w, run(plan, cuda_dev, y, v, z, 1.0, 1.0))
+    g = torch.Generator().manual_seed(5)
+    sc = torch.pow(2.0, torch.randint(-30, 31, (m,), generator=g).to(tdt))
+    va2 = va * torch.repeat_interleave(sc, (rp[1:] - rp[:-1]))
+    plan.pack(va2.to(cuda_dev))
+    ref, mag = oracle.csr(m, n, rp, ci, va2, y, v, z, 1.0, 1.0)
+    assert_parity(run(plan, cuda_dev, y, v, z, 1.0, 1.0), ref, mag, tdt, f"packed1 {dt} dynamic range")
+
+
+def test_packed1_nonfinite_and_wide_fp64(cuda_dev):
+    """Inf / NaN propagate (reading R8); an fp64 matrix too wide for one block is refused."""
+    m, n = 3000, 800
+    rp, ci, va = synth.csr(m, n, "f64", ("binomial", 0.02), seed=9)
+    y = synth.vector(n, "f64", seed=9, stream=synth.S_Y)
+    va = va.clone()
+    va[50] = float("inf")
+    va[700] = float("nan")
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, torch.float64)
+    plan.pack(va.to(cuda_dev))
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, None, None, 1.0, 0.0)
+    assert_parity(run(plan, cuda_dev, y, None, None, 1.0, 0.0), ref, mag, torch.float64, "packed1 non-finite")
+    rp, ci, va = synth.csr(200, 40_000, "f64", ("uniform", 0, 20), seed=3)
+    p64 = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), 40_000, torch.float64)
+    with pytest.raises(fp.FusedPatError):
+        p64.pack(va.to(cuda_dev))
