@@ -1240,7 +1240,7 @@ const void* pk1_pick_bs(fp_dtype dt, bool has_y) {
   return has_y ? (const void*)k_pk1<float, 1, BS1> : (const void*)k_pk1<float, 0, BS1>;
 }
 const void* pk1_pick(fp_dtype dt, bool has_y, int bs) {
-  return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y) : pk1_pick_bs<512>(dt, has_y);
+  return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y) : (bs == 768 ? pk1_pick_bs<768>(dt, has_y) : pk1_pick_bs<512>(dt, has_y));
 }
 size_t pk1_smem_n(int64_t n, fp_dtype dt, bool has_y, int bs) {
   const size_t ts = dtype_size(dt);
@@ -1300,7 +1300,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
     // measured: S3 (fp32) 0.51 ms at 1024 threads vs 0.67 at 512; C3 (fp64) 1.00 ms at 512
     // (127 registers) vs 1.21 at 1024 (64 registers: spills)
     const char* e = std::getenv("FP_PK_BS1");
-    bs = e ? (std::atoi(e) == 1024 ? 1024 : 512) : (dtype == FP_F64 ? 512 : 1024);
+    bs = e ? (std::atoi(e) == 1024 ? 1024 : (std::atoi(e) == 768 ? 768 : 512)) : (dtype == FP_F64 ? 512 : 1024);
     const void* f1 = pk1_pick(dtype, true, bs);
     set_max_dynamic_smem(f1);
     int occ = 0;
