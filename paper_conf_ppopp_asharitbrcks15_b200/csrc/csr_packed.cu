@@ -104,6 +104,14 @@ __device__ __forceinline__ void pk_ld8(const uint32_t* pc, const float* pv, uint
 __device__ __forceinline__ void st_relaxed_gpu(unsigned long long* p, unsigned long long v) {
   asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void st_relaxed_gpu2(unsigned long long* p, unsigned long long a, unsigned long long b) {
+  asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+// two 8-byte words; each is single-copy atomic on its own (its value and tag consistent)
+__device__ __forceinline__ void ld_relaxed_gpu2(const unsigned long long* p, unsigned long long& a,
+                                                unsigned long long& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
 __device__ __forceinline__ unsigned long long ld_relaxed_gpu(const unsigned long long* p) {
   unsigned long long v;
   asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -750,14 +758,12 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     }
     const float p0 = pk_lds_v(rs_base + 4 * lane), p1 = pk_lds_v(rs_base + 128 + 4 * lane);
     if constexpr (CS > 1) {
+      // lane l's two rows (l, l + 32) side by side: one 16-byte store / load per block, each
+      // 8-byte half its own (value, tag) word
       const unsigned long long tg = (unsigned long long)(tag0 + (unsigned)i) << 32;
-      unsigned long long* slot = xslot + (int64_t)(i % NS) * SW + lane;
-      st_relaxed_gpu(slot + k * kPkRows, tg | __float_as_uint(p0));
-      st_relaxed_gpu(slot + k * kPkRows + 32, tg | __float_as_uint(p1));
-      if (k == 0) {
-        st_relaxed_gpu(slot + CS * kPkRows, tg | __float_as_uint(v0));
-        st_relaxed_gpu(slot + CS * kPkRows + 32, tg | __float_as_uint(v1));
-      }
+      unsigned long long* slot = xslot + (int64_t)(i % NS) * SW + 2 * lane;
+      st_relaxed_gpu2(slot + k * kPkRows, tg | __float_as_uint(p0), tg | __float_as_uint(p1));
+      if (k == 0) st_relaxed_gpu2(slot + CS * kPkRows, tg | __float_as_uint(v0), tg | __float_as_uint(v1));
     } else {
       pown0 = p0;
       pown1 = p1;
@@ -782,26 +788,35 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     } else {
       // the exchange: value + tag in one 64-bit word, so no flag and no fence is needed
       const unsigned tag = tag0 + (unsigned)j;
-      const unsigned long long* slot = xslot + (int64_t)(j % NS) * SW + lane;
-      unsigned long long wv[2 * (CS + 1)];
+      const unsigned long long* slot = xslot + (int64_t)(j % NS) * SW + 2 * lane;
+      unsigned wv[2 * (CS + 1)];  // the values (tags checked)
       for (;;) {
         bool done = true;
 #pragma unroll
-        for (int b = 0; b < 2 * (CS + 1); ++b) {
-          wv[b] = ld_relaxed_gpu(slot + (b >> 1) * kPkRows + (b & 1) * 32);
-          done &= (unsigned)(wv[b] >> 32) == tag;
+        for (int b = 0; b <= CS; ++b) {
+          unsigned long long w0, w1;
+          ld_relaxed_gpu2(slot + b * kPkRows, w0, w1);
+          wv[2 * b] = (unsigned)w0;
+          wv[2 * b + 1] = (unsigned)w1;
+          done &= (unsigned)(w0 >> 32) == tag && (unsigned)(w1 >> 32) == tag;
         }
         if (done) break;
-        if (a.nap) __nanosleep(a.nap);
+        if (a.nap > 0) {
+          __nanosleep(a.nap);
+        } else if (a.nap < 0) {  // a busy pause: no memory traffic, the warp stays scheduled
+          const long long c0 = clock64();
+          while (clock64() - c0 < -a.nap) {
+          }
+        }
       }
       float p0 = 0.f, p1 = 0.f;
 #pragma unroll
       for (int b = 0; b < CS; ++b) {  // block order: identical in every CTA
-        p0 += __uint_as_float((unsigned)wv[2 * b]);
-        p1 += __uint_as_float((unsigned)wv[2 * b + 1]);
+        p0 += __uint_as_float(wv[2 * b]);
+        p1 += __uint_as_float(wv[2 * b + 1]);
       }
-      q0 = alpha * (__uint_as_float((unsigned)wv[2 * CS]) * p0);
-      q1 = alpha * (__uint_as_float((unsigned)wv[2 * CS + 1]) * p1);
+      q0 = alpha * (__uint_as_float(wv[2 * CS]) * p0);
+      q1 = alpha * (__uint_as_float(wv[2 * CS + 1]) * p1);
     }
     if (lane >= nr) q0 = 0.f;
     if (lane + 32 >= nr) q1 = 0.f;
