@@ -139,17 +139,18 @@ __device__ __forceinline__ uint64_t* flags_of(unsigned char* buf, size_t cap) {
   return reinterpret_cast<uint64_t*>(buf + 2 * cap);
 }
 
-// Publish this rank's arrival (epoch) into every rank's flags[rank], then wait until every
-// rank has arrived here.  One warp; release/acquire at system scope (the flags and the D
-// buffers are read over NVLink).  Gives up after ~20 s (sets *timeout_flag) rather than hang.
-__global__ void k_peer_barrier(const PeerTab t) {
+// Publish this rank's arrival (epoch) into every rank's flags[rank], then (wait = 1) wait
+// until every rank has arrived here.  One warp; release/acquire at system scope (the flags and
+// the D buffers are read over NVLink).  Gives up after ~20 s (sets *timeout_flag) rather than
+// hang.  wait = 0: publish only (single-device local groups, see peer_finish).
+__global__ void k_peer_barrier(const PeerTab t, int wait) {
   const int lane = threadIdx.x;
   __threadfence_system();
   if (lane < t.P) {
     uint64_t* f = flags_of(t.p[lane], t.cap) + t.rank;
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(t.epoch) : "memory");
   }
-  if (lane < t.P) {
+  if (wait && lane < t.P) {
     const uint64_t* f = flags_of(t.p[t.rank], t.cap) + lane;
     uint64_t t0, now, v;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
@@ -263,8 +264,22 @@ fp_status peer_begin(fp_comm* c, size_t bytes, cudaStream_t s, void** D) {
 }
 
 // Finish call e: barrier, then w = sum_k D_k + beta z.
+//
+// Single-device local groups (lsync): the ranks' kernels share one GPU, and nothing makes
+// separate launches that wait on one another run at the same time (a spinning barrier can
+// hold resources a peer's persistent or cooperative pass needs: deadlock, or a context-switch
+// timeout).  So no kernel ever waits there for a launch that has not completed: each rank
+// publishes its flag with a non-waiting launch, synchronises its stream, meets the others on
+// the host (every rank's partial and flag are then complete), and only then launches the
+// barrier, whose wait is satisfied on its first poll.  Across GPUs (IPC / NVLS) each rank's
+// barrier kernel runs on its own device and publishes + waits in one launch.
 fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double beta, void* w, cudaStream_t s) {
-  if (c->lsync) FP_REQUIRE(c->lsync->arrive_and_wait(), FP_ERR_CUDA, "local group: ranks did not meet within 30 s");
+  if (c->lsync) {
+    k_peer_barrier<<<1, 32, 0, s>>>(peer_tab(c), 0);
+    FP_CUDA(cudaGetLastError());
+    FP_CUDA(cudaStreamSynchronize(s));
+    FP_REQUIRE(c->lsync->arrive_and_wait(), FP_ERR_CUDA, "local group: ranks did not meet within 30 s");
+  }
   if (c->nvls) {
     unsigned long long* cnt_off = (unsigned long long*)(2 * c->cap);
     k_nvls_barrier<<<1, 32, 0, s>>>((unsigned long long*)(c->mc + (size_t)cnt_off),
@@ -283,7 +298,7 @@ fp_status peer_finish(fp_comm* c, int64_t n, fp_dtype dt, const void* z, double 
     return FP_OK;
   }
   const PeerTab t = peer_tab(c);
-  k_peer_barrier<<<1, 32, 0, s>>>(t);
+  k_peer_barrier<<<1, 32, 0, s>>>(t, 1);
   FP_CUDA(cudaGetLastError());
   const int grid = (int)std::min<int64_t>((n + 255) / 256, 4 * fp::device_info(c->device).sm_count);
   if (n > 0) {
@@ -664,9 +679,11 @@ fp_status fp_comm_set_mode(fp_comm* comm, int mode) {
 int fp_comm_mode(const fp_comm* comm) { return comm ? comm->mode : -1; }
 
 // Single-process group of `nranks` communicators on ONE device whose symmetric buffers are
-// plain device allocations (no IPC, no NCCL): the peer exchange exactly as across GPUs, for
-// tests and for replicas sharing a GPU.  Ranks must be driven concurrently (one host thread or
-// one stream per rank): a rank's barrier waits for the others.
+// plain device allocations (no IPC, no NCCL): the peer exchange as across GPUs (same
+// symmetric-buffer layout, epoch flags, rank-ordered sum), for tests and for replicas sharing
+// a GPU.  Ranks must be driven concurrently from one host thread each: a rank's call returns
+// after every rank reached its exchange (host rendezvous).  No device-side wait of one rank's
+// kernel on another's launch (peer_finish).
 fp_status fp_comm_init_local_group(int nranks, int device, int64_t max_bytes, fp_comm** comms) {
   FP_REQUIRE(comms && nranks >= 1 && nranks <= kMaxPeers && max_bytes > 0, FP_ERR_INVALID_ARG,
              "fp_comm_init_local_group: bad arguments (1 <= nranks <= %d)", kMaxPeers);

@@ -5,8 +5,11 @@ partials) that run across GPUs on CUDA-IPC-mapped buffers.
 
 Row a11 / SURVEY 8(e): Eq. (1) is a sum over rows (Eq. 2/3), so X row-partitioned
 over ranks needs exactly one exchange of the n-vector partials; beta*z is added once (R18).
-Each simulated rank runs in its own host thread on its own stream (its barrier waits for the
-others).  Checked: integer twins bit-exact against the full-matrix oracle, every rank holding
+Each simulated rank runs in its own host thread on its own stream.  On one device no kernel
+waits for another rank's launch (B200_PROFILING: separate launches that spin on one another may
+never run together): each rank publishes its flag, synchronises its stream and meets the others
+on the host, and only then launches its barrier, whose flags are already set (comm.cu
+peer_finish).  Checked: integer twins bit-exact against the full-matrix oracle, every rank holding
 the identical bits, three calls in a row (both parities of the double-buffered partials),
 fp_allreduce, and the CG driver with a peer communicator against the single-GPU CG.
 """
