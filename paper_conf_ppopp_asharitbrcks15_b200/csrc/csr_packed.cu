@@ -216,7 +216,7 @@ struct PkTileRes {
 struct Pk1Args {
   int64_t n;
   int64_t ntiles;
-  int64_t padidx;
+  int ns;                        // tile slots per warp in the shared-memory ring (0: no ring)
   const uint4* tile_desc;        // [ntiles]
   const int32_t* wtile;          // [ctas * 32 + 1]
   const uint32_t* cr;
@@ -225,33 +225,70 @@ struct Pk1Args {
   const void* v;                 // T
   double alpha;
   int hbits;
-  int pf;
   double* part;                  // [ctas][n]
   double* spill;                 // [n + 1]
 };
 
+constexpr int kPk1MaxNS = 4;
+constexpr uint32_t pk1_pad_word(int n) { return ((uint32_t)n * 4u) | ((uint32_t)(kPkRows - 1) << kPkRidShift); }
+
+__device__ __forceinline__ uint4 pk_lds128(unsigned addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ uint4 pk_ldg128(const void* p) {
+  uint4 v;
+  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  return v;
+}
+// 16 bytes -> 4 fp32 / 2 fp64 values of a window
+__device__ __forceinline__ void pk_put(float* x, const uint4& u) {
+  x[0] = __uint_as_float(u.x), x[1] = __uint_as_float(u.y), x[2] = __uint_as_float(u.z), x[3] = __uint_as_float(u.w);
+}
+__device__ __forceinline__ void pk_put(double* x, const uint4& u) {
+  x[0] = __hiloint2double((int)u.y, (int)u.x), x[1] = __hiloint2double((int)u.w, (int)u.z);
+}
+
 // The single-block pass (one column block, CS = 1: y and the whole partial w in each CTA's
 // shared memory, no exchange).  Every tile (<= 256 entries) is loaded ONCE: the dot, q and the
-// scatter all run from the registers that hold it (a7) -- X is read from HBM once.  A
-// longer segment (one long row) is streamed by the dot and re-read by the scatter.  fp32: the
-// partial w is one int32 per column (reading R25); fp64: a 64-bit fixed point in two native
-// int32 limbs, quantum 2^(E - 50) (the low limb's returned value gives the carry; a wrap of
-// the high limb carries 2^64 quanta into the spill).
+// scatter all run from the registers that hold it (a7) -- X is read from HBM once.
+//
+// Staging (round 2c): each warp keeps a ring of NS tile slots in shared memory, filled by TMA
+// bulk copies (cp.async.bulk, one per array, completion on the slot's mbarrier) NS tiles ahead
+// of the tile being processed, so the HBM latency of the stream is off the warp's critical
+// path (the round-2b pass loaded every tile into registers itself: 20 % of its stall samples
+// waited on that load, ncu r02c).  The window of a tile is stored lane-interleaved (pack
+// time, k_pk_interleave): the 16-byte piece k of lane l's 8 entries at (k G + l) 16 bytes, G =
+// the tile's groups of 8 -- a warp's 16-byte shared loads then touch 8 distinct bank quads per
+// phase (conflict-free), and lane l still holds the logical entries 8l..8l+7.  A longer segment
+// (one long row) is streamed from global memory by the dot and re-read by the scatter.  fp32:
+// the partial w is one int32 per column (reading R25); fp64: a 64-bit fixed point in two
+// native int32 limbs, quantum 2^(E - 50) (the low limb's returned value gives the carry; a
+// wrap of the high limb carries 2^64 quanta into the spill).
 template <typename T, int YM, int BS1>
 __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
   constexpr int NW1 = BS1 / 32;
   constexpr bool F64 = sizeof(T) == 8;
   constexpr int QB = F64 ? 50 : 26;  // bits of the first round's largest term
-  extern __shared__ __align__(16) unsigned char pk_smem[];
+  constexpr int TS = (int)sizeof(T);
+  constexpr int SLOT_CW = 256 * 4, SLOT = 256 * (4 + TS);
+  constexpr int NV = 8 * TS / 16;    // 16-byte pieces of a lane's 8 values
+  extern __shared__ __align__(128) unsigned char pk_smem[];
   __shared__ unsigned s_tmax;
+  __shared__ uint64_t s_bar[NW1][kPk1MaxNS];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int n = (int)a.n;
-  // dynamic: [rs | q / quantum | q: 3 x 32 warps x 64 rows][y: n + 1 (y[n] = 0: padding
-  // entries)][lo: n + 33][hi (fp64): n + 33] (+ a dummy word per lane)
-  T (*rs)[kPkRows] = reinterpret_cast<T (*)[kPkRows]>(pk_smem);
+  const int NS = a.ns;
+  // dynamic: [ring: NW1 x NS slots of (cw: 256 words | val: 256 values)][descriptors: NW1 x 2
+  // batches x 16][rs | q / quantum | q: 3 x NW1 warps x 64 rows][y: n + 1 (y[n] = 0: padding
+  // entries)][lo: n + 33][hi (fp64): n + 33]
+  unsigned char* ring = pk_smem + (size_t)warp * NS * SLOT;
+  uint4* sdesc = reinterpret_cast<uint4*>(pk_smem + (size_t)NW1 * NS * SLOT) + warp * 32;
+  T (*rs)[kPkRows] = reinterpret_cast<T (*)[kPkRows]>(pk_smem + (size_t)NW1 * NS * SLOT + (size_t)NW1 * 32 * 16);
   T (*qsm)[kPkRows] = rs + NW1;
   T (*qus)[kPkRows] = rs + 2 * NW1;
-  T* y_s = reinterpret_cast<T*>(pk_smem + (size_t)3 * NW1 * kPkRows * sizeof(T));
+  T* y_s = reinterpret_cast<T*>(reinterpret_cast<unsigned char*>(rs) + (size_t)3 * NW1 * kPkRows * sizeof(T));
   const int ystride = YM ? (n + 4) & ~3 : 0;
   unsigned* lo = reinterpret_cast<unsigned*>(reinterpret_cast<unsigned char*>(y_s) + (size_t)ystride * sizeof(T));
   int* hi = reinterpret_cast<int*>(lo + ((n + 36) & ~3));
@@ -261,33 +298,96 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     if (F64) hi[j] = 0;
   }
   if (threadIdx.x == 0) s_tmax = 0u;
+  if (lane == 0) {
+    for (int s = 0; s < NS; ++s) fpd::mbar_init(&s_bar[warp][s], 1);
+    fpd::fence_mbar_init();
+  }
   __syncthreads();
   const unsigned ys_base = fpd::smem_u32(y_s), lo_base = fpd::smem_u32(lo), hi_base = fpd::smem_u32(hi);
   const unsigned rs_base = fpd::smem_u32(&rs[warp][0]), qs_base = fpd::smem_u32(&qsm[warp][0]),
-                 qu_base = fpd::smem_u32(&qus[warp][0]);
-  constexpr int TS = (int)sizeof(T);
+                 qu_base = fpd::smem_u32(&qus[warp][0]), ring_base = fpd::smem_u32(ring);
   const int gq = (int)blockIdx.x * NW1 + warp;
   const int64_t t0 = a.wtile[gq];
   const int nt = a.wtile[gq + 1] - a.wtile[gq];
   const uint4* __restrict__ desc = a.tile_desc + t0;
+  const uint32_t* __restrict__ crp = a.cr;
   const T* __restrict__ val = reinterpret_cast<const T*>(a.val);
   const T* __restrict__ vv = reinterpret_cast<const T*>(a.v);
   const T alpha = (T)a.alpha;
   double* const spill = a.spill;
-  const int64_t padidx = a.padidx;
+  const uint32_t padw = pk1_pad_word(n);
   auto seg_len = [](const uint4& D) { return (int)(D.y & 0x1FFFFFFu); };
   auto seg_rows = [](const uint4& D) { return (int)(D.y >> 25); };
-  auto ld_step = [&](const uint4& D, int s0, auto keep, uint32_t (&cw)[8], T (&xv)[8]) {
-    const int o = s0 + 8 * lane;
-    const int64_t idx = o < seg_len(D) ? (int64_t)D.x * 8 + o : padidx;
-    pk_ldc<decltype(keep)::value>(a.cr + idx, cw);
-    pk_ldv<decltype(keep)::value>(val + idx, xv);
+
+  // tile descriptors in shared memory (no registers held), batches of 16 (batch b in half b & 1),
+  // one batch ahead: batch b + 1 is requested (cp.async, zero-filled beyond the warp's tiles)
+  // when tile 16 b starts and waited for at tile 16 b + 8; tiles j .. j + NS (NS <= 8) resident
+  const unsigned sdesc_base = fpd::smem_u32(sdesc);
+  auto desc_req = [&](int b) {
+    const int i = 16 * b + (lane & 15);
+    if (lane < 16)
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(sdesc_base + 16u * ((b & 1) * 16 + lane)),
+                   "l"(desc + (i < nt ? i : 0)), "r"(i < nt ? 16u : 0u)
+                   : "memory");
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  auto desc_wait = [&]() {
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+  };
+  auto desc_of = [&](int i) { return pk_lds128(sdesc_base + 16u * (unsigned)(i & 31)); };
+  desc_req(0);
+  desc_wait();
+  // fill slot s with tile i (a tile beyond the ring's window size, or none, only arrives)
+  auto issue = [&](int i, int s) {
+    if (i >= nt) return;
+    const uint4 Di = desc_of(i);
+    if (lane == 0) {
+      const unsigned len = Di.y & 0x1FFFFFFu, len8 = (len + 7u) & ~7u;
+      const unsigned cwb = len <= 256 ? len8 * 4u : 0u;
+      uint64_t* b = &s_bar[warp][s];
+      fpd::fence_proxy_async_smem();  // this warp's reads of the slot precede the copy's writes
+      fpd::mbar_arrive_expect_tx(b, cwb + cwb / 4u * TS);
+      if (cwb) {
+        unsigned char* slot = ring + (size_t)s * SLOT;
+        const int64_t e0 = (int64_t)Di.x * 8;
+        fpd::bulk_g2s(slot, crp + e0, cwb, b);
+        fpd::bulk_g2s(slot + SLOT_CW, val + e0, cwb / 4u * TS, b);
+      }
+    }
+  };
+  // the lane's 8 entries of a window with G groups: 16-byte pieces at (k G + lane) 16 bytes
+  auto win_smem = [&](int s, int G, uint32_t (&cw)[8], T (&xv)[8]) {
+    const unsigned sb = ring_base + (unsigned)s * SLOT;
+    if (lane < G) {
+      const uint4 c0 = pk_lds128(sb + 16u * lane), c1 = pk_lds128(sb + 16u * (G + lane));
+      cw[0] = c0.x, cw[1] = c0.y, cw[2] = c0.z, cw[3] = c0.w, cw[4] = c1.x, cw[5] = c1.y, cw[6] = c1.z, cw[7] = c1.w;
+#pragma unroll
+      for (int k = 0; k < NV; ++k) pk_put(xv + k * (16 / TS), pk_lds128(sb + SLOT_CW + 16u * (k * G + lane)));
+    } else {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) cw[e] = padw, xv[e] = T(0);
+    }
+  };
+  auto win_glob = [&](const uint4& D, int s0, uint32_t (&cw)[8], T (&xv)[8]) {
+    const int len8 = (seg_len(D) + 7) & ~7;
+    const int G = min(32, (len8 - s0) >> 3);
+    const int64_t e0 = (int64_t)D.x * 8 + s0;
+    if (lane < G) {
+      const uint4 c0 = pk_ldg128(crp + e0 + 4 * lane), c1 = pk_ldg128(crp + e0 + 4 * (G + lane));
+      cw[0] = c0.x, cw[1] = c0.y, cw[2] = c0.z, cw[3] = c0.w, cw[4] = c1.x, cw[5] = c1.y, cw[6] = c1.z, cw[7] = c1.w;
+#pragma unroll
+      for (int k = 0; k < NV; ++k) pk_put(xv + k * (16 / TS), pk_ldg128(val + e0 + (16 / TS) * (k * G + lane)));
+    } else {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) cw[e] = padw, xv[e] = T(0);
+    }
   };
   // y[col]: the entry word holds col * 4
   auto yaddr = [&](uint32_t w) { return ys_base + (F64 ? 2u : 1u) * (w & kPkOffMask); };
   auto qaddr = [&](unsigned base, uint32_t w) { return base + (F64 ? 2u : 1u) * (w >> 24); };
 
-  // one window of the dot into rs (as k_pk's, typed)
+  // one window of the dot into rs: in-lane runs, then one bounded segmented scan across lanes
   auto dot_win = [&](const uint32_t (&cw)[8], const T (&xv)[8], int& carry) {
     T c[8];
 #pragma unroll
@@ -356,17 +456,16 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
         const unsigned nw = (unsigned)old + (unsigned)qi;
         rare = (rare << 1) | (unsigned)(big | ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0));
       } else {
-        const bool big = !(fabs(ts) < 4.6e18);  // |term| < 2^62 quanta
+        // |term| < 2^62 quanta: both limbs always added (no branch); the high limb's wrap is
+        // detected from its returned old value
+        const bool big = !(fabs(ts) < 4.6e18);
         const long long I = big ? 0ll : __double2ll_rn(ts);
         const unsigned l = (unsigned)I;
         const unsigned ol = pk_atom_addu(lo_base + off, l);
         const int h = (int)(I >> 32) + ((ol + l < ol) ? 1 : 0);
-        bool ovf = false;
-        if (h != 0) {
-          const int oh = pk_atom_add(hi_base + off, h);
-          const unsigned nw = (unsigned)oh + (unsigned)h;
-          ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
-        }
+        const int oh = pk_atom_add(hi_base + off, h);
+        const unsigned nw = (unsigned)oh + (unsigned)h;
+        const bool ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
         rare = (rare << 1) | (unsigned)(big | ovf);
       }
     }
@@ -386,46 +485,53 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     }
   };
 
-  // ---- per tile: dot (registers), q, scatter (registers); long segments streamed twice
-  uint4 cd = make_uint4(0, 0, 0, 0);
-  auto tile = [&](int i, bool first) {
-    if ((i & 31) == 0 && i + lane < nt) cd = __ldg(desc + i + lane);
-    uint4 D;
-    D.x = __shfl_sync(0xffffffffu, cd.x, i & 31);
-    D.y = __shfl_sync(0xffffffffu, cd.y, i & 31);
-    D.z = __shfl_sync(0xffffffffu, cd.z, i & 31);
-    D.w = __shfl_sync(0xffffffffu, cd.w, i & 31);
-    {
-      const int i1 = i + 1;
-      const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
-      if ((i1 & 31) != 0 && i1 < nt && a.pf && lane == 0) {
-        const int64_t e = (int64_t)off1 * 8;
-        const unsigned ne = min(len1 & 0x1FFFFFFu, 2048u);
-        fpd::prefetch_l2(a.cr + e, ne * 4u);
-        fpd::prefetch_l2(val + e, ne * (unsigned)TS);
-      }
+  // prologue: the first NS tiles in flight; v of tile 0 in registers
+  for (int i = 0; i < NS; ++i) issue(i, i);
+  T vn0 = T(0), vn1 = T(0);
+  auto load_v = [&](int i) {  // v of tile i's rows `lane`, `lane + 32` (one tile ahead)
+    vn0 = vn1 = T(0);
+    if (i < nt) {
+      const uint4 Di = desc_of(i);
+      const int nr = seg_rows(Di);
+      const T* vp = vv + (int)Di.z;
+      vn0 = lane < nr ? (vv ? __ldg(vp + lane) : T(1)) : T(0);
+      vn1 = lane + 32 < nr ? (vv ? __ldg(vp + lane + 32) : T(1)) : T(0);
     }
-    const int len = seg_len(D), nr = seg_rows(D);
-    const T* vp = vv + (int)D.z;
-    const T v0 = lane < nr ? (vv ? __ldg(vp + lane) : T(1)) : T(0);
-    const T v1 = lane + 32 < nr ? (vv ? __ldg(vp + lane + 32) : T(1)) : T(0);
-    uint32_t cw[8];
-    T xv[8];
-    const bool one = len <= 256;
-    if (one) ld_step(D, 0, std::false_type{}, cw, xv);
+  };
+  load_v(0);
+  int slot = 0;
+  unsigned par = 0;
+
+  // FRONT of tile j: descriptor, window (ring or global), the dot, q = alpha v p into qu;
+  // `first`: the tile's largest |term| into the CTA's cap
+  auto front = [&](int j, bool first, uint4& D, bool& one, uint32_t (&cw)[8], T (&xv)[8]) {
+    if ((j & 15) == 0) desc_req((j >> 4) + 1);
+    if ((j & 15) == 8) desc_wait();
+    D = desc_of(j);
+    const int len = seg_len(D);
+    one = NS > 0 && len <= 256;
+    const T v0 = vn0, v1 = vn1;
+    if (one) {
+      fpd::mbar_wait(&s_bar[warp][slot], par);
+      win_smem(slot, ((len + 7) & ~7) >> 3, cw, xv);
+    } else if (len <= 256) {
+      win_glob(D, 0, cw, xv);
+    }
+    load_v(j + 1);
+    const bool reg = len <= 256;  // the window is in registers (else streamed)
     T q0, q1;
     if constexpr (YM != 0) {
       pk_sts(rs_base + TS * lane, T(0));
       pk_sts(rs_base + TS * (lane + 32), T(0));
       __syncwarp();
       int carry = -4;
-      if (one) {
+      if (reg) {
         if (len > 0) dot_win(cw, xv, carry);
       } else {
         for (int s0 = 0; s0 < len; s0 += 256) {
           uint32_t c2[8];
           T x2[8];
-          ld_step(D, s0, std::true_type{}, c2, x2);
+          win_glob(D, s0, c2, x2);
           dot_win(c2, x2, carry);
         }
       }
@@ -437,17 +543,16 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     }
     pk_sts(qu_base + TS * lane, q0);
     pk_sts(qu_base + TS * (lane + 32), q1);
-    // the first rounds: the CTA's cap from every warp's first tile (one barrier per round)
-    if (first) {
+    if (first) {  // the CTA's cap from every warp's first tile (one barrier per round)
       __syncwarp();
       float tm = 0.f;
       for (int s0 = 0; s0 < len; s0 += 256) {
         uint32_t c2[8];
         T x2[8];
-        if (!one) ld_step(D, s0, std::true_type{}, c2, x2);
+        if (!reg) win_glob(D, s0, c2, x2);
 #pragma unroll
         for (int e = 0; e < 8; ++e) {
-          const double t = fabs((double)((one ? xv[e] : x2[e]) * pk_lds_v(qaddr(qu_base, one ? cw[e] : c2[e]), T(0))));
+          const double t = fabs((double)((reg ? xv[e] : x2[e]) * pk_lds_v(qaddr(qu_base, reg ? cw[e] : c2[e]), T(0))));
           if (t <= 1.7976931348623157e308) tm = fmaxf(tm, (float)fmin(t, 3.0e38));
         }
       }
@@ -455,44 +560,42 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
       for (int d = 16; d > 0; d >>= 1) tm = fmaxf(tm, __shfl_xor_sync(0xffffffffu, tm, d));
       if (lane == 0 && tm > 0.f) atomicMax(&s_tmax, __float_as_uint(tm));
     }
-    return PkTileRes{D, one};
   };
-
-  // The scatter half of a tile (registers when `one`)
-  auto finish = [&](const uint4& D, bool one, const uint32_t (&cw)[8], const T (&xv)[8]) {
+  // BACK of tile j: q / quantum, the scatter (registers, or the long segment re-streamed), then
+  // the freed slot takes tile j + NS
+  auto back = [&](int j, const uint4& D, bool one, const uint32_t (&cw)[8], const T (&xv)[8]) {
     __syncwarp();
     const T s = (T)sc;
     pk_sts(qs_base + TS * lane, pk_lds_v(qu_base + TS * lane, T(0)) * s);
     pk_sts(qs_base + TS * (lane + 32), pk_lds_v(qu_base + TS * (lane + 32), T(0)) * s);
     __syncwarp();
     const int len = seg_len(D);
-    if (one) {
+    if (len <= 256) {
       if (len > 0) scat_win(cw, xv, 0, len);
     } else {
       for (int s0 = 0; s0 < len; s0 += 256) {
         uint32_t c2[8];
         T x2[8];
-        ld_step(D, s0, std::false_type{}, c2, x2);
+        win_glob(D, s0, c2, x2);
         scat_win(c2, x2, s0, len);
       }
     }
+    if (NS > 0) {
+      __syncwarp();
+      issue(j + NS, slot);
+      if (++slot == NS) slot = 0, par ^= 1u;
+    }
+    (void)one;
   };
-  (void)finish;
 
-  // Both halves share the window registers: written out per tile below.
   int j = 0;
-  for (;;) {  // first rounds (CTA-uniform loop)
+  for (;;) {  // first rounds (CTA-uniform loop): calibrate the fixed-point scale
     const bool have = j < nt;
     uint32_t cw[8];
     T xv[8];
     uint4 D = make_uint4(0, 0, 0, 0);
-    bool one = true;
-    if (have) {
-      // the tile's dot (and its cap contribution); the window is reloaded for the scatter
-      const PkTileRes r = tile(j, true);
-      D = r.D;
-      one = r.one;
-    }
+    bool one = false;
+    if (have) front(j, true, D, one, cw, xv);
     const int any = __syncthreads_or(have);
     const float mx = __uint_as_float(*(volatile unsigned*)&s_tmax);
     if (mx > 0.f) {
@@ -501,76 +604,18 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
       set_scale(e0 + a.hbits);
     }
     if (have) {
-      if (one) ld_step(D, 0, std::false_type{}, cw, xv);
-      finish(D, one, cw, xv);
+      back(j, D, one, cw, xv);
       ++j;
     }
     if (mx > 0.f || !any) break;
   }
-  for (; j < nt; ++j) {
-    // steady state: one load of the tile for dot and scatter
-    if ((j & 31) == 0 && j + lane < nt) cd = __ldg(desc + j + lane);
-    uint4 D;
-    D.x = __shfl_sync(0xffffffffu, cd.x, j & 31);
-    D.y = __shfl_sync(0xffffffffu, cd.y, j & 31);
-    D.z = __shfl_sync(0xffffffffu, cd.z, j & 31);
-    D.w = __shfl_sync(0xffffffffu, cd.w, j & 31);
-    {
-      const int i1 = j + 1;
-      const unsigned off1 = __shfl_sync(0xffffffffu, cd.x, i1 & 31), len1 = __shfl_sync(0xffffffffu, cd.y, i1 & 31);
-      if ((i1 & 31) != 0 && i1 < nt && a.pf && lane == 0) {
-        const int64_t e = (int64_t)off1 * 8;
-        const unsigned ne = min(len1 & 0x1FFFFFFu, 2048u);
-        fpd::prefetch_l2(a.cr + e, ne * 4u);
-        fpd::prefetch_l2(val + e, ne * (unsigned)TS);
-      }
-    }
-    const int len = seg_len(D), nr = seg_rows(D);
-    const T* vp = vv + (int)D.z;
-    const T v0 = lane < nr ? (vv ? __ldg(vp + lane) : T(1)) : T(0);
-    const T v1 = lane + 32 < nr ? (vv ? __ldg(vp + lane + 32) : T(1)) : T(0);
-    const bool one = len <= 256;
+  for (; j < nt; ++j) {  // steady state
     uint32_t cw[8];
     T xv[8];
-    if (one) ld_step(D, 0, std::false_type{}, cw, xv);
-    T q0, q1;
-    if constexpr (YM != 0) {
-      pk_sts(rs_base + TS * lane, T(0));
-      pk_sts(rs_base + TS * (lane + 32), T(0));
-      __syncwarp();
-      int carry = -4;
-      if (one) {
-        if (len > 0) dot_win(cw, xv, carry);
-      } else {
-        for (int s0 = 0; s0 < len; s0 += 256) {
-          uint32_t c2[8];
-          T x2[8];
-          ld_step(D, s0, std::true_type{}, c2, x2);
-          dot_win(c2, x2, carry);
-        }
-      }
-      q0 = alpha * (v0 * pk_lds_v(rs_base + TS * lane, T(0)));
-      q1 = alpha * (v1 * pk_lds_v(rs_base + TS * (lane + 32), T(0)));
-    } else {
-      q0 = alpha * v0;
-      q1 = alpha * v1;
-    }
-    const T s = (T)sc;
-    pk_sts(qu_base + TS * lane, q0);
-    pk_sts(qu_base + TS * (lane + 32), q1);
-    pk_sts(qs_base + TS * lane, q0 * s);
-    pk_sts(qs_base + TS * (lane + 32), q1 * s);
-    __syncwarp();
-    if (one) {
-      if (len > 0) scat_win(cw, xv, 0, len);
-    } else {
-      for (int s0 = 0; s0 < len; s0 += 256) {
-        uint32_t c2[8];
-        T x2[8];
-        ld_step(D, s0, std::false_type{}, c2, x2);
-        scat_win(c2, x2, s0, len);
-      }
-    }
+    uint4 D;
+    bool one;
+    front(j, false, D, one, cw, xv);
+    back(j, D, one, cw, xv);
   }
 
   __syncthreads();
@@ -1207,6 +1252,39 @@ __global__ void __launch_bounds__(256) k_pk_bankopt(int64_t nseg, const uint4* _
   }
 }
 
+// (4c) one column block (k_pk1): every 256-entry window of a segment stored lane-interleaved --
+// the 16-byte piece k of lane l's 8 entries at (k G + l) 16 bytes, G = the window's groups of 8
+// -- so the pass's 16-byte loads of a window (shared memory after the bulk copy, or global) are
+// conflict-free / coalesced while lane l still holds the logical entries 8l..8l+7.  A warp per
+// segment, in place (every lane's loads precede the stores).
+template <typename V>
+__global__ void k_pk_interleave(int64_t nseg, const uint4* __restrict__ desc, uint32_t* __restrict__ cr,
+                                V* __restrict__ pval) {
+  constexpr int PV = 16 / (int)sizeof(V);  // values per 16-byte piece
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
+  for (int64_t sg = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5); sg < nseg; sg += nw) {
+    const uint4 D = desc[sg];
+    const int len8 = (int)(((D.y & 0x1FFFFFFu) + 7u) & ~7u);
+    const int64_t base = (int64_t)D.x * 8;
+    for (int s0 = 0; s0 < len8; s0 += 256) {
+      const int G = min(32, (len8 - s0) >> 3);
+      uint32_t c[8];
+      V x[8];
+      const int64_t b = base + s0;
+      if (lane < G)
+        for (int e = 0; e < 8; ++e) c[e] = cr[b + 8 * lane + e], x[e] = pval[b + 8 * lane + e];
+      __syncwarp();
+      if (lane < G)
+        for (int e = 0; e < 8; ++e) {
+          cr[b + 4 * ((e >> 2) * G + lane) + (e & 3)] = c[e];
+          pval[b + PV * ((e / PV) * G + lane) + e % PV] = x[e];
+        }
+      __syncwarp();
+    }
+  }
+}
+
 // (5) warp-quad partition: tile ranges of equal nonzero + row cost
 __global__ void k_pk_partition(int64_t ntiles, int nq, const int64_t* __restrict__ tile_row,
                                const int64_t* __restrict__ rowptr, int32_t* __restrict__ wtile) {
@@ -1257,10 +1335,25 @@ const void* pk1_pick_bs(fp_dtype dt, bool has_y) {
 const void* pk1_pick(fp_dtype dt, bool has_y, int bs) {
   return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y) : (bs == 768 ? pk1_pick_bs<768>(dt, has_y) : pk1_pick_bs<512>(dt, has_y));
 }
-size_t pk1_smem_n(int64_t n, fp_dtype dt, bool has_y, int bs) {
+size_t pk1_slot_bytes(fp_dtype dt) { return (size_t)256 * (4 + dtype_size(dt)); }
+size_t pk1_smem_n(int64_t n, fp_dtype dt, bool has_y, int bs, int ns) {
   const size_t ts = dtype_size(dt);
   const size_t ys = has_y ? (size_t)((n + 4) & ~3) * ts : 0;
-  return (size_t)3 * (bs / 32) * kPkRows * ts + ys + (size_t)((n + 36) & ~3) * 4 * (dt == FP_F64 ? 2 : 1);
+  return (size_t)(bs / 32) * ns * pk1_slot_bytes(dt) + (size_t)(bs / 32) * 32 * 16 + (size_t)3 * (bs / 32) * kPkRows * ts + ys +
+         (size_t)((n + 36) & ~3) * 4 * (dt == FP_F64 ? 2 : 1);
+}
+// tile slots per warp of k_pk1's shared-memory ring: fp64 as many as fit (at most kPk1MaxNS)
+// next to y, the partial w and the row arrays; fp32 none (its 32 warps hide the load latency
+// themselves, and the ring's shared-memory traffic costs more).  Measured (r02c): C3 (fp64,
+// 512 threads) 0.968 ms without the ring, 0.899 / 0.897 / 0.901 ms with 2 / 3 / 4 slots; S3
+// (fp32, 1024 threads) 0.513 ms without, 0.596 with 2-4.  FP_PK1_NS (measurement) overrides.
+int pk1_ring_ns(int64_t n, fp_dtype dt, int bs) {
+  const size_t room = device_info(current_device()).smem_optin_per_block - 2048;  // - static
+  const size_t base = pk1_smem_n(n, dt, true, bs, 0);
+  const int fit = room > base ? (int)std::min<size_t>((room - base) / ((size_t)(bs / 32) * pk1_slot_bytes(dt)), kPk1MaxNS) : 0;
+  int ns = dt == FP_F64 ? fit : 0;
+  if (const char* e = std::getenv("FP_PK1_NS")) ns = std::max(0, std::min(fit, std::atoi(e)));
+  return ns;
 }
 // columns one CTA holds (y + the fixed-point partial in the opt-in shared memory)
 int packed_max_bw() {
@@ -1269,7 +1362,9 @@ int packed_max_bw() {
 }
 // the single-block pass k_pk1 (static shared memory: 3 x 32 x 64 values)
 int packed1_max_n(fp_dtype dt) {
-  const size_t stat = (size_t)3 * 16 * kPkRows * dtype_size(dt) + 1024;  // 512-thread CTAs
+  // default CTAs (fp32 1024, fp64 512 threads): row arrays + descriptor batches + static
+  const size_t nw = dt == FP_F64 ? 16 : 32;
+  const size_t stat = (size_t)3 * nw * kPkRows * dtype_size(dt) + nw * 512 + 2048;
   const size_t room = device_info(current_device()).smem_optin_per_block - stat;
   return (int)std::min<size_t>(room / (dt == FP_F64 ? 16 : 8) - 48, (kPkOffMask >> 2) - 1);
 }
@@ -1311,6 +1406,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const DeviceInfo& di = device_info(current_device());
   int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
   int bs = kPkBS;
+  int ns1 = 0;
   if (cs == 1) {  // the single-block pass: CTAs of FP_PK_BS1 (512 default) threads, as many as fit
     // measured: S3 (fp32) 0.51 ms at 1024 threads vs 0.67 at 512; C3 (fp64) 1.00 ms at 512
     // (127 registers) vs 1.21 at 1024 (64 registers: spills)
@@ -1318,8 +1414,11 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
     bs = e ? (std::atoi(e) == 1024 ? 1024 : (std::atoi(e) == 768 ? 768 : 512)) : (dtype == FP_F64 ? 512 : 1024);
     const void* f1 = pk1_pick(dtype, true, bs);
     set_max_dynamic_smem(f1);
+    ns1 = pk1_ring_ns(n, dtype, bs);
+    FP_REQUIRE(pk1_smem_n(n, dtype, true, bs, ns1) + 2048 <= di.smem_optin_per_block, FP_ERR_UNSUPPORTED,
+               "fp_csr_plan_pack: n = %lld too wide for %d-thread CTAs", (long long)n, bs);
     int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f1, bs, pk1_smem_n(n, dtype, true, bs));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f1, bs, pk1_smem_n(n, dtype, true, bs, ns1));
     groups = di.sm_count * std::max(1, occ);
   }
   if (const char* e = std::getenv("FP_PK_GROUPS")) {  // fewer CTA groups (tests: several local ranks
@@ -1337,6 +1436,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   p->rowptr = rowptr;
   p->dtype = dtype;
   p->bs = bs;
+  p->ns1 = ns1;
   const int64_t ng = (m + kPkRows - 1) / kPkRows;
   uint32_t* cnt = nullptr;
   unsigned long long* gmask = nullptr;
@@ -1431,6 +1531,13 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
     else
       k_pk_bankopt<float><<<bgrid, 256, 0, s>>>(segs, p->tile_desc, p->cr, (float*)p->val, 31);
   }
+  if (cs == 1) {  // k_pk1's lane-interleaved windows (after the bank balancing, which is by logical slot)
+    const int igrid = (int)std::min<int64_t>((segs + 7) / 8, (int64_t)di.sm_count * 16);
+    if (dtype == FP_F64)
+      k_pk_interleave<double><<<igrid, 256, 0, s>>>(segs, p->tile_desc, p->cr, (double*)p->val);
+    else
+      k_pk_interleave<float><<<igrid, 256, 0, s>>>(segs, p->tile_desc, p->cr, (float*)p->val);
+  }
   const int nq = groups * (bs / 32);
   if (ntiles >= INT32_MAX) return fail(cudaErrorInvalidValue, "too many tiles");
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
@@ -1468,7 +1575,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   return FP_OK;
 }
 
-size_t pk1_smem(const Packed* p, bool has_y) { return pk1_smem_n(p->n, p->dtype, has_y, p->bs); }
+size_t pk1_smem(const Packed* p, bool has_y) { return pk1_smem_n(p->n, p->dtype, has_y, p->bs, p->ns1); }
 
 fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   const bool has_y = a.y != nullptr;
@@ -1478,7 +1585,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     Pk1Args k{};
     k.n = p->n;
     k.ntiles = p->ntiles;
-    k.padidx = p->entries;
+    k.ns = p->ns1;
     k.tile_desc = p->tile_desc;
     k.wtile = p->wtile;
     k.cr = p->cr;
@@ -1487,8 +1594,6 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     k.v = a.v;
     k.alpha = a.alpha;
     k.hbits = pk_headroom();
-    const char* f = std::getenv("FP_PK_PF");
-    k.pf = f ? std::atoi(f) : 2;
     k.part = p->part;
     k.spill = p->spill;
     void* args[] = {&k};

@@ -87,6 +87,7 @@ struct Packed {
   void* val = nullptr;                  // [entries] fp32 / fp64
   fp_dtype dtype = FP_F32;
   int bs = 1024;                        // threads per CTA of the pass
+  int ns1 = 0;                          // cs == 1: tile slots per warp of k_pk1's shared-memory ring
   unsigned long long* xch = nullptr;    // exchange slots
   unsigned* epoch = nullptr;            // call counter
   double* part = nullptr;               // [groups][n]
