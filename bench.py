@@ -94,6 +94,11 @@ def second_ceiling(cfg, plan, nnz, kern_ms, dev):
         floor = nnz / r["gather_smem_f64"] + nnz / r["atom_smem_u32"]
         what = ("y gathers from shared memory (rate measured on fp64 words, an upper bound for fp32) + one "
                 "native int32 shared atomic per nonzero")
+    elif v == 20:  # L2-sized column blocks: every y gather and w red of a block pass hits L2
+        ops = {"l2_gathers": nnz, "l2_reds": nnz}
+        floor = nnz / r["gather_l2"] + nnz / r["red_l2"]
+        what = ("one y gather + one fp red.global per nonzero, both into the L2-resident column block "
+                "(the blocks run one after the other)")
     elif v in (4, 7, 16, 17):
         prefix = min(n, int(plan.smem_bytes) // s) if v in (16, 17) else 0
         g = int(nnz * (1.0 - prefix / n))
@@ -357,6 +362,8 @@ def run_gpu(args):
             launches_per_step = 3
         elif plan.variant == 19:  # the packed pass + the finalize
             launches_per_step = 2
+        elif plan.variant == 20:  # w init, a dot pass per block (the last fused), q, a scatter pass per block
+            launches_per_step = 2 * int(plan.cluster) + 2 if inp["y"] is not None else int(plan.cluster) + 2
         elif plan.variant in (4, 7, 16):
             s_b = 8 if cfg["dtype"] == "f64" else 4
             nrep = int(os.environ.get("FP_L2_REPLICAS", "0")) or (8 if 8 * n * s_b <= (16 << 20) else 1)

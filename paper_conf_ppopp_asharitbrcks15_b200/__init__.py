@@ -29,7 +29,8 @@ STATUS = {0: "FP_OK", 1: "FP_ERR_INVALID_ARG", 2: "FP_ERR_UNSUPPORTED", 3: "FP_E
 VARIANTS = {1: "dense_vector", 2: "dense_cta", 3: "csr_vector_smem", 4: "csr_vector_l2", 5: "csr_vector_private",
             6: "csr_flat_smem", 7: "csr_flat_l2", 8: "csr_flat_private", 9: "dense_cluster", 10: "csr_owner",
             11: "csr_vector_fixed", 12: "csr_flat_fixed", 13: "csr_colsplit_cluster",
-            14: "csr_stream_smem", 15: "csr_stream_fixed", 16: "csr_flat_l2_wide"}
+            14: "csr_stream_smem", 15: "csr_stream_fixed", 16: "csr_flat_l2_wide", 17: "csr_binned",
+            18: "csr_flat4_fixed", 19: "csr_packed", 20: "csr_l2block"}
 
 
 class FusedPatError(RuntimeError):
@@ -271,7 +272,8 @@ class CsrPlan:
         return L
 
     def pack(self, val, stream=None):
-        """fp_csr_plan_pack: the column-blocked copy of the matrix with values ``val`` (variant 19);
+        """fp_csr_plan_pack: the column-blocked copy of the matrix with values ``val`` (variant 19, or
+        variant 20's L2-sized column blocks when n is too wide for shared-memory blocks);
         afterwards ``plan(None, y, ...)`` evaluates Eq. (1) on the copy."""
         _require_cuda(val)
         if val.dtype != self.dtype or val.shape[0] != self.nnz:

@@ -1380,8 +1380,8 @@ int packed_cs(int64_t n, fp_dtype dt) {
 
 void packed_free(Packed* p) {
   if (!p) return;
-  for (void* b : {(void*)p->tile_desc, (void*)p->wtile, (void*)p->cr, (void*)p->val,
-                  (void*)p->xch, (void*)p->epoch, (void*)p->part, (void*)p->spill, (void*)p->trace})
+  for (void* b : {(void*)p->tile_desc, (void*)p->wtile, (void*)p->cr, (void*)p->val, (void*)p->xch,
+                  (void*)p->epoch, (void*)p->part, (void*)p->spill, (void*)p->trace, (void*)p->rowdot})
     if (b) cudaFree(b);
   delete p;
 }
@@ -1393,6 +1393,25 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   FP_REQUIRE(val || nnz == 0, FP_ERR_INVALID_ARG, "fp_csr_plan_pack: val is NULL");
   FP_REQUIRE(m >= 1 && n >= 1, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: empty matrix");
   FP_REQUIRE(m < INT32_MAX, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: m >= 2^31");
+  // too wide for the shared memory of a CTA group (fp64 beyond one block, fp32 beyond 8): the
+  // L2-sized column blocks of variant 20 (FP_PK_L2=1 forces them: tests, measurement)
+  const char* fl2 = std::getenv("FP_PK_L2");
+  if ((fl2 && std::atoi(fl2) != 0) || (cs_force <= 0 && packed_cs(n, dtype) == 0)) {
+    Packed* q = new (std::nothrow) Packed;
+    FP_REQUIRE(q, FP_ERR_NOMEM, "fp_csr_plan_pack: out of host memory");
+    q->m = m;
+    q->n = n;
+    q->nnz = nnz;
+    q->rowptr = rowptr;
+    q->dtype = dtype;
+    fp_status st = l2block_build(m, n, nnz, rowptr, colidx, val, dtype, q, s);
+    if (st != FP_OK) {
+      packed_free(q);
+      return st;
+    }
+    *out = q;
+    return FP_OK;
+  }
   const int cs = cs_force > 0 ? cs_force : packed_cs(n, dtype);
   FP_REQUIRE(cs == 1 || cs == 2 || cs == 4 || cs == 8, FP_ERR_UNSUPPORTED,
              "fp_csr_plan_pack: n = %lld needs more than %s column blocks", (long long)n,
@@ -1578,6 +1597,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
 size_t pk1_smem(const Packed* p, bool has_y) { return pk1_smem_n(p->n, p->dtype, has_y, p->bs, p->ns1); }
 
 fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
+  if (p->mode == 1) return l2block_exec(p, a, s);
   const bool has_y = a.y != nullptr;
   if (p->cs == 1) {
     const void* f1 = pk1_pick(p->dtype, has_y, p->bs);
@@ -1664,6 +1684,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
 }
 
 void packed_launch(const Packed* p, fp_launch* L) {
+  if (p->mode == 1) return l2block_launch(p, L);
   *L = fp_launch{};
   L->variant = FP_VAR_CSR_PACKED;
   L->vs = 32;

@@ -1,5 +1,7 @@
 // kernels.cuh -- launcher interfaces between the C-ABI layer (api.cu) and the kernel files.
 #pragma once
+#include <vector>
+
 #include "common.cuh"
 
 namespace fp {
@@ -94,7 +96,19 @@ struct Packed {
   double* spill = nullptr;              // [cs][bw + 1]
   unsigned long long* trace = nullptr;  // FP_PK_TRACE measurement buffer
   int trace_warps = 32;                 // warps per CTA of the pass (trace layout)
+  // mode 1 = variant 20 (csr_l2block.cu): cs L2-sized column blocks of bw columns, chunks
+  // (tile_desc) of block b = [l2cb[b], l2cb[b + 1]); the heaviest block is processed last (fused)
+  int mode = 0;
+  int heavy = 0;
+  std::vector<int64_t> l2cb;
+  double* rowdot = nullptr;             // [m]: row dots p, then q
 };
+// variant 20 (csr_l2block.cu)
+int64_t l2block_bw(int64_t n, fp_dtype dt);
+fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                        const void* val, fp_dtype dtype, Packed* p, cudaStream_t s);
+fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s);
+void l2block_launch(const Packed* p, fp_launch* L);
 int packed_cs(int64_t n, fp_dtype dt);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                        const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s);

@@ -14,7 +14,8 @@ Checked here, at sizes the oracle finishes in seconds:
 * IEEE propagation of Inf/NaN terms (reading R8);
 * determinism (bit-identical reruns), re-packing with new values, CUDA-graph replays (the
   per-call exchange tag lives in device memory);
-* what it refuses (fp64 wider than one block, exec without values on an unpacked plan);
+* what it refuses (exec without values on an unpacked plan); fp64 wider than one block takes
+  variant 20's L2-sized column blocks (csr_l2block.cu), tested at the end;
 * the single-block pass (k_pk1, fp32 and fp64) on C3/S3-shaped matrices.
 """
 import numpy as np
@@ -181,7 +182,7 @@ def test_packed_nonfinite_propagates(cuda_dev):
 
 def test_packed_repack_unpacked_exec_alpha0(cuda_dev):
     """pack again with new values; exec with val on a packed plan runs the unpacked path; alpha
-    = 0 writes beta z; exec without val on an unpacked plan and fp64 packing are refused."""
+    = 0 writes beta z; exec without val on an unpacked plan and a forced 16-block pack are refused."""
     m, n = 8000, 100_000
     rp, ci, va, y, v, z = make(m, n, ("powerlaw", 2.5, 13.64), seed=4, kind="int_pm12")
     plan = packed_plan(cuda_dev, rp, ci, va, n)
@@ -200,8 +201,13 @@ def test_packed_repack_unpacked_exec_alpha0(cuda_dev):
         plain(None, y.to(cuda_dev), v.to(cuda_dev), z.to(cuda_dev), 1.0, 1.0)
     rp64, ci64, va64 = synth.csr(500, 60_000, "f64", ("uniform", 0, 20), seed=3)
     p64 = fp.CsrPlan(rp64.to(cuda_dev), ci64.to(cuda_dev), 60_000, torch.float64)
-    with pytest.raises(fp.FusedPatError):  # fp64 packs one column block only
-        p64.pack(va64.to(cuda_dev))
+    with pytest.raises(fp.FusedPatError):  # more than 8 shared-memory blocks forced
+        import os
+        os.environ["FP_PK_CS"] = "16"
+        try:
+            p64.pack(va64.to(cuda_dev))
+        finally:
+            del os.environ["FP_PK_CS"]
 
 
 def test_packed_graph_replay(cuda_dev):
@@ -276,7 +282,7 @@ def test_packed1_float_parity(cuda_dev, dt):
 
 
 def test_packed1_nonfinite_and_wide_fp64(cuda_dev):
-    """Inf / NaN propagate (reading R8); an fp64 matrix too wide for one block is refused."""
+    """Inf / NaN propagate (reading R8); an fp64 matrix too wide for one block packs into L2 blocks."""
     m, n = 3000, 800
     rp, ci, va = synth.csr(m, n, "f64", ("binomial", 0.02), seed=9)
     y = synth.vector(n, "f64", seed=9, stream=synth.S_Y)
@@ -289,5 +295,106 @@ def test_packed1_nonfinite_and_wide_fp64(cuda_dev):
     assert_parity(run(plan, cuda_dev, y, None, None, 1.0, 0.0), ref, mag, torch.float64, "packed1 non-finite")
     rp, ci, va = synth.csr(200, 40_000, "f64", ("uniform", 0, 20), seed=3)
     p64 = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), 40_000, torch.float64)
-    with pytest.raises(fp.FusedPatError):
-        p64.pack(va.to(cuda_dev))
+    p64.pack(va.to(cuda_dev))  # too wide for one shared-memory block: variant 20's L2 blocks
+    assert p64.launch.variant == 20
+
+
+# ------------------------------------------------------------------ variant 20: L2-sized column blocks
+def l2_plan(dev, monkeypatch, rp, ci, va, n, bw, tdt):
+    monkeypatch.setenv("FP_PK_L2", "1")
+    monkeypatch.setenv("FP_L2B_BW", str(bw))
+    plan = fp.CsrPlan(rp.to(dev), ci.to(dev), n, tdt)
+    plan.pack(va.to(dev))
+    torch.cuda.synchronize()
+    monkeypatch.delenv("FP_PK_L2")
+    monkeypatch.delenv("FP_L2B_BW")
+    assert plan.launch.variant == 20
+    return plan
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+@pytest.mark.parametrize("n,bw", [(5000, 1000), (20_000, 3001), (4096, 4096)])
+@pytest.mark.parametrize("lengths", [("powerlaw", 2.5, 13.64), ("binomial", 0.004), ("uniform", 0, 1500)])
+def test_l2block_integer_twin_bitexact(cuda_dev, monkeypatch, dt, n, bw, lengths):
+    """Variant 20 (csr_l2block.cu): the columns in blocks of bw (here small, so that a test-sized
+    matrix spans several blocks, a ragged last block, one block), row dots accumulated over the
+    blocks, the heaviest block fused (q and its scatter from the same registers), the others
+    re-read; rows longer than a 256-entry chunk split into partial chunks; empty rows.  Integer
+    twins: every sum exact in fp64 / below 2^24 in fp32, so bit-exact whatever the red order."""
+    m = 6_007 if lengths[0] != "uniform" else 1_501
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rp, ci, va = synth.csr(m, n, dt, lengths, kind="int_pm12", seed=31)
+    y = synth.vector(n, dt, kind="int_small", seed=31, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="int_pos", seed=31, stream=synth.S_V)
+    z = synth.vector(n, dt, kind="int_small", seed=31, stream=synth.S_Z)
+    plan = l2_plan(cuda_dev, monkeypatch, rp, ci, va, n, bw, tdt)
+    assert plan.launch.cluster == (n + bw - 1) // bw
+    for args in INSTANCES(y, v, z):
+        ref, mag = oracle.csr(m, n, rp, ci, va, *args)
+        if dt == "f32" and mag.max() >= 2**24:
+            continue
+        w = run(plan, cuda_dev, *args)
+        assert_bitexact(w, ref, f"l2block {dt} n={n} bw={bw} {lengths} y={args[0] is not None}")
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+def test_l2block_float_parity_skewed(cuda_dev, monkeypatch, dt):
+    """U[-1,1) data on KDD-shaped rows (power-law lengths, Zipf-like columns: most nonzeros in
+    the first block, which then runs fused), the north_star tolerance (1e-11 fp64, 2e-5 fp32);
+    rows scaled by 2^+-30."""
+    m, n = 40_000, 200_000
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rp, ci, va = synth.csr(m, n, dt, ("powerlaw", 2.5, 9.5), seed=12, col_skew=2)
+    y = synth.vector(n, dt, seed=12, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="pos", seed=12, stream=synth.S_V)
+    z = synth.vector(n, dt, seed=12, stream=synth.S_Z)
+    plan = l2_plan(cuda_dev, monkeypatch, rp, ci, va, n, 25_000, tdt)
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    assert_parity(run(plan, cuda_dev, y, v, z, 1.0, 1.0), ref, mag, tdt, f"l2block {dt}")
+    g = torch.Generator().manual_seed(6)
+    sc = torch.pow(2.0, torch.randint(-30, 31, (m,), generator=g).to(tdt))
+    va2 = va * torch.repeat_interleave(sc, (rp[1:] - rp[:-1]))
+    plan.pack(va2.to(cuda_dev))  # re-pack unforced: fp32 -> shared-memory blocks, fp64 -> one L2 block
+    ref, mag = oracle.csr(m, n, rp, ci, va2, y, v, z, 1.0, 1.0)
+    assert_parity(run(plan, cuda_dev, y, v, z, 1.0, 1.0), ref, mag, tdt, f"l2block {dt} dynamic range")
+
+
+def test_l2block_chosen_for_wide_fp64_and_nonfinite(cuda_dev):
+    """fp64 wider than one shared-memory block packs into L2 blocks without forcing (the
+    round-2 refusal is gone); Inf / NaN propagate (reading R8)."""
+    m, n = 3000, 40_000
+    rp, ci, va = synth.csr(m, n, "f64", ("uniform", 0, 60), seed=3)
+    va = va.clone()
+    va[10] = float("inf")
+    va[4000] = float("nan")
+    y = synth.vector(n, "f64", seed=3, stream=synth.S_Y)
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, torch.float64)
+    plan.pack(va.to(cuda_dev))
+    assert plan.launch.variant == 20 and plan.launch.cluster == 1
+    ref, mag = oracle.csr(m, n, rp, ci, va, y, None, None, 1.0, 0.0)
+    assert_parity(run(plan, cuda_dev, y, None, None, 1.0, 0.0), ref, mag, torch.float64, "l2block non-finite")
+
+
+def test_l2block_graph_replay(cuda_dev, monkeypatch):
+    """The L2-block launches captured in a CUDA graph and replayed: same result each replay."""
+    m, n = 5000, 9000
+    rp, ci, va = synth.csr(m, n, "f64", ("powerlaw", 2.5, 13.64), kind="int_pm12", seed=4)
+    y = synth.vector(n, "f64", kind="int_small", seed=4, stream=synth.S_Y)
+    v = synth.vector(m, "f64", kind="int_pos", seed=4, stream=synth.S_V)
+    z = synth.vector(n, "f64", kind="int_small", seed=4, stream=synth.S_Z)
+    plan = l2_plan(cuda_dev, monkeypatch, rp, ci, va, n, 2000, torch.float64)
+    ref, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 1.0)
+    yd, vd, zd = y.to(cuda_dev), v.to(cuda_dev), z.to(cuda_dev)
+    w = torch.empty(n, dtype=torch.float64, device=cuda_dev)
+    s = torch.cuda.Stream(device=cuda_dev)
+    with torch.cuda.stream(s):
+        plan(None, yd, vd, zd, 1.0, 1.0, w=w)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        plan(None, yd, vd, zd, 1.0, 1.0, w=w)
+    for i in range(3):
+        w.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert_bitexact(w, ref, f"l2block graph replay {i}")
