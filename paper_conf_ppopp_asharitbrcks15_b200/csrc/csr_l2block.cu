@@ -22,11 +22,15 @@
 //
 // The copy (fp_csr_plan_pack, once per matrix, amortised as the paper amortises its baseline's
 // transpose): per block, the block's entries in row order, cut into CHUNKS of at most
-// 256 entries and 64 consecutive rows (one 8-entry-per-lane register window; a chunk never
-// crosses a 64-row group); a row with more than 256 entries in a block becomes a run of
-// "partial" chunks of 256.  Entry word = column in block | row in chunk << 26; chunks padded to
-// 8 entries (32-byte aligned 256-bit loads).  Descriptor per chunk: (offset / 8, length | rows
-// << 25, first row, flags).
+// 256 entries (one 8-entry-per-lane register window) and consecutive rows (at most 64 in the
+// fused block, whose q sits in shared memory; up to 1024 elsewhere, so that the sparse blocks
+// fill their windows); a row with more than 256 entries in a block becomes a run of "partial"
+// chunks of 256.  Entry word = column in block | hot flag | row in chunk; chunks padded to 8
+// entries (32-byte aligned 256-bit loads).  Descriptor per chunk: (offset / 8, length | rows
+// << 16, first row, flags).  HOT columns (more nonzeros than max(2048, nnz / 2^16): a bias
+// feature, the head of a Zipf distribution) would serialise their reds on one L2 address;
+// their entries are listed once more sorted by column and scattered by k_l2b_hot (one red per
+// 256 entries).
 #include <algorithm>
 #include <cstdlib>
 #include <new>
@@ -36,26 +40,39 @@
 
 #include "kernels.cuh"
 
+#include <cub/device/device_radix_sort.cuh>
+
 namespace fp {
 
 namespace {
 
-constexpr int kL2Win = 256;                 // entries per chunk (one window, 8 per lane)
-constexpr int kL2Rows = 64;                 // rows per chunk / per row group
-constexpr int kL2RidShift = 26;             // entry word: column in block | row in chunk << 26
-constexpr uint32_t kL2ColMask = (1u << kL2RidShift) - 1u;
-constexpr uint32_t kL2PadWord = 63u << kL2RidShift;  // padding: column 0 (never read), row 63, value 0
-constexpr unsigned kL2Partial = 1u;         // desc.w: one piece of a row longer than a window
+constexpr int kL2Win = 256;          // entries per chunk (one window, 8 per lane)
+constexpr int kL2Group = 1024;       // chunks never cross a group of 1024 rows
+constexpr int kL2HeavyRows = 64;     // rows per chunk of the fused block (its q in shared memory)
+constexpr unsigned kL2Partial = 1u;  // desc.w: one piece of a row longer than a window
 constexpr int kL2MaxBlocks = 64;
 constexpr int kL2BS = 256;
 constexpr int kL2NW = kL2BS / 32;
+constexpr int kL2MaxHot = 1 << 16;   // hot columns (scattered by column, see k_l2b_hot)
 
 enum { L2_DOT = 0, L2_FUSED = 1, L2_SCAT = 2, L2_SCAT_PARTIAL = 3 };
 
+// Entry word: column in block (cb bits) | hot flag (bit cb) | row in chunk (bits cb + 1 ..).
+// Padding: column 0, row 63, value 0 (never gathered: entries beyond a chunk's length are
+// predicated off; a run of row 63 adds 0).
+struct L2Enc {
+  unsigned cb;  // column bits
+  __host__ __device__ uint32_t colmask() const { return (1u << cb) - 1u; }
+  __host__ __device__ uint32_t hotbit() const { return 1u << cb; }
+  __host__ __device__ unsigned ridshift() const { return cb + 1; }
+  __host__ __device__ uint32_t pad() const { return 63u << (cb + 1); }
+};
+
 struct L2Args {
-  const uint4* desc;    // this block's chunks
+  const uint4* desc;    // this block's chunks: (offset / 8, length | rows << 16, first row, flags)
   int64_t nch;
   int64_t col0;         // first column of the block
+  L2Enc enc;
   const uint32_t* cr;
   const void* val;      // T
   const void* y;        // T, the full vector
@@ -65,8 +82,8 @@ struct L2Args {
   void* w;              // T
 };
 
-// 8 consecutive entries (32-byte aligned): streamed once, evict-first in L2 (the blocks of y
-// and w are what L2 should keep)
+// 8 consecutive entries (32-byte aligned): streamed, evict-first in L2 (the blocks of y and w
+// are what L2 should keep)
 __device__ __forceinline__ void l2_ldc(const uint32_t* p, uint32_t (&c)[8]) {
   asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]), "=r"(c[4]), "=r"(c[5]), "=r"(c[6]), "=r"(c[7])
@@ -101,9 +118,16 @@ __device__ __forceinline__ double l2_ldy(const double* p, uint64_t pol) {
 }
 
 // One pass over the chunks of one column block (a warp per chunk, grid-stride).
+//   DOT / FUSED: Eq. (2) on the window -- in-lane runs of a row, one bounded segmented scan
+//     across lanes; the lane that closes a row's run owns its window sum.  DOT (and the partial
+//     chunks of the fused block): the owner adds it into p[row] (fp64 red).  FUSED (rows <= 64):
+//     the sums go to shared memory, p[row] is completed, q = alpha v p, and the scatter runs
+//     from the registers that hold the window (a7).
+//   SCAT: q[row] = p[row] after k_l2b_q; SCAT_PARTIAL: the fused block's partial chunks.
+// Hot entries (columns scattered by column in k_l2b_hot) take part in the dot, not the scatter.
 template <typename T, int MODE>
 __global__ void __launch_bounds__(kL2BS) k_l2b(const L2Args a) {
-  __shared__ double s_rs[kL2NW][kL2Rows];
+  __shared__ double s_rs[kL2NW][kL2HeavyRows];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   double* rs = s_rs[wi];
   const T* __restrict__ y = reinterpret_cast<const T*>(a.y) + a.col0;
@@ -111,14 +135,17 @@ __global__ void __launch_bounds__(kL2BS) k_l2b(const L2Args a) {
   const T* __restrict__ val = reinterpret_cast<const T*>(a.val);
   T* w = reinterpret_cast<T*>(a.w) + a.col0;
   double* p = a.p;
+  const uint32_t cmask = a.enc.colmask(), hot = a.enc.hotbit();
+  const unsigned rsh = a.enc.ridshift();
+  const uint32_t padw = a.enc.pad();
   const uint64_t keep = l2_keep_policy();
   const int64_t nw = (int64_t)gridDim.x * kL2NW;
   for (int64_t c = (int64_t)blockIdx.x * kL2NW + wi; c < a.nch; c += nw) {
     const uint4 D = __ldg(a.desc + c);
     const bool partial = (D.w & kL2Partial) != 0;
     if (MODE == L2_SCAT_PARTIAL && !partial) continue;
-    const int len = (int)(D.y & 0x1FFFFFFu), rows = (int)(D.y >> 25);
-    const int64_t r0 = (int64_t)D.z;
+    const int len = (int)(D.y & 0xFFFFu), rows = (int)(D.y >> 16);
+    double* pr0 = p + D.z;
     const int o = 8 * lane;
     uint32_t cw[8];
     T xv[8];
@@ -128,36 +155,42 @@ __global__ void __launch_bounds__(kL2BS) k_l2b(const L2Args a) {
       l2_ldv(val + e0, xv);
     } else {
 #pragma unroll
-      for (int e = 0; e < 8; ++e) cw[e] = kL2PadWord, xv[e] = T(0);
+      for (int e = 0; e < 8; ++e) cw[e] = padw, xv[e] = T(0);
     }
-    bool fused_scatter = false;
+    bool fused = false;
     if constexpr (MODE == L2_DOT || MODE == L2_FUSED) {
-      // Eq. (2) on the window: in-lane runs of a row, then one bounded segmented scan across
-      // lanes; each row's window sum lands in rs[row] exactly once
-      rs[lane] = 0.0;
-      rs[lane + 32] = 0.0;
-      __syncwarp();
+      fused = MODE == L2_FUSED && !partial;
+      if (fused) {
+        rs[lane] = 0.0;
+        rs[lane + 32] = 0.0;
+        __syncwarp();
+      }
+      // the owner of a row's window sum: the shared slot (fused) or a red into p
+      auto put = [&](unsigned r, T sum) {
+        if (fused) rs[r] = (double)sum;
+        else if ((int)r < rows) atomicAdd(pr0 + r, (double)sum);
+      };
       T cs_[8];
 #pragma unroll
       for (int e = 0; e < 8; ++e) {
-        const T pr = o + e < len ? xv[e] * l2_ldy(y + (cw[e] & kL2ColMask), keep) : T(0);
-        cs_[e] = (e == 0 || (cw[e] >> kL2RidShift) != (cw[e - 1] >> kL2RidShift)) ? pr : cs_[e - 1] + pr;
+        const T pr = o + e < len ? xv[e] * l2_ldy(y + (cw[e] & cmask), keep) : T(0);
+        cs_[e] = (e == 0 || (cw[e] >> rsh) != (cw[e - 1] >> rsh)) ? pr : cs_[e - 1] + pr;
       }
-      const int last = (int)(cw[7] >> kL2RidShift);
+      const int last = (int)(cw[7] >> rsh);
       int prev = __shfl_up_sync(0xffffffffu, last, 1);
       if (lane == 0) prev = -1;
-      const bool h0 = (int)(cw[0] >> kL2RidShift) != prev;
+      const bool h0 = (int)(cw[0] >> rsh) != prev;
       bool seen = h0;
 #pragma unroll
       for (int e = 0; e < 7; ++e) {
-        const bool h = (cw[e + 1] >> kL2RidShift) != (cw[e] >> kL2RidShift);
-        if (h && seen) rs[cw[e] >> kL2RidShift] = (double)cs_[e];
+        const bool h = (cw[e + 1] >> rsh) != (cw[e] >> rsh);
+        if (h && seen) put(cw[e] >> rsh, cs_[e]);
         seen |= h;
       }
       T P = cs_[7];
 #pragma unroll
       for (int e = 7; e >= 1; --e)
-        if ((cw[e] >> kL2RidShift) != (cw[e - 1] >> kL2RidShift)) P = cs_[e - 1];
+        if ((cw[e] >> rsh) != (cw[e - 1] >> rsh)) P = cs_[e - 1];
       if (h0) P = T(0);
       const unsigned hl = __ballot_sync(0xffffffffu, seen) >> lane;
       const int dist = hl ? __ffs(hl) : 32 - lane;
@@ -169,34 +202,55 @@ __global__ void __launch_bounds__(kL2BS) k_l2b(const L2Args a) {
       }
       T rn = __shfl_down_sync(0xffffffffu, r, 1);
       if (lane == 31) rn = T(0);
-      if (seen) rs[last] = (double)(cs_[7] + rn);
-      __syncwarp();
-      if (MODE == L2_DOT || partial) {
-        // the block's share of the row dots (a partial chunk: its piece of one long row)
-        if (lane < rows) atomicAdd(p + r0 + lane, rs[lane]);
-        if (lane + 32 < rows) atomicAdd(p + r0 + lane + 32, rs[lane + 32]);
-      } else {
-        // the heaviest block, processed last: p complete -> q = alpha v p, kept for the scatter
+      if (seen) put((unsigned)last, cs_[7] + rn);
+      if (fused) {
+        // the fused block, processed last: p complete -> q = alpha v p, kept for the scatter
+        __syncwarp();
         for (int k = lane; k < rows; k += 32) {
-          const double pt = p[r0 + k] + rs[k];
-          p[r0 + k] = pt;
-          const double vr = vv ? (double)vv[r0 + k] : 1.0;
+          const double pt = pr0[k] + rs[k];
+          pr0[k] = pt;
+          const double vr = vv ? (double)vv[D.z + k] : 1.0;
           rs[k] = a.alpha * (vr * pt);
         }
-        fused_scatter = true;
+        __syncwarp();
       }
-    } else {
-      // q of the chunk's rows (k_l2b_q converted p in place)
-      for (int k = lane; k < rows; k += 32) rs[k] = p[r0 + k];
     }
-    if (MODE == L2_SCAT || MODE == L2_SCAT_PARTIAL || fused_scatter) {
-      __syncwarp();
+    if (MODE == L2_SCAT || MODE == L2_SCAT_PARTIAL || fused) {
       // Eq. (3) from the registers that hold the window: one red per nonzero into the block of w
+      const double q1 = MODE == L2_SCAT_PARTIAL ? __ldg(pr0) : 0.0;
 #pragma unroll
       for (int e = 0; e < 8; ++e)
-        if (o + e < len) atomicAdd(w + (cw[e] & kL2ColMask), (T)((double)xv[e] * rs[cw[e] >> kL2RidShift]));
+        if (o + e < len && !(cw[e] & hot)) {
+          const double q = MODE == L2_SCAT_PARTIAL ? q1 : (fused ? rs[cw[e] >> rsh] : __ldg(pr0 + (cw[e] >> rsh)));
+          atomicAdd(w + (cw[e] & cmask), (T)((double)xv[e] * q));
+        }
     }
     __syncwarp();
+  }
+}
+
+// Hot columns (a column with more nonzeros than the threshold of l2block_build, e.g. the bias
+// feature every row of a KDD-like matrix has): one red per nonzero would serialise on one L2
+// address (K1: ~15M reds into the first columns).  Their entries are kept a second time sorted
+// by column; a warp sums 256 of them, x q[row], and adds ONE red per item (Eq. 3 by column).
+template <typename T>
+__global__ void __launch_bounds__(kL2BS) k_l2b_hot(const uint4* __restrict__ items, int64_t nitems,
+                                                   const uint32_t* __restrict__ hrow, const T* __restrict__ hval,
+                                                   const int32_t* __restrict__ hcol, const double* __restrict__ q,
+                                                   T* w) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * kL2NW;
+  for (int64_t it = (int64_t)blockIdx.x * kL2NW + (threadIdx.x >> 5); it < nitems; it += nw) {
+    const uint4 I = __ldg(items + it);  // (first entry, count, hot slot)
+    double s = 0.0;
+#pragma unroll
+    for (int k = 0; k < kL2Win / 32; ++k) {
+      const int e = k * 32 + lane;
+      if (e < (int)I.y) s += (double)hval[I.x + e] * __ldg(q + hrow[I.x + e]);
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
+    if (lane == 0) atomicAdd(w + hcol[I.z], (T)s);
   }
 }
 
@@ -220,47 +274,70 @@ __global__ void k_l2b_init(int64_t n, T* __restrict__ w, const T* __restrict__ z
 }
 
 // ---------------------------------------------------------------- the copy (pack time)
-// (1) entries of row r in block b: cnt[b m + r] (zeroed before)
+// (1) entries of row r in block b (cnt[b m + r]), entries of column c (colcnt[c]), per block
 __global__ void k_l2b_count(int64_t m, const int64_t* __restrict__ rowptr, const int32_t* __restrict__ colidx,
-                            int64_t bw, uint32_t* __restrict__ cnt) {
+                            int64_t bw, uint32_t* __restrict__ cnt, uint32_t* __restrict__ colcnt,
+                            unsigned long long* __restrict__ blocktot) {
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
     const int64_t e = rowptr[r + 1];
-    for (int64_t i = rowptr[r]; i < e; ++i) cnt[(int64_t)(colidx[i] / bw) * m + r] += 1u;
+    for (int64_t i = rowptr[r]; i < e; ++i) {
+      const int64_t b = colidx[i] / bw;
+      cnt[b * m + r] += 1u;
+      atomicAdd(colcnt + colidx[i], 1u);
+      atomicAdd(blocktot + b, 1ull);
+    }
   }
 }
 
-// (2) the chunks of one (block, 64-row group): a thread walks the group's rows.  COUNT: number
-// of chunks and padded entries; WRITE: the descriptors, and per (block, row) the entry offset
-// of the row's first block-b entry and its row-in-chunk.
+// (2) hot columns: more than `thr` nonzeros -> a slot (at most kL2MaxHot)
+__global__ void k_l2b_hotsel(int64_t n, const uint32_t* __restrict__ colcnt, uint32_t thr, int32_t* __restrict__ slot,
+                             int32_t* __restrict__ hcol, unsigned* __restrict__ nhot) {
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
+    int32_t sl = -1;
+    if (colcnt[c] > thr) {
+      const unsigned k = atomicAdd(nhot, 1u);
+      if (k < (unsigned)kL2MaxHot) {
+        sl = (int32_t)k;
+        hcol[k] = (int32_t)c;
+      }
+    }
+    slot[c] = sl;
+  }
+}
+
+// (3) the chunks of one (block, 1024-row group): a thread walks the group's rows.  COUNT:
+// number of chunks and padded entries; WRITE: the descriptors, and per (block, row) the entry
+// offset of the row's first block-b entry and its row in the chunk.  A chunk: <= 256 entries,
+// <= rowcap rows (64 in the fused block, else as many as the entry word's row field holds).
 template <bool WRITE>
-__global__ void k_l2b_walk(int64_t m, int cs, const uint32_t* __restrict__ cnt, int64_t* __restrict__ nchunk,
-                           int64_t* __restrict__ nent, const int64_t* __restrict__ cbase,
+__global__ void k_l2b_walk(int64_t m, int cs, int heavy, int rowcap, const uint32_t* __restrict__ cnt,
+                           int64_t* __restrict__ nchunk, int64_t* __restrict__ nent, const int64_t* __restrict__ cbase,
                            const int64_t* __restrict__ ebase, uint4* __restrict__ desc, uint32_t* __restrict__ rowoff,
-                           uint8_t* __restrict__ rid) {
-  const int64_t ng = (m + kL2Rows - 1) / kL2Rows;
+                           uint16_t* __restrict__ rid) {
+  const int64_t ng = (m + kL2Group - 1) / kL2Group;
   for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < (int64_t)cs * ng;
        t += (int64_t)gridDim.x * blockDim.x) {
     const int b = (int)(t / ng);
     const int64_t g = t % ng;
+    const int cap = b == heavy ? kL2HeavyRows : rowcap;
     int64_t ci = WRITE ? cbase[t] : 0, ei = WRITE ? ebase[t] : 0;
     int64_t nc = 0, ne = 0;
-    int64_t r0 = -1;
+    int64_t r0 = -1, last_row = -1;
     int len = 0;
     auto emit = [&](int64_t first, int rows, int l, unsigned flags) {
-      if (WRITE) desc[ci++] = make_uint4((unsigned)(ei / 8), (unsigned)l | ((unsigned)rows << 25), (unsigned)first, flags);
+      if (WRITE) desc[ci++] = make_uint4((unsigned)(ei / 8), (unsigned)l | ((unsigned)rows << 16), (unsigned)first, flags);
       ++nc;
       const int64_t al = (l + 7) & ~7;
       ne += al;
       ei += al;
     };
-    int64_t last_row = -1;
     auto flush = [&]() {
       if (r0 >= 0) emit(r0, (int)(last_row - r0 + 1), len, 0u);
       r0 = -1;
       len = 0;
     };
-    for (int i = 0; i < kL2Rows && g * kL2Rows + i < m; ++i) {
-      const int64_t r = g * kL2Rows + i;
+    for (int i = 0; i < kL2Group && g * kL2Group + i < m; ++i) {
+      const int64_t r = g * kL2Group + i;
       const uint32_t c = cnt[(int64_t)b * m + r];
       if (c == 0) continue;
       if (c > (uint32_t)kL2Win) {  // a run of partial chunks of 256 (contiguous entries)
@@ -272,11 +349,11 @@ __global__ void k_l2b_walk(int64_t m, int cs, const uint32_t* __restrict__ cnt, 
         for (uint32_t k = 0; k < c; k += kL2Win) emit(r, 1, (int)std::min<uint32_t>(kL2Win, c - k), kL2Partial);
         continue;
       }
-      if (r0 >= 0 && len + (int)c > kL2Win) flush();
+      if (r0 >= 0 && (len + (int)c > kL2Win || r - r0 >= cap)) flush();
       if (r0 < 0) r0 = r;
       if (WRITE) {
         rowoff[(int64_t)b * m + r] = (uint32_t)(ei + len);
-        rid[(int64_t)b * m + r] = (uint8_t)(r - r0);
+        rid[(int64_t)b * m + r] = (uint16_t)(r - r0);
       }
       len += (int)c;
       last_row = r;
@@ -289,13 +366,14 @@ __global__ void k_l2b_walk(int64_t m, int cs, const uint32_t* __restrict__ cnt, 
   }
 }
 
-// (3) the entries: a thread per row, running count per block (stable order: non-canonical rows
-// are packed as given, reading R7)
+// (4) the entries: a thread per row, running count per block (stable order: non-canonical rows
+// are packed as given, reading R7); hot entries flagged and listed once more (key: slot, row)
 template <typename V>
-__global__ void k_l2b_scatter(int64_t m, int cs, int64_t bw, const int64_t* __restrict__ rowptr,
+__global__ void k_l2b_scatter(int64_t m, int cs, int64_t bw, L2Enc enc, const int64_t* __restrict__ rowptr,
                               const int32_t* __restrict__ colidx, const V* __restrict__ val,
-                              const uint32_t* __restrict__ rowoff, const uint8_t* __restrict__ rid,
-                              uint32_t* __restrict__ cr, V* __restrict__ pval) {
+                              const uint32_t* __restrict__ rowoff, const uint16_t* __restrict__ rid,
+                              const int32_t* __restrict__ slot, uint32_t* __restrict__ cr, V* __restrict__ pval,
+                              unsigned long long* __restrict__ hkey, V* __restrict__ hv, unsigned long long* __restrict__ hn) {
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
     uint32_t k[kL2MaxBlocks];
     for (int b = 0; b < cs; ++b) k[b] = 0;
@@ -304,8 +382,15 @@ __global__ void k_l2b_scatter(int64_t m, int cs, int64_t bw, const int64_t* __re
       const int col = colidx[i];
       const int b = (int)(col / bw);
       const int64_t pos = (int64_t)rowoff[(int64_t)b * m + r] + k[b]++;
-      cr[pos] = (uint32_t)(col - b * bw) | ((uint32_t)rid[(int64_t)b * m + r] << kL2RidShift);
+      const int32_t sl = slot ? slot[col] : -1;
+      cr[pos] = (uint32_t)(col - b * bw) | (sl >= 0 ? enc.hotbit() : 0u) |
+                ((uint32_t)rid[(int64_t)b * m + r] << enc.ridshift());
       pval[pos] = val[i];
+      if (sl >= 0) {
+        const unsigned long long h = atomicAdd(hn, 1ull);
+        hkey[h] = ((unsigned long long)sl << 32) | (unsigned long long)r;
+        hv[h] = val[i];
+      }
     }
   }
 }
@@ -313,16 +398,31 @@ __global__ void k_l2b_scatter(int64_t m, int cs, int64_t bw, const int64_t* __re
 __global__ void k_l2b_fill(int64_t n, uint32_t* __restrict__ p, uint32_t v) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
 }
+__global__ void k_l2b_gather(int64_t n, const int32_t* __restrict__ idx, const uint32_t* __restrict__ src,
+                             uint32_t* __restrict__ dst) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = src[idx[i]];
+}
+__global__ void k_l2b_rows(int64_t n, const unsigned long long* __restrict__ key, uint32_t* __restrict__ row) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    row[i] = (uint32_t)key[i];
+}
+
+unsigned bits_for(int64_t v) {  // bits to hold 0 .. v - 1
+  unsigned b = 1;
+  while (((int64_t)1 << b) < v) ++b;
+  return b;
+}
 
 }  // namespace
 
 // columns per L2 block: y and w of a block take 32 MB (fp64: 2M columns, fp32: 4M); FP_L2B_BW
-// (measurement / tests) overrides; at most kL2MaxBlocks blocks
+// (measurement / tests) overrides; at most kL2MaxBlocks blocks, at most 2^24 columns a block
 int64_t l2block_bw(int64_t n, fp_dtype dt) {
   int64_t bw = dt == FP_F64 ? (int64_t)1 << 21 : (int64_t)1 << 22;
   if (const char* e = std::getenv("FP_L2B_BW")) bw = std::max<int64_t>(1, std::atoll(e));
   bw = std::max<int64_t>(bw, (n + kL2MaxBlocks - 1) / kL2MaxBlocks);
-  return std::min<int64_t>(bw, (int64_t)kL2ColMask + 1);
+  return std::min<int64_t>(std::min<int64_t>(bw, n), (int64_t)1 << 24);
 }
 
 fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
@@ -331,16 +431,23 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   const int cs = (int)((n + bw - 1) / bw);
   FP_REQUIRE(cs <= kL2MaxBlocks, FP_ERR_UNSUPPORTED, "fp_csr_plan_pack: n = %lld needs more than %d L2 blocks",
              (long long)n, kL2MaxBlocks);
+  const L2Enc enc{bits_for(bw)};
+  const int rowcap = (int)std::min<int64_t>(kL2Group, (int64_t)1 << (31 - enc.cb));
   const DeviceInfo& di = device_info(current_device());
-  const int64_t ng = (m + kL2Rows - 1) / kL2Rows;
+  const int64_t ng = (m + kL2Group - 1) / kL2Group;
   const int64_t nt = (int64_t)cs * ng;
-  uint32_t* cnt = nullptr;
-  uint32_t* rowoff = nullptr;
-  uint8_t* rid = nullptr;
+  const size_t vs = dtype_size(dtype);
+  uint32_t *cnt = nullptr, *colcnt = nullptr, *rowoff = nullptr;
+  uint16_t* rid = nullptr;
+  int32_t* slot = nullptr;
+  unsigned long long *blocktot = nullptr, *hkey = nullptr, *hkey2 = nullptr, *hn = nullptr;
+  void *hv = nullptr, *tmp = nullptr;
+  unsigned* nhot = nullptr;
   int64_t *nchunk = nullptr, *nent = nullptr, *cbase = nullptr, *ebase = nullptr;
-  void* tmp = nullptr;
   auto cleanup = [&]() {
-    for (void* b : {(void*)cnt, (void*)rowoff, (void*)rid, (void*)nchunk, (void*)nent, (void*)cbase, (void*)ebase, tmp})
+    for (void* b : {(void*)cnt, (void*)colcnt, (void*)rowoff, (void*)rid, (void*)slot, (void*)blocktot, (void*)hkey,
+                    (void*)hkey2, (void*)hn, hv, tmp, (void*)nhot, (void*)nchunk, (void*)nent, (void*)cbase,
+                    (void*)ebase})
       if (b) cudaFree(b);
   };
   auto fail = [&](cudaError_t e, const char* what) {
@@ -355,25 +462,48 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
     if (e_ != cudaSuccess) return fail(e_, what);   \
   } while (0)
   const int tb = 256;
-  const int grid_r = (int)std::min<int64_t>((m + tb - 1) / tb, (int64_t)di.sm_count * 32);
-  const int grid_t = (int)std::min<int64_t>((nt + tb - 1) / tb, (int64_t)di.sm_count * 32);
+  auto grid_of = [&](int64_t k) { return (int)std::max<int64_t>(1, std::min<int64_t>((k + tb - 1) / tb, (int64_t)di.sm_count * 32)); };
   L2_TRY(cudaMalloc((void**)&cnt, (size_t)cs * m * 4), "alloc");
+  L2_TRY(cudaMalloc((void**)&colcnt, (size_t)n * 4), "alloc");
+  L2_TRY(cudaMalloc((void**)&blocktot, (size_t)cs * 8), "alloc");
   L2_TRY(cudaMemsetAsync(cnt, 0, (size_t)cs * m * 4, s), "memset");
-  k_l2b_count<<<grid_r, tb, 0, s>>>(m, rowptr, colidx, bw, cnt);
+  L2_TRY(cudaMemsetAsync(colcnt, 0, (size_t)n * 4, s), "memset");
+  L2_TRY(cudaMemsetAsync(blocktot, 0, (size_t)cs * 8, s), "memset");
+  k_l2b_count<<<grid_of(m), tb, 0, s>>>(m, rowptr, colidx, bw, cnt, colcnt, blocktot);
+  // the heaviest block runs last, fused
+  std::vector<unsigned long long> hbt(cs);
+  L2_TRY(cudaMemcpyAsync(hbt.data(), blocktot, (size_t)cs * 8, cudaMemcpyDeviceToHost, s), "copy");
+  // hot columns: more than max(2048, nnz / 2^16) nonzeros (FP_L2B_HOT overrides; 0 = none)
+  uint32_t thr = (uint32_t)std::max<int64_t>(2048, nnz >> 16);
+  if (const char* e = std::getenv("FP_L2B_HOT")) thr = (uint32_t)std::max<long long>(0, std::atoll(e));
+  L2_TRY(cudaMalloc((void**)&slot, (size_t)n * 4), "alloc");
+  L2_TRY(cudaMalloc((void**)&p->hcol, (size_t)kL2MaxHot * 4), "alloc");
+  L2_TRY(cudaMalloc((void**)&nhot, 4), "alloc");
+  L2_TRY(cudaMemsetAsync(nhot, 0, 4, s), "memset");
+  const bool use_hot = thr > 0;
+  if (use_hot) k_l2b_hotsel<<<grid_of(n), tb, 0, s>>>(n, colcnt, thr, slot, p->hcol, nhot);
+  unsigned hnh = 0;
+  L2_TRY(cudaMemcpyAsync(&hnh, nhot, 4, cudaMemcpyDeviceToHost, s), "copy");
+  L2_TRY(cudaStreamSynchronize(s), "sync");
+  const int nh = (int)std::min<unsigned>(hnh, (unsigned)kL2MaxHot);
+  int heavy = 0;
+  for (int b = 1; b < cs; ++b)
+    if (hbt[b] > hbt[heavy]) heavy = b;
+  // chunks
   L2_TRY(cudaMalloc((void**)&nchunk, (size_t)(nt + 1) * 8), "alloc");
   L2_TRY(cudaMalloc((void**)&nent, (size_t)(nt + 1) * 8), "alloc");
   L2_TRY(cudaMalloc((void**)&cbase, (size_t)(nt + 1) * 8), "alloc");
   L2_TRY(cudaMalloc((void**)&ebase, (size_t)(nt + 1) * 8), "alloc");
   L2_TRY(cudaMemsetAsync(nchunk + nt, 0, 8, s), "memset");
   L2_TRY(cudaMemsetAsync(nent + nt, 0, 8, s), "memset");
-  k_l2b_walk<false><<<grid_t, tb, 0, s>>>(m, cs, cnt, nchunk, nent, nullptr, nullptr, nullptr, nullptr, nullptr);
-  size_t tb_bytes = 0;
+  k_l2b_walk<false><<<grid_of(nt), tb, 0, s>>>(m, cs, heavy, rowcap, cnt, nchunk, nent, nullptr, nullptr, nullptr,
+                                               nullptr, nullptr);
+  size_t tb_bytes = 0, tmp_bytes = 0;
   L2_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, nchunk, cbase, nt + 1, s), "scan");
-  L2_TRY(cudaMalloc(&tmp, tb_bytes), "alloc");
+  tmp_bytes = tb_bytes;
+  L2_TRY(cudaMalloc(&tmp, tmp_bytes), "alloc");
   L2_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb_bytes, nchunk, cbase, nt + 1, s), "scan");
   L2_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb_bytes, nent, ebase, nt + 1, s), "scan");
-  // chunk ranges of the blocks (block b's chunks are [cbase[b ng], cbase[(b + 1) ng])) and the
-  // entries of every block (the heaviest is processed last, fused)
   std::vector<int64_t> hcb(cs + 1), heb(cs + 1);
   for (int b = 0; b <= cs; ++b) {
     L2_TRY(cudaMemcpyAsync(&hcb[b], cbase + (int64_t)b * ng, 8, cudaMemcpyDeviceToHost, s), "copy");
@@ -381,24 +511,80 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   }
   L2_TRY(cudaStreamSynchronize(s), "sync");
   const int64_t nch = hcb[cs], total = heb[cs];
-  if (total >= (int64_t)UINT32_MAX) return fail(cudaErrorInvalidValue, "too many entries for 32-bit offsets");
+  if (total >= (int64_t)UINT32_MAX * 8) return fail(cudaErrorInvalidValue, "too many entries for 32-bit offsets");
+  if (total >= (int64_t)UINT32_MAX) return fail(cudaErrorInvalidValue, "too many entries for 32-bit row offsets");
   L2_TRY(cudaMalloc((void**)&p->tile_desc, (size_t)std::max<int64_t>(nch, 1) * sizeof(uint4)), "alloc");
   L2_TRY(cudaMalloc((void**)&rowoff, (size_t)cs * m * 4), "alloc");
-  L2_TRY(cudaMalloc((void**)&rid, (size_t)cs * m), "alloc");
-  k_l2b_walk<true><<<grid_t, tb, 0, s>>>(m, cs, cnt, nullptr, nullptr, cbase, ebase, p->tile_desc, rowoff, rid);
+  L2_TRY(cudaMalloc((void**)&rid, (size_t)cs * m * 2), "alloc");
+  k_l2b_walk<true><<<grid_of(nt), tb, 0, s>>>(m, cs, heavy, rowcap, cnt, nullptr, nullptr, cbase, ebase, p->tile_desc,
+                                              rowoff, rid);
   const int64_t cap = total + 8;
-  const size_t vs = dtype_size(dtype);
   L2_TRY(cudaMalloc((void**)&p->cr, (size_t)cap * 4), "alloc");
   L2_TRY(cudaMalloc((void**)&p->val, (size_t)cap * vs), "alloc");
-  k_l2b_fill<<<(int)std::min<int64_t>((cap + tb - 1) / tb, (int64_t)di.sm_count * 32), tb, 0, s>>>(cap, p->cr,
-                                                                                                   kL2PadWord);
+  k_l2b_fill<<<grid_of(cap), tb, 0, s>>>(cap, p->cr, enc.pad());
   L2_TRY(cudaMemsetAsync(p->val, 0, (size_t)cap * vs, s), "memset");
+  // hot entries: exactly the nonzeros of the hot columns
+  int64_t nhe = 0;
+  if (nh > 0) {
+    std::vector<uint32_t> hcnt(nh);
+      L2_TRY(cudaMalloc((void**)&hkey, (size_t)nh * 4), "alloc");  // (scratch: the hot columns' counts)
+    k_l2b_gather<<<grid_of(nh), tb, 0, s>>>(nh, p->hcol, colcnt, (uint32_t*)hkey);
+    L2_TRY(cudaMemcpyAsync(hcnt.data(), hkey, (size_t)nh * 4, cudaMemcpyDeviceToHost, s), "copy");
+    L2_TRY(cudaStreamSynchronize(s), "sync");
+    cudaFree(hkey);
+    hkey = nullptr;
+    // work items: <= 256 entries of one hot column, in slot order (the sort below)
+    std::vector<uint4> items;
+    int64_t off = 0;
+    for (int k = 0; k < nh; ++k) {
+      for (uint32_t e = 0; e < hcnt[k]; e += kL2Win)
+        items.push_back(make_uint4((unsigned)(off + e), std::min<uint32_t>(kL2Win, hcnt[k] - e), (unsigned)k, 0u));
+      off += hcnt[k];
+    }
+    nhe = off;
+    L2_TRY(cudaMalloc((void**)&hkey, (size_t)nhe * 8), "alloc");
+    L2_TRY(cudaMalloc((void**)&hkey2, (size_t)nhe * 8), "alloc");
+    L2_TRY(cudaMalloc(&hv, (size_t)nhe * vs), "alloc");
+    L2_TRY(cudaMalloc((void**)&p->hval, (size_t)nhe * vs), "alloc");
+    L2_TRY(cudaMalloc((void**)&p->hrow, (size_t)nhe * 4), "alloc");
+    L2_TRY(cudaMalloc((void**)&hn, 8), "alloc");
+    L2_TRY(cudaMemsetAsync(hn, 0, 8, s), "memset");
+    L2_TRY(cudaMalloc((void**)&p->hitems, items.size() * sizeof(uint4)), "alloc");
+    L2_TRY(cudaMemcpyAsync(p->hitems, items.data(), items.size() * sizeof(uint4), cudaMemcpyHostToDevice, s), "copy");
+    L2_TRY(cudaStreamSynchronize(s), "sync");
+    p->nhitems = (int64_t)items.size();
+  }
   if (dtype == FP_F64)
-    k_l2b_scatter<double><<<grid_r, tb, 0, s>>>(m, cs, bw, rowptr, colidx, (const double*)val, rowoff, rid, p->cr,
-                                                (double*)p->val);
+    k_l2b_scatter<double><<<grid_of(m), tb, 0, s>>>(m, cs, bw, enc, rowptr, colidx, (const double*)val, rowoff, rid,
+                                                    nh > 0 ? slot : nullptr, p->cr, (double*)p->val, hkey,
+                                                    (double*)hv, hn);
   else
-    k_l2b_scatter<float><<<grid_r, tb, 0, s>>>(m, cs, bw, rowptr, colidx, (const float*)val, rowoff, rid, p->cr,
-                                               (float*)p->val);
+    k_l2b_scatter<float><<<grid_of(m), tb, 0, s>>>(m, cs, bw, enc, rowptr, colidx, (const float*)val, rowoff, rid,
+                                                   nh > 0 ? slot : nullptr, p->cr, (float*)p->val, hkey, (float*)hv,
+                                                   hn);
+  if (nhe > 0) {  // sort the hot entries by (slot, row): each column's entries contiguous, in row order
+    size_t sb = 0;
+    const int end_bit = 32 + (int)bits_for(nh + 1);
+    if (dtype == FP_F64)
+      L2_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sb, hkey, hkey2, (const double*)hv, (double*)p->hval, nhe, 0,
+                                             end_bit, s), "sort");
+    else
+      L2_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sb, hkey, hkey2, (const float*)hv, (float*)p->hval, nhe, 0,
+                                             end_bit, s), "sort");
+    if (sb > tmp_bytes) {
+      cudaFree(tmp);
+      tmp = nullptr;
+      tmp_bytes = sb;
+      L2_TRY(cudaMalloc(&tmp, tmp_bytes), "alloc");
+    }
+    if (dtype == FP_F64)
+      L2_TRY(cub::DeviceRadixSort::SortPairs(tmp, sb, hkey, hkey2, (const double*)hv, (double*)p->hval, nhe, 0,
+                                             end_bit, s), "sort");
+    else
+      L2_TRY(cub::DeviceRadixSort::SortPairs(tmp, sb, hkey, hkey2, (const float*)hv, (float*)p->hval, nhe, 0,
+                                             end_bit, s), "sort");
+    k_l2b_rows<<<grid_of(nhe), tb, 0, s>>>(nhe, hkey2, p->hrow);
+  }
   L2_TRY(cudaMalloc((void**)&p->rowdot, (size_t)std::max<int64_t>(m, 1) * 8), "alloc");
   L2_TRY(cudaStreamSynchronize(s), "sync");
 #undef L2_TRY
@@ -406,15 +592,13 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   p->mode = 1;
   p->cs = cs;
   p->bw = (int)bw;
+  p->cbits = (int)enc.cb;
   p->ntiles = nch;
   p->entries = total;
   p->groups = 0;
+  p->nhot = nh;
   p->l2cb.assign(hcb.begin(), hcb.end());
-  int heavy = 0;
-  for (int b = 1; b < cs; ++b)
-    if (heb[b + 1] - heb[b] > heb[heavy + 1] - heb[heavy]) heavy = b;
   p->heavy = heavy;
-  (void)nnz;
   return FP_OK;
 }
 
@@ -423,8 +607,9 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   const bool has_y = a.y != nullptr;
   const int64_t m = p->m, n = p->n;
   const int tb = 256;
+  const bool f64 = p->dtype == FP_F64;
   const int gn = (int)std::min<int64_t>((n + tb - 1) / tb, (int64_t)di.sm_count * 8);
-  if (p->dtype == FP_F64)
+  if (f64)
     k_l2b_init<double><<<gn, tb, 0, s>>>(n, (double*)a.w, (const double*)a.z, a.beta, a.add_beta_z ? 1 : 0,
                                          a.accumulate ? 1 : 0);
   else
@@ -438,6 +623,7 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     if (k.nch == 0) return FP_OK;
     k.desc = p->tile_desc + p->l2cb[b];
     k.col0 = (int64_t)b * p->bw;
+    k.enc = L2Enc{(unsigned)p->cbits};
     k.cr = p->cr;
     k.val = p->val;
     k.y = a.y;
@@ -446,7 +632,6 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     k.p = p->rowdot;
     k.w = a.w;
     const int grid = (int)std::min<int64_t>((k.nch + kL2NW - 1) / kL2NW, (int64_t)di.sm_count * 8);
-    const bool f64 = p->dtype == FP_F64;
 #define L2_LAUNCH(M)                                                    \
   if (f64) k_l2b<double, M><<<grid, kL2BS, 0, s>>>(k);                  \
   else k_l2b<float, M><<<grid, kL2BS, 0, s>>>(k);
@@ -468,7 +653,7 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     if (st != FP_OK) return st;
   }
   const int gm = (int)std::min<int64_t>((m + tb - 1) / tb, (int64_t)di.sm_count * 8);
-  if (p->dtype == FP_F64)
+  if (f64)
     k_l2b_q<double><<<gm, tb, 0, s>>>(m, p->rowdot, (const double*)a.v, a.alpha, has_y ? 1 : 0);
   else
     k_l2b_q<float><<<gm, tb, 0, s>>>(m, p->rowdot, (const float*)a.v, a.alpha, has_y ? 1 : 0);
@@ -476,6 +661,16 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   for (int b = 0; b < p->cs && st == FP_OK; ++b)
     if (b != p->heavy) st = pass(b, L2_SCAT);
   if (st == FP_OK) st = pass(p->heavy, has_y ? L2_SCAT_PARTIAL : L2_SCAT);
+  if (st == FP_OK && p->nhitems > 0) {
+    const int gh = (int)std::min<int64_t>((p->nhitems + kL2NW - 1) / kL2NW, (int64_t)di.sm_count * 8);
+    if (f64)
+      k_l2b_hot<double><<<gh, kL2BS, 0, s>>>(p->hitems, p->nhitems, p->hrow, (const double*)p->hval, p->hcol,
+                                             p->rowdot, (double*)a.w);
+    else
+      k_l2b_hot<float><<<gh, kL2BS, 0, s>>>(p->hitems, p->nhitems, p->hrow, (const float*)p->hval, p->hcol,
+                                            p->rowdot, (float*)a.w);
+    FP_CUDA(cudaGetLastError());
+  }
   return st;
 }
 
@@ -487,7 +682,7 @@ void l2block_launch(const Packed* p, fp_launch* L) {
   L->bs = kL2BS;
   L->grid = device_info(current_device()).sm_count * 8;
   L->cluster = p->cs;
-  L->smem_bytes = kL2NW * kL2Rows * 8;
+  L->smem_bytes = kL2NW * kL2HeavyRows * 8;
   L->blocks_per_sm = 8;
   cudaFuncAttributes fa{};
   const void* f = p->dtype == FP_F64 ? (const void*)k_l2b<double, L2_FUSED> : (const void*)k_l2b<float, L2_FUSED>;

@@ -102,6 +102,13 @@ struct Packed {
   int heavy = 0;
   std::vector<int64_t> l2cb;
   double* rowdot = nullptr;             // [m]: row dots p, then q
+  int cbits = 0;                        // column bits of the entry word
+  int nhot = 0;                         // hot columns: hcol[slot], entries hrow / hval by column,
+  int32_t* hcol = nullptr;              //   work items hitems (first entry, count, slot)
+  uint32_t* hrow = nullptr;
+  void* hval = nullptr;
+  uint4* hitems = nullptr;
+  int64_t nhitems = 0;
 };
 // variant 20 (csr_l2block.cu)
 int64_t l2block_bw(int64_t n, fp_dtype dt);

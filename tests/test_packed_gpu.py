@@ -314,16 +314,21 @@ def l2_plan(dev, monkeypatch, rp, ci, va, n, bw, tdt):
 
 @pytest.mark.parametrize("dt", ["f32", "f64"])
 @pytest.mark.parametrize("n,bw", [(5000, 1000), (20_000, 3001), (4096, 4096)])
-@pytest.mark.parametrize("lengths", [("powerlaw", 2.5, 13.64), ("binomial", 0.004), ("uniform", 0, 1500)])
-def test_l2block_integer_twin_bitexact(cuda_dev, monkeypatch, dt, n, bw, lengths):
+@pytest.mark.parametrize("lengths,skew", [(("powerlaw", 2.5, 13.64), 0), (("binomial", 0.004), 0),
+                                          (("uniform", 0, 1500), 0), (("powerlaw", 2.5, 9.5), 2)])
+@pytest.mark.parametrize("hot", [None, "40"])
+def test_l2block_integer_twin_bitexact(cuda_dev, monkeypatch, dt, n, bw, lengths, skew, hot):
     """Variant 20 (csr_l2block.cu): the columns in blocks of bw (here small, so that a test-sized
     matrix spans several blocks, a ragged last block, one block), row dots accumulated over the
     blocks, the heaviest block fused (q and its scatter from the same registers), the others
-    re-read; rows longer than a 256-entry chunk split into partial chunks; empty rows.  Integer
-    twins: every sum exact in fp64 / below 2^24 in fp32, so bit-exact whatever the red order."""
+    re-read; rows longer than a 256-entry chunk split into partial chunks; empty rows; Zipf-like
+    columns (skew); hot columns (more than `hot` nonzeros: scattered by column).  Integer twins:
+    every sum exact in fp64 / below 2^24 in fp32, so bit-exact whatever the red order."""
     m = 6_007 if lengths[0] != "uniform" else 1_501
     tdt = torch.float64 if dt == "f64" else torch.float32
-    rp, ci, va = synth.csr(m, n, dt, lengths, kind="int_pm12", seed=31)
+    if hot is not None:
+        monkeypatch.setenv("FP_L2B_HOT", hot)
+    rp, ci, va = synth.csr(m, n, dt, lengths, kind="int_pm12", seed=31, col_skew=skew)
     y = synth.vector(n, dt, kind="int_small", seed=31, stream=synth.S_Y)
     v = synth.vector(m, dt, kind="int_pos", seed=31, stream=synth.S_V)
     z = synth.vector(n, dt, kind="int_small", seed=31, stream=synth.S_Z)
