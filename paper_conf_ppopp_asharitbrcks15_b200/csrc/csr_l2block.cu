@@ -100,7 +100,9 @@ __device__ __forceinline__ void l2_ldv(const double* p, double (&x)[8]) {
   asm("ld.global.nc.L1::no_allocate.L2::evict_first.v4.f64 {%0,%1,%2,%3}, [%4];"
       : "=d"(x[4]), "=d"(x[5]), "=d"(x[6]), "=d"(x[7]) : "l"(p + 4));
 }
-// y of the block: kept in L2 (an evict_last cache policy), not in L1 (little reuse per SM)
+// y of the block: kept in L2 (an evict_last cache policy) and cached in L1 -- the hot columns'
+// y values are read by most rows: without L1 every such read goes to the one L2 slice that
+// holds the word (K1's fused block: 3.99 ms with L1::no_allocate, ncu r02c)
 __device__ __forceinline__ uint64_t l2_keep_policy() {
   uint64_t pol;
   asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
@@ -108,12 +110,12 @@ __device__ __forceinline__ uint64_t l2_keep_policy() {
 }
 __device__ __forceinline__ float l2_ldy(const float* p, uint64_t pol) {
   float v;
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+  asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
   return v;
 }
 __device__ __forceinline__ double l2_ldy(const double* p, uint64_t pol) {
   double v;
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol));
+  asm("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol));
   return v;
 }
 
@@ -274,18 +276,36 @@ __global__ void k_l2b_init(int64_t n, T* __restrict__ w, const T* __restrict__ z
 }
 
 // ---------------------------------------------------------------- the copy (pack time)
-// (1) entries of row r in block b (cnt[b m + r]), entries of column c (colcnt[c]), per block
+// (1) entries of row r in block b (cnt[b m + r]) and of column c (colcnt[c]); a warp per row
+// (its lanes on distinct columns of the row)
 __global__ void k_l2b_count(int64_t m, const int64_t* __restrict__ rowptr, const int32_t* __restrict__ colidx,
-                            int64_t bw, uint32_t* __restrict__ cnt, uint32_t* __restrict__ colcnt,
-                            unsigned long long* __restrict__ blocktot) {
-  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
+                            int64_t bw, uint32_t* __restrict__ cnt, uint32_t* __restrict__ colcnt) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
+  for (int64_t r = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); r < m; r += nw) {
     const int64_t e = rowptr[r + 1];
-    for (int64_t i = rowptr[r]; i < e; ++i) {
-      const int64_t b = colidx[i] / bw;
-      cnt[b * m + r] += 1u;
+    for (int64_t i = rowptr[r] + lane; i < e; i += 32) {
+      atomicAdd(cnt + (int64_t)(colidx[i] / bw) * m + r, 1u);
       atomicAdd(colcnt + colidx[i], 1u);
-      atomicAdd(blocktot + b, 1ull);
     }
+  }
+}
+// entries per block: sum of cnt over the rows (one CTA per (block, slice), a red per CTA)
+__global__ void k_l2b_blocktot(int64_t m, const uint32_t* __restrict__ cnt, unsigned long long* __restrict__ tot) {
+  const int b = blockIdx.y;
+  unsigned long long s = 0;
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x)
+    s += cnt[(int64_t)b * m + r];
+  for (int d = 16; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
+  if ((threadIdx.x & 31) == 0) atomicAdd(tot + b, s);
+}
+// hot entries of each row (their offsets: an exclusive scan)
+__global__ void k_l2b_hotrows(int64_t m, const int64_t* __restrict__ rowptr, const int32_t* __restrict__ colidx,
+                              const int32_t* __restrict__ slot, int64_t* __restrict__ hr) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
+    int64_t k = 0;
+    for (int64_t i = rowptr[r]; i < rowptr[r + 1]; ++i) k += slot[colidx[i]] >= 0;
+    hr[r] = k;
   }
 }
 
@@ -373,11 +393,12 @@ __global__ void k_l2b_scatter(int64_t m, int cs, int64_t bw, L2Enc enc, const in
                               const int32_t* __restrict__ colidx, const V* __restrict__ val,
                               const uint32_t* __restrict__ rowoff, const uint16_t* __restrict__ rid,
                               const int32_t* __restrict__ slot, uint32_t* __restrict__ cr, V* __restrict__ pval,
-                              unsigned long long* __restrict__ hkey, V* __restrict__ hv, unsigned long long* __restrict__ hn) {
+                              unsigned long long* __restrict__ hkey, V* __restrict__ hv, const int64_t* __restrict__ hroff) {
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (int64_t)gridDim.x * blockDim.x) {
     uint32_t k[kL2MaxBlocks];
     for (int b = 0; b < cs; ++b) k[b] = 0;
     const int64_t e = rowptr[r + 1];
+    int64_t h = slot ? hroff[r] : 0;
     for (int64_t i = rowptr[r]; i < e; ++i) {
       const int col = colidx[i];
       const int b = (int)(col / bw);
@@ -387,9 +408,8 @@ __global__ void k_l2b_scatter(int64_t m, int cs, int64_t bw, L2Enc enc, const in
                 ((uint32_t)rid[(int64_t)b * m + r] << enc.ridshift());
       pval[pos] = val[i];
       if (sl >= 0) {
-        const unsigned long long h = atomicAdd(hn, 1ull);
         hkey[h] = ((unsigned long long)sl << 32) | (unsigned long long)r;
-        hv[h] = val[i];
+        hv[h++] = val[i];
       }
     }
   }
@@ -443,11 +463,11 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   unsigned long long *blocktot = nullptr, *hkey = nullptr, *hkey2 = nullptr, *hn = nullptr;
   void *hv = nullptr, *tmp = nullptr;
   unsigned* nhot = nullptr;
-  int64_t *nchunk = nullptr, *nent = nullptr, *cbase = nullptr, *ebase = nullptr;
+  int64_t *nchunk = nullptr, *nent = nullptr, *cbase = nullptr, *ebase = nullptr, *hroff = nullptr;
   auto cleanup = [&]() {
     for (void* b : {(void*)cnt, (void*)colcnt, (void*)rowoff, (void*)rid, (void*)slot, (void*)blocktot, (void*)hkey,
                     (void*)hkey2, (void*)hn, hv, tmp, (void*)nhot, (void*)nchunk, (void*)nent, (void*)cbase,
-                    (void*)ebase})
+                    (void*)ebase, (void*)hroff})
       if (b) cudaFree(b);
   };
   auto fail = [&](cudaError_t e, const char* what) {
@@ -469,13 +489,14 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   L2_TRY(cudaMemsetAsync(cnt, 0, (size_t)cs * m * 4, s), "memset");
   L2_TRY(cudaMemsetAsync(colcnt, 0, (size_t)n * 4, s), "memset");
   L2_TRY(cudaMemsetAsync(blocktot, 0, (size_t)cs * 8, s), "memset");
-  k_l2b_count<<<grid_of(m), tb, 0, s>>>(m, rowptr, colidx, bw, cnt, colcnt, blocktot);
+  k_l2b_count<<<grid_of(m * 32), tb, 0, s>>>(m, rowptr, colidx, bw, cnt, colcnt);
+  k_l2b_blocktot<<<dim3((unsigned)std::min<int64_t>((m + tb - 1) / tb, 256), (unsigned)cs), tb, 0, s>>>(m, cnt, blocktot);
   // the heaviest block runs last, fused
   std::vector<unsigned long long> hbt(cs);
   L2_TRY(cudaMemcpyAsync(hbt.data(), blocktot, (size_t)cs * 8, cudaMemcpyDeviceToHost, s), "copy");
   // hot columns: more than max(2048, nnz / 2^16) nonzeros (FP_L2B_HOT overrides; 0 = none)
   uint32_t thr = (uint32_t)std::max<int64_t>(2048, nnz >> 16);
-  if (const char* e = std::getenv("FP_L2B_HOT")) thr = (uint32_t)std::max<long long>(0, std::atoll(e));
+  if (const char* e = std::getenv("FP_L2B_HOT"); e && *e) thr = (uint32_t)std::max<long long>(0, std::atoll(e));
   L2_TRY(cudaMalloc((void**)&slot, (size_t)n * 4), "alloc");
   L2_TRY(cudaMalloc((void**)&p->hcol, (size_t)kL2MaxHot * 4), "alloc");
   L2_TRY(cudaMalloc((void**)&nhot, 4), "alloc");
@@ -547,8 +568,20 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
     L2_TRY(cudaMalloc(&hv, (size_t)nhe * vs), "alloc");
     L2_TRY(cudaMalloc((void**)&p->hval, (size_t)nhe * vs), "alloc");
     L2_TRY(cudaMalloc((void**)&p->hrow, (size_t)nhe * 4), "alloc");
-    L2_TRY(cudaMalloc((void**)&hn, 8), "alloc");
-    L2_TRY(cudaMemsetAsync(hn, 0, 8, s), "memset");
+    // each row's hot entries at an offset of its own (no shared counter)
+    L2_TRY(cudaMalloc((void**)&hn, (size_t)(m + 1) * 8), "alloc");
+    L2_TRY(cudaMalloc((void**)&hroff, (size_t)(m + 1) * 8), "alloc");
+    L2_TRY(cudaMemsetAsync(hn + m, 0, 8, s), "memset");
+    k_l2b_hotrows<<<grid_of(m), tb, 0, s>>>(m, rowptr, colidx, slot, (int64_t*)hn);
+    size_t hb = 0;
+    L2_TRY(cub::DeviceScan::ExclusiveSum(nullptr, hb, (int64_t*)hn, hroff, m + 1, s), "scan");
+    if (hb > tmp_bytes) {
+      cudaFree(tmp);
+      tmp = nullptr;
+      tmp_bytes = hb;
+      L2_TRY(cudaMalloc(&tmp, tmp_bytes), "alloc");
+    }
+    L2_TRY(cub::DeviceScan::ExclusiveSum(tmp, hb, (int64_t*)hn, hroff, m + 1, s), "scan");
     L2_TRY(cudaMalloc((void**)&p->hitems, items.size() * sizeof(uint4)), "alloc");
     L2_TRY(cudaMemcpyAsync(p->hitems, items.data(), items.size() * sizeof(uint4), cudaMemcpyHostToDevice, s), "copy");
     L2_TRY(cudaStreamSynchronize(s), "sync");
@@ -557,11 +590,11 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   if (dtype == FP_F64)
     k_l2b_scatter<double><<<grid_of(m), tb, 0, s>>>(m, cs, bw, enc, rowptr, colidx, (const double*)val, rowoff, rid,
                                                     nh > 0 ? slot : nullptr, p->cr, (double*)p->val, hkey,
-                                                    (double*)hv, hn);
+                                                    (double*)hv, hroff);
   else
     k_l2b_scatter<float><<<grid_of(m), tb, 0, s>>>(m, cs, bw, enc, rowptr, colidx, (const float*)val, rowoff, rid,
                                                    nh > 0 ? slot : nullptr, p->cr, (float*)p->val, hkey, (float*)hv,
-                                                   hn);
+                                                   hroff);
   if (nhe > 0) {  // sort the hot entries by (slot, row): each column's entries contiguous, in row order
     size_t sb = 0;
     const int end_bit = 32 + (int)bits_for(nh + 1);

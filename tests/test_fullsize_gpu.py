@@ -1,5 +1,6 @@
-"""Full-size parity at BASELINE.json's configs (C1-C5), in the launch configuration bench.py
-times (same entry point, same plan): the device-generated input is copied to the host and
+"""Full-size parity at BASELINE.json's configs (C1-C5, plus S3 and the KDD-shaped K1), in the
+launch configuration bench.py times (same entry point, same plan: the packed copy for CSR) and
+through the unpacked chooser plan: the device-generated input is copied to the host and
 the fp64 oracle evaluates the whole matrix on the host cores.  fp64 integer twins of C1, C3
 and C5 are exact in any summation order and must match bit for bit; the fp32 configs (C2,
 C4) are checked against the north_star tolerance."""
@@ -71,6 +72,41 @@ def test_fullsize_integer_twin_bitexact(cuda_dev, name):
     del d
     torch.cuda.empty_cache()
     assert_bitexact(w, ref, f"{name} integer twin")
+
+
+def run_gpu_packed(cfg, d):
+    """bench.py's CSR launch: a plan (fp_csr_plan_create) with its packed copy (fp_csr_plan_pack:
+    variant 19's shared-memory column blocks, or variant 20's L2 blocks when n is wider)."""
+    plan = fp.CsrPlan(d["rp"], d["ci"], cfg["n"], d["va"].dtype)
+    plan.pack(d["va"])
+    w = plan(None, d["y"], d["v"], d["z"], cfg["alpha"], cfg["beta"])
+    torch.cuda.synchronize()
+    return w.cpu(), plan.launch.variant
+
+
+@pytest.mark.parametrize("name,variant", [("C3", 19), ("C4", 19), ("S3", 19), ("K1", 20)])
+def test_fullsize_packed_parity(cuda_dev, name, variant):
+    """The packed plans bench.py times, at full size, against the fp64 oracle (north_star
+    tolerance); K1 is the KDD-shaped 15M x 29.9M matrix on variant 20."""
+    cfg, d = gen(name, cuda_dev)
+    w, var = run_gpu_packed(cfg, d)
+    assert var == variant
+    ref, mag = run_oracle(cfg, d)
+    del d
+    torch.cuda.empty_cache()
+    assert_parity(w, ref, mag, w.dtype, f"{name} packed full size")
+
+
+@pytest.mark.parametrize("name", ["C3", "K1"])
+def test_fullsize_packed_integer_twin_bitexact(cuda_dev, name):
+    """fp64 packed plans on integer twins: exact in any order (K1: the hot-column sums stay below
+    2^53), so bit-exact against the oracle."""
+    cfg, d = gen(name, cuda_dev, kind="int_pm12")
+    w, _ = run_gpu_packed(cfg, d)
+    ref, _ = run_oracle(cfg, d)
+    del d
+    torch.cuda.empty_cache()
+    assert_bitexact(w, ref, f"{name} packed integer twin")
 
 
 def test_generator_host_equals_device(cuda_dev):
