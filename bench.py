@@ -362,8 +362,12 @@ def run_gpu(args):
             launches_per_step = 3
         elif plan.variant == 19:  # the packed pass + the finalize
             launches_per_step = 2
-        elif plan.variant == 20:  # w init, a dot pass per block (the last fused), q, a scatter pass per block
-            launches_per_step = 2 * int(plan.cluster) + 2 if inp["y"] is not None else int(plan.cluster) + 2
+        elif plan.variant == 20:  # w init, a dot launch per other block, fused, q, a scatter launch per
+            # other block, the fused block's partial chunks, hot columns (+ a memset)
+            nb = int(plan.cluster) - 1
+            if os.environ.get("FP_L2B_MERGE", "0") not in ("", "0"):
+                nb = 2
+            launches_per_step = 2 * nb + 5 if inp["y"] is not None else nb + 4
         elif plan.variant in (4, 7, 16):
             s_b = 8 if cfg["dtype"] == "f64" else 4
             nrep = int(os.environ.get("FP_L2_REPLICAS", "0")) or (8 if 8 * n * s_b <= (16 << 20) else 1)

@@ -69,9 +69,9 @@ struct L2Enc {
 };
 
 struct L2Args {
-  const uint4* desc;    // this block's chunks: (offset / 8, length | rows << 16, first row, flags)
+  const uint4* desc;    // chunks (offset / 8, length | rows << 16, first row, flags | block << 8)
   int64_t nch;
-  int64_t col0;         // first column of the block
+  int64_t bw;           // columns per block (block b starts at column b bw)
   L2Enc enc;
   const uint32_t* cr;
   const void* val;      // T
@@ -132,10 +132,10 @@ __global__ void __launch_bounds__(kL2BS) k_l2b(const L2Args a) {
   __shared__ double s_rs[kL2NW][kL2HeavyRows];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   double* rs = s_rs[wi];
-  const T* __restrict__ y = reinterpret_cast<const T*>(a.y) + a.col0;
+  const T* __restrict__ yall = reinterpret_cast<const T*>(a.y);
   const T* __restrict__ vv = reinterpret_cast<const T*>(a.v);
   const T* __restrict__ val = reinterpret_cast<const T*>(a.val);
-  T* w = reinterpret_cast<T*>(a.w) + a.col0;
+  T* wall = reinterpret_cast<T*>(a.w);
   double* p = a.p;
   const uint32_t cmask = a.enc.colmask(), hot = a.enc.hotbit();
   const unsigned rsh = a.enc.ridshift();
@@ -148,6 +148,9 @@ __global__ void __launch_bounds__(kL2BS) k_l2b(const L2Args a) {
     if (MODE == L2_SCAT_PARTIAL && !partial) continue;
     const int len = (int)(D.y & 0xFFFFu), rows = (int)(D.y >> 16);
     double* pr0 = p + D.z;
+    const int64_t col0 = (int64_t)(D.w >> 8) * a.bw;  // the chunk's block (a launch may span several)
+    const T* __restrict__ y = yall + col0;
+    T* w = wall + col0;
     const int o = 8 * lane;
     uint32_t cw[8];
     T xv[8];
@@ -345,7 +348,9 @@ __global__ void k_l2b_walk(int64_t m, int cs, int heavy, int rowcap, const uint3
     int64_t r0 = -1, last_row = -1;
     int len = 0;
     auto emit = [&](int64_t first, int rows, int l, unsigned flags) {
-      if (WRITE) desc[ci++] = make_uint4((unsigned)(ei / 8), (unsigned)l | ((unsigned)rows << 16), (unsigned)first, flags);
+      if (WRITE)
+        desc[ci++] = make_uint4((unsigned)(ei / 8), (unsigned)l | ((unsigned)rows << 16), (unsigned)first,
+                                flags | ((unsigned)b << 8));
       ++nc;
       const int64_t al = (l + 7) & ~7;
       ne += al;
@@ -650,12 +655,14 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
                                         a.accumulate ? 1 : 0);
   FP_CUDA(cudaGetLastError());
   if (has_y) FP_CUDA(cudaMemsetAsync(p->rowdot, 0, (size_t)m * 8, s));
-  auto pass = [&](int b, int mode) -> fp_status {
-    L2Args k{};
-    k.nch = p->l2cb[b + 1] - p->l2cb[b];
-    if (k.nch == 0) return FP_OK;
-    k.desc = p->tile_desc + p->l2cb[b];
-    k.col0 = (int64_t)b * p->bw;
+  // one launch per phase over a range of chunks [c0, c1): the chunks are stored block by block
+  // and a grid-stride loop walks them in order, so the SMs work on one or two blocks at a time
+  // (their y / w stay in L2) without a launch per block
+  auto pass = [&](int64_t c0, int64_t c1, int mode) -> fp_status {
+    L2Args k{};  // (an empty range still launches: a fixed launch count per call)
+    k.nch = std::max<int64_t>(0, c1 - c0);
+    k.desc = p->tile_desc + c0;
+    k.bw = p->bw;
     k.enc = L2Enc{(unsigned)p->cbits};
     k.cr = p->cr;
     k.val = p->val;
@@ -664,7 +671,7 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     k.alpha = a.alpha;
     k.p = p->rowdot;
     k.w = a.w;
-    const int grid = (int)std::min<int64_t>((k.nch + kL2NW - 1) / kL2NW, (int64_t)di.sm_count * 8);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((k.nch + kL2NW - 1) / kL2NW, (int64_t)di.sm_count * 8));
 #define L2_LAUNCH(M)                                                    \
   if (f64) k_l2b<double, M><<<grid, kL2BS, 0, s>>>(k);                  \
   else k_l2b<float, M><<<grid, kL2BS, 0, s>>>(k);
@@ -678,11 +685,28 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     FP_CUDA(cudaGetLastError());
     return FP_OK;
   };
+  const std::vector<int64_t>& cb = p->l2cb;
+  const int H = p->heavy, cs = p->cs;
+  static const bool merge = [] {  // FP_L2B_MERGE=1: one launch per phase over all blocks (measurement)
+    const char* e = std::getenv("FP_L2B_MERGE");
+    return e && std::atoi(e) != 0;
+  }();
+  auto others = [&](int mode) -> fp_status {  // every block but the fused one
+    if (merge) {
+      fp_status st = pass(cb[0], cb[H], mode);
+      return st != FP_OK ? st : pass(cb[H + 1], cb[cs], mode);
+    }
+    for (int b = 0; b < cs; ++b)
+      if (b != H) {
+        fp_status st = pass(cb[b], cb[b + 1], mode);
+        if (st != FP_OK) return st;
+      }
+    return FP_OK;
+  };
   fp_status st = FP_OK;
   if (has_y) {
-    for (int b = 0; b < p->cs && st == FP_OK; ++b)
-      if (b != p->heavy) st = pass(b, L2_DOT);
-    if (st == FP_OK) st = pass(p->heavy, L2_FUSED);
+    st = others(L2_DOT);
+    if (st == FP_OK) st = pass(cb[H], cb[H + 1], L2_FUSED);
     if (st != FP_OK) return st;
   }
   const int gm = (int)std::min<int64_t>((m + tb - 1) / tb, (int64_t)di.sm_count * 8);
@@ -691,11 +715,10 @@ fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
   else
     k_l2b_q<float><<<gm, tb, 0, s>>>(m, p->rowdot, (const float*)a.v, a.alpha, has_y ? 1 : 0);
   FP_CUDA(cudaGetLastError());
-  for (int b = 0; b < p->cs && st == FP_OK; ++b)
-    if (b != p->heavy) st = pass(b, L2_SCAT);
-  if (st == FP_OK) st = pass(p->heavy, has_y ? L2_SCAT_PARTIAL : L2_SCAT);
-  if (st == FP_OK && p->nhitems > 0) {
-    const int gh = (int)std::min<int64_t>((p->nhitems + kL2NW - 1) / kL2NW, (int64_t)di.sm_count * 8);
+  st = others(L2_SCAT);
+  if (st == FP_OK) st = pass(cb[H], cb[H + 1], has_y ? L2_SCAT_PARTIAL : L2_SCAT);
+  if (st == FP_OK) {
+    const int gh = (int)std::max<int64_t>(1, std::min<int64_t>((p->nhitems + kL2NW - 1) / kL2NW, (int64_t)di.sm_count * 8));
     if (f64)
       k_l2b_hot<double><<<gh, kL2BS, 0, s>>>(p->hitems, p->nhitems, p->hrow, (const double*)p->hval, p->hcol,
                                              p->rowdot, (double*)a.w);
