@@ -214,6 +214,7 @@ struct PkTileRes {
 };
 
 struct Pk1Args {
+  int64_t m;
   int64_t n;
   int64_t ntiles;
   int ns;                        // tile slots per warp in the shared-memory ring (0: no ring)
@@ -272,7 +273,8 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
   constexpr bool F64 = sizeof(T) == 8;
   constexpr int QB = F64 ? 50 : 26;  // bits of the first round's largest term
   constexpr int TS = (int)sizeof(T);
-  constexpr int SLOT_CW = 256 * 4, SLOT = 256 * (4 + TS);
+  // a slot: cw (256 words) | values (256) | v of the tile's rows (a 16-byte aligned superset)
+  constexpr int SLOT_CW = 256 * 4, SLOT_V = 256 * (4 + TS), SLOT = SLOT_V + kPkRows * TS + 16;
   constexpr int NV = 8 * TS / 16;    // 16-byte pieces of a lane's 8 values
   extern __shared__ __align__(128) unsigned char pk_smem[];
   __shared__ unsigned s_tmax;
@@ -316,6 +318,10 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
   const T alpha = (T)a.alpha;
   double* const spill = a.spill;
   const uint32_t padw = pk1_pad_word(n);
+  // v rides with the tile's copy when 16-byte aligned: rows whose v lies below vlim (the last
+  // 16-byte boundary of v) come from the slot, the few beyond it from global memory
+  const bool vring = vv != nullptr && NS > 0 && ((uintptr_t)vv & 15u) == 0;
+  const int64_t vlim = ((int64_t)a.m * TS) & ~(int64_t)15;
   auto seg_len = [](const uint4& D) { return (int)(D.y & 0x1FFFFFFu); };
   auto seg_rows = [](const uint4& D) { return (int)(D.y >> 25); };
 
@@ -345,14 +351,18 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     if (lane == 0) {
       const unsigned len = Di.y & 0x1FFFFFFu, len8 = (len + 7u) & ~7u;
       const unsigned cwb = len <= 256 ? len8 * 4u : 0u;
+      int64_t v0b = (int64_t)Di.z * TS & ~(int64_t)15;
+      const int64_t v1b = std::min<int64_t>(((int64_t)(Di.z + (Di.y >> 25)) * TS + 15) & ~(int64_t)15, vlim);
+      const unsigned vb = (vring && cwb && v1b > v0b) ? (unsigned)(v1b - v0b) : 0u;
       uint64_t* b = &s_bar[warp][s];
       fpd::fence_proxy_async_smem();  // this warp's reads of the slot precede the copy's writes
-      fpd::mbar_arrive_expect_tx(b, cwb + cwb / 4u * TS);
+      fpd::mbar_arrive_expect_tx(b, cwb + cwb / 4u * TS + vb);
       if (cwb) {
         unsigned char* slot = ring + (size_t)s * SLOT;
         const int64_t e0 = (int64_t)Di.x * 8;
         fpd::bulk_g2s(slot, crp + e0, cwb, b);
         fpd::bulk_g2s(slot + SLOT_CW, val + e0, cwb / 4u * TS, b);
+        if (vb) fpd::bulk_g2s(slot + SLOT_V, reinterpret_cast<const unsigned char*>(vv) + v0b, vb, b);
       }
     }
   };
@@ -485,20 +495,18 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     }
   };
 
-  // prologue: the first NS tiles in flight; v of tile 0 in registers
+  // prologue: the first NS tiles in flight
   for (int i = 0; i < NS; ++i) issue(i, i);
-  T vn0 = T(0), vn1 = T(0);
-  auto load_v = [&](int i) {  // v of tile i's rows `lane`, `lane + 32` (one tile ahead)
-    vn0 = vn1 = T(0);
-    if (i < nt) {
-      const uint4 Di = desc_of(i);
-      const int nr = seg_rows(Di);
-      const T* vp = vv + (int)Di.z;
-      vn0 = lane < nr ? (vv ? __ldg(vp + lane) : T(1)) : T(0);
-      vn1 = lane + 32 < nr ? (vv ? __ldg(vp + lane + 32) : T(1)) : T(0);
+  // v of row D.z + k of a tile (k < rows): from the slot when it came with the copy
+  auto v_of = [&](const uint4& D, int k, bool from_slot, int s) {
+    if (!vv) return T(1);
+    const int64_t row = (int64_t)D.z + k;
+    if (from_slot && (row + 1) * TS <= vlim) {
+      const int64_t v0b = (int64_t)D.z * TS & ~(int64_t)15;
+      return pk_lds_v(ring_base + (unsigned)s * SLOT + SLOT_V + (unsigned)(row * TS - v0b), T(0));
     }
+    return __ldg(vv + row);
   };
-  load_v(0);
   int slot = 0;
   unsigned par = 0;
 
@@ -510,14 +518,15 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     D = desc_of(j);
     const int len = seg_len(D);
     one = NS > 0 && len <= 256;
-    const T v0 = vn0, v1 = vn1;
     if (one) {
       fpd::mbar_wait(&s_bar[warp][slot], par);
       win_smem(slot, ((len + 7) & ~7) >> 3, cw, xv);
     } else if (len <= 256) {
       win_glob(D, 0, cw, xv);
     }
-    load_v(j + 1);
+    const int nr = seg_rows(D);
+    const T v0 = lane < nr ? v_of(D, lane, one && vring, slot) : T(0);
+    const T v1 = lane + 32 < nr ? v_of(D, lane + 32, one && vring, slot) : T(0);
     const bool reg = len <= 256;  // the window is in registers (else streamed)
     T q0, q1;
     if constexpr (YM != 0) {
@@ -1335,7 +1344,7 @@ const void* pk1_pick_bs(fp_dtype dt, bool has_y) {
 const void* pk1_pick(fp_dtype dt, bool has_y, int bs) {
   return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y) : (bs == 768 ? pk1_pick_bs<768>(dt, has_y) : pk1_pick_bs<512>(dt, has_y));
 }
-size_t pk1_slot_bytes(fp_dtype dt) { return (size_t)256 * (4 + dtype_size(dt)); }
+size_t pk1_slot_bytes(fp_dtype dt) { return (size_t)256 * (4 + dtype_size(dt)) + (size_t)kPkRows * dtype_size(dt) + 16; }
 size_t pk1_smem_n(int64_t n, fp_dtype dt, bool has_y, int bs, int ns) {
   const size_t ts = dtype_size(dt);
   const size_t ys = has_y ? (size_t)((n + 4) & ~3) * ts : 0;
@@ -1604,6 +1613,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     const void* f1 = pk1_pick(p->dtype, has_y, p->bs);
     set_max_dynamic_smem(f1);
     Pk1Args k{};
+    k.m = p->m;
     k.n = p->n;
     k.ntiles = p->ntiles;
     k.ns = p->ns1;
