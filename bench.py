@@ -71,7 +71,7 @@ def traffic_for(config, variant):
     return e.get("dram_bytes_per_step", e.get("dram_bytes_per_launch")), src
 
 
-def second_ceiling(cfg, plan, nnz, kern_ms, dev):
+def second_ceiling(cfg, plan, nnz, kern_ms, dev, detail=None):
     """SURVEY 8(d) C4 'second ceiling': the random on-chip accesses of the CSR paths (y gathers
     that miss the shared-memory copy of y, w updates) at the rates the device sustains, measured
     live by fp_probe_rates in this run.  floor_ms = the time those accesses alone need;
@@ -95,10 +95,12 @@ def second_ceiling(cfg, plan, nnz, kern_ms, dev):
         what = ("y gathers from shared memory (rate measured on fp64 words, an upper bound for fp32) + one "
                 "native int32 shared atomic per nonzero")
     elif v == 20:  # L2-sized column blocks: every y gather and w red of a block pass hits L2
-        ops = {"l2_gathers": nnz, "l2_reds": nnz}
-        floor = nnz / r["gather_l2"] + nnz / r["red_l2"]
-        what = ("one y gather + one fp red.global per nonzero, both into the L2-resident column block "
-                "(the blocks run one after the other)")
+        hot = int((detail or {}).get("hot_entries", 0))
+        ops = {"l2_gathers": nnz - hot, "l2_reds": nnz - hot, "hot_entries_by_column": hot}
+        floor = (nnz - hot) / r["gather_l2"] + (nnz - hot) / r["red_l2"]
+        what = ("one y gather + one fp red.global per nonzero into the L2-resident column block (the blocks "
+                "run one after the other); the hot columns' nonzeros are summed by column (one red per 256) "
+                "and their y words are L1 hits, so they are left out; reds measured on fp32 words")
     elif v in (4, 7, 16, 17):
         prefix = min(n, int(plan.smem_bytes) // s) if v in (16, 17) else 0
         g = int(nnz * (1.0 - prefix / n))
@@ -294,6 +296,7 @@ def run_gpu(args):
     plan = None
     plan_ms = None
     pack_info = None
+    pack_detail = None
     if name == "C5":
         iters = args.cg_iters
 
@@ -345,6 +348,8 @@ def run_gpu(args):
             pack_ms = (time.perf_counter() - t0) * 1e3
             if packed:
                 pack_info = dict(cplan.pack_info, pack_ms=round(pack_ms, 1))
+                pack_detail = cplan.pack_detail
+                pack_info["detail"] = pack_detail
 
         def step():
             if comm is None:
@@ -363,11 +368,10 @@ def run_gpu(args):
         elif plan.variant == 19:  # the packed pass + the finalize
             launches_per_step = 2
         elif plan.variant == 20:  # w init, a dot launch per other block, fused, q, a scatter launch per
-            # other block, the fused block's partial chunks, hot columns (+ a memset)
-            nb = int(plan.cluster) - 1
+            # other block, the fused block's partial chunks, hot columns (+ a memset): the library's count
+            launches_per_step = int(pack_detail["launches"])
             if os.environ.get("FP_L2B_MERGE", "0") not in ("", "0"):
-                nb = 2
-            launches_per_step = 2 * nb + 5 if inp["y"] is not None else nb + 4
+                launches_per_step = 9
         elif plan.variant in (4, 7, 16):
             s_b = 8 if cfg["dtype"] == "f64" else 4
             nrep = int(os.environ.get("FP_L2_REPLICAS", "0")) or (8 if 8 * n * s_b <= (16 << 20) else 1)
@@ -455,7 +459,7 @@ def run_gpu(args):
     achieved = alg_local * passes_per_step / (kern_ms / 1e3) / 1e9   # per-GPU kernel bytes / kernel time
     variant = None if plan is None else int(plan.variant)
     traffic, traffic_src = traffic_for(name, variant)
-    sc = None if world > 1 else second_ceiling(cfg, plan, nnz_all or 0, kern_ms, dev)
+    sc = None if world > 1 else second_ceiling(cfg, plan, nnz_all or 0, kern_ms, dev, pack_detail)
     frac = achieved / peak
     # what binds: HBM when the step runs near the copy peak; else the random on-chip accesses
     # when they alone account for most of the step; else latency / issue (profiles/)

@@ -91,6 +91,7 @@ _SIGS = {
     "fp_csr_plan_pack": (_int, [_vp, _vp, _vp]),
     "fp_csr_plan_dist": (_int, [_vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _vp]),
     "fp_csr_plan_pack_info": (_int, [_vp, _P(_i64), _P(_i64), _P(_int), _P(_int)]),
+    "fp_csr_plan_pack_detail": (_int, [_vp, _P(_i64)]),
     "fp_dense_host": (_int, [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_csr_host": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _dbl, _dbl, _vp, _int, _int]),
     "fp_release_workspace": (_int, []),
@@ -287,6 +288,15 @@ class CsrPlan:
         _call("fp_csr_plan_pack_info", self._h, ctypes.byref(nt), ctypes.byref(ne), ctypes.byref(cs),
               ctypes.byref(gr))
         return {"tiles": nt.value, "entries": ne.value, "blocks": cs.value, "groups": gr.value}
+
+    @property
+    def pack_detail(self):
+        """fp_csr_plan_pack_detail: what one exec of the packed copy does (the roofline's inputs)."""
+        out = (ctypes.c_int64 * 8)()
+        _call("fp_csr_plan_pack_detail", self._h, out)
+        keys = ("variant", "blocks", "fused_block", "hot_columns", "hot_entries", "entries_streamed",
+                "launches", "reserved")
+        return dict(zip(keys, (int(x) for x in out)))
 
     def __call__(self, val, y=None, v=None, z=None, alpha=1.0, beta=0.0, w=None, stream=None):
         """Eq. (1) on the plan's matrix with values ``val``; ``val=None`` uses the packed copy."""

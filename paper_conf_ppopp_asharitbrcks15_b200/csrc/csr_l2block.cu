@@ -637,7 +637,28 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
   p->nhot = nh;
   p->l2cb.assign(hcb.begin(), hcb.end());
   p->heavy = heavy;
+  p->hot_entries = nhe;
+  p->heavy_entries = heb[heavy + 1] - heb[heavy];
   return FP_OK;
+}
+
+void packed_detail(const Packed* p, int64_t out[8]) {
+  for (int i = 0; i < 8; ++i) out[i] = 0;
+  if (p->mode == 1) {
+    out[0] = FP_VAR_CSR_L2BLOCK;
+    out[1] = p->cs;
+    out[2] = p->heavy;
+    out[3] = p->nhot;
+    out[4] = p->hot_entries;
+    out[5] = 2 * p->entries - p->heavy_entries + p->hot_entries;
+    out[6] = 2 * (p->cs - 1) + 5;  // init, a dot launch per other block, fused, q, scatters, partial, hot
+  } else {
+    out[0] = FP_VAR_CSR_PACKED;
+    out[1] = p->cs;
+    out[2] = -1;
+    out[5] = p->entries;
+    out[6] = 2;  // the pass + the finalize
+  }
 }
 
 fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {

@@ -219,6 +219,13 @@ fp_status fp_csr_plan_pack_info(const fp_csr_plan* p, int64_t* ntiles, int64_t* 
   return FP_OK;
 }
 
+fp_status fp_csr_plan_pack_detail(const fp_csr_plan* p, int64_t out[8]) {
+  FP_REQUIRE(p && out, FP_ERR_INVALID_ARG, "fp_csr_plan_pack_detail: NULL argument");
+  FP_REQUIRE(p->packed, FP_ERR_INVALID_ARG, "fp_csr_plan_pack_detail: the plan is not packed");
+  fp::packed_detail(p->packed, out);
+  return FP_OK;
+}
+
 fp_status fp_csr_plan_destroy(fp_csr_plan* p) {
   if (!p) return FP_OK;
   if (p->soff) cudaFree(p->soff);

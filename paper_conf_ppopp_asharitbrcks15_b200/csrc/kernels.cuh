@@ -109,6 +109,8 @@ struct Packed {
   void* hval = nullptr;
   uint4* hitems = nullptr;
   int64_t nhitems = 0;
+  int64_t hot_entries = 0;
+  int64_t heavy_entries = 0;            // stored entries of the fused block
 };
 // variant 20 (csr_l2block.cu)
 int64_t l2block_bw(int64_t n, fp_dtype dt);
@@ -116,6 +118,7 @@ fp_status l2block_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr
                         const void* val, fp_dtype dtype, Packed* p, cudaStream_t s);
 fp_status l2block_exec(Packed* p, const PatternArgs& a, cudaStream_t s);
 void l2block_launch(const Packed* p, fp_launch* L);
+void packed_detail(const Packed* p, int64_t out[8]);  // fp_csr_plan_pack_detail
 int packed_cs(int64_t n, fp_dtype dt);  // column blocks (1, 2, 4, 8) for n columns, 0 if too wide
 fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                        const void* val, fp_dtype dtype, int cs_force, Packed** out, cudaStream_t s);

@@ -403,3 +403,27 @@ def test_l2block_graph_replay(cuda_dev, monkeypatch):
         g.replay()
         torch.cuda.synchronize()
         assert_bitexact(w, ref, f"l2block graph replay {i}")
+
+
+def test_pack_detail_counts(cuda_dev, monkeypatch):
+    """fp_csr_plan_pack_detail reports what an exec does: variant 20's hot columns and their
+    nonzeros equal a host count of the columns above the threshold; the entries streamed count
+    the fused block once and the others twice; variant 19 streams its copy once in 2 launches."""
+    m, n, thr = 6000, 30_000, 120
+    rp, ci, va = synth.csr(m, n, "f64", ("powerlaw", 2.5, 9.5), seed=17, col_skew=2)
+    monkeypatch.setenv("FP_L2B_HOT", str(thr))
+    plan = l2_plan(cuda_dev, monkeypatch, rp, ci, va, n, 7000, torch.float64)
+    d, info = plan.pack_detail, plan.pack_info
+    counts = np.bincount(ci.numpy(), minlength=n)
+    assert d["variant"] == 20 and d["blocks"] == info["blocks"] == 5
+    assert d["hot_columns"] == int((counts > thr).sum()) > 0
+    assert d["hot_entries"] == int(counts[counts > thr].sum())
+    per_block = np.bincount(ci.numpy() // 7000, minlength=5)
+    assert d["fused_block"] == int(np.argmax(per_block))
+    assert info["entries"] < d["entries_streamed"] <= 2 * info["entries"] + d["hot_entries"]
+    assert d["launches"] == 2 * (5 - 1) + 5
+    rp, ci, va = synth.csr(m, 1000, "f32", ("binomial", 0.01), seed=17)
+    p19 = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), 1000, torch.float32)
+    p19.pack(va.to(cuda_dev))
+    d = p19.pack_detail
+    assert d["variant"] == 19 and d["entries_streamed"] == p19.pack_info["entries"] and d["launches"] == 2

@@ -69,6 +69,9 @@ def full(rep, config, alg_bytes, variant=None, rnd=None):
     # consumer, finalize): the step's traffic is the sum of their per-launch means
     kern = {k: int(sum(v) / len(v)) for k, v in per_kernel.items()}
     step = sum(kern.values())
+    if os.environ.get("NCU_STEP_ALL"):  # the capture is exactly one step (variant 20: a launch per block)
+        kern = {k: int(sum(v)) for k, v in per_kernel.items()}
+        step = int(sum(traffic_all))
     print(f"\nDRAM traffic per step (sum over the {len(kern)} kernels): {step / 1e9:.4f} GB; "
           f"traffic / algorithmic = {step / alg_bytes:.4f}\n")
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
