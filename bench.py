@@ -30,6 +30,10 @@ import sys
 import threading
 import time
 
+# stdout carries exactly one JSON line: NCCL's version banner (NCCL_DEBUG=VERSION) would add one
+if os.environ.get("NCCL_DEBUG", "").upper() == "VERSION":
+    os.environ["NCCL_DEBUG"] = "WARN"
+
 import numpy as np
 import torch
 
