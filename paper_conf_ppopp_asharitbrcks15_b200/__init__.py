@@ -488,7 +488,8 @@ def probe_rates(n, smem_elems=1000, device=None):
 class LocalGroup:
     """fp_comm_init_local_group: `nranks` peer-exchange communicators on ONE device (a single
     process, no NCCL) -- the same fused exchange as across GPUs, between plain allocations.
-    Drive the ranks concurrently (one host thread per rank): each rank's barrier waits for all."""
+    Drive the ranks concurrently (one host thread per rank): a rank's call returns once every
+    rank reached its exchange (they meet on the host; no kernel waits for another rank's launch)."""
 
     def __init__(self, nranks, device=0, max_bytes=1 << 22):
         arr = (ctypes.c_void_p * nranks)()

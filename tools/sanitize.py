@@ -3,7 +3,8 @@
 family once -- dense vector / CTA / cluster, CSR vector (shared / L2 / private / owner /
 fixed-point / cp.async stream), flat (shared / L2 / private / fixed / 1024-thread with a y
 prefix), flat-4 with the fixed-point partial (18), the binned scatter (17: producer, consumer,
-finalize), the peer exchange (one-rank local group), the L2-replica fold, the column-split plan, the row epilogues, CG and TRON drivers --
+finalize), the packed plans (19: k_pk1 with its TMA ring, the cooperative k_pk; 20: L2 blocks
+with hot columns and long rows, and their pack kernels), the peer exchange (one-rank local group), the L2-replica fold, the column-split plan, the row epilogues, CG and TRON drivers --
 on tiny inputs.
 
   compute-sanitizer --tool memcheck python tools/sanitize.py
@@ -62,6 +63,33 @@ def main():
                 L.variant, L.vs, L.tl, L.bs, L.grid, L.cluster = 17, 32, 8, 1024, 5, nb
                 fp.csr(rpb, cib, vab, nn, yb, vb, zb, 1.0, 1.0, launch=L)
                 fp.csr(rpb, cib, vab, nn, None, vb, None, 2.0, 0.0, launch=L)
+        # packed plans: variant 19 (one block: k_pk1 with the TMA tile ring; fp32 two blocks: the
+        # cooperative k_pk) and variant 20 (L2 blocks, forced small; hot columns; long rows)
+        rpp, cip, vap = synth.csr(3000, 1500, dt, ("uniform", 0, 700), seed=8, device=dev)
+        yp = synth.vector(1500, dt, seed=8, device=dev)
+        vp = synth.vector(3000, dt, kind="pos", seed=8, stream=synth.S_V, device=dev)
+        P1 = fp.CsrPlan(rpp, cip, 1500, vap.dtype)
+        P1.pack(vap)
+        P1(None, yp, vp, yp, 1.0, 1.0)
+        P1(None, None, vp, None, 2.0, 0.0)
+        if dt == "f32":
+            rq, cq, vq = synth.csr(4000, 60000, dt, ("powerlaw", 2.0, 3.0), seed=9, device=dev)
+            yq = synth.vector(60000, dt, seed=9, device=dev)
+            os.environ["FP_PK_GROUPS"] = "2"
+            P2 = fp.CsrPlan(rq, cq, 60000, vq.dtype)
+            P2.pack(vq)
+            del os.environ["FP_PK_GROUPS"]
+            P2(None, yq, None, yq, 1.0, 1.0)
+        rl, cl, vl = synth.csr(3000, 20000, dt, ("powerlaw", 2.5, 9.5), seed=10, device=dev, col_skew=2)
+        yl = synth.vector(20000, dt, seed=10, device=dev)
+        vl2 = synth.vector(3000, dt, kind="pos", seed=10, stream=synth.S_V, device=dev)
+        os.environ.update(FP_PK_L2="1", FP_L2B_BW="6000", FP_L2B_HOT="50")
+        P3 = fp.CsrPlan(rl, cl, 20000, vl.dtype)
+        P3.pack(vl)
+        for k in ("FP_PK_L2", "FP_L2B_BW", "FP_L2B_HOT"):
+            del os.environ[k]
+        P3(None, yl, vl2, yl, 1.0, 1.0)
+        P3(None, None, vl2, None, 1.0, 0.0)
         # the peer exchange (one-rank local group: the same kernels, a trivially met barrier)
         g = fp.LocalGroup(1, 0, max_bytes=700 * 8)
         fp.csr_dist(g.comms[0], rp, ci, va, 700, y, v, z, 1.0, 1.0)
