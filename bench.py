@@ -285,6 +285,19 @@ def run_gpu(args):
         except fp.FusedPatError as e:
             print(f"[bench] rank {rank}: {exchange} exchange unavailable ({e})", file=sys.stderr)
             ok = 0
+        # the exchange checks itself once (an allreduce of rank + 1 everywhere: every element must
+        # be N (N + 1) / 2 and no barrier may have timed out) before anything is timed
+        if ok and exchange != "nccl":
+            try:
+                chk = torch.full((4096,), float(rank + 1), dtype=torch.float64, device=dev)
+                comm.allreduce(chk)
+                torch.cuda.synchronize()
+                ok = int(bool((chk == world * (world + 1) / 2).all()) and not comm.timed_out())
+            except fp.FusedPatError as e:
+                print(f"[bench] rank {rank}: {exchange} exchange self-check failed ({e})", file=sys.stderr)
+                ok = 0
+            if not ok:
+                print(f"[bench] rank {rank}: {exchange} exchange self-check failed", file=sys.stderr)
         # every rank must use the same exchange: fall back to NCCL together if any rank failed
         import torch.distributed as dist
 

@@ -456,6 +456,10 @@ class Comm:
         _call("fp_allreduce", self.handle, _ptr(t), t.numel(), _dt(t), _stream(t.device, stream))
         return t
 
+    def timed_out(self):
+        """fp_comm_timed_out: True if a peer / NVLS barrier of this communicator gave up waiting."""
+        return lib().fp_comm_timed_out(self.handle) == 1
+
     def enable_peer(self, max_bytes, stream=None):
         """Collective: switch this communicator to the fused peer-memory exchange
         (FP_COMM_PEER, include/fusedpat.h) for vectors of up to max_bytes."""
