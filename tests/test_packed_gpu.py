@@ -427,3 +427,29 @@ def test_pack_detail_counts(cuda_dev, monkeypatch):
     p19.pack(va.to(cuda_dev))
     d = p19.pack_detail
     assert d["variant"] == 19 and d["entries_streamed"] == p19.pack_info["entries"] and d["launches"] == 2
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+def test_packed1_unaligned_v_and_w_alias_z(cuda_dev, dt):
+    """k_pk1 takes v with its tile copy only when v is 16-byte aligned: a v that starts one
+    element into its buffer runs the global-load path, same bits; w may alias z (in place)."""
+    m, n = 7_001, 1000
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rp, ci, va = synth.csr(m, n, dt, ("binomial", 0.01), kind="int_pm12", seed=23)
+    y = synth.vector(n, dt, kind="int_small", seed=23, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="int_pos", seed=23, stream=synth.S_V)
+    z = synth.vector(n, dt, kind="int_small", seed=23, stream=synth.S_Z)
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, tdt)
+    plan.pack(va.to(cuda_dev))
+    ref, _ = oracle.csr(m, n, rp, ci, va, y, v, z, 1.0, 2.0)
+    vbuf = torch.zeros(m + 1, dtype=tdt, device=cuda_dev)
+    vbuf[1:] = v.to(cuda_dev)
+    vu = vbuf[1:]
+    assert vu.data_ptr() % 16 != 0
+    w = plan(None, y.to(cuda_dev), vu, z.to(cuda_dev), 1.0, 2.0)
+    torch.cuda.synchronize()
+    assert_bitexact(w, ref, f"packed1 {dt} unaligned v")
+    zw = z.to(cuda_dev).clone()
+    plan(None, y.to(cuda_dev), v.to(cuda_dev), zw, 1.0, 2.0, w=zw)
+    torch.cuda.synchronize()
+    assert_bitexact(zw, ref, f"packed1 {dt} w aliases z")

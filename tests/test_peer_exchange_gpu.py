@@ -140,9 +140,9 @@ def test_peer_cg_matches_single_gpu(cuda_dev):
 
 
 @pytest.mark.parametrize("P", [2, 4])
-@pytest.mark.parametrize("packed", [True, False])
+@pytest.mark.parametrize("packed", [True, False, "l2"])
 def test_peer_plan_dist_bitexact(cuda_dev, monkeypatch, P, packed):
-    """fp_csr_plan_dist: every rank runs its shard's plan (packed copy: variant 19, or the
+    """fp_csr_plan_dist: every rank runs its shard's plan (packed copy: variant 19 or 20, or the
     unpacked plan) and the peer exchange; every rank bit-identical and bit-exact against the
     full-matrix oracle on an integer twin, over three calls.  The ranks share one GPU here, so
     the packed passes (cooperative launches) use 4 CTA groups each (FP_PK_GROUPS)."""
@@ -155,6 +155,10 @@ def test_peer_plan_dist_bitexact(cuda_dev, monkeypatch, P, packed):
     b = fp.shard_rows_csr(rp, P)
     shards = [tuple(t.contiguous().to(cuda_dev) for t in fp.shard_slice_csr(rp, ci, va, v, b, r)) for r in range(P)]
     monkeypatch.setenv("FP_PK_GROUPS", "4")
+    if packed == "l2":  # variant 20 (L2-sized column blocks, forced small) on every rank's shard
+        monkeypatch.setenv("FP_PK_L2", "1")
+        monkeypatch.setenv("FP_L2B_BW", "7000")
+        monkeypatch.setenv("FP_L2B_HOT", "40")
     plans = []
     for lrp, lci, lva, lv in shards:
         pl = fp.CsrPlan(lrp, lci, n, torch.float32)
