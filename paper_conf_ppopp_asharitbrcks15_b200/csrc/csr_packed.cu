@@ -664,18 +664,21 @@ __global__ void k_pk1_finalize(int64_t n, int ctas, const double* __restrict__ p
 // own work.  Padding entries (column = the block's zero / dummy slot, row 63, value 0) fill the
 // segments to 8 entries and the lanes beyond a segment load a padding block: no per-entry
 // predicates.
-template <int CS, int YM>
-__global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
+template <int CS, int YM, int BS>
+__global__ void __launch_bounds__(BS, 1) k_pk(const PkArgs a) {
+  constexpr int NW = BS / 32;
+  // BS <= 768: 85 registers -- the scatter's first window is loaded before the exchange poll
+  constexpr bool PFS = BS <= 768;
   // pipeline depth: measured on C4, D = 1 6.22 ms, D = 2 7.05 ms (the segments of 3 tiles per warp
   // in flight between dot and scatter overflow L2: the re-reads miss), D = 0 13.5 ms (exchange latency)
   constexpr int D = (CS > 1 && YM != 0) ? 1 : 0;
   constexpr int NS = PkSlots<D>::NS;
   static_assert(kPkRing >= D + 1, "descriptor ring");
   extern __shared__ __align__(16) unsigned char pk_smem[];
-  __shared__ float rs[kPkNW][kPkRows];   // the tile's block partials of the row dots (by row in tile)
-  __shared__ float qsm[kPkNW][kPkRows];  // q / quantum of the tile's rows
-  __shared__ float qus[kPkNW][kPkRows];  // q of the tile's rows (spill path, first rounds)
-  __shared__ uint4 ring[kPkNW][kPkRing]; // descriptors of the tiles between DOT and SCATTER
+  __shared__ float rs[NW][kPkRows];   // the tile's block partials of the row dots (by row in tile)
+  __shared__ float qsm[NW][kPkRows];  // q / quantum of the tile's rows
+  __shared__ float qus[NW][kPkRows];  // q of the tile's rows (spill path, first rounds)
+  __shared__ uint4 ring[NW][kPkRing]; // descriptors of the tiles between DOT and SCATTER
   __shared__ unsigned s_tmax;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int k = CS == 1 ? 0 : (int)(blockIdx.x % CS);
@@ -689,7 +692,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   const int ystride = YM ? (bw + 4) & ~3 : 0;
   float* y_s = reinterpret_cast<float*>(pk_smem);
   int* acc = reinterpret_cast<int*>(pk_smem) + ystride;
-  for (int j = threadIdx.x; j <= bw + 32; j += kPkBS) {
+  for (int j = threadIdx.x; j <= bw + 32; j += BS) {
     if (YM && j <= bw) y_s[j] = j < bwk ? a.y[c0 + j] : 0.f;
     acc[j] = 0;
   }
@@ -701,7 +704,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
 
   unsigned long long tr0 = 0, tr1 = 0;
   if (a.trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr0));
-  const int gq = g * kPkNW + warp;
+  const int gq = g * NW + warp;
   const int64_t t0 = a.wtile[gq];
   const int nt = a.wtile[gq + 1] - a.wtile[gq];
   const uint4* __restrict__ desc = a.tile_desc + (int64_t)k * a.ntiles + t0;
@@ -890,7 +893,9 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   // ---- SCAT(j): Eq. (3) from the segment, re-read.  SAFE (every |x q| of the tile below the
   // cap, from the plan's max |x| of the tile): no per-entry checks; else terms beyond the cap
   // and non-finite terms are flagged too.  Flagged entries (and int32 wraps) spill after.
-  auto scatter = [&](const uint4& T) {
+  // pf: the segment's first window, loaded by the caller before the exchange poll (its load
+  // latency hides behind the wait; ncu r02c: 13 % of k_pk's stall samples sat on that load)
+  auto scatter = [&](const uint4& T, const uint32_t (&pcw)[8], const float (&pxv)[8], bool pf) {
     __syncwarp();
     const float q0 = pk_lds_v(qu_base + 4 * lane), q1 = pk_lds_v(qu_base + 128 + 4 * lane);
     const float qs0 = q0 * sc, qs1 = q1 * sc;
@@ -904,7 +909,12 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
       for (int s0 = 0; s0 < len; s0 += 256) {
         uint32_t cw[8];
         float xv[8];
-        ld_step(T, s0, std::false_type{}, cw, xv);
+        if (pf && s0 == 0) {
+#pragma unroll
+          for (int e = 0; e < 8; ++e) cw[e] = pcw[e], xv[e] = pxv[e];
+        } else {
+          ld_step(T, s0, std::false_type{}, cw, xv);
+        }
         const unsigned abase = acc_base + (s0 + 8 * lane < len ? 0u : 4u * (lane + 1));  // lane's dummy
         unsigned rare = 0;
 #pragma unroll
@@ -985,7 +995,9 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
     }
     // (while every finite term so far is 0, the provisional scale adds zeros; non-finite terms spill)
     if (have) {
-      scatter(T);
+      uint32_t pcw[8];
+      float pxv[8];
+      scatter(T, pcw, pxv, false);
       ++j;
     }
     if (mx > 0.f || !any) break;
@@ -996,13 +1008,16 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
   for (; j < nt; ++j) {
     if (j + D < nt) dot(j + D);
     const uint4 T = ring[warp][j % kPkRing];
+    uint32_t pcw[8];
+    float pxv[8];
+    if constexpr (PFS) ld_step(T, 0, std::false_type{}, pcw, pxv);  // in flight during the poll
     qcalc(T, j);
-    scatter(T);
+    scatter(T, pcw, pxv, PFS);
   }
   if (a.trace && lane == 0) {
     unsigned long long tr2;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr2));
-    unsigned long long* tp = a.trace + ((int64_t)blockIdx.x * kPkNW + warp) * 8;
+    unsigned long long* tp = a.trace + ((int64_t)blockIdx.x * NW + warp) * 8;
     tp[0] = tr0;
     tp[1] = tr2;
     tp[2] = (unsigned long long)nt;
@@ -1012,7 +1027,7 @@ __global__ void __launch_bounds__(kPkBS, 1) k_pk(const PkArgs a) {
 
   __syncthreads();
   double* dst = a.part + (int64_t)g * a.n + c0;
-  for (int i = threadIdx.x; i < bwk; i += kPkBS) dst[i] = (double)acc[i] * quantum;
+  for (int i = threadIdx.x; i < bwk; i += BS) dst[i] = (double)acc[i] * quantum;
 }
 
 __global__ void k_pk_finalize(int64_t n, int bw, int groups, const double* __restrict__ part,
@@ -1362,15 +1377,14 @@ __global__ void k_pk_partition(int64_t ntiles, int nq, const int64_t* __restrict
 }
 
 template <int CS, int YM>
-const void* pk_kernel() {
-  return (const void*)k_pk<CS, YM>;
+const void* pk_kernel(int bs) {
+  return bs == 768 ? (const void*)k_pk<CS, YM, 768> : (const void*)k_pk<CS, YM, 1024>;
 }
-const void* pk_pick(int cs, bool has_y) {
+const void* pk_pick(int cs, bool has_y, int bs) {
   switch (cs) {
-    case 1: return has_y ? pk_kernel<1, 1>() : pk_kernel<1, 0>();
-    case 2: return has_y ? pk_kernel<2, 1>() : pk_kernel<2, 0>();
-    case 4: return has_y ? pk_kernel<4, 1>() : pk_kernel<4, 0>();
-    case 8: return has_y ? pk_kernel<8, 1>() : pk_kernel<8, 0>();
+    case 2: return has_y ? pk_kernel<2, 1>(bs) : pk_kernel<2, 0>(bs);
+    case 4: return has_y ? pk_kernel<4, 1>(bs) : pk_kernel<4, 0>(bs);
+    case 8: return has_y ? pk_kernel<8, 1>(bs) : pk_kernel<8, 0>(bs);
   }
   return nullptr;
 }
@@ -1484,7 +1498,10 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const int span = cs == 1 ? 256 : kPkLong;  // one block: a tile is one window (loaded once)
   const DeviceInfo& di = device_info(current_device());
   int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
+  // column-block groups (cs > 1): CTAs of FP_PK_BSN threads (1024 default; 768: 85 registers,
+  // the scatter's first window prefetched before the exchange poll)
   int bs = kPkBS;
+  if (const char* e = std::getenv("FP_PK_BSN"); e && cs > 1 && std::atoi(e) == 768) bs = 768;
   int ns1 = 0;
   if (cs == 1) {  // the single-block pass: CTAs of FP_PK_BS1 (512 default) threads, as many as fit
     // measured: S3 (fp32) 0.51 ms at 1024 threads vs 0.67 at 512; C3 (fp64) 1.00 ms at 512
@@ -1515,6 +1532,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   p->rowptr = rowptr;
   p->dtype = dtype;
   p->bs = bs;
+  p->trace_warps = bs / 32;
   p->ns1 = ns1;
   const int64_t ng = (m + kPkRows - 1) / kPkRows;
   uint32_t* cnt = nullptr;
@@ -1624,7 +1642,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile);
   // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
   const int ns = cs > 1 ? PkSlots<1>::NS : 1;
-  const size_t xbytes = (size_t)groups * kPkNW * ns * (cs + 1) * kPkRows * 8;
+  const size_t xbytes = (size_t)groups * (bs / 32) * ns * (cs + 1) * kPkRows * 8;
   PK_TRY(cudaMalloc((void**)&p->xch, xbytes), "alloc");
   PK_TRY(cudaMemsetAsync(p->xch, 0, xbytes, s), "memset");
   PK_TRY(cudaMalloc((void**)&p->epoch, 16), "alloc");
@@ -1691,7 +1709,7 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     FP_CUDA(cudaGetLastError());
     return FP_OK;
   }
-  const void* f = pk_pick(p->cs, has_y);
+  const void* f = pk_pick(p->cs, has_y, p->bs);
   FP_REQUIRE(f, FP_ERR_UNSUPPORTED, "fp_csr_plan_exec: no packed kernel for %d blocks", p->cs);
   set_max_dynamic_smem(f);
   PkArgs k{};
@@ -1721,14 +1739,14 @@ fp_status packed_exec(Packed* p, const PatternArgs& a, cudaStream_t s) {
     k.nap = n ? std::atoi(n) : 0;
   }
   if (std::getenv("FP_PK_TRACE")) {  // measurement: per-warp timing of the pass (kept in the plan)
-    if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * kPkNW * 64);
+    if (!p->trace) cudaMalloc((void**)&p->trace, (size_t)p->groups * p->cs * (p->bs / 32) * 64);
     k.trace = p->trace;
   }
   const size_t smem = ((has_y ? (size_t)((p->bw + 4) & ~3) : 0) + (size_t)p->bw + 33) * 4;
   void* args[] = {&k};
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(p->groups * p->cs);
-  cfg.blockDim = dim3(kPkBS);
+  cfg.blockDim = dim3(p->bs);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
@@ -1758,7 +1776,7 @@ void packed_launch(const Packed* p, fp_launch* L) {
   L->tl = p->cs == 1 ? 256 : kPkLong;
   L->blocks_per_sm = 1;
   cudaFuncAttributes fa{};
-  if (cudaFuncGetAttributes(&fa, p->cs == 1 ? pk1_pick(p->dtype, true, p->bs) : pk_pick(p->cs, true)) == cudaSuccess)
+  if (cudaFuncGetAttributes(&fa, p->cs == 1 ? pk1_pick(p->dtype, true, p->bs) : pk_pick(p->cs, true, p->bs)) == cudaSuccess)
     L->regs_per_thread = fa.numRegs;
   else cudaGetLastError();
 }
