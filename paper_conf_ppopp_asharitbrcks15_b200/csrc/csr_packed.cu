@@ -1406,7 +1406,9 @@ const void* pk1_pick_bs(fp_dtype dt, bool has_y) {
   return has_y ? (const void*)k_pk1<float, 1, BS1> : (const void*)k_pk1<float, 0, BS1>;
 }
 const void* pk1_pick(fp_dtype dt, bool has_y, int bs) {
-  return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y) : (bs == 768 ? pk1_pick_bs<768>(dt, has_y) : pk1_pick_bs<512>(dt, has_y));
+  return bs == 1024 ? pk1_pick_bs<1024>(dt, has_y)
+                    : (bs == 768 ? pk1_pick_bs<768>(dt, has_y)
+                                 : (bs == 640 ? pk1_pick_bs<640>(dt, has_y) : pk1_pick_bs<512>(dt, has_y)));
 }
 size_t pk1_slot_bytes(fp_dtype dt) { return (size_t)256 * (4 + dtype_size(dt)) + (size_t)kPkRows * dtype_size(dt) + 16; }
 size_t pk1_smem_n(int64_t n, fp_dtype dt, bool has_y, int bs, int ns) {
@@ -1505,9 +1507,12 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   int ns1 = 0;
   if (cs == 1) {  // the single-block pass: CTAs of FP_PK_BS1 (512 default) threads, as many as fit
     // measured: S3 (fp32) 0.51 ms at 1024 threads vs 0.67 at 512; C3 (fp64) 1.00 ms at 512
-    // (127 registers) vs 1.21 at 1024 (64 registers: spills)
+    // (127 registers) vs 1.21 at 1024 (64 registers: spills).  Round 2c (ring, v in the slot):
+    // C3 512 / 640 / 768 / 1024 threads 0.890 / 0.922 / 1.075 / 1.467 ms; S3 0.654 / 0.565 /
+    // 0.517 / 0.490 ms
     const char* e = std::getenv("FP_PK_BS1");
-    bs = e ? (std::atoi(e) == 1024 ? 1024 : (std::atoi(e) == 768 ? 768 : 512)) : (dtype == FP_F64 ? 512 : 1024);
+    const int eb = e ? std::atoi(e) : 0;
+    bs = (eb == 1024 || eb == 768 || eb == 640 || eb == 512) ? eb : (dtype == FP_F64 ? 512 : 1024);
     const void* f1 = pk1_pick(dtype, true, bs);
     set_max_dynamic_smem(f1);
     ns1 = pk1_ring_ns(n, dtype, bs);
