@@ -231,6 +231,10 @@ struct Pk1Args {
 };
 
 constexpr int kPk1MaxNS = 4;
+#ifndef FP_PK1_FG
+#define FP_PK1_FG 8
+#endif
+constexpr int kPk1FG = FP_PK1_FG;  // fp64 scatter: terms whose low limbs are added before their high limbs
 constexpr uint32_t pk1_pad_word(int n) { return ((uint32_t)n * 4u) | ((uint32_t)(kPkRows - 1) << kPkRidShift); }
 
 __device__ __forceinline__ uint4 pk_lds128(unsigned addr) {
@@ -455,28 +459,48 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
   auto scat_win = [&](const uint32_t (&cw)[8], const T (&xv)[8], int s0, int len) {
     const unsigned dm = (s0 + 8 * lane < len) ? 0u : 4u * (lane + 1);  // lane's dummy beyond the segment
     unsigned rare = 0;
+    if constexpr (!F64) {
 #pragma unroll
-    for (int e = 0; e < 8; ++e) {
-      const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
-      const unsigned off = dm + (cw[e] & kPkOffMask);
-      if constexpr (!F64) {
+      for (int e = 0; e < 8; ++e) {
+        const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
+        const unsigned off = dm + (cw[e] & kPkOffMask);
         const bool big = !(fabsf(ts) < kPkCap);
         const int qi = big ? 0 : __float2int_rn(ts);
         const int old = pk_atom_add(lo_base + off, qi);
         const unsigned nw = (unsigned)old + (unsigned)qi;
         rare = (rare << 1) | (unsigned)(big | ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0));
-      } else {
-        // |term| < 2^62 quanta: both limbs always added (no branch); the high limb's wrap is
-        // detected from its returned old value
-        const bool big = !(fabs(ts) < 4.6e18);
-        const long long I = big ? 0ll : __double2ll_rn(ts);
-        const unsigned l = (unsigned)I;
-        const unsigned ol = pk_atom_addu(lo_base + off, l);
-        const int h = (int)(I >> 32) + ((ol + l < ol) ? 1 : 0);
-        const int oh = pk_atom_add(hi_base + off, h);
-        const unsigned nw = (unsigned)oh + (unsigned)h;
-        const bool ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
-        rare = (rare << 1) | (unsigned)(big | ovf);
+      }
+    } else {
+      // |term| < 2^62 quanta: both limbs always added (no branch); the high limb's wrap is
+      // detected from its returned old value.  The low limbs of a group of PG terms go first:
+      // a high limb's operand waits for its low limb's returned value (the carry) and the
+      // volatile atomics keep program order, so alternating lo / hi per term would chain 16
+      // shared-memory round trips per window
+#pragma unroll
+      for (int g0 = 0; g0 < 8; g0 += kPk1FG) {
+        unsigned l[kPk1FG], ol[kPk1FG], off[kPk1FG];
+        int hh[kPk1FG];
+        bool big[kPk1FG];
+#pragma unroll
+        for (int k = 0; k < kPk1FG; ++k) {
+          const int e = g0 + k;
+          const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
+          off[k] = dm + (cw[e] & kPkOffMask);
+          big[k] = !(fabs(ts) < 4.6e18);
+          const long long I = big[k] ? 0ll : __double2ll_rn(ts);
+          l[k] = (unsigned)I;
+          hh[k] = (int)(I >> 32);
+        }
+#pragma unroll
+        for (int k = 0; k < kPk1FG; ++k) ol[k] = pk_atom_addu(lo_base + off[k], l[k]);
+#pragma unroll
+        for (int k = 0; k < kPk1FG; ++k) {
+          const int h = hh[k] + ((ol[k] + l[k] < ol[k]) ? 1 : 0);
+          const int oh = pk_atom_add(hi_base + off[k], h);
+          const unsigned nw = (unsigned)oh + (unsigned)h;
+          const bool ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
+          rare = (rare << 1) | (unsigned)(big[k] | ovf);
+        }
       }
     }
     if (rare) {  // bit 7 - e flags entry e
