@@ -1093,16 +1093,16 @@ __device__ __forceinline__ bool pk_is_long(const uint32_t* cnt, int64_t m, int c
     if (cnt[(int64_t)kk * m + r] > (uint32_t)span) return true;
   return false;
 }
-__global__ void k_pk_tiles(int64_t m, int cs, int span, const uint32_t* __restrict__ cnt,
+__global__ void k_pk_tiles(int64_t m, int gr, int cs, int span, const uint32_t* __restrict__ cnt,
                            unsigned long long* __restrict__ gmask, int64_t* __restrict__ gcount) {
-  const int64_t ng = (m + kPkRows - 1) / kPkRows;
+  const int64_t ng = (m + gr - 1) / gr;
   for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
     uint32_t accs[kPkMaxCS] = {};
     unsigned long long mask = 0;
     int ntl = 0;
     bool fresh = true;  // the next row starts a tile
-    for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
-      const int64_t r = gi * kPkRows + i;
+    for (int i = 0; i < gr && gi * gr + i < m; ++i) {
+      const int64_t r = gi * gr + i;
       if (pk_is_long(cnt, m, cs, r, span)) {
         mask |= 1ull << i;
         ++ntl;
@@ -1125,10 +1125,10 @@ __global__ void k_pk_tiles(int64_t m, int cs, int span, const uint32_t* __restri
 }
 
 // (3) tile rows and segment lengths; al = the lengths rounded up to 8 (scanned into offsets)
-__global__ void k_pk_tile_rows(int64_t m, int cs, int64_t ntiles, const uint32_t* __restrict__ cnt,
+__global__ void k_pk_tile_rows(int64_t m, int gr, int cs, int64_t ntiles, const uint32_t* __restrict__ cnt,
                                const unsigned long long* __restrict__ gmask, const int64_t* __restrict__ gbase,
                                int64_t* __restrict__ tile_row, uint32_t* __restrict__ tlen, int64_t* __restrict__ al) {
-  const int64_t ng = (m + kPkRows - 1) / kPkRows;
+  const int64_t ng = (m + gr - 1) / gr;
   for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < ng; gi += (int64_t)gridDim.x * blockDim.x) {
     const unsigned long long mask = gmask[gi];
     int64_t t = gbase[gi] - 1;
@@ -1141,8 +1141,8 @@ __global__ void k_pk_tile_rows(int64_t m, int cs, int64_t ntiles, const uint32_t
         len[kk] = 0;
       }
     };
-    for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
-      const int64_t r = gi * kPkRows + i;
+    for (int i = 0; i < gr && gi * gr + i < m; ++i) {
+      const int64_t r = gi * gr + i;
       if ((mask >> i) & 1ull) {
         flush();
         ++t;
@@ -1174,13 +1174,13 @@ __global__ void k_pk_fill(int64_t n, uint32_t* __restrict__ p, uint32_t v) {
 // byte offset of the column inside its block | row inside the tile << 26.  Also the largest
 // |x| of every (tile, block) segment (+Inf if a value is not finite): the scatter's no-check test.
 template <typename V>
-__global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const int64_t* __restrict__ rowptr,
+__global__ void k_pk_scatter(int64_t m, int gr, int cs, int bw, int64_t ntiles, const int64_t* __restrict__ rowptr,
                              const int32_t* __restrict__ colidx, const V* __restrict__ val,
                              const unsigned long long* __restrict__ gmask, const int64_t* __restrict__ gbase,
                              uint4* __restrict__ desc, uint32_t* __restrict__ cr, V* __restrict__ pval) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = pk_lanemask_lt();
-  const int64_t ng = (m + kPkRows - 1) / kPkRows;
+  const int64_t ng = (m + gr - 1) / gr;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
   for (int64_t gi = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5); gi < ng; gi += nw) {
     const unsigned long long mask = gmask[gi];
@@ -1198,8 +1198,8 @@ __global__ void k_pk_scatter(int64_t m, int cs, int bw, int64_t ntiles, const in
         xm[kk] = 0.f;
       }
     };
-    for (int i = 0; i < kPkRows && gi * kPkRows + i < m; ++i) {
-      const int64_t r = gi * kPkRows + i;
+    for (int i = 0; i < gr && gi * gr + i < m; ++i) {
+      const int64_t r = gi * gr + i;
       if ((mask >> i) & 1ull) {
         flush();
         ++t;
@@ -1521,7 +1521,12 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   FP_REQUIRE(cs == 1 ? n <= packed1_max_n(dtype) : bw <= packed_max_bw(), FP_ERR_UNSUPPORTED,
              "fp_csr_plan_pack: n = %lld too wide for %d blocks", (long long)n, cs);
   const size_t vs = dtype_size(dtype);
-  const int span = cs == 1 ? 256 : kPkLong;  // one block: a tile is one window (loaded once)
+  // one block: a tile is one window (loaded once); measurement knobs (cs > 1): FP_PK_SPAN (entries
+  // per block segment before a row goes alone), FP_PK_ROWS (rows per tile: 16 / 32 / 64)
+  int span = cs == 1 ? 256 : kPkLong;
+  if (const char* e = std::getenv("FP_PK_SPAN"); e && cs > 1 && std::atoi(e) >= 256) span = std::atoi(e);
+  int gr = kPkRows;
+  if (const char* e = std::getenv("FP_PK_ROWS"); e && (std::atoi(e) == 16 || std::atoi(e) == 32)) gr = std::atoi(e);
   const DeviceInfo& di = device_info(current_device());
   int groups = cs == 1 ? di.sm_count : di.sm_count / cs;
   // column-block groups (cs > 1): CTAs of FP_PK_BSN threads (1024 default; 768: 85 registers,
@@ -1563,7 +1568,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   p->bs = bs;
   p->trace_warps = bs / 32;
   p->ns1 = ns1;
-  const int64_t ng = (m + kPkRows - 1) / kPkRows;
+  const int64_t ng = (m + gr - 1) / gr;
   uint32_t* cnt = nullptr;
   unsigned long long* gmask = nullptr;
   int64_t* gcount = nullptr;
@@ -1598,7 +1603,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const int grid_r = (int)std::min<int64_t>((m + tb - 1) / tb, (int64_t)di.sm_count * 32);
   const int grid_g = (int)std::min<int64_t>((ng + tb - 1) / tb, (int64_t)di.sm_count * 32);
   k_pk_count<<<grid_r, tb, 0, s>>>(m, rowptr, colidx, cs, bw, cnt);
-  k_pk_tiles<<<grid_g, tb, 0, s>>>(m, cs, span, cnt, gmask, gcount);
+  k_pk_tiles<<<grid_g, tb, 0, s>>>(m, gr, cs, span, cnt, gmask, gcount);
   size_t tb_bytes = 0;
   PK_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, gcount, gbase, ng, s), "scan");
   size_t tmp_bytes = tb_bytes;
@@ -1615,7 +1620,7 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   PK_TRY(cudaMalloc((void**)&tlen, (size_t)segs * 4), "alloc");
   PK_TRY(cudaMalloc((void**)&al, (size_t)segs * 8), "alloc");
   PK_TRY(cudaMalloc((void**)&off, (size_t)segs * 8), "alloc");
-  k_pk_tile_rows<<<grid_g, tb, 0, s>>>(m, cs, ntiles, cnt, gmask, gbase, tile_row, tlen, al);
+  k_pk_tile_rows<<<grid_g, tb, 0, s>>>(m, gr, cs, ntiles, cnt, gmask, gbase, tile_row, tlen, al);
   PK_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb_bytes, al, off, segs, s), "scan");
   if (tb_bytes > tmp_bytes) {
     cudaFree(tmp);
@@ -1644,10 +1649,10 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   PK_TRY(cudaMemsetAsync(p->val, 0, (size_t)cap * vs, s), "memset");
   const int sgrid = (int)std::min<int64_t>((ng + 7) / 8, (int64_t)di.sm_count * 16);
   if (dtype == FP_F64)
-    k_pk_scatter<double><<<sgrid, 256, 0, s>>>(m, cs, bw, ntiles, rowptr, colidx, (const double*)val, gmask, gbase,
+    k_pk_scatter<double><<<sgrid, 256, 0, s>>>(m, gr, cs, bw, ntiles, rowptr, colidx, (const double*)val, gmask, gbase,
                                               p->tile_desc, p->cr, (double*)p->val);
   else
-    k_pk_scatter<float><<<sgrid, 256, 0, s>>>(m, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase,
+    k_pk_scatter<float><<<sgrid, 256, 0, s>>>(m, gr, cs, bw, ntiles, rowptr, colidx, (const float*)val, gmask, gbase,
                                              p->tile_desc, p->cr, (float*)p->val);
   if (std::getenv("FP_PK_NOBANK") == nullptr)  // measurement: FP_PK_NOBANK=1 keeps the row order
   {
