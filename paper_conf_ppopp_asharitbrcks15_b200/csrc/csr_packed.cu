@@ -1481,7 +1481,7 @@ void packed_free(Packed* p) {
   if (!p) return;
   for (void* b : {(void*)p->tile_desc, (void*)p->wtile, (void*)p->cr, (void*)p->val, (void*)p->xch,
                   (void*)p->epoch, (void*)p->part, (void*)p->spill, (void*)p->trace, (void*)p->rowdot,
-                  (void*)p->hcol, (void*)p->hrow, p->hval, (void*)p->hitems})
+                  (void*)p->hcol, (void*)p->hrow, p->hval, (void*)p->hitems, (void*)p->dotlist})
     if (b) cudaFree(b);
   delete p;
 }

@@ -110,6 +110,8 @@ struct Packed {
   uint4* hitems = nullptr;
   int64_t nhitems = 0;
   int64_t hot_entries = 0;
+  uint32_t* dotlist = nullptr;          // variant 20: the dot phase's chunks in (row panel, block) order
+  int64_t ndot = 0;
   int64_t heavy_entries = 0;            // stored entries of the fused block
 };
 // variant 20 (csr_l2block.cu)

@@ -421,7 +421,7 @@ def test_pack_detail_counts(cuda_dev, monkeypatch):
     per_block = np.bincount(ci.numpy() // 7000, minlength=5)
     assert d["fused_block"] == int(np.argmax(per_block))
     assert info["entries"] < d["entries_streamed"] <= 2 * info["entries"] + d["hot_entries"]
-    assert d["launches"] == 2 * (5 - 1) + 5
+    assert d["launches"] == 2 * (5 - 1) + 5  # init, 4 dots, fused, q, 4 scatters, partial, hot
     rp, ci, va = synth.csr(m, 1000, "f32", ("binomial", 0.01), seed=17)
     p19 = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), 1000, torch.float32)
     p19.pack(va.to(cuda_dev))
