@@ -91,11 +91,6 @@ __device__ __forceinline__ unsigned lanemask_lt() {
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
   return r;
 }
-__device__ __forceinline__ unsigned lanemask_le() {
-  unsigned r;
-  asm("mov.u32 %0, %%lanemask_le;" : "=r"(r));
-  return r;
-}
 
 // E with max|t| < 2^E (frexp), 0 for an all-zero call
 __device__ __forceinline__ int bin_exponent(const unsigned* gmax) {

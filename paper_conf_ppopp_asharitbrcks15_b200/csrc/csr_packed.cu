@@ -208,10 +208,6 @@ __device__ __forceinline__ void pk_ldc(const uint32_t* pc, uint32_t* c) {
         : "l"(pc));
 }
 
-struct PkTileRes {
-  uint4 D;
-  bool one;
-};
 
 struct Pk1Args {
   int64_t m;
