@@ -5,7 +5,7 @@
 // Why.  With n = 29.9M fp64, y and w are 240 MB each: every nonzero of the flat path (variant 7)
 // is a random 32-byte gather of y plus a random red.global into w that mostly miss the 126 MB
 // L2, so the pass is bound by random HBM sectors (K1: 42 ms, 0.022 of the copy peak).  Split
-// the COLUMNS into L2-sized blocks instead (bw = 2M fp64 columns: y and w of a block are 32 MB)
+// the COLUMNS into L2-sized blocks instead (bw = 4M columns: y and w of a fp64 block are 64 MB)
 // and process the blocks one after the other, so that every gather and every red of a block
 // pass hits L2:
 //   DOT(b)   for every block but the heaviest H: p[r] += sum over row r's block-b entries of
@@ -442,10 +442,13 @@ unsigned bits_for(int64_t v) {  // bits to hold 0 .. v - 1
 
 }  // namespace
 
-// columns per L2 block: y and w of a block take 32 MB (fp64: 2M columns, fp32: 4M); FP_L2B_BW
-// (measurement / tests) overrides; at most kL2MaxBlocks blocks, at most 2^24 columns a block
+// columns per L2 block: fp64 4M (y and w of a block: 64 MB) -- measured on K1 (per-block
+// launches, hot columns by column, y cached in L1): 1M / 2M / 3M / 4M / 6M / 8M / 12M columns
+// 6.43 / 5.62 / 5.30 / 5.17 / 5.33 / 6.34 / 8.65 ms; fp32 4M (32 MB, unmeasured: no fp32
+// config is this wide).  FP_L2B_BW (measurement / tests) overrides; at most kL2MaxBlocks
+// blocks, at most 2^24 columns a block
 int64_t l2block_bw(int64_t n, fp_dtype dt) {
-  int64_t bw = dt == FP_F64 ? (int64_t)1 << 21 : (int64_t)1 << 22;
+  int64_t bw = (int64_t)1 << 22;
   if (const char* e = std::getenv("FP_L2B_BW")) bw = std::max<int64_t>(1, std::atoll(e));
   bw = std::max<int64_t>(bw, (n + kL2MaxBlocks - 1) / kL2MaxBlocks);
   return std::min<int64_t>(std::min<int64_t>(bw, n), (int64_t)1 << 24);
