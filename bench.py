@@ -30,9 +30,18 @@ import sys
 import threading
 import time
 
-# stdout carries exactly one JSON line: NCCL's version banner (NCCL_DEBUG=VERSION) would add one
-if os.environ.get("NCCL_DEBUG", "").upper() == "VERSION":
-    os.environ["NCCL_DEBUG"] = "WARN"
+# stdout carries exactly one JSON line.  Native libraries (NCCL's version banner with any
+# NCCL_DEBUG level) write to fd 1 directly, so fd 1 is pointed at stderr for the whole run and
+# the JSON line goes to a duplicate of the original stdout (emit()).
+_JSON_OUT = os.fdopen(os.dup(1), "w")
+sys.stdout.flush()
+os.dup2(2, 1)
+
+
+def emit(obj):
+    _JSON_OUT.write(json.dumps(obj) + "\n")
+    _JSON_OUT.flush()
+
 
 import numpy as np
 import torch
@@ -533,7 +542,7 @@ def run_gpu(args):
             "e2e": e2e,
             "cpu_baseline": cpu,
         }
-        print(json.dumps(out), flush=True)
+        emit(out)
     if comm is not None:
         comm.close()
         import torch.distributed as dist
@@ -669,7 +678,7 @@ def run_reference(args):
            "cpu_baseline": {"value": round(val, 4), "unit": "GB/s", "kind": "oracle", "cores": threads,
                             "sample": sample},
            "e2e": {"value": round(val, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(out), flush=True)
+    emit(out)
 
 
 def run_unfused(args):
@@ -728,7 +737,7 @@ def run_unfused(args):
            "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
            "config": {"workload": f"{name}: {cfg['desc']}", "m": cfg["m"], "n": n,
                       "chain": "torch.mv (cuBLAS gemv / cuSPARSE SpMV) x2 + elementwise"}}
-    print(json.dumps(out), flush=True)
+    emit(out)
 
 
 def main():
