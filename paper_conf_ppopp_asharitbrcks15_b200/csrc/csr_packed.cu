@@ -452,53 +452,60 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
 
   // one window of the scatter: every x q into the fixed-point partial; terms beyond the
   // int32 / int64 range, non-finite terms and wraps spill (rare)
-  auto scat_win = [&](const uint32_t (&cw)[8], const T (&xv)[8], int s0, int len) {
+  // SAFE (the tile's max |x| times every |q / quantum| of its rows below the limb range, from the
+  // plan's per-tile max |x|): no per-entry range checks -- only wraps can be rare
+  auto scat_win = [&](const uint32_t (&cw)[8], const T (&xv)[8], int s0, int len, bool safe) {
     const unsigned dm = (s0 + 8 * lane < len) ? 0u : 4u * (lane + 1);  // lane's dummy beyond the segment
     unsigned rare = 0;
-    if constexpr (!F64) {
+    auto body = [&](auto SAFE) {
+      constexpr bool S = decltype(SAFE)::value;
+      if constexpr (!F64) {
 #pragma unroll
-      for (int e = 0; e < 8; ++e) {
-        const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
-        const unsigned off = dm + (cw[e] & kPkOffMask);
-        const bool big = !(fabsf(ts) < kPkCap);
-        const int qi = big ? 0 : __float2int_rn(ts);
-        const int old = pk_atom_add(lo_base + off, qi);
-        const unsigned nw = (unsigned)old + (unsigned)qi;
-        rare = (rare << 1) | (unsigned)(big | ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0));
-      }
-    } else {
-      // |term| < 2^62 quanta: both limbs always added (no branch); the high limb's wrap is
-      // detected from its returned old value.  The low limbs of a group of PG terms go first:
-      // a high limb's operand waits for its low limb's returned value (the carry) and the
-      // volatile atomics keep program order, so alternating lo / hi per term would chain 16
-      // shared-memory round trips per window
-#pragma unroll
-      for (int g0 = 0; g0 < 8; g0 += kPk1FG) {
-        unsigned l[kPk1FG], ol[kPk1FG], off[kPk1FG];
-        int hh[kPk1FG];
-        bool big[kPk1FG];
-#pragma unroll
-        for (int k = 0; k < kPk1FG; ++k) {
-          const int e = g0 + k;
+        for (int e = 0; e < 8; ++e) {
           const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
-          off[k] = dm + (cw[e] & kPkOffMask);
-          big[k] = !(fabs(ts) < 4.6e18);
-          const long long I = big[k] ? 0ll : __double2ll_rn(ts);
-          l[k] = (unsigned)I;
-          hh[k] = (int)(I >> 32);
+          const unsigned off = dm + (cw[e] & kPkOffMask);
+          const bool big = S ? false : !(fabsf(ts) < kPkCap);
+          const int qi = big ? 0 : __float2int_rn(ts);
+          const int old = pk_atom_add(lo_base + off, qi);
+          const unsigned nw = (unsigned)old + (unsigned)qi;
+          rare = (rare << 1) | (unsigned)(big | ((int)(((unsigned)old ^ nw) & ((unsigned)qi ^ nw)) < 0));
         }
+      } else {
+        // |term| < 2^62 quanta: both limbs always added (no branch); the high limb's wrap is
+        // detected from its returned old value.  The low limbs of a group of PG terms go first:
+        // a high limb's operand waits for its low limb's returned value (the carry) and the
+        // volatile atomics keep program order, so alternating lo / hi per term would chain 16
+        // shared-memory round trips per window
 #pragma unroll
-        for (int k = 0; k < kPk1FG; ++k) ol[k] = pk_atom_addu(lo_base + off[k], l[k]);
+        for (int g0 = 0; g0 < 8; g0 += kPk1FG) {
+          unsigned l[kPk1FG], ol[kPk1FG], off[kPk1FG];
+          int hh[kPk1FG];
+          bool big[kPk1FG];
 #pragma unroll
-        for (int k = 0; k < kPk1FG; ++k) {
-          const int h = hh[k] + ((ol[k] + l[k] < ol[k]) ? 1 : 0);
-          const int oh = pk_atom_add(hi_base + off[k], h);
-          const unsigned nw = (unsigned)oh + (unsigned)h;
-          const bool ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
-          rare = (rare << 1) | (unsigned)(big[k] | ovf);
+          for (int k = 0; k < kPk1FG; ++k) {
+            const int e = g0 + k;
+            const T ts = xv[e] * pk_lds(qaddr(qs_base, cw[e]), T(0));
+            off[k] = dm + (cw[e] & kPkOffMask);
+            big[k] = S ? false : !(fabs(ts) < 4.6e18);
+            const long long I = big[k] ? 0ll : __double2ll_rn(ts);
+            l[k] = (unsigned)I;
+            hh[k] = (int)(I >> 32);
+          }
+#pragma unroll
+          for (int k = 0; k < kPk1FG; ++k) ol[k] = pk_atom_addu(lo_base + off[k], l[k]);
+#pragma unroll
+          for (int k = 0; k < kPk1FG; ++k) {
+            const int h = hh[k] + ((ol[k] + l[k] < ol[k]) ? 1 : 0);
+            const int oh = pk_atom_add(hi_base + off[k], h);
+            const unsigned nw = (unsigned)oh + (unsigned)h;
+            const bool ovf = (int)(((unsigned)oh ^ nw) & ((unsigned)h ^ nw)) < 0;
+            rare = (rare << 1) | (unsigned)(big[k] | ovf);
+          }
         }
       }
-    }
+    };
+    if (safe) body(std::true_type{});
+    else body(std::false_type{});
     if (rare) {  // bit 7 - e flags entry e
 #pragma unroll
       for (int e = 0; e < 8; ++e) {
@@ -599,14 +606,22 @@ __global__ void __launch_bounds__(BS1, 1) k_pk1(const Pk1Args a) {
     pk_sts(qs_base + TS * (lane + 32), pk_lds_v(qu_base + TS * (lane + 32), T(0)) * s);
     __syncwarp();
     const int len = seg_len(D);
+    // fp64 only (C3 0.821 -> 0.785 ms); the fp32 pass at 64 registers spills with both paths
+    // (S3 0.487 -> 0.501 ms), so it keeps the checked one
+    bool safe = false;
+    if constexpr (F64) {
+      const double xm = (double)__uint_as_float(D.w);  // the tile's max |x| (+Inf if not finite)
+      safe = __all_sync(0xffffffffu, fabs(pk_lds_v(qs_base + TS * lane, T(0))) * xm < 4.0e18 &&
+                                         fabs(pk_lds_v(qs_base + TS * (lane + 32), T(0))) * xm < 4.0e18);
+    }
     if (len <= 256) {
-      if (len > 0) scat_win(cw, xv, 0, len);
+      if (len > 0) scat_win(cw, xv, 0, len, safe);
     } else {
       for (int s0 = 0; s0 < len; s0 += 256) {
         uint32_t c2[8];
         T x2[8];
         win_glob(D, s0, c2, x2);
-        scat_win(c2, x2, s0, len);
+        scat_win(c2, x2, s0, len, safe);
       }
     }
     if (NS > 0) {
