@@ -255,11 +255,12 @@ __device__ __forceinline__ void pk_put(double* x, const uint4& u) {
 // shared memory, no exchange).  Every tile (<= 256 entries) is loaded ONCE: the dot, q and the
 // scatter all run from the registers that hold it (a7) -- X is read from HBM once.
 //
-// Staging (round 2c): each warp keeps a ring of NS tile slots in shared memory, filled by TMA
-// bulk copies (cp.async.bulk, one per array, completion on the slot's mbarrier) NS tiles ahead
-// of the tile being processed, so the HBM latency of the stream is off the warp's critical
-// path (the round-2b pass loaded every tile into registers itself: 20 % of its stall samples
-// waited on that load, ncu r02c).  The window of a tile is stored lane-interleaved (pack
+// Staging (round 2c; fp64 -- fp32's 32 warps hide the load themselves): each warp keeps a
+// ring of NS tile slots in shared memory, filled by TMA bulk copies (cp.async.bulk of the
+// tile's column words, values and the v of its rows, completion on the slot's mbarrier) NS
+// tiles ahead of the tile being processed, so the HBM latency of the stream is off the warp's
+// critical path (the round-2b pass loaded every tile into registers itself: 20 % of its stall
+// samples waited on that load, ncu r02c).  Descriptors arrive in batches of 16 by cp.async.  The window of a tile is stored lane-interleaved (pack
 // time, k_pk_interleave): the 16-byte piece k of lane l's 8 entries at (k G + l) 16 bytes, G =
 // the tile's groups of 8 -- a warp's 16-byte shared loads then touch 8 distinct bank quads per
 // phase (conflict-free), and lane l still holds the logical entries 8l..8l+7.  A longer segment
