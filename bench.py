@@ -31,16 +31,26 @@ import threading
 import time
 
 # stdout carries exactly one JSON line.  Native libraries (NCCL's version banner with any
-# NCCL_DEBUG level) write to fd 1 directly, so fd 1 is pointed at stderr for the whole run and
-# the JSON line goes to a duplicate of the original stdout (emit()).
-_JSON_OUT = os.fdopen(os.dup(1), "w")
-sys.stdout.flush()
-os.dup2(2, 1)
+# NCCL_DEBUG level) write to fd 1 directly, so when bench.py runs as the program, fd 1 is
+# pointed at stderr for the whole run and the JSON line goes to a duplicate of the original
+# stdout (emit()); tools that import bench keep their stdout.
+_JSON_OUT = None
+
+
+def _stdout_to_stderr():
+    global _JSON_OUT
+    sys.stdout.flush()
+    _JSON_OUT = os.fdopen(os.dup(1), "w")
+    os.dup2(2, 1)
 
 
 def emit(obj):
-    _JSON_OUT.write(json.dumps(obj) + "\n")
-    _JSON_OUT.flush()
+    line = json.dumps(obj)
+    if _JSON_OUT is None:
+        print(line, flush=True)
+    else:
+        _JSON_OUT.write(line + "\n")
+        _JSON_OUT.flush()
 
 
 import numpy as np
@@ -741,6 +751,7 @@ def run_unfused(args):
 
 
 def main():
+    _stdout_to_stderr()
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
