@@ -453,3 +453,27 @@ def test_packed1_unaligned_v_and_w_alias_z(cuda_dev, dt):
     plan(None, y.to(cuda_dev), v.to(cuda_dev), zw, 1.0, 2.0, w=zw)
     torch.cuda.synchronize()
     assert_bitexact(zw, ref, f"packed1 {dt} w aliases z")
+
+
+@pytest.mark.parametrize("dt,n,ns", [("f64", 1000, "0"), ("f64", 1000, "1"), ("f64", 1000, "2"), ("f32", 1000, "2"),
+                                     ("f64", 12_000, None), ("f32", 23_000, None)])
+def test_packed1_ring_depths_and_widest_block(cuda_dev, monkeypatch, dt, n, ns):
+    """k_pk1 with every ring depth (0: windows from global memory, fp64 too) and at the widest
+    single block (the ring no longer fits next to y and the partial w): integer twins bit-exact,
+    long rows included."""
+    m = 3_001
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rp, ci, va = synth.csr(m, n, dt, ("uniform", 0, 400), kind="int_pm12", seed=29)
+    y = synth.vector(n, dt, kind="int_small", seed=29, stream=synth.S_Y)
+    v = synth.vector(m, dt, kind="int_pos", seed=29, stream=synth.S_V)
+    z = synth.vector(n, dt, kind="int_small", seed=29, stream=synth.S_Z)
+    if ns is not None:
+        monkeypatch.setenv("FP_PK1_NS", ns)
+    plan = fp.CsrPlan(rp.to(cuda_dev), ci.to(cuda_dev), n, tdt)
+    plan.pack(va.to(cuda_dev))
+    assert plan.launch.variant == 19 and plan.launch.cluster == 1
+    for args in ((y, v, z, 1.0, 1.0), (None, v, z, -1.0, 0.5)):
+        ref, mag = oracle.csr(m, n, rp, ci, va, *args)
+        if dt == "f32" and mag.max() >= 2**24:
+            continue
+        assert_bitexact(run(plan, cuda_dev, *args), ref, f"packed1 {dt} n={n} ns={ns}")
