@@ -1397,10 +1397,11 @@ __global__ void k_pk_interleave(int64_t nseg, const uint4* __restrict__ desc, ui
 
 // (5) warp-quad partition: tile ranges of equal nonzero + row cost
 __global__ void k_pk_partition(int64_t ntiles, int nq, const int64_t* __restrict__ tile_row,
-                               const int64_t* __restrict__ rowptr, int32_t* __restrict__ wtile) {
+                               const int64_t* __restrict__ rowptr, int32_t* __restrict__ wtile, int rc, int tc) {
   const int qi = blockIdx.x * blockDim.x + threadIdx.x;
   if (qi > nq) return;
-  auto cost = [&](int64_t t) { const int64_t r = tile_row[t]; return rowptr[r] - rowptr[0] + kPkRowCost * r; };
+  // work before tile t: its nonzeros + rc per row + tc per tile
+  auto cost = [&](int64_t t) { const int64_t r = tile_row[t]; return rowptr[r] - rowptr[0] + rc * r + tc * t; };
   const int64_t total = cost(ntiles);
   const int64_t target = (int64_t)((__int128)total * qi / nq);
   int64_t lo = 0, hi = ntiles;  // smallest t with cost(t) >= target
@@ -1685,7 +1686,12 @@ fp_status packed_build(int64_t m, int64_t n, int64_t nnz, const int64_t* rowptr,
   const int nq = groups * (bs / 32);
   if (ntiles >= INT32_MAX) return fail(cudaErrorInvalidValue, "too many tiles");
   PK_TRY(cudaMalloc((void**)&p->wtile, (size_t)(nq + 1) * 4), "alloc");
-  k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile);
+  {  // measurement knobs: FP_PK_ROWCOST (default kPkRowCost), FP_PK_TILECOST (default 0)
+    const char* r = std::getenv("FP_PK_ROWCOST");
+    const char* t = std::getenv("FP_PK_TILECOST");
+    k_pk_partition<<<(nq + 1 + 127) / 128, 128, 0, s>>>(ntiles, nq, tile_row, rowptr, p->wtile,
+                                                         r ? std::atoi(r) : kPkRowCost, t ? std::atoi(t) : 0);
+  }
   // per-call state: exchange slots (zero), the call counter (starts at 1), partials, spill (zero)
   const int ns = cs > 1 ? PkSlots<1>::NS : 1;
   const size_t xbytes = (size_t)groups * (bs / 32) * ns * (cs + 1) * kPkRows * 8;
